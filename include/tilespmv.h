@@ -1,0 +1,150 @@
+/*
+ * tilespmv.h -- C ABI of the B200-native TileSpMV hot path.
+ *
+ * Operation (Alg. 1): y = A * x in fp64
+ * (P:237), A sparse m x n given in CSR, converted to the paper's
+ * two-level 16x16 tiled storage with per-tile formats chosen by
+ * the TileSpMV_ADPT rules and, by default, the DeferredCOO
+ * extraction of all COO data into a CSR remainder.  The
+ * preprocess-then-multiply split follows P:285-289.
+ *
+ * Conventions for every entry point
+ *   - plain pointers and sizes only; `stream` is a cudaStream_t passed as
+ *     void* (NULL = the legacy default stream);
+ *   - "d_" pointers are device memory on the device current at create time,
+ *     "h_" pointers are host memory;
+ *   - every call returns an int status: TILESPMV_OK (0) or a negative code
+ *     below.  Nothing throws or aborts across the ABI; the last error message
+ *     of the calling thread is available from tilespmv_last_error().
+ */
+#ifndef TILESPMV_H
+#define TILESPMV_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* status codes */
+#define TILESPMV_OK 0
+#define TILESPMV_INVALID_ARG (-1)       /* null pointer, negative size, bad mode/array id,
+                                           x/y overlap, handle used on another device   */
+#define TILESPMV_NOT_CANONICAL (-2)     /* rowptr not monotone / not 0..nnz, column out of
+                                           range, or columns not strictly increasing      */
+#define TILESPMV_OVERFLOW (-3)          /* nnz >= 2^31, m or n >= 2^31, payload >= 64 GiB */
+#define TILESPMV_OOM (-4)               /* device or host allocation failed               */
+#define TILESPMV_CUDA (-5)              /* any other CUDA runtime error                   */
+
+/* methods of P:177 (+ the size switch of P:235) */
+#define TILESPMV_MODE_ADPT 0      /* TileSpMV_ADPT: adaptive format per tile, no extraction */
+#define TILESPMV_MODE_DEFERRED 1  /* TileSpMV_DeferredCOO: COO data -> CSR remainder (default) */
+#define TILESPMV_MODE_AUTO 2      /* DEFERRED iff nnz >= 1.8e6 (reading R18), else ADPT */
+#define TILESPMV_MODE_FORCE_CSR 3 /* TileSpMV_CSR: every tile CSR */
+
+/* tile format codes, in the order of P:20 / P:96 */
+#define TILESPMV_FMT_CSR 0
+#define TILESPMV_FMT_COO 1
+#define TILESPMV_FMT_ELL 2
+#define TILESPMV_FMT_HYB 3
+#define TILESPMV_FMT_DNS 4
+#define TILESPMV_FMT_DNSROW 5
+#define TILESPMV_FMT_DNSCOL 6
+
+/* arrays for tilespmv_export (canonical layout, DESIGN.md §"Canonical layout") */
+#define TILESPMV_ARR_TILEPTR 0    /* int32  [tilem+1]   tiles per tile row, prefix        */
+#define TILESPMV_ARR_TILECOLIDX 1 /* int32  [numtile]   tile column index                 */
+#define TILESPMV_ARR_TILENNZ 2    /* int32  [numtile+1] prefix of nonzeros held per tile  */
+#define TILESPMV_ARR_TILEFMT 3    /* uint8  [numtile]   format code                               */
+#define TILESPMV_ARR_TILEAUX 4    /* uint8  [numtile]   ELL/HYB width, DnsRow/DnsCol count, else 0 */
+#define TILESPMV_ARR_TILEOFF 5    /* uint32 [numtile+1] payload offset in 16-byte units          */
+#define TILESPMV_ARR_PAYLOAD 6    /* uint8  [payload_bytes] level-2 per-tile payloads */
+#define TILESPMV_ARR_REMROWPTR 7  /* int32  [m+1]       remainder CSR; empty if no extraction */
+#define TILESPMV_ARR_REMCOL 8     /* int32  [rem_nnz]   global column indices                     */
+#define TILESPMV_ARR_REMVAL 9     /* double [rem_nnz]                                             */
+
+typedef struct tilespmv_matrix *tilespmv_handle_t; /* opaque; owns all its device storage */
+
+typedef struct {
+    int32_t mode;     /* TILESPMV_MODE_*; default DEFERRED                               */
+    int32_t validate; /* 1 (default): check the CSR is canonical; 0: trust the caller   */
+} tilespmv_opts_t;
+
+typedef struct {
+    int64_t m, n, nnz;
+    int64_t tilem, tilen; /* ceil(m/16), ceil(n/16) */
+    int64_t numtile;      /* tiles stored (after extraction) */
+    int32_t mode;         /* resolved mode (AUTO never appears here) */
+    int32_t device;
+    int64_t sel_tiles[7], sel_nnz[7];   /* formats chosen by the ADPT rules, before extraction */
+    int64_t kept_tiles[7], kept_nnz[7]; /* tiles stored and the nonzeros they hold */
+    int64_t rem_nnz;                    /* nonzeros in the CSR remainder */
+    int64_t payload_bytes;              /* level-2 payload (16-byte aligned per tile) */
+    int64_t meta_bytes;                 /* level-1 arrays read per SpMV */
+    int64_t alg_bytes;                  /* algorithmic bytes per SpMV (DESIGN.md §"Bytes model") */
+    int64_t flops;                      /* 2 * nnz */
+    int64_t num_items;                  /* warp work items of the SpMV schedule */
+    int64_t num_split_rows;             /* tile rows split over several items */
+    int64_t device_bytes;               /* device memory owned by the handle */
+    double create_ms;                   /* wall time of tilespmv_create_from_csr */
+} tilespmv_info_t;
+
+/* Build a tiled matrix from a canonical device CSR ("converting a basic
+ * CSR matrix to our tile form").  All preprocessing runs on the GPU.
+ *   m, n        rows / columns (0 allowed; m,n < 2^31)
+ *   nnz         number of stored entries (< 2^31); must equal d_rowptr[m]
+ *   d_rowptr    int32[m+1], d_colidx int32[nnz], d_val double[nnz]: device,
+ *               caller-owned, read only during this call.  Explicit zeros
+ *               are entries.  d_colidx/d_val may be NULL when nnz == 0.
+ *   opts        NULL = defaults {DEFERRED, validate=1}
+ *   stream      work is queued on it; the call synchronises it before return,
+ *               so the inputs may be freed immediately afterwards.
+ * On success *out receives a handle bound to the current device.
+ * Errors: INVALID_ARG, NOT_CANONICAL (only detected with validate=1),
+ * OVERFLOW, OOM, CUDA.  On error *out is set to NULL and nothing leaks.     */
+int tilespmv_create_from_csr(tilespmv_handle_t *out, int64_t m, int64_t n, int64_t nnz,
+                             const int32_t *d_rowptr, const int32_t *d_colidx,
+                             const double *d_val, const tilespmv_opts_t *opts, void *stream);
+
+/* y = A * x (Alg. 1: y_i <- 0, then y_i += a_ij * x_j).
+ *   d_x double[n] device, read; must be finite (reading R19).
+ *   d_y double[m] device, fully overwritten (no alpha/beta); must not overlap x.
+ * Asynchronous on `stream`: one kernel launch, no host synchronisation.
+ * The result is bitwise deterministic run to run.  Runs on the same handle
+ * must be serialised (the handle owns one split-row workspace).             */
+int tilespmv_run(tilespmv_handle_t h, const double *d_x, double *d_y, void *stream);
+
+/* Host-buffer variant: copies h_x (double[n]) to a handle-owned device
+ * buffer, runs, copies y back to h_y (double[m]) and synchronises `stream`.
+ * h_x / h_y should be page-locked for asynchronous copies.                  */
+int tilespmv_run_host(tilespmv_handle_t h, const double *h_x, double *h_y, void *stream);
+
+/* Release all device storage; NULL is a no-op returning TILESPMV_OK. */
+int tilespmv_destroy(tilespmv_handle_t h);
+
+/* Statistics of the tiled matrix (format histogram P:229, space P:279). */
+int tilespmv_get_info(tilespmv_handle_t h, tilespmv_info_t *info);
+
+/* Size in bytes of an exported array (TILESPMV_ARR_*), or a negative status. */
+int64_t tilespmv_export_size(tilespmv_handle_t h, int32_t which);
+
+/* Copy one array of the canonical tiled layout to host memory (synchronous);
+ * `bytes` must equal tilespmv_export_size(h, which).  Used for bit-exact
+ * parity against the reference tiler.                                        */
+int tilespmv_export(tilespmv_handle_t h, int32_t which, void *host_dst, size_t bytes);
+
+/* Static description of a status code. */
+const char *tilespmv_status_string(int status);
+
+/* Message of the last failing call on this thread ("" if none). */
+const char *tilespmv_last_error(void);
+
+/* Name of the SpMV kernel symbol (for profiler filters) and its launch shape
+ * for this handle: grid CTAs, threads per CTA, dynamic shared memory bytes. */
+int tilespmv_launch_shape(tilespmv_handle_t h, int32_t *grid, int32_t *block, int32_t *smem_bytes);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* TILESPMV_H */

@@ -1,0 +1,87 @@
+// internal.cuh -- shared definitions of the CUDA product path (tiler, SpMV
+// kernel, C ABI).  Nothing here is shared with oracle/.
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <string>
+
+#include "../../include/tilespmv.h"
+
+namespace tsp {
+
+constexpr int kTile = 16;  // P:20 "the size is always 16 by 16"
+
+// Format codes (same numbering as the ABI, P:96 order).
+enum : uint8_t { F_CSR = 0, F_COO = 1, F_ELL = 2, F_HYB = 3, F_DNS = 4, F_DNSROW = 5, F_DNSCOL = 6 };
+
+// ---------------------------------------------------------------------------
+// SpMV schedule.  A work item is a byte-bounded piece of one tile row: a run
+// of at most kItemTiles consecutive tiles whose payload fits kItemPayload
+// bytes, and/or at most kItemRem remainder entries of the tile row's 16 rows.
+// A tile row split over several items writes per-item partials that the last
+// finishing item sums in item order (deterministic; replaces the atomic
+// merge of tbalance).  Item boundaries depend only on the tile row's
+// own content, so a tile-row-sharded run reproduces the 1-GPU y bitwise.
+// ---------------------------------------------------------------------------
+constexpr int kItemTiles = 16;
+constexpr int kItemPayload = 10240;  // bytes; one FEM tile row = 5 Dns tiles
+constexpr int kItemRem = 256;        // remainder entries per item
+constexpr int kShortRow = 8;         // remainder rows up to this length: 2 lanes per row
+
+struct __align__(16) Item {
+    int32_t I;        // tile row
+    int32_t tb;       // first tile
+    int32_t kb, ke;   // remainder entry range
+    uint32_t offb;    // payload offset of tile tb (16-byte units)
+    uint32_t offe;    // payload offset one past the last tile
+    int32_t split;    // split-row index, or -1 if the item covers its whole tile row
+    int32_t part_nt;  // (part index within the split row) | (number of tiles << 24)
+};
+
+struct Matrix {
+    int device = 0;
+    int64_t m = 0, n = 0, nnz = 0, tilem = 0, tilen = 0, numtile = 0;
+    int32_t mode = TILESPMV_MODE_DEFERRED;
+    // level 1 + format bytes + payload offsets
+    int32_t *tilePtr = nullptr, *tileColIdx = nullptr, *tileNnz = nullptr;
+    uint8_t *tileFmt = nullptr, *tileAux = nullptr;
+    uint32_t *tileOff = nullptr;
+    // level 2
+    uint8_t *payload = nullptr;
+    int64_t payload_bytes = 0;
+    // DeferredCOO remainder
+    int32_t *remRowPtr = nullptr, *remCol = nullptr;
+    double *remVal = nullptr;
+    int64_t rem_nnz = 0;
+    // SpMV schedule
+    Item *items = nullptr;
+    int64_t num_items = 0;
+    int2 *split_info = nullptr;  // {first partial slot, number of parts}
+    int64_t num_split = 0;
+    double *partials = nullptr;
+    int32_t *counters = nullptr;
+    // host-staging buffers for tilespmv_run_host
+    double *xstage = nullptr, *ystage = nullptr;
+    // statistics
+    int64_t sel_tiles[7] = {0}, sel_nnz[7] = {0}, kept_tiles[7] = {0}, kept_nnz[7] = {0};
+    int64_t device_bytes = 0;
+    double create_ms = 0;
+    // launch shape
+    int grid = 0, block = 0, smem = 0;
+};
+
+// status helpers (thread-local last error)
+int set_error(int status, const std::string &msg);
+int cuda_status(cudaError_t e, const char *what);
+
+// tiler.cu
+int build_tiled(Matrix &M, const int32_t *d_rowptr, const int32_t *d_colidx, const double *d_val,
+                int validate, cudaStream_t stream);
+// spmv.cu
+int build_schedule(Matrix &M, cudaStream_t stream);
+int configure_launch(Matrix &M);
+int launch_spmv(const Matrix &M, const double *d_x, double *d_y, cudaStream_t stream);
+
+}  // namespace tsp

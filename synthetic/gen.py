@@ -184,21 +184,25 @@ def lap2d(nx: int = 64, ny: int | None = None, values: str = "stencil",
 # ----------------------------------------------------------------------------
 
 def stencil27(nx: int = 200, values: str = "uniform", seed: int = 7,
-              ny: int | None = None, nz: int | None = None) -> CSR:
+              ny: int | None = None, nz: int | None = None,
+              row_range: tuple[int, int] | None = None) -> CSR:
     """Row i = x + nx*y + nx*ny*z.  values='stencil' puts 26 on the diagonal
-    and -1 on the 26 neighbours; 'uniform'/'int' use the counter RNG."""
+    and -1 on the 26 neighbours; 'uniform'/'int' use the counter RNG.
+    row_range=(r0, r1) generates only rows [r0, r1) (rebased, n unchanged),
+    identical to the same rows of the full matrix."""
     ny = nx if ny is None else ny
     nz = nx if nz is None else nz
-    m = nx * ny * nz
+    n = nx * ny * nz
+    r0, r1 = (0, n) if row_range is None else row_range
     plane = nx * ny
     # column order is increasing in (dz, dy, dx) lexicographic order
     offsets = [(dz, dy, dx) for dz in (-1, 0, 1) for dy in (-1, 0, 1)
                for dx in (-1, 0, 1)]
     rows_out, cols_out, vals_out = [], [], []
-    zchunk = max(1, (1 << 22) // max(plane, 1))
-    for z0 in range(0, nz, zchunk):
-        z1 = min(nz, z0 + zchunk)
-        i = np.arange(z0 * plane, z1 * plane, dtype=np.int64)
+    chunk = 1 << 22
+    for c0 in range(r0, r1, chunk):
+        c1 = min(r1, c0 + chunk)
+        i = np.arange(c0, c1, dtype=np.int64)
         x = i % nx
         y = (i // nx) % ny
         z = i // plane
@@ -219,15 +223,15 @@ def stencil27(nx: int = 200, values: str = "uniform", seed: int = 7,
         if values == "stencil":
             v = np.where(r == c, 26.0, -1.0)
         else:
-            v = values_for(seed, r, c, m, values)
-        rows_out.append(r.astype(np.int32))
+            v = values_for(seed, r, c, n, values)
+        rows_out.append((r - r0).astype(np.int32))
         cols_out.append(c.astype(np.int32))
         vals_out.append(v)
-    rows = np.concatenate(rows_out)
-    cols = np.concatenate(cols_out)
-    vals = np.concatenate(vals_out)
+    rows = np.concatenate(rows_out) if rows_out else np.zeros(0, np.int32)
+    cols = np.concatenate(cols_out) if cols_out else np.zeros(0, np.int32)
+    vals = np.concatenate(vals_out) if vals_out else np.zeros(0)
     del rows_out, cols_out, vals_out
-    return csr_from_sorted(m, m, rows, cols, vals, f"stencil27_{nx}x{ny}x{nz}")
+    return csr_from_sorted(r1 - r0, n, rows, cols, vals, f"stencil27_{nx}x{ny}x{nz}")
 
 
 # ----------------------------------------------------------------------------

@@ -1,0 +1,85 @@
+"""CPU-side checks of the boundary: the C-ABI library loads and exports every
+symbol include/tilespmv.h declares; the product package never touches
+oracle/; without a CUDA device the product path fails loudly."""
+import ast
+import os
+import re
+import subprocess
+
+import pytest
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+HEADER = os.path.join(ROOT, "include", "tilespmv.h")
+PKG = os.path.join(ROOT, "paper_conf_ipps_niuldj0t21_b200")
+
+
+def declared_functions():
+    src = open(HEADER).read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    return sorted(set(re.findall(r"\b(tilespmv_[a-z_]+)\s*\(", src)))
+
+
+def test_header_declares_the_boundary():
+    names = declared_functions()
+    for required in ("tilespmv_create_from_csr", "tilespmv_run", "tilespmv_destroy"):
+        assert required in names
+
+
+def test_library_exports_every_declared_symbol():
+    from paper_conf_ipps_niuldj0t21_b200 import EXPORTED_SYMBOLS, load
+    L = load()
+    names = declared_functions()
+    assert sorted(EXPORTED_SYMBOLS) == names
+    for n in names:
+        assert hasattr(L, n), n
+    out = subprocess.run(["nm", "-D", "--defined-only", L._name], capture_output=True, text=True).stdout
+    for n in names:
+        assert re.search(rf"\bT {n}$", out, flags=re.M), n
+
+
+def test_status_strings_without_gpu():
+    from paper_conf_ipps_niuldj0t21_b200 import load
+    L = load()
+    assert L.tilespmv_status_string(0) == b"ok"
+    assert L.tilespmv_status_string(-2) == b"input CSR is not canonical"
+    assert L.tilespmv_destroy(None) == 0
+
+
+def test_null_arguments_rejected_without_gpu():
+    import ctypes
+    from paper_conf_ipps_niuldj0t21_b200 import load
+    L = load()
+    assert L.tilespmv_create_from_csr(None, 1, 1, 0, None, None, None, None, None) == -1
+    h = ctypes.c_void_p()
+    assert L.tilespmv_create_from_csr(ctypes.byref(h), -1, 1, 0, None, None, None, None, None) == -1
+    assert L.tilespmv_create_from_csr(ctypes.byref(h), 1 << 31, 1, 0, None, None, None, None, None) == -3
+    assert L.tilespmv_run(None, None, None, None) == -1
+
+
+def test_product_package_does_not_import_oracle():
+    for dirpath, _, files in os.walk(PKG):
+        for f in files:
+            path = os.path.join(dirpath, f)
+            if f.endswith(".py"):
+                tree = ast.parse(open(path).read())
+                for node in ast.walk(tree):
+                    if isinstance(node, ast.Import):
+                        assert not any(a.name.startswith("oracle") for a in node.names), path
+                    if isinstance(node, ast.ImportFrom):
+                        assert not (node.module or "").startswith("oracle"), path
+            if f.endswith((".cu", ".cuh", ".h", ".cpp")):
+                for line in open(path):
+                    if line.lstrip().startswith("#include"):
+                        assert "oracle" not in line, path
+
+
+def test_no_cpu_fallback():
+    import numpy as np
+    import torch
+    if torch.cuda.is_available():
+        pytest.skip("a GPU is present")
+    from paper_conf_ipps_niuldj0t21_b200 import TiledMatrix, TileSpMVError
+    from synthetic import gen
+    with pytest.raises(TileSpMVError, match="no CUDA device"):
+        TiledMatrix.from_host_csr(gen.identity(4))
+    assert np  # silence
