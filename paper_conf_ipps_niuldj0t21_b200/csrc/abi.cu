@@ -36,7 +36,7 @@ static void free_matrix(tilespmv_matrix *M) {
     if (cur != M->device) cudaSetDevice(M->device);
     void *ptrs[] = {M->tilePtr, M->tileColIdx, M->tileNnz, M->tileFmt, M->tileAux, M->tileOff,
                     M->payload, M->remRowPtr, M->remCol, M->remVal, M->items, M->split_info,
-                    M->partials, M->counters, M->xstage, M->ystage};
+                    M->partials, M->counters, M->xstage, M->ystage, M->tdesc, M->cta_begin};
     for (void *p : ptrs)
         if (p) cudaFree(p);
     if (cur >= 0 && cur != M->device) cudaSetDevice(cur);
@@ -111,6 +111,7 @@ int tilespmv_create_from_csr(tilespmv_handle_t *out, int64_t m, int64_t n, int64
                                            : o.mode;
     int rc = build_tiled(*M, d_rowptr, d_colidx, d_val, o.validate, st);
     if (!rc) rc = build_schedule(*M, st);
+    if (!rc) rc = build_tdesc(*M, st);
     if (!rc) rc = configure_launch(*M);
     if (!rc) {
         cudaError_t e = cudaStreamSynchronize(st);

@@ -68,7 +68,11 @@ struct Matrix {
     int64_t sel_tiles[7] = {0}, sel_nnz[7] = {0}, kept_tiles[7] = {0}, kept_nnz[7] = {0};
     int64_t device_bytes = 0;
     double create_ms = 0;
+    // v2 kernel inputs derived from the canonical arrays
+    uint2 *tdesc = nullptr;        // 8-byte packed tile descriptors
+    int64_t *cta_begin = nullptr;  // contiguous item chunk per CTA
     // launch shape
+    int kernel_version = 2;
     int grid = 0, block = 0, smem = 0;
 };
 
@@ -81,6 +85,7 @@ int build_tiled(Matrix &M, const int32_t *d_rowptr, const int32_t *d_colidx, con
                 int validate, cudaStream_t stream);
 // spmv.cu
 int build_schedule(Matrix &M, cudaStream_t stream);
+int build_tdesc(Matrix &M, cudaStream_t stream);
 int configure_launch(Matrix &M);
 int launch_spmv(const Matrix &M, const double *d_x, double *d_y, cudaStream_t stream);
 

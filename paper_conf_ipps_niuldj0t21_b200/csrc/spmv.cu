@@ -59,6 +59,8 @@ struct Params {
     const double *x;
     double *y;
     int64_t m, n;
+    const uint2 *tdesc;        // v2: packed tile descriptors
+    const int64_t *cta_begin;  // v2: contiguous item chunk per CTA
 };
 
 // ---------------------------------------------------------------- PTX -----
@@ -99,6 +101,7 @@ __device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
     while (!mbar_try_wait(bar, parity)) {
     }
 }
+__device__ __forceinline__ int64_t imin64(int64_t a, int64_t b) { return a < b ? a : b; }
 __device__ __forceinline__ int nib(const uint8_t *base, int idx) {
     return (base[idx >> 1] >> ((idx & 1) * 4)) & 15;
 }
@@ -191,18 +194,28 @@ __device__ __forceinline__ void tile_spmv(int fmt, int aux, int nz, const uint8_
         }
         break;
     }
-    case F_CSR: {  // two lanes per row (Alg. 2)
+    case F_CSR: {  // two lanes per row (Alg. 2); warp-uniform trip count
         const uint8_t *rp = P + 8 * nz;
         const uint8_t *ci = rp + 16;
-        int beg = rp[r], end = r < 15 ? rp[r + 1] : nz;
-        for (int j = beg + h; j < end; j += 2) acc = fma(V[j], X[nib(ci, j)], acc);
+        const int beg = rp[r] + h, end = r < 15 ? rp[r + 1] : nz;
+        const int trips = __reduce_max_sync(FULL, (unsigned)max(0, (end - beg + 1) >> 1));
+#pragma unroll 2
+        for (int i = 0; i < trips; ++i) {
+            const int j = beg + 2 * i;
+            if (j < end) acc = fma(V[j], X[nib(ci, j)], acc);
+        }
         break;
     }
     case F_COO: {  // lanes of row r pick their entries, no atomics
         const uint8_t *rc = P + 8 * nz;
-        for (int j = h; j < nz; j += 2) {
-            int b = rc[j];
-            if ((b >> 4) == r) acc = fma(V[j], X[b & 15], acc);
+        const int trips = (nz + 1) >> 1;
+#pragma unroll 2
+        for (int i = 0; i < trips; ++i) {
+            const int j = h + 2 * i;
+            if (j < nz) {
+                const int b = rc[j];
+                if ((b >> 4) == r) acc = fma(V[j], X[b & 15], acc);
+            }
         }
         break;
     }
@@ -215,9 +228,14 @@ __device__ __forceinline__ void tile_spmv(int fmt, int aux, int nz, const uint8_
             int s = lane + 32 * i;
             if (s < 16 * w) acc = fma(V[s], X[nib(ei, s)], acc);
         }
-        for (int j = h; j < kc; j += 2) {
-            int b = rc[j];
-            if ((b >> 4) == r) acc = fma(CV[j], X[b & 15], acc);
+        const int trips = (kc + 1) >> 1;
+#pragma unroll 2
+        for (int i = 0; i < trips; ++i) {
+            const int j = h + 2 * i;
+            if (j < kc) {
+                const int b = rc[j];
+                if ((b >> 4) == r) acc = fma(CV[j], X[b & 15], acc);
+            }
         }
         break;
     }
@@ -339,6 +357,312 @@ __global__ void __launch_bounds__(kWarps * 32) tilespmv_fp64_kernel(const Params
         }
         __syncwarp();  // shared slot free before the next item's bulk copy
     }
+}
+
+
+// ======================================================================
+// v2: warp-specialised persistent kernel.  Per CTA (one per SM): one
+// producer warp streams the CTA's contiguous chunk of work items into a
+// shared-memory byte ring with TMA bulk copies (payload, packed 8-byte tile
+// descriptors, remainder rowptr/col/val), signalling a per-slot "full"
+// mbarrier through its transaction count; C consumer warps compute from
+// shared memory and release the slot through its "empty" mbarrier.  Slot s
+// is always served by consumer s mod C (S is a multiple of C), so every
+// consumer waits on its own slots in order and parity waits cannot alias.
+// ======================================================================
+
+// bytes of one item in the ring: payload | descriptors | rowptr | col | val
+struct RingParts {
+    uint32_t pay, dsc, rp, col, val, total;
+    uint32_t dsc_skew, col_skew, val_skew;
+};
+
+__device__ __forceinline__ uint32_t up16(uint32_t v) { return (v + 15u) & ~15u; }
+
+__device__ __forceinline__ RingParts ring_parts(const Item &it, int64_t m) {
+    RingParts r;
+    const int nt = it.part_nt >> 24;
+    r.pay = (it.offe - it.offb) * 16u;
+    r.dsc_skew = (it.tb & 1) * 8u;                       // tdesc[tb] may sit mid 16-byte line
+    r.dsc = nt ? up16(r.dsc_skew + 8u * nt) : 0u;
+    if (it.ke > it.kb) {
+        const int64_t rows = imin64(16, m - 16 * (int64_t)it.I);
+        r.rp = up16((uint32_t)(rows + 1) * 4u);            // remRowPtr[16I .. 16I+rows], 64I-aligned
+        r.col_skew = ((uint32_t)it.kb * 4u) & 15u;
+        r.col = up16(r.col_skew + 4u * (it.ke - it.kb));
+        r.val_skew = ((uint32_t)it.kb * 8u) & 15u;
+        r.val = up16(r.val_skew + 8u * (it.ke - it.kb));
+    } else {
+        r.rp = r.col = r.val = r.col_skew = r.val_skew = 0u;
+    }
+    r.total = r.pay + r.dsc + r.rp + r.col + r.val;
+    return r;
+}
+
+// the largest item: payload + 16 descriptors + rowptr + kItemRem col/val
+constexpr uint32_t kItemMaxBytes =
+    kItemPayload + ((8 * kItemTiles + 8 + 15) & ~15) + 80 + ((4 * kItemRem + 12 + 15) & ~15) +
+    ((8 * kItemRem + 8 + 15) & ~15);
+
+template <int C, int S>
+struct RingCfg {
+    static_assert(S % C == 0, "slot s must always map to consumer s mod C");
+    static constexpr uint32_t kRing = (S + 1) * kItemMaxBytes;   // no live item can be overwritten
+    static constexpr uint32_t kX = C * 16 * kItemTiles * 8;       // per-consumer x segments
+    static constexpr uint32_t kSlots = S * (uint32_t)sizeof(Item) + S * 4;
+    static constexpr uint32_t kBars = 2 * S * 8;
+    static constexpr uint32_t kSmem = kRing + kX + ((kSlots + 15) & ~15u) + kBars;
+    static constexpr int kThreads = 32 * (C + 1);
+};
+
+__device__ __forceinline__ void mbar_arrive(uint32_t bar) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(bar) : "memory");
+}
+
+// remainder rows staged in shared memory (rowptr, col, val), x gathered from L2
+__device__ __forceinline__ void remainder_rows_smem(const Params &p, int64_t I, int kb, int ke,
+                                                    const int *rpS, const int *colS, const double *valS,
+                                                    int lane, double &acc) {
+    const int r = lane & 15, h = lane >> 4;
+    const int mr = (int)imin64(16, p.m - 16 * I);
+    int b = rpS[min(r, mr)], e = rpS[min(r + 1, mr)];
+    b = max(b, kb);
+    e = min(e, ke);
+    const int len = max(e - b, 0);
+    const bool is_short = len <= kShortRow;
+    {
+        int cs[kShortRow / 2];
+        double vs[kShortRow / 2];
+#pragma unroll
+        for (int i = 0; i < kShortRow / 2; ++i) {
+            int k = b + h + 2 * i;
+            bool ok = is_short && k < e;
+            cs[i] = ok ? colS[k - kb] : 0;
+            vs[i] = ok ? valS[k - kb] : 0.0;
+        }
+        double xs[kShortRow / 2];
+#pragma unroll
+        for (int i = 0; i < kShortRow / 2; ++i) {
+            int k = b + h + 2 * i;
+            xs[i] = (is_short && k < e) ? __ldg(p.x + cs[i]) : 0.0;
+        }
+#pragma unroll
+        for (int i = 0; i < kShortRow / 2; ++i) {
+            int k = b + h + 2 * i;
+            if (is_short && k < e) acc = fma(vs[i], xs[i], acc);
+        }
+    }
+    unsigned longs = __ballot_sync(FULL, lane < 16 && !is_short);
+    while (longs) {
+        const int rr = __ffs(longs) - 1;
+        longs &= longs - 1;
+        const int bb = __shfl_sync(FULL, b, rr), ee = __shfl_sync(FULL, e, rr);
+        double s = 0.0;
+        for (int k0 = bb; k0 < ee; k0 += 128) {
+            int cs[4];
+            double vs[4], xv[4];
+#pragma unroll
+            for (int i = 0; i < 4; ++i) {
+                int k = k0 + lane + 32 * i;
+                cs[i] = k < ee ? colS[k - kb] : 0;
+                vs[i] = k < ee ? valS[k - kb] : 0.0;
+            }
+#pragma unroll
+            for (int i = 0; i < 4; ++i) xv[i] = (k0 + lane + 32 * i < ee) ? __ldg(p.x + cs[i]) : 0.0;
+#pragma unroll
+            for (int i = 0; i < 4; ++i)
+                if (k0 + lane + 32 * i < ee) s = fma(vs[i], xv[i], s);
+        }
+#pragma unroll
+        for (int o = 16; o >= 1; o >>= 1) s += __shfl_xor_sync(FULL, s, o);
+        if (lane == rr) acc += s;
+    }
+}
+
+__device__ __forceinline__ void write_rows(const Params &p, const Item &item, int lane, double acc) {
+    const int64_t row = 16 * (int64_t)item.I + lane;
+    if (item.split < 0) {
+        if (lane < 16 && row < p.m) p.y[row] = acc;
+        return;
+    }
+    const int2 si = p.split_info[item.split];
+    const int part = item.part_nt & 0xFFFFFF;
+    if (lane < 16) __stcg(p.partials + (int64_t)(si.x + part) * 16 + lane, acc);
+    __threadfence();
+    __syncwarp();
+    int old = 0;
+    if (lane == 0) old = atomicAdd(p.counters + item.split, 1);
+    old = __shfl_sync(FULL, old, 0);
+    if (old == si.y - 1) {  // last part of this tile row: sum the parts in item order
+        __threadfence();
+        const int r = lane & 15, hh = lane >> 4;
+        double s = 0.0;
+        for (int q = hh; q < si.y; q += 2) s += __ldcg(p.partials + (int64_t)(si.x + q) * 16 + r);
+        s += __shfl_xor_sync(FULL, s, 16);
+        if (lane < 16 && row < p.m) p.y[row] = s;
+        if (lane == 0) p.counters[item.split] = 0;  // ready for the next run
+    }
+}
+
+template <int C, int S>
+__global__ void __launch_bounds__(RingCfg<C, S>::kThreads, 1) tilespmv_fp64_ring_kernel(const Params p) {
+    using Cfg = RingCfg<C, S>;
+    extern __shared__ __align__(128) uint8_t smem[];
+    uint8_t *ring = smem;
+    double *xs_all = reinterpret_cast<double *>(smem + Cfg::kRing);
+    Item *slot_item = reinterpret_cast<Item *>(smem + Cfg::kRing + Cfg::kX);
+    uint32_t *slot_pos = reinterpret_cast<uint32_t *>(slot_item + S);
+    uint64_t *bars = reinterpret_cast<uint64_t *>(smem + Cfg::kRing + Cfg::kX + ((Cfg::kSlots + 15) & ~15u));
+    const uint32_t full0 = smem_u32(bars), empty0 = smem_u32(bars + S);
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < S; ++s) {
+            mbar_init(full0 + 8 * s, 1);
+            mbar_init(empty0 + 8 * s, 1);
+        }
+        fence_mbar_init();
+    }
+    __syncthreads();
+    const int64_t beg = p.cta_begin[blockIdx.x], end = p.cta_begin[blockIdx.x + 1];
+    const uint32_t ring_s = smem_u32(ring);
+
+    if (warp == 0) {
+        // ---------------------------------------------------- producer ----
+        uint32_t pos = 0;
+        for (int64_t k0 = beg; k0 < end; k0 += 32) {
+            const int cnt = (int)imin64(32, end - k0);
+            int4 ia = make_int4(0, 0, 0, 0), ib = ia;
+            if (lane < cnt) {
+                const int4 *src = reinterpret_cast<const int4 *>(p.items + k0 + lane);
+                ia = __ldg(src);
+                ib = __ldg(src + 1);
+            }
+            for (int j = 0; j < cnt; ++j) {
+                Item it;
+                it.I = __shfl_sync(FULL, ia.x, j);
+                it.tb = __shfl_sync(FULL, ia.y, j);
+                it.kb = __shfl_sync(FULL, ia.z, j);
+                it.ke = __shfl_sync(FULL, ia.w, j);
+                it.offb = (uint32_t)__shfl_sync(FULL, ib.x, j);
+                it.offe = (uint32_t)__shfl_sync(FULL, ib.y, j);
+                it.split = __shfl_sync(FULL, ib.z, j);
+                it.part_nt = __shfl_sync(FULL, ib.w, j);
+                if (lane == 0) {
+                    const int64_t q = k0 + j - beg;
+                    const int slot = (int)(q % S);
+                    const uint32_t round = (uint32_t)(q / S);
+                    if (round > 0) mbar_wait(empty0 + 8 * slot, (round - 1) & 1u);
+                    const RingParts rp = ring_parts(it, p.m);
+                    if (pos + rp.total > Cfg::kRing) pos = 0;
+                    slot_item[slot] = it;
+                    slot_pos[slot] = pos;
+                    const uint32_t bar = full0 + 8 * slot;
+                    fence_proxy_async();
+                    mbar_expect_tx(bar, rp.total);
+                    uint32_t d = ring_s + pos;
+                    if (rp.pay) bulk_g2s(d, p.payload + (size_t)it.offb * 16, rp.pay, bar);
+                    d += rp.pay;
+                    if (rp.dsc) bulk_g2s(d, reinterpret_cast<const uint8_t *>(p.tdesc + it.tb) - rp.dsc_skew, rp.dsc, bar);
+                    d += rp.dsc;
+                    if (rp.rp) {
+                        bulk_g2s(d, p.remRowPtr + 16 * (int64_t)it.I, rp.rp, bar);
+                        d += rp.rp;
+                        bulk_g2s(d, reinterpret_cast<const uint8_t *>(p.remCol + it.kb) - rp.col_skew, rp.col, bar);
+                        d += rp.col;
+                        bulk_g2s(d, reinterpret_cast<const uint8_t *>(p.remVal + it.kb) - rp.val_skew, rp.val, bar);
+                    }
+                    pos += rp.total;
+                }
+                __syncwarp();
+            }
+        }
+        return;
+    }
+    // -------------------------------------------------------- consumers ---
+    const int c = warp - 1;
+    double *xs = xs_all + c * 16 * kItemTiles;
+    for (int64_t q = c; beg + q < end; q += C) {
+        const int slot = (int)(q % S);
+        const uint32_t round = (uint32_t)(q / S);
+        mbar_wait(full0 + 8 * slot, round & 1u);
+        const Item it = slot_item[slot];
+        const uint32_t pos = slot_pos[slot];
+        const RingParts rp = ring_parts(it, p.m);
+        const uint8_t *pay = ring + pos;
+        const uint2 *dsc = reinterpret_cast<const uint2 *>(pay + rp.pay + rp.dsc_skew);
+        const int nt = it.part_nt >> 24;
+        // x segments of the item's tiles (x stays in L2; 128-byte lines)
+        {
+            double xv[kItemTiles / 2];
+#pragma unroll
+            for (int k = 0; k < kItemTiles / 2; ++k) {
+                const int t = 2 * k + (lane >> 4);
+                xv[k] = 0.0;
+                if (t < nt) {
+                    const int64_t col = 16 * (int64_t)(dsc[t].x & 0x7FFFFFFu) + (lane & 15);
+                    if (col < p.n) xv[k] = __ldg(p.x + col);
+                }
+            }
+#pragma unroll
+            for (int k = 0; k < kItemTiles / 2; ++k) xs[(2 * k + (lane >> 4)) * 16 + (lane & 15)] = xv[k];
+        }
+        double acc = 0.0;
+        if (rp.rp) {
+            const uint8_t *rb = pay + rp.pay + rp.dsc;
+            remainder_rows_smem(p, it.I, it.kb, it.ke, reinterpret_cast<const int *>(rb),
+                                reinterpret_cast<const int *>(rb + rp.rp + rp.col_skew),
+                                reinterpret_cast<const double *>(rb + rp.rp + rp.col + rp.val_skew), lane, acc);
+        }
+        __syncwarp();
+        uint32_t off = 0;
+        for (int t = 0; t < nt; ++t) {
+            const uint2 d = dsc[t];
+            const int fmt = (int)(d.x >> 27);
+            const int aux = (int)(d.y & 31u), nz = (int)((d.y >> 5) & 511u);
+            tile_spmv(fmt, aux, nz, pay + off, xs + 16 * t, lane, acc);
+            off += ((d.y >> 14) & 255u) * 16u;
+        }
+        acc += __shfl_xor_sync(FULL, acc, 16);
+        write_rows(p, it, lane, acc);
+        __syncwarp();
+        if (lane == 0) mbar_arrive(empty0 + 8 * slot);
+    }
+}
+
+// 8-byte tile descriptor read by the v2 kernel, derived from the canonical
+// level-1 arrays: x = J | fmt << 27 ; y = aux | nnz << 5 | size16 << 14.
+__global__ void k_build_tdesc(const int32_t *tileColIdx, const uint8_t *tileFmt, const uint8_t *tileAux,
+                              const int32_t *tileNnz, const uint32_t *tileOff, int64_t numtile, uint2 *tdesc) {
+    int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (t >= numtile) return;
+    uint2 d;
+    d.x = (uint32_t)tileColIdx[t] | ((uint32_t)tileFmt[t] << 27);
+    d.y = (uint32_t)tileAux[t] | ((uint32_t)(tileNnz[t + 1] - tileNnz[t]) << 5) |
+          ((tileOff[t + 1] - tileOff[t]) << 14);
+    tdesc[t] = d;
+}
+
+// item cost for the CTA chunking: bytes moved + a fixed per-item overhead
+__global__ void k_item_cost(const Item *items, int64_t n, int64_t *cost) {
+    int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (k >= n) return;
+    const Item it = items[k];
+    cost[k] = (int64_t)(it.offe - it.offb) * 16 + 12 * (int64_t)(it.ke - it.kb) + 8 * (it.part_nt >> 24) + 256;
+}
+
+__global__ void k_cta_begin(const int64_t *incl, int64_t n, int G, int64_t *cta_begin) {
+    int b = blockIdx.x * blockDim.x + threadIdx.x;
+    if (b > G) return;
+    if (b == G) { cta_begin[b] = n; return; }
+    const int64_t total = n ? incl[n - 1] : 0;
+    const int64_t target = total * b / G;   // first item whose prefix-before >= target
+    int64_t lo = 0, hi = n;
+    while (lo < hi) {
+        int64_t mid = (lo + hi) / 2;
+        int64_t before = mid ? incl[mid - 1] : 0;
+        if (before < target) lo = mid + 1; else hi = mid;
+    }
+    cta_begin[b] = lo;
 }
 
 // ----------------------------------------------------------- schedule -----
@@ -480,18 +804,86 @@ done:
     return rc;
 }
 
+using KernelFn = void (*)(Params);
+
+struct KernelChoice {
+    const char *name;
+    KernelFn fn;
+    int threads, smem, ctas_per_sm;
+};
+
+template <int C, int S>
+KernelChoice ring_choice(const char *name) {
+    return {name, tilespmv_fp64_ring_kernel<C, S>, RingCfg<C, S>::kThreads, (int)RingCfg<C, S>::kSmem, 1};
+}
+
+static KernelChoice choose_kernel(int version) {
+    switch (version) {
+    case 1: return {"v1", tilespmv_fp64_kernel, kWarps * 32, kSmemBytes, 0};
+    case 2: return ring_choice<6, 12>("ring_c6_s12");
+    case 3: return ring_choice<4, 8>("ring_c4_s8");
+    case 4: return ring_choice<4, 12>("ring_c4_s12");
+    case 5: return ring_choice<8, 8>("ring_c8_s8");
+    case 6: return ring_choice<3, 12>("ring_c3_s12");
+    default: return ring_choice<6, 12>("ring_c6_s12");
+    }
+}
+
 int configure_launch(Matrix &M) {
-    TSP_CK(cudaFuncSetAttribute(tilespmv_fp64_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                kSmemBytes));
+    int version = 2;
+    if (const char *e = getenv("TILESPMV_KERNEL")) version = atoi(e);
+    const KernelChoice kc = choose_kernel(version);
+    TSP_CK(cudaFuncSetAttribute(kc.fn, cudaFuncAttributeMaxDynamicSharedMemorySize, kc.smem));
     int sms = 0, per_sm = 0;
     TSP_CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, M.device));
-    TSP_CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, tilespmv_fp64_kernel, kWarps * 32,
-                                                         kSmemBytes));
-    per_sm = std::max(per_sm, 1);
-    const int64_t need = (M.num_items + kWarps - 1) / kWarps;
-    M.grid = (int)std::max<int64_t>(1, std::min<int64_t>(need, (int64_t)sms * per_sm));
-    M.block = kWarps * 32;
-    M.smem = kSmemBytes;
+    TSP_CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kc.fn, kc.threads, kc.smem));
+    if (per_sm < 1) return set_error(TILESPMV_CUDA, "SpMV kernel does not fit on an SM");
+    M.kernel_version = version;
+    M.block = kc.threads;
+    M.smem = kc.smem;
+    if (version == 1) {
+        const int64_t need = (M.num_items + kWarps - 1) / kWarps;
+        M.grid = (int)std::max<int64_t>(1, std::min<int64_t>(need, (int64_t)sms * per_sm));
+        return 0;
+    }
+    // v2: one CTA per SM, each owning a contiguous, cost-balanced item chunk
+    const int G = (int)std::max<int64_t>(1, std::min<int64_t>((int64_t)sms * kc.ctas_per_sm, M.num_items));
+    M.grid = G;
+    if (M.cta_begin) cudaFree(M.cta_begin);
+    M.cta_begin = nullptr;
+    TSP_CK(cudaMalloc(&M.cta_begin, (G + 1) * sizeof(int64_t)));
+    M.device_bytes += (G + 1) * 8;
+    if (M.num_items > 0) {
+        int64_t *cost = nullptr, *incl = nullptr;
+        void *tmp = nullptr;
+        size_t tb = 0;
+        TSP_CK(cudaMalloc(&cost, M.num_items * sizeof(int64_t)));
+        TSP_CK(cudaMalloc(&incl, M.num_items * sizeof(int64_t)));
+        k_item_cost<<<(unsigned)((M.num_items + 255) / 256), 256>>>(M.items, M.num_items, cost);
+        TSP_CK(cub::DeviceScan::InclusiveSum(nullptr, tb, cost, incl, (int)M.num_items));
+        TSP_CK(cudaMalloc(&tmp, tb));
+        TSP_CK(cub::DeviceScan::InclusiveSum(tmp, tb, cost, incl, (int)M.num_items));
+        k_cta_begin<<<(G + 1 + 255) / 256, 256>>>(incl, M.num_items, G, M.cta_begin);
+        TSP_CK(cudaGetLastError());
+        TSP_CK(cudaDeviceSynchronize());
+        cudaFree(cost);
+        cudaFree(incl);
+        cudaFree(tmp);
+    } else {
+        TSP_CK(cudaMemset(M.cta_begin, 0, (G + 1) * sizeof(int64_t)));
+    }
+    return 0;
+}
+
+int build_tdesc(Matrix &M, cudaStream_t st) {
+    TSP_CK(cudaMalloc(&M.tdesc, (M.numtile + 2) * sizeof(uint2)));
+    M.device_bytes += (M.numtile + 2) * 8;
+    if (M.numtile > 0) {
+        k_build_tdesc<<<(unsigned)((M.numtile + 255) / 256), 256, 0, st>>>(M.tileColIdx, M.tileFmt, M.tileAux,
+                                                                           M.tileNnz, M.tileOff, M.numtile,
+                                                                           M.tdesc);
+        TSP_CK(cudaGetLastError());
+    }
     return 0;
 }
 
@@ -516,7 +908,10 @@ int launch_spmv(const Matrix &M, const double *d_x, double *d_y, cudaStream_t st
     p.y = d_y;
     p.m = M.m;
     p.n = M.n;
-    tilespmv_fp64_kernel<<<M.grid, M.block, M.smem, st>>>(p);
+    p.tdesc = M.tdesc;
+    p.cta_begin = M.cta_begin;
+    const KernelChoice kc = choose_kernel(M.kernel_version);
+    kc.fn<<<M.grid, M.block, M.smem, st>>>(p);
     TSP_CK(cudaGetLastError());
     return 0;
 }

@@ -481,7 +481,7 @@ int build_tiled_k(Matrix &M, const int32_t *d_rowptr, const int32_t *d_colidx, c
         if (int rc = read_scalar(pos.p + nnz, &nrem, st)) return rc;
         M.rem_nnz = nrem;
         if (nrem > 0) {
-            TSP_CK(cudaMalloc(&M.remRowPtr, (M.m + 1) * sizeof(int32_t)));
+            TSP_CK(cudaMalloc(&M.remRowPtr, (M.m + 1 + 8) * sizeof(int32_t)));  // + bulk-copy slack
             TSP_CK(cudaMalloc(&M.remCol, (nrem + 4) * sizeof(int32_t)));
             TSP_CK(cudaMalloc(&M.remVal, (nrem + 2) * sizeof(double)));
             M.device_bytes += (M.m + 1) * 4 + (nrem + 4) * 4 + (nrem + 2) * 8;

@@ -1,0 +1,100 @@
+"""World-size-2 CPU tests (gloo) of the tile-row sharding and the y
+all-gather assembly used for N > 1 (paper_conf_ipps_niuldj0t21_b200/sharded.py).
+Each rank's "SpMV" is the CPU oracle on its row slice (a CPU fake of the GPU
+kernel), so the partition/assembly logic is tested without GPUs: the gathered
+vector must equal the unsharded oracle y bitwise."""
+import os
+import socket
+
+import numpy as np
+import pytest
+import torch
+import torch.distributed as dist
+import torch.multiprocessing as mp
+
+from paper_conf_ipps_niuldj0t21_b200.sharded import ShardedSpMV, partition_tile_rows
+
+
+def _port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _worker(rank, world, port, name, weighted, iters, q):
+    try:
+        from oracle import oracle as O
+        from synthetic import gen
+        os.environ["MASTER_ADDR"] = "127.0.0.1"
+        os.environ["MASTER_PORT"] = str(port)
+        dist.init_process_group("gloo", rank=rank, world_size=world)
+        A, x = gen.make(name)
+        w = None
+        if weighted:
+            idx = np.minimum(np.arange(0, A.m + 16, 16), A.m)
+            w = np.diff(A.rowptr[idx].astype(np.int64))
+        b = partition_tile_rows(A.m, world, w)
+        S = A.row_slice(b[rank], b[rank + 1])
+
+        def spmv(xf, yout):
+            y, _ = O.spmv(S, xf.numpy())
+            yout.copy_(torch.from_numpy(y))
+
+        sh = ShardedSpMV(spmv, b, rank, world, device="cpu")
+        xk = torch.from_numpy(x.copy())
+        outs = []
+        for _ in range(iters):
+            xk = sh.step(xk).clone()
+            outs.append(xk.numpy().copy())
+        q.put((rank, b, outs))
+        dist.destroy_process_group()
+    except Exception as e:  # pragma: no cover
+        q.put((rank, None, repr(e)))
+
+
+@pytest.mark.parametrize("name,weighted", [("stencil27_21", False), ("rmat12", True),
+                                           ("lap2d_37x29", True)])
+def test_sharded_allgather_equals_unsharded(name, weighted):
+    from oracle import oracle as O
+    from synthetic import gen
+    world, iters = 2, 3
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _port()
+    procs = [ctx.Process(target=_worker, args=(r, world, port, name, weighted, iters, q))
+             for r in range(world)]
+    for p in procs:
+        p.start()
+    res = [q.get(timeout=300) for _ in range(world)]
+    for p in procs:
+        p.join(timeout=60)
+    for r, b, outs in res:
+        assert b is not None, outs
+    A, x = gen.make(name)
+    # reference: the unsharded oracle iterate x_{k+1} = A x_k
+    ref = []
+    xk = x.copy()
+    for _ in range(iters):
+        xk, _ = O.spmv(A, xk)
+        ref.append(xk.copy())
+    for r, b, outs in res:
+        assert b[0] == 0 and b[-1] == A.m and all(v % 16 == 0 for v in b[:-1])
+        for k in range(iters):
+            assert np.array_equal(outs[k].view(np.uint64), ref[k].view(np.uint64)), (name, r, k)
+
+
+def test_partition_properties():
+    for m, P in [(8_000_000, 8), (100, 3), (17, 4), (16, 2), (1, 2), (0, 2)]:
+        b = partition_tile_rows(m, P)
+        assert len(b) == P + 1 and b[0] == 0 and b[-1] == m
+        assert all(b[i] <= b[i + 1] for i in range(P))
+        assert all(v % 16 == 0 for v in b[:-1])
+    b = partition_tile_rows(8_000_000, 8)
+    assert b == [1_000_000 * i for i in range(9)]   # C5: 62,500 tile rows per rank
+    w = np.ones(100)
+    w[:10] = 50
+    b = partition_tile_rows(1600, 4, w)
+    loads = [w[b[i] // 16:b[i + 1] // 16].sum() for i in range(4)]
+    assert max(loads) <= 1.5 * (w.sum() / 4) + 50
