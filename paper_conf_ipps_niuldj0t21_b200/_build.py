@@ -7,8 +7,10 @@ import subprocess
 PKG = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(PKG)
 LIB = os.path.join(PKG, "libtilespmv.so")
-SOURCES = [os.path.join(PKG, "csrc", f) for f in ("abi.cu", "tiler.cu", "spmv.cu")]
-HEADERS = [os.path.join(PKG, "csrc", "internal.cuh"), os.path.join(ROOT, "include", "tilespmv.h")]
+SOURCES = [os.path.join(PKG, "csrc", f)
+           for f in ("abi.cu", "tiler.cu", "schedule.cu", "spmv_v1.cu", "spmv_ring.cu")]
+HEADERS = [os.path.join(PKG, "csrc", f) for f in ("internal.cuh", "spmv_common.cuh")] + \
+          [os.path.join(ROOT, "include", "tilespmv.h")]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-lineinfo", "-O3", "-std=c++17",
          "-Xcompiler", "-fPIC", "-shared", "-t", "3"]

@@ -18,17 +18,18 @@ enum : uint8_t { F_CSR = 0, F_COO = 1, F_ELL = 2, F_HYB = 3, F_DNS = 4, F_DNSROW
 
 // ---------------------------------------------------------------------------
 // SpMV schedule.  A work item is a byte-bounded piece of one tile row: a run
-// of at most kItemTiles consecutive tiles whose payload fits kItemPayload
-// bytes, and/or at most kItemRem remainder entries of the tile row's 16 rows.
-// A tile row split over several items writes per-item partials that the last
-// finishing item sums in item order (deterministic; replaces the atomic
-// merge of tbalance).  Item boundaries depend only on the tile row's
-// own content, so a tile-row-sharded run reproduces the 1-GPU y bitwise.
+// of at most kItemTiles consecutive tiles and/or a range of remainder entries
+// of the tile row's 16 rows, such that everything the kernel stages for it
+// (payloads, 8-byte tile descriptors, remainder rowptr/col/val) fits one
+// kItemBytes shared-memory slot.  A tile row split over several items writes
+// per-item partials that the last finishing item sums in item order
+// (deterministic; replaces the atomic merge of tbalance).  Item
+// boundaries depend only on the tile row's own content, so a tile-row-sharded
+// run reproduces the 1-GPU y bitwise.
 // ---------------------------------------------------------------------------
 constexpr int kItemTiles = 16;
-constexpr int kItemPayload = 10240;  // bytes; one FEM tile row = 5 Dns tiles
-constexpr int kItemRem = 256;        // remainder entries per item
-constexpr int kShortRow = 8;         // remainder rows up to this length: 2 lanes per row
+constexpr int kItemBytes = 8192;  // one shared-memory slot
+constexpr int kShortRow = 8;      // remainder rows up to this length: 2 lanes per row
 
 struct __align__(16) Item {
     int32_t I;        // tile row

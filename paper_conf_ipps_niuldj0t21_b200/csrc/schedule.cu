@@ -1,0 +1,279 @@
+// schedule.cu -- create-time SpMV schedule and launch dispatch.
+//   * work items: byte-bounded pieces of one tile row (internal.cuh), built
+//     by one thread per tile row in two passes (count, scan, write);
+//   * 8-byte tile descriptors derived from the canonical level-1 arrays;
+//   * contiguous, cost-balanced item chunks per CTA for the ring kernels;
+//   * kernel choice (TILESPMV_KERNEL env: 1 = v1 baseline, else ring variant).
+#include <cub/cub.cuh>
+
+#include <algorithm>
+#include <cstdlib>
+
+#include "spmv_common.cuh"
+
+namespace tsp {
+
+#define TSP_CK(call)                                                   \
+    do {                                                               \
+        cudaError_t e_ = (call);                                       \
+        if (e_ != cudaSuccess) return cuda_status(e_, #call);          \
+    } while (0)
+
+namespace {
+
+// Greedy split of tile row I into items whose staged bytes (item_parts)
+// never exceed kItemBytes: tiles first (at most kItemTiles), then the tile
+// row's remainder entries.  Depends only on the tile row's own content.
+template <bool WRITE>
+__device__ int items_for_row(int64_t I, const int32_t *tilePtr, const uint32_t *tileOff, const int32_t *remRowPtr,
+                             int64_t m, Item *out, int split) {
+    const int tp0 = tilePtr[I], tp1 = tilePtr[I + 1];
+    int k0 = 0, k1 = 0;
+    if (remRowPtr) {
+        k0 = remRowPtr[16 * I];
+        k1 = remRowPtr[16 * I + 16 < m ? 16 * I + 16 : m];
+    }
+    const int64_t rows = imin64(16, m - 16 * I);
+    const uint32_t rp_bytes = up16((uint32_t)(rows + 1) * 4u);
+    int t = tp0, k = k0, cnt = 0;
+    do {
+        const int tb = t;
+        uint32_t used = 0;
+        while (t < tp1 && t - tb < kItemTiles) {
+            const uint32_t pay = (tileOff[t + 1] - tileOff[tb]) * 16u;
+            const uint32_t dsc = up16((uint32_t)(tb & 1) * 8u + 8u * (uint32_t)(t - tb + 1));
+            if (pay + dsc > (uint32_t)kItemBytes) break;
+            used = pay + dsc;
+            t++;
+        }
+        if (t == tb && t < tp1) {  // unreachable: one tile (<= 2176 B) always fits
+            used = (tileOff[t + 1] - tileOff[tb]) * 16u + 16u;
+            t++;
+        }
+        int kb = k, ke = k;
+        if (t == tp1 && k < k1) {
+            const int64_t avail = (int64_t)kItemBytes - used - rp_bytes - 64;  // 2 x 32 B skew slack
+            const int64_t e = imin64(avail > 0 ? avail / 12 : 0, k1 - k);
+            if (e > 0) {
+                ke = k + (int)e;
+                k = ke;
+            }
+        }
+        if (WRITE) {
+            Item it;
+            it.I = (int32_t)I;
+            it.tb = tb;
+            it.kb = kb;
+            it.ke = ke;
+            it.offb = tileOff[tb];
+            it.offe = tileOff[t];
+            it.split = split;
+            it.part_nt = (split >= 0 ? cnt : 0) | ((t - tb) << 24);
+            out[cnt] = it;
+        }
+        cnt++;
+    } while (t < tp1 || k < k1);
+    return cnt;
+}
+
+__global__ void k_items_count(const int32_t *tilePtr, const uint32_t *tileOff, const int32_t *remRowPtr, int64_t m,
+                              int64_t tilem, int32_t *nitems, int32_t *nsplit, int32_t *parts) {
+    int64_t I = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (I >= tilem) return;
+    const int c = items_for_row<false>(I, tilePtr, tileOff, remRowPtr, m, nullptr, -1);
+    nitems[I] = c;
+    nsplit[I] = c > 1 ? 1 : 0;
+    parts[I] = c > 1 ? c : 0;
+}
+
+__global__ void k_items_write(const int32_t *tilePtr, const uint32_t *tileOff, const int32_t *remRowPtr, int64_t m,
+                              int64_t tilem, const int32_t *itemBase, const int32_t *splitId, const int32_t *nitems,
+                              const int32_t *partBase, Item *items, int2 *split_info) {
+    int64_t I = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (I >= tilem) return;
+    const bool split = nitems[I] > 1;
+    const int sid = split ? splitId[I] : -1;
+    items_for_row<true>(I, tilePtr, tileOff, remRowPtr, m, items + itemBase[I], sid);
+    if (split) split_info[sid] = make_int2(partBase[I], nitems[I]);
+}
+
+// x = J | fmt << 27 ; y = aux | nnz << 5 | size16 << 14
+__global__ void k_build_tdesc(const int32_t *tileColIdx, const uint8_t *tileFmt, const uint8_t *tileAux,
+                              const int32_t *tileNnz, const uint32_t *tileOff, int64_t numtile, uint2 *tdesc) {
+    int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (t >= numtile) return;
+    uint2 d;
+    d.x = (uint32_t)tileColIdx[t] | ((uint32_t)tileFmt[t] << 27);
+    d.y = (uint32_t)tileAux[t] | ((uint32_t)(tileNnz[t + 1] - tileNnz[t]) << 5) | ((tileOff[t + 1] - tileOff[t]) << 14);
+    tdesc[t] = d;
+}
+
+// item cost for the CTA chunking: bytes staged + a fixed per-item overhead
+__global__ void k_item_cost(const Item *items, int64_t n, int64_t m, int64_t *cost) {
+    int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (k >= n) return;
+    const Item it = items[k];
+    cost[k] = (int64_t)item_parts(it, m).total + 40 * (it.part_nt >> 24) + 512;
+}
+
+__global__ void k_cta_begin(const int64_t *incl, int64_t n, int G, int64_t *cta_begin) {
+    const int b = blockIdx.x * blockDim.x + threadIdx.x;
+    if (b > G) return;
+    if (b == G) {
+        cta_begin[b] = n;
+        return;
+    }
+    const int64_t total = n ? incl[n - 1] : 0;
+    const int64_t target = total * b / G;  // first item whose prefix-before >= target
+    int64_t lo = 0, hi = n;
+    while (lo < hi) {
+        const int64_t mid = (lo + hi) / 2;
+        const int64_t before = mid ? incl[mid - 1] : 0;
+        if (before < target) lo = mid + 1;
+        else hi = mid;
+    }
+    cta_begin[b] = lo;
+}
+
+template <class F>
+int scan(F &&f) {
+    size_t bytes = 0;
+    TSP_CK(f(nullptr, bytes));
+    void *tmp = nullptr;
+    TSP_CK(cudaMalloc(&tmp, std::max<size_t>(bytes, 1)));
+    cudaError_t e = f(tmp, bytes);
+    cudaFree(tmp);
+    TSP_CK(e);
+    return 0;
+}
+
+KernelChoice choose(int version) { return version == 1 ? kernel_v1() : kernel_ring(version); }
+
+}  // namespace
+
+int build_schedule(Matrix &M, cudaStream_t st) {
+    const int TB = 256;
+    const int64_t T = M.tilem;
+    if (T == 0) return 0;
+    auto blocks = [&](int64_t n) { return (unsigned)std::max<int64_t>(1, (n + TB - 1) / TB); };
+    int32_t *buf = nullptr;
+    TSP_CK(cudaMalloc(&buf, 6 * (T + 1) * sizeof(int32_t)));
+    int32_t *nitems = buf, *nsplit = buf + (T + 1), *parts = buf + 2 * (T + 1), *itemBase = buf + 3 * (T + 1),
+            *splitId = buf + 4 * (T + 1), *partBase = buf + 5 * (T + 1);
+    int rc = 0;
+    do {
+        if (cudaMemsetAsync(buf, 0, 3 * (T + 1) * sizeof(int32_t), st) != cudaSuccess) { rc = cuda_status(cudaGetLastError(), "memset"); break; }
+        k_items_count<<<blocks(T), TB, 0, st>>>(M.tilePtr, M.tileOff, M.remRowPtr, M.m, T, nitems, nsplit, parts);
+        if ((rc = scan([&](void *t, size_t &b) { return cub::DeviceScan::ExclusiveSum(t, b, nitems, itemBase, (int)(T + 1), st); }))) break;
+        if ((rc = scan([&](void *t, size_t &b) { return cub::DeviceScan::ExclusiveSum(t, b, nsplit, splitId, (int)(T + 1), st); }))) break;
+        if ((rc = scan([&](void *t, size_t &b) { return cub::DeviceScan::ExclusiveSum(t, b, parts, partBase, (int)(T + 1), st); }))) break;
+        int32_t h[3];
+        cudaMemcpyAsync(&h[0], itemBase + T, 4, cudaMemcpyDeviceToHost, st);
+        cudaMemcpyAsync(&h[1], splitId + T, 4, cudaMemcpyDeviceToHost, st);
+        cudaMemcpyAsync(&h[2], partBase + T, 4, cudaMemcpyDeviceToHost, st);
+        if (cudaStreamSynchronize(st) != cudaSuccess) { rc = cuda_status(cudaGetLastError(), "schedule sizes"); break; }
+        M.num_items = h[0];
+        M.num_split = h[1];
+        const int64_t nparts = h[2];
+        if (cudaMalloc(&M.items, std::max<int64_t>(M.num_items, 1) * sizeof(Item)) != cudaSuccess ||
+            cudaMalloc(&M.split_info, std::max<int64_t>(M.num_split, 1) * sizeof(int2)) != cudaSuccess ||
+            cudaMalloc(&M.counters, std::max<int64_t>(M.num_split, 1) * sizeof(int32_t)) != cudaSuccess ||
+            cudaMalloc(&M.partials, std::max<int64_t>(nparts, 1) * 16 * sizeof(double)) != cudaSuccess) {
+            rc = cuda_status(cudaGetLastError(), "cudaMalloc(schedule)");
+            break;
+        }
+        M.device_bytes += M.num_items * (int64_t)sizeof(Item) + M.num_split * 12 + nparts * 128;
+        cudaMemsetAsync(M.counters, 0, std::max<int64_t>(M.num_split, 1) * sizeof(int32_t), st);
+        k_items_write<<<blocks(T), TB, 0, st>>>(M.tilePtr, M.tileOff, M.remRowPtr, M.m, T, itemBase, splitId, nitems,
+                                                partBase, M.items, M.split_info);
+        if (cudaStreamSynchronize(st) != cudaSuccess) rc = cuda_status(cudaGetLastError(), "k_items_write");
+    } while (0);
+    cudaFree(buf);
+    return rc;
+}
+
+int build_tdesc(Matrix &M, cudaStream_t st) {
+    TSP_CK(cudaMalloc(&M.tdesc, (M.numtile + 2) * sizeof(uint2)));  // +2: 16-byte superset reads
+    M.device_bytes += (M.numtile + 2) * 8;
+    if (M.numtile > 0) {
+        k_build_tdesc<<<(unsigned)((M.numtile + 255) / 256), 256, 0, st>>>(M.tileColIdx, M.tileFmt, M.tileAux, M.tileNnz,
+                                                                           M.tileOff, M.numtile, M.tdesc);
+        TSP_CK(cudaGetLastError());
+    }
+    return 0;
+}
+
+int configure_launch(Matrix &M) {
+    int version = 2;
+    if (const char *e = getenv("TILESPMV_KERNEL")) version = atoi(e);
+    const KernelChoice kc = choose(version);
+    TSP_CK(cudaFuncSetAttribute(kc.fn, cudaFuncAttributeMaxDynamicSharedMemorySize, kc.smem));
+    int sms = 0, per_sm = 0;
+    TSP_CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, M.device));
+    TSP_CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kc.fn, kc.threads, kc.smem));
+    if (per_sm < 1) return set_error(TILESPMV_CUDA, "SpMV kernel does not fit on an SM");
+    M.kernel_version = version;
+    M.block = kc.threads;
+    M.smem = kc.smem;
+    if (!kc.ring) {
+        const int64_t warps = kc.threads / 32;
+        const int64_t need = (M.num_items + warps - 1) / warps;
+        M.grid = (int)std::max<int64_t>(1, std::min<int64_t>(need, (int64_t)sms * per_sm));
+        return 0;
+    }
+    // ring kernels: one CTA per SM, each owning a contiguous cost-balanced chunk
+    const int G = (int)std::max<int64_t>(1, std::min<int64_t>((int64_t)sms * kc.ctas_per_sm, M.num_items));
+    M.grid = G;
+    if (M.cta_begin) cudaFree(M.cta_begin);
+    M.cta_begin = nullptr;
+    TSP_CK(cudaMalloc(&M.cta_begin, (G + 1) * sizeof(int64_t)));
+    M.device_bytes += (G + 1) * 8;
+    if (M.num_items > 0) {
+        int64_t *cost = nullptr;
+        TSP_CK(cudaMalloc(&cost, 2 * M.num_items * sizeof(int64_t)));
+        int64_t *incl = cost + M.num_items;
+        k_item_cost<<<(unsigned)((M.num_items + 255) / 256), 256>>>(M.items, M.num_items, M.m, cost);
+        int rc = scan([&](void *t, size_t &b) { return cub::DeviceScan::InclusiveSum(t, b, cost, incl, (int)M.num_items); });
+        if (!rc) {
+            k_cta_begin<<<(G + 1 + 255) / 256, 256>>>(incl, M.num_items, G, M.cta_begin);
+            cudaError_t e = cudaDeviceSynchronize();
+            if (e != cudaSuccess) rc = cuda_status(e, "k_cta_begin");
+        }
+        cudaFree(cost);
+        if (rc) return rc;
+    } else {
+        TSP_CK(cudaMemset(M.cta_begin, 0, (G + 1) * sizeof(int64_t)));
+    }
+    return 0;
+}
+
+int launch_spmv(const Matrix &M, const double *d_x, double *d_y, cudaStream_t st) {
+    if (M.m == 0) return 0;
+    Params p;
+    p.items = M.items;
+    p.num_items = M.num_items;
+    p.tileColIdx = M.tileColIdx;
+    p.tileFmt = M.tileFmt;
+    p.tileAux = M.tileAux;
+    p.tileNnz = M.tileNnz;
+    p.tileOff = M.tileOff;
+    p.payload = M.payload;
+    p.remRowPtr = M.remRowPtr;
+    p.remCol = M.remCol;
+    p.remVal = M.remVal;
+    p.split_info = M.split_info;
+    p.partials = M.partials;
+    p.counters = M.counters;
+    p.x = d_x;
+    p.y = d_y;
+    p.m = M.m;
+    p.n = M.n;
+    p.tdesc = M.tdesc;
+    p.cta_begin = M.cta_begin;
+    const KernelChoice kc = choose(M.kernel_version);
+    kc.fn<<<M.grid, M.block, M.smem, st>>>(p);
+    TSP_CK(cudaGetLastError());
+    return 0;
+}
+
+}  // namespace tsp
