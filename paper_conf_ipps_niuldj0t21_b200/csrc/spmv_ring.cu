@@ -4,22 +4,23 @@
 //
 // Warp-specialised persistent kernel, one CTA per SM, each CTA owning a
 // contiguous, cost-balanced chunk of work items:
-//   * producer warp: lane j streams item (k0 + j) of a batch of S items into
-//     shared-memory slot j with TMA bulk copies (cp.async.bulk, 1-D):
-//     tile payloads, 8-byte tile descriptors, remainder rowptr/col/val.
-//     Completion is counted in bytes on the slot's "full" mbarrier.
+//   * producer warp: lane j owns shared-memory slot j and streams items
+//     beg + j, beg + j + S, ... into it with TMA bulk copies
+//     (cp.async.bulk, 1-D): tile payloads, 8-byte tile descriptors,
+//     remainder rowptr/col/val.  Completion is counted in bytes on the
+//     slot's "full" mbarrier; the slot is reused after its "empty" mbarrier.
 //   * C consumer warps: consumer c serves slots c, c+C, ... (S % C == 0, so
-//     every slot has one consumer and mbarrier parities cannot alias).  It
-//     stages the x segments of the item's tiles (one 128-byte line each) in
-//     shared memory, runs the format routines and writes y, then releases
-//     the slot on its "empty" mbarrier.
-//   * Tiles are processed TWO AT A TIME: after a warp ballot groups the
-//     item's tiles by format, each half-warp takes one tile of a same-format
-//     pair with one lane per tile row (the per-row decomposition of the
-//     paper's CSR/ELL/DnsCol routines), so the per-tile
-//     dispatch and setup cost is shared by two tiles and every loop has a
-//     warp-uniform trip count with predicated FMAs (no divergent branches).
-//     Row r's two half sums meet in acc(r) + acc(r + 16).
+//     every slot has exactly one consumer and mbarrier parities cannot
+//     alias).  Per item it stages the x segment of every tile (one 128-byte
+//     line) in shared memory, lists the tiles grouped by format, runs the
+//     format routines and writes y, then releases the slot.
+//   * Tiles run TWO AT A TIME: each half-warp takes one tile of a
+//     same-format pair, one lane per tile row (the per-row decomposition of
+//     the paper's CSR/ELL/DnsCol routines), so dispatch
+//     and setup are shared by two tiles and every loop has a warp-uniform
+//     trip count with predicated FMAs.  Row r's two half sums meet in
+//     acc(r) + acc(r + 16).  All shared-memory traffic uses 32-bit shared
+//     addresses with immediate offsets.
 //   * No floating-point atomics: y is bitwise deterministic.
 #include "spmv_common.cuh"
 
@@ -31,45 +32,76 @@ struct RingCfg {
     static_assert(S % C == 0, "slot s must always be served by consumer s mod C");
     static_assert(S <= 32, "one producer lane per slot");
     static constexpr uint32_t kRing = (uint32_t)S * kItemBytes;
-    static constexpr uint32_t kX = (uint32_t)C * kItemTiles * 16 * 8;
+    static constexpr uint32_t kXPer = kItemTiles * 16 * 8;  // x segments per consumer
+    static constexpr uint32_t kListPer = 128;               // tile list per consumer
+    static constexpr uint32_t kX = (uint32_t)C * kXPer;
+    static constexpr uint32_t kList = (uint32_t)C * kListPer;
     static constexpr uint32_t kSlots = (uint32_t)S * sizeof(Item);
     static constexpr uint32_t kBars = 2u * S * 8u;
-    static constexpr uint32_t kSmem = kRing + kX + kSlots + kBars + 64;  // +64: loads may overrun a slot
+    static constexpr uint32_t kSmem = kRing + kX + kList + kSlots + kBars + 256;  // +256: loads may overrun a slot
     static constexpr int kThreads = 32 * (C + 1);
 };
+
+// ------------------------------------------------- shared-memory access ----
+__device__ __forceinline__ double lds_f64(uint32_t a) {
+    double v;
+    asm volatile("ld.shared.f64 %0, [%1];" : "=d"(v) : "r"(a));
+    return v;
+}
+__device__ __forceinline__ uint32_t lds_u8(uint32_t a) {
+    uint32_t v;
+    asm volatile("ld.shared.u8 %0, [%1];" : "=r"(v) : "r"(a));
+    return v;
+}
+__device__ __forceinline__ int lds_s32(uint32_t a) {
+    int v;
+    asm volatile("ld.shared.s32 %0, [%1];" : "=r"(v) : "r"(a));
+    return v;
+}
+__device__ __forceinline__ uint2 lds_v2u32(uint32_t a) {
+    uint2 v;
+    asm volatile("ld.shared.v2.u32 {%0, %1}, [%2];" : "=r"(v.x), "=r"(v.y) : "r"(a));
+    return v;
+}
+__device__ __forceinline__ void sts_u32(uint32_t a, uint32_t v) {
+    asm volatile("st.shared.u32 [%0], %1;" ::"r"(a), "r"(v) : "memory");
+}
+__device__ __forceinline__ void sts_f64(uint32_t a, double v) {
+    asm volatile("st.shared.f64 [%0], %1;" ::"r"(a), "d"(v) : "memory");
+}
 
 // ------------------------------------------------ remainder (from smem) ----
 // rows of at most kShortRow entries: two lanes per row; longer rows: the
 // whole warp strides the row and reduces with a butterfly (fixed order).
-__device__ __forceinline__ void remainder_rows(const Params &p, int64_t I, int kb, int ke, const int *rpS,
-                                               const int *colS, const double *valS, int lane, double &acc) {
+// rpS/colS/valS: shared addresses of remRowPtr[16I..], remCol[kb..], remVal[kb..]
+__device__ __forceinline__ void remainder_rows(const Params &p, int rows, int kb, int ke, uint32_t rpS, uint32_t colS,
+                                               uint32_t valS, int lane, double &acc) {
     const int r = lane & 15, h = lane >> 4;
-    const int mr = (int)imin64(16, p.m - 16 * I);
-    int b = rpS[min(r, mr)], e = rpS[min(r + 1, mr)];
-    b = max(b, kb);
-    e = min(e, ke);
+    int b = lds_s32(rpS + 4 * min(r, rows)), e = lds_s32(rpS + 4 * min(r + 1, rows));
+    b = max(b, kb) - kb;
+    e = min(e, ke) - kb;
     const int len = max(e - b, 0);
     const bool is_short = len <= kShortRow;
-    {
+    const int nshort = is_short ? len : 0;
+    const int trips = (int)__reduce_max_sync(FULL, (unsigned)((nshort + 1 - h) >> 1));
+    if (trips > 0) {
         int cs[kShortRow / 2];
         double vs[kShortRow / 2], xs[kShortRow / 2];
 #pragma unroll
         for (int i = 0; i < kShortRow / 2; ++i) {
             const int k = b + h + 2 * i;
-            const bool ok = is_short && k < e;
-            cs[i] = ok ? colS[k - kb] : 0;
-            vs[i] = ok ? valS[k - kb] : 0.0;
+            const bool ok = i < trips && k < b + nshort;
+            cs[i] = ok ? lds_s32(colS + 4 * k) : 0;
+            vs[i] = ok ? lds_f64(valS + 8 * k) : 0.0;
         }
 #pragma unroll
         for (int i = 0; i < kShortRow / 2; ++i) {
-            const int k = b + h + 2 * i;
-            xs[i] = (is_short && k < e) ? __ldg(p.x + cs[i]) : 0.0;
+            const bool ok = i < trips && b + h + 2 * i < b + nshort;
+            xs[i] = ok ? __ldg(p.x + (uint32_t)cs[i]) : 0.0;
         }
 #pragma unroll
-        for (int i = 0; i < kShortRow / 2; ++i) {
-            const int k = b + h + 2 * i;
-            if (is_short && k < e) acc = fma(vs[i], xs[i], acc);
-        }
+        for (int i = 0; i < kShortRow / 2; ++i)
+            if (i < trips && b + h + 2 * i < b + nshort) acc = fma(vs[i], xs[i], acc);
     }
     unsigned longs = __ballot_sync(FULL, lane < 16 && !is_short);
     while (longs) {
@@ -83,11 +115,11 @@ __device__ __forceinline__ void remainder_rows(const Params &p, int64_t I, int k
 #pragma unroll
             for (int i = 0; i < 4; ++i) {
                 const int k = k0 + lane + 32 * i;
-                cs[i] = k < ee ? colS[k - kb] : 0;
-                vs[i] = k < ee ? valS[k - kb] : 0.0;
+                cs[i] = k < ee ? lds_s32(colS + 4 * k) : 0;
+                vs[i] = k < ee ? lds_f64(valS + 8 * k) : 0.0;
             }
 #pragma unroll
-            for (int i = 0; i < 4; ++i) xv[i] = (k0 + lane + 32 * i < ee) ? __ldg(p.x + cs[i]) : 0.0;
+            for (int i = 0; i < 4; ++i) xv[i] = (k0 + lane + 32 * i < ee) ? __ldg(p.x + (uint32_t)cs[i]) : 0.0;
 #pragma unroll
             for (int i = 0; i < 4; ++i)
                 if (k0 + lane + 32 * i < ee) s = fma(vs[i], xv[i], s);
@@ -99,136 +131,135 @@ __device__ __forceinline__ void remainder_rows(const Params &p, int64_t I, int k
 }
 
 // --------------------------------------------- half-warp tile routines -----
-// Lane r of a half owns row r of its tile.  P: payload, X: 16 x values,
-// ok: the half has a tile.  All loops have warp-uniform trip counts; the
-// unconditional shared-memory loads past a tile's end stay inside the CTA's
-// shared memory and are masked out of the FMA.
+// Lane r of a half owns row r of its tile.  P: shared address of the tile's
+// payload, X: of its 16 x values; ok: the half has a tile (else it runs the
+// other half's tile with its FMAs masked).  Loads past a tile's end stay
+// inside the CTA's shared memory and are masked out of the FMA.
 
 // CSR: csrVal row-major | csrRowPtr[16] u8 | 4-bit columns (Alg. 2)
-__device__ __forceinline__ void half_csr(const uint8_t *P, int nz, const double *X, int r, bool ok, double &acc) {
-    const double *V = reinterpret_cast<const double *>(P);
-    const uint8_t *rp = P + 8 * nz;
-    const uint8_t *ci = rp + 16;
-    const int beg = ok ? rp[r] : 0;
-    const int end = ok ? (r < 15 ? rp[r + 1] : nz) : 0;
-    const int len = end - beg;
+__device__ __forceinline__ void half_csr(uint32_t P, int nz, uint32_t X, int r, bool ok, double &acc) {
+    const uint32_t rp = P + 8 * nz;
+    const int beg = (int)lds_u8(rp + r);
+    const int end = r < 15 ? (int)lds_u8(rp + r + 1) : nz;
+    const int len = ok ? end - beg : 0;
     const int trips = (int)__reduce_max_sync(FULL, (unsigned)len);
-    const double *Vb = V + beg;
+    // nibble of entry beg+i: byte (beg+i)>>1 = b_even + i/2 (i even) or
+    // b_odd + i/2 (i odd), shifted by s_even / s_odd
+    const uint32_t cb = rp + 16 + (beg >> 1);
+    const uint32_t odd = beg & 1;
+    const uint32_t b_odd = cb + odd;
+    const uint32_t s_even = 4 * odd, s_odd = 4 - 4 * odd;
+    const uint32_t V = P + 8 * beg;
 #pragma unroll 4
     for (int i = 0; i < trips; ++i) {
-        const int j = beg + i;
-        const double v = Vb[i];
-        const double xv = X[nib(ci, j)];
+        const uint32_t byte = (i & 1) ? lds_u8(b_odd + (i >> 1)) : lds_u8(cb + (i >> 1));
+        const uint32_t c = (byte >> ((i & 1) ? s_odd : s_even)) & 15u;
+        const double v = lds_f64(V + 8 * i);
+        const double xv = lds_f64(X + 8 * c);
         if (i < len) acc = fma(v, xv, acc);
     }
 }
 
 // ELL: slots k*16 + r column-major | 4-bit columns (Alg. 4).
 // Pads (k >= 1 with column 0, reading R26) are skipped.
-__device__ __forceinline__ void half_ell(const uint8_t *P, int w, const double *X, int r, bool ok, double &acc) {
-    const double *V = reinterpret_cast<const double *>(P);
-    const uint8_t *ci = P + 128 * w;
+__device__ __forceinline__ void half_ell(uint32_t P, int w, uint32_t X, int r, bool ok, double &acc) {
     const int wq = ok ? w : 0;
     const int trips = (int)__reduce_max_sync(FULL, (unsigned)wq);
-    const int sh = 4 * (r & 1);
+    const uint32_t ci = P + 128 * w + (r >> 1);
+    const uint32_t sh = 4 * (r & 1);
+    const uint32_t V = P + 8 * r;
 #pragma unroll 4
     for (int k = 0; k < trips; ++k) {
-        const double v = V[16 * k + r];
-        const int c = (ci[8 * k + (r >> 1)] >> sh) & 15;
-        const double xv = X[c];
+        const uint32_t c = (lds_u8(ci + 8 * k) >> sh) & 15u;
+        const double v = lds_f64(V + 128 * k);
+        const double xv = lds_f64(X + 8 * c);
         if (k < wq && (k == 0 || c != 0)) acc = fma(v, xv, acc);
     }
 }
 
 // Dns: 256 values column-major
-__device__ __forceinline__ void half_dns(const uint8_t *P, const double *X, int r, bool ok, double &acc) {
-    const double *V = reinterpret_cast<const double *>(P) + r;
+__device__ __forceinline__ void half_dns(uint32_t P, uint32_t X, int r, bool ok, double &acc) {
+    const uint32_t V = P + 8 * r;
     double a0 = 0.0, a1 = 0.0;
 #pragma unroll
     for (int c = 0; c < 16; c += 2) {
-        a0 = fma(V[16 * c], X[c], a0);
-        a1 = fma(V[16 * c + 16], X[c + 1], a1);
+        a0 = fma(lds_f64(V + 128 * c), lds_f64(X + 8 * c), a0);
+        a1 = fma(lds_f64(V + 128 * c + 128), lds_f64(X + 8 * c + 8), a1);
     }
     if (ok) acc += a0 + a1;
 }
 
 // DnsCol: full column q holds value q*16 + r, column id colid[q]
-__device__ __forceinline__ void half_dnscol(const uint8_t *P, int nc, const double *X, int r, bool ok, double &acc) {
-    const double *V = reinterpret_cast<const double *>(P);
-    const uint8_t *cid = P + 128 * nc;
+__device__ __forceinline__ void half_dnscol(uint32_t P, int nc, uint32_t X, int r, bool ok, double &acc) {
     const int nq = ok ? nc : 0;
     const int trips = (int)__reduce_max_sync(FULL, (unsigned)nq);
+    const uint32_t cid = P + 128 * nc;
     for (int q = 0; q < trips; ++q) {
-        const double v = V[16 * q + r];
-        const double xv = X[cid[q] & 15];
+        const double v = lds_f64(P + 8 * (16 * q + r));
+        const double xv = lds_f64(X + 8 * (lds_u8(cid + q) & 15u));
         if (q < nq) acc = fma(v, xv, acc);
     }
 }
 
 // DnsRow: full row q (id rowid[q]) holds values q*16 + c; the
 // lane of row rowid[q] sums the 16 products of its row.
-__device__ __forceinline__ void half_dnsrow(const uint8_t *P, int nr, const double *X, int r, bool ok, double &acc) {
-    const double *V = reinterpret_cast<const double *>(P);
-    const uint8_t *rid = P + 128 * nr;
+__device__ __forceinline__ void half_dnsrow(uint32_t P, int nr, uint32_t X, int r, bool ok, double &acc) {
+    const uint32_t rid = P + 128 * nr;
     int q_r = -1;
     const int nq = ok ? nr : 0;
     for (int q = 0; q < 7; ++q)
-        if (q < nq && rid[q] == r) q_r = q;
+        if (q < nq && (int)lds_u8(rid + q) == r) q_r = q;
     const bool mine = q_r >= 0;
-    const double *Vr = V + 16 * (mine ? q_r : 0);
-    const bool any = __any_sync(FULL, mine);
-    if (any) {
+    if (__any_sync(FULL, mine)) {
+        const uint32_t Vr = P + 128 * (mine ? q_r : 0);
         double a0 = 0.0, a1 = 0.0;
 #pragma unroll
         for (int c = 0; c < 16; c += 2) {
-            a0 = fma(Vr[c], X[c], a0);
-            a1 = fma(Vr[c + 1], X[c + 1], a1);
+            a0 = fma(lds_f64(Vr + 8 * c), lds_f64(X + 8 * c), a0);
+            a1 = fma(lds_f64(Vr + 8 * c + 8), lds_f64(X + 8 * c + 8), a1);
         }
         if (mine) acc += a0 + a1;
     }
 }
 
-// COO part: value j, packed (row << 4 | col) byte (Alg. 3); the lane
+// COO entries: value j, packed (row << 4 | col) byte (Alg. 3); the lane
 // of the entry's row adds it (no atomics, fixed order)
-__device__ __forceinline__ void half_coo(const double *V, const uint8_t *rc, int n, const double *X, int r, bool ok,
-                                         double &acc) {
+__device__ __forceinline__ void half_coo(uint32_t V, uint32_t rc, int n, uint32_t X, int r, bool ok, double &acc) {
     const int nq = ok ? n : 0;
     const int trips = (int)__reduce_max_sync(FULL, (unsigned)nq);
 #pragma unroll 2
     for (int j = 0; j < trips; ++j) {
-        const int b = rc[j];
-        const double v = V[j];
-        const double xv = X[b & 15];
-        if (j < nq && (b >> 4) == r) acc = fma(v, xv, acc);
+        const uint32_t b = lds_u8(rc + j);
+        const double v = lds_f64(V + 8 * j);
+        const double xv = lds_f64(X + 8 * (b & 15u));
+        if (j < nq && (int)(b >> 4) == r) acc = fma(v, xv, acc);
     }
 }
 
 // HYB: ELL(w) values | COO values | ELL 4-bit columns | COO (row<<4|col)
-__device__ __forceinline__ void half_hyb(const uint8_t *P, int w, int nz, const double *X, int r, bool ok,
-                                         double &acc) {
-    const double *V = reinterpret_cast<const double *>(P);
+__device__ __forceinline__ void half_hyb(uint32_t P, int w, int nz, uint32_t X, int r, bool ok, double &acc) {
     const int kc = nz - 16 * w;
-    const uint8_t *ei = P + 128 * w + 8 * kc;
+    const uint32_t ei = P + 128 * w + 8 * kc;
     const int wq = ok ? w : 0;
     const int trips = (int)__reduce_max_sync(FULL, (unsigned)wq);
-    const int sh = 4 * (r & 1);
+    const uint32_t sh = 4 * (r & 1);
     for (int k = 0; k < trips; ++k) {
-        const double v = V[16 * k + r];
-        const double xv = X[(ei[8 * k + (r >> 1)] >> sh) & 15];
+        const double v = lds_f64(P + 8 * (16 * k + r));
+        const double xv = lds_f64(X + 8 * ((lds_u8(ei + 8 * k + (r >> 1)) >> sh) & 15u));
         if (k < wq) acc = fma(v, xv, acc);
     }
-    half_coo(V + 16 * w, ei + 8 * w, kc, X, r, ok, acc);
+    half_coo(P + 128 * w, ei + 8 * w, kc, X, r, ok, acc);
 }
 
 // ------------------------------------------------------------ kernel -------
+// tile-list entry: t | aux << 4 | nz << 9 | off16 << 18 | invalid << 27 | fmt << 28
 template <int C, int S>
 __global__ void __launch_bounds__(RingCfg<C, S>::kThreads, 1) tilespmv_fp64_ring(const Params p) {
     using Cfg = RingCfg<C, S>;
     extern __shared__ __align__(128) uint8_t smem[];
-    uint8_t *ring = smem;
-    double *xs_all = reinterpret_cast<double *>(smem + Cfg::kRing);
-    Item *slot_item = reinterpret_cast<Item *>(smem + Cfg::kRing + Cfg::kX);
-    uint64_t *bars = reinterpret_cast<uint64_t *>(smem + Cfg::kRing + Cfg::kX + Cfg::kSlots);
+    Item *slot_item = reinterpret_cast<Item *>(smem + Cfg::kRing + Cfg::kX + Cfg::kList);
+    uint64_t *bars = reinterpret_cast<uint64_t *>(smem + Cfg::kRing + Cfg::kX + Cfg::kList + Cfg::kSlots);
+    const uint32_t sbase = smem_u32(smem);
     const uint32_t full0 = smem_u32(bars), empty0 = smem_u32(bars + S);
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     if (threadIdx.x < S) {
@@ -237,16 +268,15 @@ __global__ void __launch_bounds__(RingCfg<C, S>::kThreads, 1) tilespmv_fp64_ring
     }
     if (threadIdx.x == 0) fence_mbar_init();
     __syncthreads();
-    const int64_t beg = p.cta_begin[blockIdx.x], end = p.cta_begin[blockIdx.x + 1];
+    const int beg = (int)p.cta_begin[blockIdx.x], end = (int)p.cta_begin[blockIdx.x + 1];
 
     if (warp == 0) {
         // ---------------------------------------------------- producer ----
-        // lane j owns slot j: items beg + j, beg + j + S, beg + j + 2S, ...
         if (lane < S) {
             const uint32_t full = full0 + 8 * lane, empty = empty0 + 8 * lane;
-            const uint32_t dst0 = smem_u32(ring) + (uint32_t)lane * kItemBytes;
+            const uint32_t dst0 = sbase + (uint32_t)lane * kItemBytes;
             uint32_t round = 0;
-            for (int64_t k = beg + lane; k < end; k += S, ++round) {
+            for (int k = beg + lane; k < end; k += S, ++round) {
                 const int4 *src = reinterpret_cast<const int4 *>(p.items + k);
                 const int4 a = __ldg(src), b = __ldg(src + 1);
                 Item it;
@@ -278,85 +308,101 @@ __global__ void __launch_bounds__(RingCfg<C, S>::kThreads, 1) tilespmv_fp64_ring
     // -------------------------------------------------------- consumers ---
     const int c = warp - 1;
     const int h = lane >> 4, r = lane & 15;
-    double *xs = xs_all + c * 16 * kItemTiles;
-    for (int64_t q = c; beg + q < end; q += C) {
-        const int slot = (int)(q % S);
-        mbar_wait(full0 + 8 * slot, (uint32_t)(q / S) & 1u);
+    const uint32_t xs = sbase + Cfg::kRing + (uint32_t)c * Cfg::kXPer;
+    const uint32_t list = sbase + Cfg::kRing + Cfg::kX + (uint32_t)c * Cfg::kListPer;
+    const uint32_t n32 = (uint32_t)p.n;
+    const unsigned lt_mask = (1u << lane) - 1u;
+    int slot = c;
+    uint32_t round = 0;
+    for (int k = beg + c; k < end; k += C) {
+        mbar_wait(full0 + 8 * slot, round & 1u);
         const Item it = slot_item[slot];
         const ItemParts pt = item_parts(it, p.m);
-        const uint8_t *pay = ring + (uint32_t)slot * kItemBytes;
+        const uint32_t pay = sbase + (uint32_t)slot * kItemBytes;
         const int nt = it.part_nt >> 24;
         // per-lane tile descriptor (lane t < nt holds tile tb + t)
-        uint2 d = make_uint2(0u, 7u << 27);
-        if (lane < nt) d = reinterpret_cast<const uint2 *>(pay + pt.pay + pt.dsc_skew)[lane];
-        const int fmt = (int)(d.y >> 27) == 0 ? (int)(d.x >> 27) : 7;  // 7: no tile
-        const int aux = (int)(d.y & 31u), nz = (int)((d.y >> 5) & 511u);
-        // byte offset of each tile in the payload: exclusive warp scan of sizes
-        int off = (int)((d.y >> 14) & 255u) * 16;
+        uint2 d = make_uint2(0u, 0u);
+        if (lane < nt) d = lds_v2u32(pay + pt.pay + pt.dsc_skew + 8 * lane);
+        const bool has = lane < nt;
+        const int fmt = has ? (int)(d.x >> 27) : 7;
+        const uint32_t sz16 = (d.y >> 14) & 255u;
+        // payload offset of each tile (16-byte units): exclusive warp scan
+        uint32_t off16 = sz16;
 #pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-            const int v = __shfl_up_sync(FULL, off, o);
-            if (lane >= o) off += v;
+        for (int o = 1; o < 16; o <<= 1) {
+            const uint32_t v = __shfl_up_sync(FULL, off16, o);
+            if (lane >= o) off16 += v;
         }
-        off -= (int)((d.y >> 14) & 255u) * 16;
+        off16 -= sz16;
         // x segments: lane l loads x[16 J_t + (l & 15)] for tiles t = 2k + h
         {
             const uint32_t J = d.x & 0x7FFFFFFu;
             double xv[kItemTiles / 2];
 #pragma unroll
-            for (int k = 0; k < kItemTiles / 2; ++k) {
-                const int t = 2 * k + h;
-                const int64_t col = 16 * (int64_t)__shfl_sync(FULL, J, t) + r;
-                xv[k] = (t < nt && col < p.n) ? __ldg(p.x + col) : 0.0;
+            for (int kk = 0; kk < kItemTiles / 2; ++kk) {
+                const int t = 2 * kk + h;
+                const uint32_t col = 16u * __shfl_sync(FULL, J, t) + (uint32_t)r;
+                xv[kk] = (t < nt && col < n32) ? __ldg(p.x + col) : 0.0;
             }
 #pragma unroll
-            for (int k = 0; k < kItemTiles / 2; ++k) xs[(2 * k + h) * 16 + r] = xv[k];
+            for (int kk = 0; kk < kItemTiles / 2; ++kk) sts_f64(xs + 8 * ((2 * kk + h) * 16 + r), xv[kk]);
+        }
+        // tile list grouped by format, each group padded to an even length
+        int npairs = 0;
+        {
+            const uint32_t entry = (uint32_t)lane | ((d.y & 31u) << 4) | (((d.y >> 5) & 511u) << 9) |
+                                   (off16 << 18) | ((uint32_t)fmt << 28);
+            int base = 0;
+#pragma unroll
+            for (int f = 0; f < 7; ++f) {
+                const unsigned mf = __ballot_sync(FULL, fmt == f);
+                const int cnt = __popc(mf);
+                if (fmt == f) {
+                    const int pos = base + __popc(mf & lt_mask);
+                    sts_u32(list + 4 * pos, entry);
+                    if (pos == base + cnt - 1 && (cnt & 1))  // odd group: invalid partner
+                        sts_u32(list + 4 * (pos + 1), entry | (1u << 27));
+                }
+                base += (cnt + 1) & ~1;
+            }
+            npairs = base >> 1;
         }
         double acc = 0.0;
         if (pt.rp) {
-            const uint8_t *rb = pay + pt.pay + pt.dsc;
-            remainder_rows(p, it.I, it.kb, it.ke, reinterpret_cast<const int *>(rb),
-                           reinterpret_cast<const int *>(rb + pt.rp + pt.col_skew),
-                           reinterpret_cast<const double *>(rb + pt.rp + pt.col + pt.val_skew), lane, acc);
+            const uint32_t rb = pay + pt.pay + pt.dsc;
+            remainder_rows(p, (int)imin64(16, p.m - 16 * (int64_t)it.I), it.kb, it.ke, rb, rb + pt.rp + pt.col_skew,
+                           rb + pt.rp + pt.col + pt.val_skew, lane, acc);
         }
         __syncwarp();
-        // tiles, grouped by format, two at a time (one per half-warp)
-        const unsigned present = __reduce_or_sync(FULL, lane < nt ? 1u << fmt : 0u);
 #pragma unroll 1
-        for (int f = 0; f < 7; ++f) {
-            if (!((present >> f) & 1u)) continue;
-            unsigned mask = __ballot_sync(FULL, fmt == f);
-            while (mask) {
-                const int t0 = __ffs(mask) - 1;
-                mask &= mask - 1;
-                const int t1 = mask ? __ffs(mask) - 1 : -1;
-                if (t1 >= 0) mask &= mask - 1;
-                const int th = h ? t1 : t0;
-                const bool ok = th >= 0;
-                const int src = ok ? th : t0;
-                const int a = __shfl_sync(FULL, aux, src);
-                const int n_ = __shfl_sync(FULL, nz, src);
-                const int o = __shfl_sync(FULL, off, src);
-                const uint8_t *P = pay + o;
-                const double *X = xs + 16 * src;
-                switch (f) {
-                case F_CSR: half_csr(P, n_, X, r, ok, acc); break;
-                case F_ELL: half_ell(P, a, X, r, ok, acc); break;
-                case F_DNS: half_dns(P, X, r, ok, acc); break;
-                case F_DNSCOL: half_dnscol(P, a, X, r, ok, acc); break;
-                case F_DNSROW: half_dnsrow(P, a, X, r, ok, acc); break;
-                case F_COO:
-                    half_coo(reinterpret_cast<const double *>(P), P + 8 * n_, n_, X, r, ok, acc);
-                    break;
-                case F_HYB: half_hyb(P, a, n_, X, r, ok, acc); break;
-                default: break;
-                }
+        for (int q = 0; q < npairs; ++q) {
+            const uint32_t e = (uint32_t)lds_s32(list + 8 * q + 4 * h);
+            const int f = (int)(e >> 28);  // same for both halves by construction
+            const bool ok = !((e >> 27) & 1u);
+            const int a = (int)((e >> 4) & 31u);
+            const int nz = (int)((e >> 9) & 511u);
+            const uint32_t P = pay + 16 * ((e >> 18) & 511u);
+            const uint32_t X = xs + 128 * (e & 15u);
+            switch (f) {
+            case F_CSR: half_csr(P, nz, X, r, ok, acc); break;
+            case F_ELL: half_ell(P, a, X, r, ok, acc); break;
+            case F_DNS: half_dns(P, X, r, ok, acc); break;
+            case F_DNSCOL: half_dnscol(P, a, X, r, ok, acc); break;
+            case F_DNSROW: half_dnsrow(P, a, X, r, ok, acc); break;
+            case F_COO: half_coo(P, P + 8 * nz, nz, X, r, ok, acc); break;
+            case F_HYB: half_hyb(P, a, nz, X, r, ok, acc); break;
+            default: break;
             }
         }
         acc += __shfl_xor_sync(FULL, acc, 16);
         write_rows(p, it, lane, acc);
         __syncwarp();
         if (lane == 0) mbar_arrive(empty0 + 8 * slot);
+        slot += C;
+        if (slot >= S) {
+            slot -= S;
+            ++round;
+        }
     }
 }
 
@@ -374,6 +420,7 @@ KernelChoice kernel_ring(int variant) {
     case 5: return ring_choice<12, 24>("ring_c12_s24");
     case 6: return ring_choice<4, 24>("ring_c4_s24");
     case 7: return ring_choice<10, 20>("ring_c10_s20");
+    case 8: return ring_choice<11, 22>("ring_c11_s22");
     default: return ring_choice<12, 24>("ring_c12_s24");
     }
 }
