@@ -70,66 +70,6 @@ __device__ __forceinline__ void sts_f64(uint32_t a, double v) {
     asm volatile("st.shared.f64 [%0], %1;" ::"r"(a), "d"(v) : "memory");
 }
 
-// ------------------------------------------------ remainder (from smem) ----
-// rows of at most kShortRow entries: two lanes per row; longer rows: the
-// whole warp strides the row and reduces with a butterfly (fixed order).
-// rpS/colS/valS: shared addresses of remRowPtr[16I..], remCol[kb..], remVal[kb..]
-__device__ __forceinline__ void remainder_rows(const Params &p, int rows, int kb, int ke, uint32_t rpS, uint32_t colS,
-                                               uint32_t valS, int lane, double &acc) {
-    const int r = lane & 15, h = lane >> 4;
-    int b = lds_s32(rpS + 4 * min(r, rows)), e = lds_s32(rpS + 4 * min(r + 1, rows));
-    b = max(b, kb) - kb;
-    e = min(e, ke) - kb;
-    const int len = max(e - b, 0);
-    const bool is_short = len <= kShortRow;
-    const int nshort = is_short ? len : 0;
-    const int trips = (int)__reduce_max_sync(FULL, (unsigned)((nshort + 1 - h) >> 1));
-    if (trips > 0) {
-        int cs[kShortRow / 2];
-        double vs[kShortRow / 2], xs[kShortRow / 2];
-#pragma unroll
-        for (int i = 0; i < kShortRow / 2; ++i) {
-            const int k = b + h + 2 * i;
-            const bool ok = i < trips && k < b + nshort;
-            cs[i] = ok ? lds_s32(colS + 4 * k) : 0;
-            vs[i] = ok ? lds_f64(valS + 8 * k) : 0.0;
-        }
-#pragma unroll
-        for (int i = 0; i < kShortRow / 2; ++i) {
-            const bool ok = i < trips && b + h + 2 * i < b + nshort;
-            xs[i] = ok ? __ldg(p.x + (uint32_t)cs[i]) : 0.0;
-        }
-#pragma unroll
-        for (int i = 0; i < kShortRow / 2; ++i)
-            if (i < trips && b + h + 2 * i < b + nshort) acc = fma(vs[i], xs[i], acc);
-    }
-    unsigned longs = __ballot_sync(FULL, lane < 16 && !is_short);
-    while (longs) {
-        const int rr = __ffs(longs) - 1;
-        longs &= longs - 1;
-        const int bb = __shfl_sync(FULL, b, rr), ee = __shfl_sync(FULL, e, rr);
-        double s = 0.0;
-        for (int k0 = bb; k0 < ee; k0 += 128) {
-            int cs[4];
-            double vs[4], xv[4];
-#pragma unroll
-            for (int i = 0; i < 4; ++i) {
-                const int k = k0 + lane + 32 * i;
-                cs[i] = k < ee ? lds_s32(colS + 4 * k) : 0;
-                vs[i] = k < ee ? lds_f64(valS + 8 * k) : 0.0;
-            }
-#pragma unroll
-            for (int i = 0; i < 4; ++i) xv[i] = (k0 + lane + 32 * i < ee) ? __ldg(p.x + (uint32_t)cs[i]) : 0.0;
-#pragma unroll
-            for (int i = 0; i < 4; ++i)
-                if (k0 + lane + 32 * i < ee) s = fma(vs[i], xv[i], s);
-        }
-#pragma unroll
-        for (int o = 16; o >= 1; o >>= 1) s += __shfl_xor_sync(FULL, s, o);
-        if (lane == rr) acc += s;
-    }
-}
-
 // --------------------------------------------- half-warp tile routines -----
 // Lane r of a half owns row r of its tile.  P: shared address of the tile's
 // payload, X: of its 16 x values; ok: the half has a tile (else it runs the
@@ -150,14 +90,17 @@ __device__ __forceinline__ void half_csr(uint32_t P, int nz, uint32_t X, int r, 
     const uint32_t b_odd = cb + odd;
     const uint32_t s_even = 4 * odd, s_odd = 4 - 4 * odd;
     const uint32_t V = P + 8 * beg;
-#pragma unroll 4
-    for (int i = 0; i < trips; ++i) {
-        const uint32_t byte = (i & 1) ? lds_u8(b_odd + (i >> 1)) : lds_u8(cb + (i >> 1));
-        const uint32_t c = (byte >> ((i & 1) ? s_odd : s_even)) & 15u;
-        const double v = lds_f64(V + 8 * i);
-        const double xv = lds_f64(X + 8 * c);
-        if (i < len) acc = fma(v, xv, acc);
+    double a1 = 0.0;
+#pragma unroll 1
+    for (int i = 0; i < trips; i += 2) {  // two independent FMA chains
+        const uint32_t c0 = (lds_u8(cb + (i >> 1)) >> s_even) & 15u;
+        const uint32_t c1 = (lds_u8(b_odd + (i >> 1)) >> s_odd) & 15u;
+        const double v0 = lds_f64(V + 8 * i), v1 = lds_f64(V + 8 * i + 8);
+        const double x0 = lds_f64(X + 8 * c0), x1 = lds_f64(X + 8 * c1);
+        if (i < len) acc = fma(v0, x0, acc);
+        if (i + 1 < len) a1 = fma(v1, x1, a1);
     }
+    acc += a1;
 }
 
 // ELL: slots k*16 + r column-major | 4-bit columns (Alg. 4).
@@ -306,27 +249,82 @@ __global__ void __launch_bounds__(RingCfg<C, S>::kThreads, 1) tilespmv_fp64_ring
     }
 
     // -------------------------------------------------------- consumers ---
+    // Software pipeline: while item k is computed, the global x loads of
+    // item k + C (this consumer's next item) are already in flight.
     const int c = warp - 1;
     const int h = lane >> 4, r = lane & 15;
     const uint32_t xs = sbase + Cfg::kRing + (uint32_t)c * Cfg::kXPer;
     const uint32_t list = sbase + Cfg::kRing + Cfg::kX + (uint32_t)c * Cfg::kListPer;
     const uint32_t n32 = (uint32_t)p.n;
     const unsigned lt_mask = (1u << lane) - 1u;
+
+    struct Prep {
+        Item it;
+        ItemParts pt;
+        uint32_t pay;
+        uint2 d;
+        double xt[kItemTiles / 2];  // x[16 J_t + r] for tiles t = 2k + h
+        double xr[kShortRow / 2];   // x of this lane's short remainder entries
+    };
+    auto prepare = [&](Prep &P, int slot, uint32_t round) {
+        mbar_wait(full0 + 8 * slot, round & 1u);
+        P.it = slot_item[slot];
+        P.pt = item_parts(P.it, p.m);
+        P.pay = sbase + (uint32_t)slot * kItemBytes;
+        const int nt = P.it.part_nt >> 24;
+        P.d = make_uint2(0u, 0u);
+        if (lane < nt) P.d = lds_v2u32(P.pay + P.pt.pay + P.pt.dsc_skew + 8 * lane);
+        const uint32_t J = P.d.x & 0x7FFFFFFu;
+#pragma unroll
+        for (int kk = 0; kk < kItemTiles / 2; ++kk) {
+            const int t = 2 * kk + h;
+            const uint32_t col = 16u * __shfl_sync(FULL, J, t) + (uint32_t)r;
+            P.xt[kk] = (t < nt && col < n32) ? __ldg(p.x + col) : 0.0;
+        }
+#pragma unroll
+        for (int i = 0; i < kShortRow / 2; ++i) P.xr[i] = 0.0;
+        if (P.pt.rp) {  // x of the short remainder rows (two lanes per row)
+            const uint32_t rb = P.pay + P.pt.pay + P.pt.dsc;
+            const int rows = (int)imin64(16, p.m - 16 * (int64_t)P.it.I);
+            int b = lds_s32(rb + 4 * min(r, rows)), e = lds_s32(rb + 4 * min(r + 1, rows));
+            b = max(b, P.it.kb) - P.it.kb;
+            e = min(e, P.it.ke) - P.it.kb;
+            const uint32_t colS = rb + P.pt.rp + P.pt.col_skew;
+            if (e - b <= kShortRow) {
+#pragma unroll
+                for (int i = 0; i < kShortRow / 2; ++i) {
+                    const int kq = b + h + 2 * i;
+                    if (kq < e) P.xr[i] = __ldg(p.x + (uint32_t)lds_s32(colS + 4 * kq));
+                }
+            }
+        }
+    };
+
+    int k = beg + c;
+    if (k >= end) return;
     int slot = c;
     uint32_t round = 0;
-    for (int k = beg + c; k < end; k += C) {
-        mbar_wait(full0 + 8 * slot, round & 1u);
-        const Item it = slot_item[slot];
-        const ItemParts pt = item_parts(it, p.m);
-        const uint32_t pay = sbase + (uint32_t)slot * kItemBytes;
+    Prep cur;
+    prepare(cur, slot, round);
+    for (;;) {
+        // next item of this consumer: issue its loads before computing this one
+        int nslot = slot + C;
+        uint32_t nround = round;
+        if (nslot >= S) {
+            nslot -= S;
+            ++nround;
+        }
+        const bool has_next = k + C < end;
+        Prep nxt;
+        if (has_next) prepare(nxt, nslot, nround);
+
+        const Item &it = cur.it;
+        const ItemParts &pt = cur.pt;
+        const uint32_t pay = cur.pay;
         const int nt = it.part_nt >> 24;
-        // per-lane tile descriptor (lane t < nt holds tile tb + t)
-        uint2 d = make_uint2(0u, 0u);
-        if (lane < nt) d = lds_v2u32(pay + pt.pay + pt.dsc_skew + 8 * lane);
         const bool has = lane < nt;
-        const int fmt = has ? (int)(d.x >> 27) : 7;
-        const uint32_t sz16 = (d.y >> 14) & 255u;
-        // payload offset of each tile (16-byte units): exclusive warp scan
+        const int fmt = has ? (int)(cur.d.x >> 27) : 7;
+        const uint32_t sz16 = (cur.d.y >> 14) & 255u;
         uint32_t off16 = sz16;
 #pragma unroll
         for (int o = 1; o < 16; o <<= 1) {
@@ -334,23 +332,12 @@ __global__ void __launch_bounds__(RingCfg<C, S>::kThreads, 1) tilespmv_fp64_ring
             if (lane >= o) off16 += v;
         }
         off16 -= sz16;
-        // x segments: lane l loads x[16 J_t + (l & 15)] for tiles t = 2k + h
-        {
-            const uint32_t J = d.x & 0x7FFFFFFu;
-            double xv[kItemTiles / 2];
 #pragma unroll
-            for (int kk = 0; kk < kItemTiles / 2; ++kk) {
-                const int t = 2 * kk + h;
-                const uint32_t col = 16u * __shfl_sync(FULL, J, t) + (uint32_t)r;
-                xv[kk] = (t < nt && col < n32) ? __ldg(p.x + col) : 0.0;
-            }
-#pragma unroll
-            for (int kk = 0; kk < kItemTiles / 2; ++kk) sts_f64(xs + 8 * ((2 * kk + h) * 16 + r), xv[kk]);
-        }
+        for (int kk = 0; kk < kItemTiles / 2; ++kk) sts_f64(xs + 8 * ((2 * kk + h) * 16 + r), cur.xt[kk]);
         // tile list grouped by format, each group padded to an even length
-        int npairs = 0;
+        int npairs;
         {
-            const uint32_t entry = (uint32_t)lane | ((d.y & 31u) << 4) | (((d.y >> 5) & 511u) << 9) |
+            const uint32_t entry = (uint32_t)lane | ((cur.d.y & 31u) << 4) | (((cur.d.y >> 5) & 511u) << 9) |
                                    (off16 << 18) | ((uint32_t)fmt << 28);
             int base = 0;
 #pragma unroll
@@ -360,8 +347,7 @@ __global__ void __launch_bounds__(RingCfg<C, S>::kThreads, 1) tilespmv_fp64_ring
                 if (fmt == f) {
                     const int pos = base + __popc(mf & lt_mask);
                     sts_u32(list + 4 * pos, entry);
-                    if (pos == base + cnt - 1 && (cnt & 1))  // odd group: invalid partner
-                        sts_u32(list + 4 * (pos + 1), entry | (1u << 27));
+                    if (pos == base + cnt - 1 && (cnt & 1)) sts_u32(list + 4 * (pos + 1), entry | (1u << 27));
                 }
                 base += (cnt + 1) & ~1;
             }
@@ -370,8 +356,44 @@ __global__ void __launch_bounds__(RingCfg<C, S>::kThreads, 1) tilespmv_fp64_ring
         double acc = 0.0;
         if (pt.rp) {
             const uint32_t rb = pay + pt.pay + pt.dsc;
-            remainder_rows(p, (int)imin64(16, p.m - 16 * (int64_t)it.I), it.kb, it.ke, rb, rb + pt.rp + pt.col_skew,
-                           rb + pt.rp + pt.col + pt.val_skew, lane, acc);
+            const int rows = (int)imin64(16, p.m - 16 * (int64_t)it.I);
+            int b = lds_s32(rb + 4 * min(r, rows)), e = lds_s32(rb + 4 * min(r + 1, rows));
+            b = max(b, it.kb) - it.kb;
+            e = min(e, it.ke) - it.kb;
+            const uint32_t colS = rb + pt.rp + pt.col_skew, valS = rb + pt.rp + pt.col + pt.val_skew;
+            const bool is_short = e - b <= kShortRow;
+            if (is_short) {
+#pragma unroll
+                for (int i = 0; i < kShortRow / 2; ++i) {
+                    const int kq = b + h + 2 * i;
+                    if (kq < e) acc = fma(lds_f64(valS + 8 * kq), cur.xr[i], acc);
+                }
+            }
+            unsigned longs = __ballot_sync(FULL, lane < 16 && !is_short);
+            while (longs) {  // rows longer than kShortRow: the whole warp strides the row
+                const int rr = __ffs(longs) - 1;
+                longs &= longs - 1;
+                const int bb = __shfl_sync(FULL, b, rr), ee = __shfl_sync(FULL, e, rr);
+                double s = 0.0;
+                for (int k0 = bb; k0 < ee; k0 += 128) {
+                    int cs[4];
+                    double vs[4], xv[4];
+#pragma unroll
+                    for (int i = 0; i < 4; ++i) {
+                        const int kq = k0 + lane + 32 * i;
+                        cs[i] = kq < ee ? lds_s32(colS + 4 * kq) : 0;
+                        vs[i] = kq < ee ? lds_f64(valS + 8 * kq) : 0.0;
+                    }
+#pragma unroll
+                    for (int i = 0; i < 4; ++i) xv[i] = (k0 + lane + 32 * i < ee) ? __ldg(p.x + (uint32_t)cs[i]) : 0.0;
+#pragma unroll
+                    for (int i = 0; i < 4; ++i)
+                        if (k0 + lane + 32 * i < ee) s = fma(vs[i], xv[i], s);
+                }
+#pragma unroll
+                for (int o = 16; o >= 1; o >>= 1) s += __shfl_xor_sync(FULL, s, o);
+                if (lane == rr) acc += s;
+            }
         }
         __syncwarp();
 #pragma unroll 1
@@ -398,11 +420,11 @@ __global__ void __launch_bounds__(RingCfg<C, S>::kThreads, 1) tilespmv_fp64_ring
         write_rows(p, it, lane, acc);
         __syncwarp();
         if (lane == 0) mbar_arrive(empty0 + 8 * slot);
-        slot += C;
-        if (slot >= S) {
-            slot -= S;
-            ++round;
-        }
+        if (!has_next) break;
+        k += C;
+        slot = nslot;
+        round = nround;
+        cur = nxt;
     }
 }
 
