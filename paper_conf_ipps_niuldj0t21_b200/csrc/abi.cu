@@ -110,6 +110,7 @@ int tilespmv_create_from_csr(tilespmv_handle_t *out, int64_t m, int64_t n, int64
     M->mode = o.mode == TILESPMV_MODE_AUTO ? (nnz >= 1800000 ? TILESPMV_MODE_DEFERRED : TILESPMV_MODE_ADPT)
                                            : o.mode;
     int rc = build_tiled(*M, d_rowptr, d_colidx, d_val, o.validate, st);
+    if (!rc) rc = choose_kernel(*M);
     if (!rc) rc = build_schedule(*M, st);
     if (!rc) rc = build_tdesc(*M, st);
     if (!rc) rc = configure_launch(*M);

@@ -21,14 +21,14 @@ enum : uint8_t { F_CSR = 0, F_COO = 1, F_ELL = 2, F_HYB = 3, F_DNS = 4, F_DNSROW
 // of at most kItemTiles consecutive tiles and/or a range of remainder entries
 // of the tile row's 16 rows, such that everything the kernel stages for it
 // (payloads, 8-byte tile descriptors, remainder rowptr/col/val) fits one
-// kItemBytes shared-memory slot.  A tile row split over several items writes
+// shared-memory slot (the kernel's slot size, <= kItemBytesMax).  A tile row split over several items writes
 // per-item partials that the last finishing item sums in item order
 // (deterministic; replaces the atomic merge of tbalance).  Item
 // boundaries depend only on the tile row's own content, so a tile-row-sharded
 // run reproduces the 1-GPU y bitwise.
 // ---------------------------------------------------------------------------
 constexpr int kItemTiles = 16;
-constexpr int kItemBytes = 8192;  // one shared-memory slot
+constexpr int kItemBytesMax = 8192;  // largest shared-memory slot of any kernel
 constexpr int kShortRow = 8;      // remainder rows up to this length: 2 lanes per row
 
 struct __align__(16) Item {
@@ -74,6 +74,7 @@ struct Matrix {
     int64_t *cta_begin = nullptr;  // contiguous item chunk per CTA
     // launch shape
     int kernel_version = 2;
+    int item_bytes = kItemBytesMax;  // slot size the schedule was built for
     int grid = 0, block = 0, smem = 0;
 };
 
@@ -85,6 +86,7 @@ int cuda_status(cudaError_t e, const char *what);
 int build_tiled(Matrix &M, const int32_t *d_rowptr, const int32_t *d_colidx, const double *d_val,
                 int validate, cudaStream_t stream);
 // spmv.cu
+int choose_kernel(Matrix &M);
 int build_schedule(Matrix &M, cudaStream_t stream);
 int build_tdesc(Matrix &M, cudaStream_t stream);
 int configure_launch(Matrix &M);

@@ -22,11 +22,11 @@ namespace tsp {
 namespace {
 
 // Greedy split of tile row I into items whose staged bytes (item_parts)
-// never exceed kItemBytes: tiles first (at most kItemTiles), then the tile
+// never exceed the kernel's slot size (budget): tiles first (at most kItemTiles), then the tile
 // row's remainder entries.  Depends only on the tile row's own content.
 template <bool WRITE>
 __device__ int items_for_row(int64_t I, const int32_t *tilePtr, const uint32_t *tileOff, const int32_t *remRowPtr,
-                             int64_t m, Item *out, int split) {
+                             int64_t m, int budget, Item *out, int split) {
     const int tp0 = tilePtr[I], tp1 = tilePtr[I + 1];
     int k0 = 0, k1 = 0;
     if (remRowPtr) {
@@ -42,7 +42,7 @@ __device__ int items_for_row(int64_t I, const int32_t *tilePtr, const uint32_t *
         while (t < tp1 && t - tb < kItemTiles) {
             const uint32_t pay = (tileOff[t + 1] - tileOff[tb]) * 16u;
             const uint32_t dsc = up16((uint32_t)(tb & 1) * 8u + 8u * (uint32_t)(t - tb + 1));
-            if (pay + dsc > (uint32_t)kItemBytes) break;
+            if (pay + dsc > (uint32_t)budget) break;
             used = pay + dsc;
             t++;
         }
@@ -52,7 +52,7 @@ __device__ int items_for_row(int64_t I, const int32_t *tilePtr, const uint32_t *
         }
         int kb = k, ke = k;
         if (t == tp1 && k < k1) {
-            const int64_t avail = (int64_t)kItemBytes - used - rp_bytes - 64;  // 2 x 32 B skew slack
+            const int64_t avail = (int64_t)budget - used - rp_bytes - 64;  // 2 x 32 B skew slack
             const int64_t e = imin64(avail > 0 ? avail / 12 : 0, k1 - k);
             if (e > 0) {
                 ke = k + (int)e;
@@ -77,23 +77,23 @@ __device__ int items_for_row(int64_t I, const int32_t *tilePtr, const uint32_t *
 }
 
 __global__ void k_items_count(const int32_t *tilePtr, const uint32_t *tileOff, const int32_t *remRowPtr, int64_t m,
-                              int64_t tilem, int32_t *nitems, int32_t *nsplit, int32_t *parts) {
+                              int budget, int64_t tilem, int32_t *nitems, int32_t *nsplit, int32_t *parts) {
     int64_t I = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     if (I >= tilem) return;
-    const int c = items_for_row<false>(I, tilePtr, tileOff, remRowPtr, m, nullptr, -1);
+    const int c = items_for_row<false>(I, tilePtr, tileOff, remRowPtr, m, budget, nullptr, -1);
     nitems[I] = c;
     nsplit[I] = c > 1 ? 1 : 0;
     parts[I] = c > 1 ? c : 0;
 }
 
 __global__ void k_items_write(const int32_t *tilePtr, const uint32_t *tileOff, const int32_t *remRowPtr, int64_t m,
-                              int64_t tilem, const int32_t *itemBase, const int32_t *splitId, const int32_t *nitems,
+                              int budget, int64_t tilem, const int32_t *itemBase, const int32_t *splitId, const int32_t *nitems,
                               const int32_t *partBase, Item *items, int2 *split_info) {
     int64_t I = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     if (I >= tilem) return;
     const bool split = nitems[I] > 1;
     const int sid = split ? splitId[I] : -1;
-    items_for_row<true>(I, tilePtr, tileOff, remRowPtr, m, items + itemBase[I], sid);
+    items_for_row<true>(I, tilePtr, tileOff, remRowPtr, m, budget, items + itemBase[I], sid);
     if (split) split_info[sid] = make_int2(partBase[I], nitems[I]);
 }
 
@@ -163,7 +163,7 @@ int build_schedule(Matrix &M, cudaStream_t st) {
     int rc = 0;
     do {
         if (cudaMemsetAsync(buf, 0, 3 * (T + 1) * sizeof(int32_t), st) != cudaSuccess) { rc = cuda_status(cudaGetLastError(), "memset"); break; }
-        k_items_count<<<blocks(T), TB, 0, st>>>(M.tilePtr, M.tileOff, M.remRowPtr, M.m, T, nitems, nsplit, parts);
+        k_items_count<<<blocks(T), TB, 0, st>>>(M.tilePtr, M.tileOff, M.remRowPtr, M.m, M.item_bytes, T, nitems, nsplit, parts);
         if ((rc = scan([&](void *t, size_t &b) { return cub::DeviceScan::ExclusiveSum(t, b, nitems, itemBase, (int)(T + 1), st); }))) break;
         if ((rc = scan([&](void *t, size_t &b) { return cub::DeviceScan::ExclusiveSum(t, b, nsplit, splitId, (int)(T + 1), st); }))) break;
         if ((rc = scan([&](void *t, size_t &b) { return cub::DeviceScan::ExclusiveSum(t, b, parts, partBase, (int)(T + 1), st); }))) break;
@@ -184,7 +184,7 @@ int build_schedule(Matrix &M, cudaStream_t st) {
         }
         M.device_bytes += M.num_items * (int64_t)sizeof(Item) + M.num_split * 12 + nparts * 128;
         cudaMemsetAsync(M.counters, 0, std::max<int64_t>(M.num_split, 1) * sizeof(int32_t), st);
-        k_items_write<<<blocks(T), TB, 0, st>>>(M.tilePtr, M.tileOff, M.remRowPtr, M.m, T, itemBase, splitId, nitems,
+        k_items_write<<<blocks(T), TB, 0, st>>>(M.tilePtr, M.tileOff, M.remRowPtr, M.m, M.item_bytes, T, itemBase, splitId, nitems,
                                                 partBase, M.items, M.split_info);
         if (cudaStreamSynchronize(st) != cudaSuccess) rc = cuda_status(cudaGetLastError(), "k_items_write");
     } while (0);
@@ -203,16 +203,22 @@ int build_tdesc(Matrix &M, cudaStream_t st) {
     return 0;
 }
 
-int configure_launch(Matrix &M) {
-    int version = 2;
+int choose_kernel(Matrix &M) {
+    int version = 0;
     if (const char *e = getenv("TILESPMV_KERNEL")) version = atoi(e);
+    M.kernel_version = version;
+    M.item_bytes = choose(version).slot_bytes;
+    return 0;
+}
+
+int configure_launch(Matrix &M) {
+    const int version = M.kernel_version;
     const KernelChoice kc = choose(version);
     TSP_CK(cudaFuncSetAttribute(kc.fn, cudaFuncAttributeMaxDynamicSharedMemorySize, kc.smem));
     int sms = 0, per_sm = 0;
     TSP_CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, M.device));
     TSP_CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kc.fn, kc.threads, kc.smem));
     if (per_sm < 1) return set_error(TILESPMV_CUDA, "SpMV kernel does not fit on an SM");
-    M.kernel_version = version;
     M.block = kc.threads;
     M.smem = kc.smem;
     if (!kc.ring) {

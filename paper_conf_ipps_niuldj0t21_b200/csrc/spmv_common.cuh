@@ -146,6 +146,7 @@ struct KernelChoice {
     void (*fn)(Params);
     int threads, smem, ctas_per_sm;
     bool ring;
+    int slot_bytes;  // item budget the schedule must respect
 };
 KernelChoice kernel_v1();
 KernelChoice kernel_ring(int variant);

@@ -27,11 +27,13 @@
 namespace tsp {
 namespace {
 
-template <int C, int S>
+template <int C, int S, int SLOT>
 struct RingCfg {
     static_assert(S % C == 0, "slot s must always be served by consumer s mod C");
     static_assert(S <= 32, "one producer lane per slot");
-    static constexpr uint32_t kRing = (uint32_t)S * kItemBytes;
+    static_assert(SLOT % 16 == 0 && SLOT <= kItemBytesMax, "slot size");
+    static constexpr uint32_t kItemBytes = SLOT;
+    static constexpr uint32_t kRing = (uint32_t)S * SLOT;
     static constexpr uint32_t kXPer = kItemTiles * 16 * 8;  // x segments per consumer
     static constexpr uint32_t kListPer = 128;               // tile list per consumer
     static constexpr uint32_t kX = (uint32_t)C * kXPer;
@@ -196,9 +198,10 @@ __device__ __forceinline__ void half_hyb(uint32_t P, int w, int nz, uint32_t X, 
 
 // ------------------------------------------------------------ kernel -------
 // tile-list entry: t | aux << 4 | nz << 9 | off16 << 18 | invalid << 27 | fmt << 28
-template <int C, int S>
-__global__ void __launch_bounds__(RingCfg<C, S>::kThreads, 1) tilespmv_fp64_ring(const Params p) {
-    using Cfg = RingCfg<C, S>;
+template <int C, int S, int SLOT>
+__global__ void __launch_bounds__(RingCfg<C, S, SLOT>::kThreads, 1) tilespmv_fp64_ring(const Params p) {
+    using Cfg = RingCfg<C, S, SLOT>;
+    constexpr uint32_t kItemBytes = Cfg::kItemBytes;
     extern __shared__ __align__(128) uint8_t smem[];
     Item *slot_item = reinterpret_cast<Item *>(smem + Cfg::kRing + Cfg::kX + Cfg::kList);
     uint64_t *bars = reinterpret_cast<uint64_t *>(smem + Cfg::kRing + Cfg::kX + Cfg::kList + Cfg::kSlots);
@@ -428,22 +431,26 @@ __global__ void __launch_bounds__(RingCfg<C, S>::kThreads, 1) tilespmv_fp64_ring
     }
 }
 
-template <int C, int S>
+template <int C, int S, int SLOT>
 KernelChoice ring_choice(const char *name) {
-    return {name, tilespmv_fp64_ring<C, S>, RingCfg<C, S>::kThreads, (int)RingCfg<C, S>::kSmem, 1, true};
+    using Cfg = RingCfg<C, S, SLOT>;
+    return {name, tilespmv_fp64_ring<C, S, SLOT>, Cfg::kThreads, (int)Cfg::kSmem, 1, true, SLOT};
 }
 
 }  // namespace
 
+// consumers C, slots S (S/C slots per consumer: >= 3 lets the next item's x
+// loads overlap the current item), slot size SLOT bytes
 KernelChoice kernel_ring(int variant) {
     switch (variant) {
-    case 3: return ring_choice<8, 24>("ring_c8_s24");
-    case 4: return ring_choice<6, 24>("ring_c6_s24");
-    case 5: return ring_choice<12, 24>("ring_c12_s24");
-    case 6: return ring_choice<4, 24>("ring_c4_s24");
-    case 7: return ring_choice<10, 20>("ring_c10_s20");
-    case 8: return ring_choice<11, 22>("ring_c11_s22");
-    default: return ring_choice<12, 24>("ring_c12_s24");
+    case 3: return ring_choice<8, 24, 8192>("ring_c8_s24_8k");
+    case 4: return ring_choice<10, 30, 5120>("ring_c10_s30_5k");
+    case 5: return ring_choice<8, 32, 6144>("ring_c8_s32_6k");
+    case 6: return ring_choice<12, 24, 8192>("ring_c12_s24_8k");
+    case 7: return ring_choice<9, 27, 6144>("ring_c9_s27_6k");
+    case 8: return ring_choice<7, 28, 6144>("ring_c7_s28_6k");
+    case 9: return ring_choice<10, 30, 6144>("ring_c10_s30_6k");
+    default: return ring_choice<10, 30, 5120>("ring_c10_s30_5k");
     }
 }
 

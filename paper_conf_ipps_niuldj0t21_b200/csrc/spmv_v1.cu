@@ -11,7 +11,7 @@ namespace {
 
 constexpr int kWarps = 4;                                   // warps per CTA
 constexpr int kXBytes = kItemTiles * 16 * 8;                // x segments per item
-constexpr int kWarpSmem = kItemBytes + kXBytes + 128;       // + mbarrier slot
+constexpr int kWarpSmem = kItemBytesMax + kXBytes + 128;       // + mbarrier slot
 constexpr int kSmemBytes = kWarps * kWarpSmem;
 
 // ------------------------------------------------------- remainder rows ---
@@ -180,8 +180,8 @@ __global__ void __launch_bounds__(kWarps * 32) tilespmv_fp64_kernel(const Params
     extern __shared__ __align__(128) uint8_t smem[];
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     uint8_t *buf = smem + warp * kWarpSmem;
-    double *sx = reinterpret_cast<double *>(buf + kItemBytes);
-    const uint32_t bar = smem_u32(buf + kItemBytes + kXBytes);
+    double *sx = reinterpret_cast<double *>(buf + kItemBytesMax);
+    const uint32_t bar = smem_u32(buf + kItemBytesMax + kXBytes);
     const uint32_t buf_s = smem_u32(buf);
     if (lane == 0) {
         mbar_init(bar, 1);
@@ -272,7 +272,7 @@ __global__ void __launch_bounds__(kWarps * 32) tilespmv_fp64_kernel(const Params
 }  // namespace
 
 KernelChoice kernel_v1() {
-    return {"v1_warp_staged", tilespmv_fp64_kernel, kWarps * 32, kSmemBytes, 0, false};
+    return {"v1_warp_staged", tilespmv_fp64_kernel, kWarps * 32, kSmemBytes, 0, false, kItemBytesMax};
 }
 
 }  // namespace tsp
