@@ -39,6 +39,9 @@ struct __align__(16) Item {
     uint32_t offe;    // payload offset one past the last tile
     int32_t split;    // split-row index, or -1 if the item covers its whole tile row
     int32_t part_nt;  // (part index within the split row) | (number of tiles << 24)
+    int32_t dbeg;     // first entry of the item's tile-descriptor list (dlist)
+    int32_t ndsc;     // entries: the item's tiles grouped by format, groups padded to even length
+    int32_t pad0, pad1;
 };
 
 struct Matrix {
@@ -70,7 +73,8 @@ struct Matrix {
     int64_t device_bytes = 0;
     double create_ms = 0;
     // v2 kernel inputs derived from the canonical arrays
-    uint2 *tdesc = nullptr;        // 8-byte packed tile descriptors
+    uint2 *tdesc = nullptr;        // per-item tile-descriptor lists (dlist)
+    int64_t num_dsc = 0;
     int64_t *cta_begin = nullptr;  // contiguous item chunk per CTA
     // launch shape
     int kernel_version = 2;

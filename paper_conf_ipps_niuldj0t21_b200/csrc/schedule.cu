@@ -41,13 +41,14 @@ __device__ int items_for_row(int64_t I, const int32_t *tilePtr, const uint32_t *
         uint32_t used = 0;
         while (t < tp1 && t - tb < kItemTiles) {
             const uint32_t pay = (tileOff[t + 1] - tileOff[tb]) * 16u;
-            const uint32_t dsc = up16((uint32_t)(tb & 1) * 8u + 8u * (uint32_t)(t - tb + 1));
+            // descriptor list: <= ntiles + 7 pad entries, 8 B each, + 8 B skew
+            const uint32_t dsc = up16(8u + 8u * (uint32_t)(t - tb + 1 + 7));
             if (pay + dsc > (uint32_t)budget) break;
             used = pay + dsc;
             t++;
         }
         if (t == tb && t < tp1) {  // unreachable: one tile (<= 2176 B) always fits
-            used = (tileOff[t + 1] - tileOff[tb]) * 16u + 16u;
+            used = (tileOff[t + 1] - tileOff[tb]) * 16u + 80u;
             t++;
         }
         int kb = k, ke = k;
@@ -69,6 +70,9 @@ __device__ int items_for_row(int64_t I, const int32_t *tilePtr, const uint32_t *
             it.offe = tileOff[t];
             it.split = split;
             it.part_nt = (split >= 0 ? cnt : 0) | ((t - tb) << 24);
+            it.dbeg = 0;
+            it.ndsc = 0;
+            it.pad0 = it.pad1 = 0;
             out[cnt] = it;
         }
         cnt++;
@@ -97,15 +101,50 @@ __global__ void k_items_write(const int32_t *tilePtr, const uint32_t *tileOff, c
     if (split) split_info[sid] = make_int2(partBase[I], nitems[I]);
 }
 
-// x = J | fmt << 27 ; y = aux | nnz << 5 | size16 << 14
-__global__ void k_build_tdesc(const int32_t *tileColIdx, const uint8_t *tileFmt, const uint8_t *tileAux,
-                              const int32_t *tileNnz, const uint32_t *tileOff, int64_t numtile, uint2 *tdesc) {
-    int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
-    if (t >= numtile) return;
-    uint2 d;
-    d.x = (uint32_t)tileColIdx[t] | ((uint32_t)tileFmt[t] << 27);
-    d.y = (uint32_t)tileAux[t] | ((uint32_t)(tileNnz[t + 1] - tileNnz[t]) << 5) | ((tileOff[t + 1] - tileOff[t]) << 14);
-    tdesc[t] = d;
+// Per-item tile-descriptor list: the item's tiles grouped by format (format
+// order, tile order inside a group), every odd group padded with a copy of
+// its last entry marked invalid, so a half-warp pair never mixes formats.
+// Entry: x = J | fmt << 27 ; y = aux | nnz << 5 | off16 << 14 | t << 23 | invalid << 27
+// (off16: payload offset inside the item in 16-byte units, t: tile index in the item).
+__global__ void k_dsc_count(Item *items, int64_t n, const uint8_t *tileFmt, int32_t *ndsc) {
+    int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (k >= n) return;
+    const Item it = items[k];
+    const int nt = it.part_nt >> 24;
+    int cnt[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+    for (int t = 0; t < nt; ++t) cnt[tileFmt[it.tb + t] & 7]++;
+    int total = 0;
+    for (int f = 0; f < 7; ++f) total += (cnt[f] + 1) & ~1;
+    ndsc[k] = total;
+}
+
+__global__ void k_dsc_write(Item *items, int64_t n, const int32_t *dbeg, const int32_t *ndsc, const int32_t *tileColIdx,
+                            const uint8_t *tileFmt, const uint8_t *tileAux, const int32_t *tileNnz,
+                            const uint32_t *tileOff, uint2 *dlist) {
+    int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (k >= n) return;
+    Item it = items[k];
+    const int nt = it.part_nt >> 24;
+    int pos = dbeg[k];
+    it.dbeg = pos;
+    it.ndsc = ndsc[k];
+    items[k] = it;
+    for (int f = 0; f < 7; ++f) {
+        uint2 last = make_uint2(0u, 0u);
+        int c = 0;
+        for (int t = 0; t < nt; ++t) {
+            const int g = it.tb + t;
+            if (tileFmt[g] != f) continue;
+            uint2 d;
+            d.x = (uint32_t)tileColIdx[g] | ((uint32_t)f << 27);
+            d.y = (uint32_t)tileAux[g] | ((uint32_t)(tileNnz[g + 1] - tileNnz[g]) << 5) |
+                  ((tileOff[g] - it.offb) << 14) | ((uint32_t)t << 23);
+            dlist[pos++] = d;
+            last = d;
+            c++;
+        }
+        if (c & 1) dlist[pos++] = make_uint2(last.x, last.y | (1u << 27));
+    }
 }
 
 // item cost for the CTA chunking: bytes staged + a fixed per-item overhead
@@ -193,14 +232,32 @@ int build_schedule(Matrix &M, cudaStream_t st) {
 }
 
 int build_tdesc(Matrix &M, cudaStream_t st) {
-    TSP_CK(cudaMalloc(&M.tdesc, (M.numtile + 2) * sizeof(uint2)));  // +2: 16-byte superset reads
-    M.device_bytes += (M.numtile + 2) * 8;
-    if (M.numtile > 0) {
-        k_build_tdesc<<<(unsigned)((M.numtile + 255) / 256), 256, 0, st>>>(M.tileColIdx, M.tileFmt, M.tileAux, M.tileNnz,
-                                                                           M.tileOff, M.numtile, M.tdesc);
-        TSP_CK(cudaGetLastError());
+    const int64_t n = M.num_items;
+    if (n == 0) {
+        TSP_CK(cudaMalloc(&M.tdesc, 4 * sizeof(uint2)));
+        return 0;
     }
-    return 0;
+    int32_t *cnt = nullptr;
+    TSP_CK(cudaMalloc(&cnt, 2 * (n + 1) * sizeof(int32_t)));
+    int32_t *beg = cnt + (n + 1);
+    const unsigned nb = (unsigned)((n + 255) / 256);
+    int rc = 0;
+    do {
+        if (cudaMemsetAsync(cnt + n, 0, sizeof(int32_t), st) != cudaSuccess) { rc = cuda_status(cudaGetLastError(), "memset"); break; }
+        k_dsc_count<<<nb, 256, 0, st>>>(M.items, n, M.tileFmt, cnt);
+        if ((rc = scan([&](void *t, size_t &b) { return cub::DeviceScan::ExclusiveSum(t, b, cnt, beg, (int)(n + 1), st); }))) break;
+        int32_t total = 0;
+        cudaMemcpyAsync(&total, beg + n, 4, cudaMemcpyDeviceToHost, st);
+        if (cudaStreamSynchronize(st) != cudaSuccess) { rc = cuda_status(cudaGetLastError(), "dsc sizes"); break; }
+        M.num_dsc = total;
+        if (cudaMalloc(&M.tdesc, (total + 4) * sizeof(uint2)) != cudaSuccess) { rc = cuda_status(cudaGetLastError(), "cudaMalloc(dlist)"); break; }
+        M.device_bytes += (total + 4) * 8;
+        k_dsc_write<<<nb, 256, 0, st>>>(M.items, n, beg, cnt, M.tileColIdx, M.tileFmt, M.tileAux, M.tileNnz, M.tileOff,
+                                         M.tdesc);
+        if (cudaStreamSynchronize(st) != cudaSuccess) rc = cuda_status(cudaGetLastError(), "k_dsc_write");
+    } while (0);
+    cudaFree(cnt);
+    return rc;
 }
 
 int choose_kernel(Matrix &M) {

@@ -27,7 +27,7 @@ struct Params {
     const double *x;
     double *y;
     int64_t m, n;
-    const uint2 *tdesc;        // packed tile descriptors (schedule.cu)
+    const uint2 *tdesc;        // per-item tile-descriptor lists (schedule.cu)
     const int64_t *cta_begin;  // contiguous item chunk per CTA (ring kernels)
 };
 
@@ -93,10 +93,9 @@ struct ItemParts {
 
 __host__ __device__ __forceinline__ ItemParts item_parts(const Item &it, int64_t m) {
     ItemParts r;
-    const int nt = it.part_nt >> 24;
     r.pay = (it.offe - it.offb) * 16u;
-    r.dsc_skew = (uint32_t)(it.tb & 1) * 8u;
-    r.dsc = nt ? up16(r.dsc_skew + 8u * (uint32_t)nt) : 0u;
+    r.dsc_skew = (uint32_t)(it.dbeg & 1) * 8u;
+    r.dsc = it.ndsc ? up16(r.dsc_skew + 8u * (uint32_t)it.ndsc) : 0u;
     if (it.ke > it.kb) {
         const int64_t rows = imin64(16, m - 16 * (int64_t)it.I);
         r.rp = up16((uint32_t)(rows + 1) * 4u);

@@ -92,15 +92,22 @@ __device__ __forceinline__ void half_csr(uint32_t P, int nz, uint32_t X, int r, 
     const uint32_t b_odd = cb + odd;
     const uint32_t s_even = 4 * odd, s_odd = 4 - 4 * odd;
     const uint32_t V = P + 8 * beg;
+    // four entries per iteration: independent load chains, two FMA chains
     double a1 = 0.0;
 #pragma unroll 1
-    for (int i = 0; i < trips; i += 2) {  // two independent FMA chains
+    for (int i = 0; i < trips; i += 4) {
         const uint32_t c0 = (lds_u8(cb + (i >> 1)) >> s_even) & 15u;
         const uint32_t c1 = (lds_u8(b_odd + (i >> 1)) >> s_odd) & 15u;
+        const uint32_t c2 = (lds_u8(cb + (i >> 1) + 1) >> s_even) & 15u;
+        const uint32_t c3 = (lds_u8(b_odd + (i >> 1) + 1) >> s_odd) & 15u;
         const double v0 = lds_f64(V + 8 * i), v1 = lds_f64(V + 8 * i + 8);
+        const double v2 = lds_f64(V + 8 * i + 16), v3 = lds_f64(V + 8 * i + 24);
         const double x0 = lds_f64(X + 8 * c0), x1 = lds_f64(X + 8 * c1);
+        const double x2 = lds_f64(X + 8 * c2), x3 = lds_f64(X + 8 * c3);
         if (i < len) acc = fma(v0, x0, acc);
         if (i + 1 < len) a1 = fma(v1, x1, a1);
+        if (i + 2 < len) acc = fma(v2, x2, acc);
+        if (i + 3 < len) a1 = fma(v3, x3, a1);
     }
     acc += a1;
 }
@@ -197,7 +204,7 @@ __device__ __forceinline__ void half_hyb(uint32_t P, int w, int nz, uint32_t X, 
 }
 
 // ------------------------------------------------------------ kernel -------
-// tile-list entry: t | aux << 4 | nz << 9 | off16 << 18 | invalid << 27 | fmt << 28
+// descriptor entries: see k_dsc_write (schedule.cu)
 template <int C, int S, int SLOT>
 __global__ void __launch_bounds__(RingCfg<C, S, SLOT>::kThreads, 1) tilespmv_fp64_ring(const Params p) {
     using Cfg = RingCfg<C, S, SLOT>;
@@ -224,10 +231,11 @@ __global__ void __launch_bounds__(RingCfg<C, S, SLOT>::kThreads, 1) tilespmv_fp6
             uint32_t round = 0;
             for (int k = beg + lane; k < end; k += S, ++round) {
                 const int4 *src = reinterpret_cast<const int4 *>(p.items + k);
-                const int4 a = __ldg(src), b = __ldg(src + 1);
+                const int4 a = __ldg(src), b = __ldg(src + 1), e = __ldg(src + 2);
                 Item it;
                 it.I = a.x; it.tb = a.y; it.kb = a.z; it.ke = a.w;
                 it.offb = (uint32_t)b.x; it.offe = (uint32_t)b.y; it.split = b.z; it.part_nt = b.w;
+                it.dbeg = e.x; it.ndsc = e.y; it.pad0 = e.z; it.pad1 = e.w;
                 if (round > 0) mbar_wait(empty, (round - 1) & 1u);
                 slot_item[lane] = it;
                 const ItemParts pt = item_parts(it, p.m);
@@ -237,7 +245,7 @@ __global__ void __launch_bounds__(RingCfg<C, S, SLOT>::kThreads, 1) tilespmv_fp6
                 if (pt.pay) bulk_g2s(d, p.payload + (size_t)it.offb * 16, pt.pay, full);
                 d += pt.pay;
                 if (pt.dsc)
-                    bulk_g2s(d, reinterpret_cast<const uint8_t *>(p.tdesc + it.tb) - pt.dsc_skew, pt.dsc, full);
+                    bulk_g2s(d, reinterpret_cast<const uint8_t *>(p.tdesc + it.dbeg) - pt.dsc_skew, pt.dsc, full);
                 d += pt.dsc;
                 if (pt.rp) {
                     bulk_g2s(d, p.remRowPtr + 16 * (int64_t)it.I, pt.rp, full);
@@ -259,30 +267,34 @@ __global__ void __launch_bounds__(RingCfg<C, S, SLOT>::kThreads, 1) tilespmv_fp6
     const uint32_t xs = sbase + Cfg::kRing + (uint32_t)c * Cfg::kXPer;
     const uint32_t list = sbase + Cfg::kRing + Cfg::kX + (uint32_t)c * Cfg::kListPer;
     const uint32_t n32 = (uint32_t)p.n;
-    const unsigned lt_mask = (1u << lane) - 1u;
 
     struct Prep {
         Item it;
         ItemParts pt;
         uint32_t pay;
-        uint2 d;
         double xt[kItemTiles / 2];  // x[16 J_t + r] for tiles t = 2k + h
         double xr[kShortRow / 2];   // x of this lane's short remainder entries
     };
+    // list = per-consumer scratch: J of each tile by tile index (64 B)
     auto prepare = [&](Prep &P, int slot, uint32_t round) {
         mbar_wait(full0 + 8 * slot, round & 1u);
         P.it = slot_item[slot];
         P.pt = item_parts(P.it, p.m);
         P.pay = sbase + (uint32_t)slot * kItemBytes;
         const int nt = P.it.part_nt >> 24;
-        P.d = make_uint2(0u, 0u);
-        if (lane < nt) P.d = lds_v2u32(P.pay + P.pt.pay + P.pt.dsc_skew + 8 * lane);
-        const uint32_t J = P.d.x & 0x7FFFFFFu;
+        if (lane < P.it.ndsc) {
+            const uint2 d = lds_v2u32(P.pay + P.pt.pay + P.pt.dsc_skew + 8 * lane);
+            if (!((d.y >> 27) & 1u)) sts_u32(list + 4 * ((d.y >> 23) & 15u), d.x & 0x7FFFFFFu);
+        }
+        __syncwarp();
 #pragma unroll
         for (int kk = 0; kk < kItemTiles / 2; ++kk) {
             const int t = 2 * kk + h;
-            const uint32_t col = 16u * __shfl_sync(FULL, J, t) + (uint32_t)r;
-            P.xt[kk] = (t < nt && col < n32) ? __ldg(p.x + col) : 0.0;
+            P.xt[kk] = 0.0;
+            if (t < nt) {
+                const uint32_t col = 16u * (uint32_t)lds_s32(list + 4 * t) + (uint32_t)r;
+                if (col < n32) P.xt[kk] = __ldg(p.x + col);
+            }
         }
 #pragma unroll
         for (int i = 0; i < kShortRow / 2; ++i) P.xr[i] = 0.0;
@@ -301,6 +313,7 @@ __global__ void __launch_bounds__(RingCfg<C, S, SLOT>::kThreads, 1) tilespmv_fp6
                 }
             }
         }
+        __syncwarp();  // list scratch reusable
     };
 
     int k = beg + c;
@@ -324,38 +337,10 @@ __global__ void __launch_bounds__(RingCfg<C, S, SLOT>::kThreads, 1) tilespmv_fp6
         const Item &it = cur.it;
         const ItemParts &pt = cur.pt;
         const uint32_t pay = cur.pay;
-        const int nt = it.part_nt >> 24;
-        const bool has = lane < nt;
-        const int fmt = has ? (int)(cur.d.x >> 27) : 7;
-        const uint32_t sz16 = (cur.d.y >> 14) & 255u;
-        uint32_t off16 = sz16;
-#pragma unroll
-        for (int o = 1; o < 16; o <<= 1) {
-            const uint32_t v = __shfl_up_sync(FULL, off16, o);
-            if (lane >= o) off16 += v;
-        }
-        off16 -= sz16;
 #pragma unroll
         for (int kk = 0; kk < kItemTiles / 2; ++kk) sts_f64(xs + 8 * ((2 * kk + h) * 16 + r), cur.xt[kk]);
-        // tile list grouped by format, each group padded to an even length
-        int npairs;
-        {
-            const uint32_t entry = (uint32_t)lane | ((cur.d.y & 31u) << 4) | (((cur.d.y >> 5) & 511u) << 9) |
-                                   (off16 << 18) | ((uint32_t)fmt << 28);
-            int base = 0;
-#pragma unroll
-            for (int f = 0; f < 7; ++f) {
-                const unsigned mf = __ballot_sync(FULL, fmt == f);
-                const int cnt = __popc(mf);
-                if (fmt == f) {
-                    const int pos = base + __popc(mf & lt_mask);
-                    sts_u32(list + 4 * pos, entry);
-                    if (pos == base + cnt - 1 && (cnt & 1)) sts_u32(list + 4 * (pos + 1), entry | (1u << 27));
-                }
-                base += (cnt + 1) & ~1;
-            }
-            npairs = base >> 1;
-        }
+        const int npairs = it.ndsc >> 1;
+        const uint32_t dsc = pay + pt.pay + pt.dsc_skew;
         double acc = 0.0;
         if (pt.rp) {
             const uint32_t rb = pay + pt.pay + pt.dsc;
@@ -401,13 +386,13 @@ __global__ void __launch_bounds__(RingCfg<C, S, SLOT>::kThreads, 1) tilespmv_fp6
         __syncwarp();
 #pragma unroll 1
         for (int q = 0; q < npairs; ++q) {
-            const uint32_t e = (uint32_t)lds_s32(list + 8 * q + 4 * h);
-            const int f = (int)(e >> 28);  // same for both halves by construction
-            const bool ok = !((e >> 27) & 1u);
-            const int a = (int)((e >> 4) & 31u);
-            const int nz = (int)((e >> 9) & 511u);
-            const uint32_t P = pay + 16 * ((e >> 18) & 511u);
-            const uint32_t X = xs + 128 * (e & 15u);
+            const uint2 e = lds_v2u32(dsc + 16 * q + 8 * h);
+            const int f = (int)(e.x >> 27);  // same for both halves by construction
+            const bool ok = !((e.y >> 27) & 1u);
+            const int a = (int)(e.y & 31u);
+            const int nz = (int)((e.y >> 5) & 511u);
+            const uint32_t P = pay + 16 * ((e.y >> 14) & 511u);
+            const uint32_t X = xs + 128 * ((e.y >> 23) & 15u);
             switch (f) {
             case F_CSR: half_csr(P, nz, X, r, ok, acc); break;
             case F_ELL: half_ell(P, a, X, r, ok, acc); break;
@@ -450,6 +435,9 @@ KernelChoice kernel_ring(int variant) {
     case 7: return ring_choice<9, 27, 6144>("ring_c9_s27_6k");
     case 8: return ring_choice<7, 28, 6144>("ring_c7_s28_6k");
     case 9: return ring_choice<10, 30, 6144>("ring_c10_s30_6k");
+    case 10: return ring_choice<16, 32, 5632>("ring_c16_s32_5.5k");
+    case 11: return ring_choice<14, 28, 6144>("ring_c14_s28_6k");
+    case 12: return ring_choice<13, 26, 6656>("ring_c13_s26_6.5k");
     default: return ring_choice<10, 30, 5120>("ring_c10_s30_5k");
     }
 }
