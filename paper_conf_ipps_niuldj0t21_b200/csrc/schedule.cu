@@ -186,7 +186,11 @@ int scan(F &&f) {
     return 0;
 }
 
-KernelChoice choose(int version) { return version == 1 ? kernel_v1() : kernel_ring(version); }
+KernelChoice choose(int version) {
+    if (version == 1) return kernel_v1();
+    if (version >= 20 && version < 30) return kernel_warp(version);
+    return kernel_ring(version);
+}
 
 }  // namespace
 

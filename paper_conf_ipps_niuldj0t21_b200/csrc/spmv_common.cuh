@@ -149,5 +149,6 @@ struct KernelChoice {
 };
 KernelChoice kernel_v1();
 KernelChoice kernel_ring(int variant);
+KernelChoice kernel_warp(int variant);
 
 }  // namespace tsp

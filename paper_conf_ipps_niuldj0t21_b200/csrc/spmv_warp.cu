@@ -1,0 +1,177 @@
+// spmv_warp.cu -- high-occupancy variant of the tiled SpMV (TILESPMV_KERNEL
+// 20+): every warp is its own producer and consumer.  Per work item, lane 0
+// stages the item (tile payloads, descriptor list, remainder rowptr/col/val)
+// into the warp's shared-memory slot with TMA bulk copies on the warp's
+// mbarrier; the warp then gathers the x segments, runs the half-warp tile
+// routines of spmv_tiles.cuh and writes y.  Latency is hidden by warp count
+// (~32 warps/SM with small slots) instead of by a deep per-CTA ring; the next
+// item's descriptor is prefetched into registers.
+#include "spmv_tiles.cuh"
+
+namespace tsp {
+namespace {
+
+template <int WARPS, int SLOT>
+struct WarpCfg {
+    static_assert(SLOT % 16 == 0 && SLOT <= kItemBytesMax, "slot size");
+    static constexpr uint32_t kX = kItemTiles * 16 * 8;
+    static constexpr uint32_t kPer = SLOT + kX + 64 + 16;  // slot | x | J scratch | mbarrier
+    static constexpr uint32_t kSmem = WARPS * kPer + 256;   // +256: loads may overrun a slot
+    static constexpr int kThreads = 32 * WARPS;
+};
+
+__device__ __forceinline__ Item load_item(const Item *items, int k) {
+    const int4 *src = reinterpret_cast<const int4 *>(items + k);
+    const int4 a = __ldg(src), b = __ldg(src + 1), e = __ldg(src + 2);
+    Item it;
+    it.I = a.x; it.tb = a.y; it.kb = a.z; it.ke = a.w;
+    it.offb = (uint32_t)b.x; it.offe = (uint32_t)b.y; it.split = b.z; it.part_nt = b.w;
+    it.dbeg = e.x; it.ndsc = e.y; it.pad0 = e.z; it.pad1 = e.w;
+    return it;
+}
+
+template <int WARPS, int SLOT, int MINB>
+__global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, MINB) tilespmv_fp64_warp(const Params p) {
+    using Cfg = WarpCfg<WARPS, SLOT>;
+    extern __shared__ __align__(128) uint8_t smem[];
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int h = lane >> 4, r = lane & 15;
+    const uint32_t base = smem_u32(smem) + (uint32_t)warp * Cfg::kPer;
+    const uint32_t slot = base, xs = base + SLOT, jt = xs + Cfg::kX, bar = jt + 64;
+    if (lane == 0) {
+        mbar_init(bar, 1);
+        fence_mbar_init();
+    }
+    __syncwarp();
+    const uint32_t n32 = (uint32_t)p.n;
+    // contiguous item chunk per warp (x segments of neighbouring tile rows are shared)
+    const int64_t gw = (int64_t)blockIdx.x * WARPS + warp, nw = (int64_t)gridDim.x * WARPS;
+    const int kbeg = (int)(p.num_items * gw / nw), kend = (int)(p.num_items * (gw + 1) / nw);
+    uint32_t phase = 0;
+    Item nxt;
+    if (kbeg < kend) nxt = load_item(p.items, kbeg);
+    for (int k = kbeg; k < kend; ++k) {
+        const Item it = nxt;
+        if (k + 1 < kend) nxt = load_item(p.items, k + 1);  // in flight during this item
+        const ItemParts pt = item_parts(it, p.m);
+        if (lane == 0 && pt.total) {
+            fence_proxy_async();
+            mbar_expect_tx(bar, pt.total);
+            uint32_t d = slot;
+            if (pt.pay) bulk_g2s(d, p.payload + (size_t)it.offb * 16, pt.pay, bar);
+            d += pt.pay;
+            if (pt.dsc) bulk_g2s(d, reinterpret_cast<const uint8_t *>(p.tdesc + it.dbeg) - pt.dsc_skew, pt.dsc, bar);
+            d += pt.dsc;
+            if (pt.rp) {
+                bulk_g2s(d, p.remRowPtr + 16 * (int64_t)it.I, pt.rp, bar);
+                d += pt.rp;
+                bulk_g2s(d, reinterpret_cast<const uint8_t *>(p.remCol + it.kb) - pt.col_skew, pt.col, bar);
+                d += pt.col;
+                bulk_g2s(d, reinterpret_cast<const uint8_t *>(p.remVal + it.kb) - pt.val_skew, pt.val, bar);
+            }
+        }
+        if (pt.total) {
+            mbar_wait(bar, phase);
+            phase ^= 1u;
+        }
+        const int nt = it.part_nt >> 24;
+        const uint32_t dsc = slot + pt.pay + pt.dsc_skew;
+        // J of every tile by tile index, then the x segments (lane: tile 2k+h, element r)
+        if (lane < it.ndsc) {
+            const uint2 d = lds_v2u32(dsc + 8 * lane);
+            if (!((d.y >> 27) & 1u)) sts_u32(jt + 4 * ((d.y >> 23) & 15u), d.x & 0x7FFFFFFu);
+        }
+        __syncwarp();
+        {
+            double xv[kItemTiles / 2];
+#pragma unroll
+            for (int kk = 0; kk < kItemTiles / 2; ++kk) {
+                const int t = 2 * kk + h;
+                xv[kk] = 0.0;
+                if (t < nt) {
+                    const uint32_t col = 16u * (uint32_t)lds_s32(jt + 4 * t) + (uint32_t)r;
+                    if (col < n32) xv[kk] = __ldg(p.x + col);
+                }
+            }
+#pragma unroll
+            for (int kk = 0; kk < kItemTiles / 2; ++kk) sts_f64(xs + 8 * ((2 * kk + h) * 16 + r), xv[kk]);
+        }
+        double acc = 0.0;
+        if (pt.rp) {  // fused CSR remainder: two lanes per short row, warp per long row
+            const uint32_t rb = slot + pt.pay + pt.dsc;
+            const int rows = (int)imin64(16, p.m - 16 * (int64_t)it.I);
+            int b = lds_s32(rb + 4 * min(r, rows)), e = lds_s32(rb + 4 * min(r + 1, rows));
+            b = max(b, it.kb) - it.kb;
+            e = min(e, it.ke) - it.kb;
+            const uint32_t colS = rb + pt.rp + pt.col_skew, valS = rb + pt.rp + pt.col + pt.val_skew;
+            const bool is_short = e - b <= kShortRow;
+            if (is_short) {
+                int cs[kShortRow / 2];
+                double vs[kShortRow / 2], xr[kShortRow / 2];
+#pragma unroll
+                for (int i = 0; i < kShortRow / 2; ++i) {
+                    const int kq = b + h + 2 * i;
+                    cs[i] = kq < e ? lds_s32(colS + 4 * kq) : 0;
+                    vs[i] = kq < e ? lds_f64(valS + 8 * kq) : 0.0;
+                }
+#pragma unroll
+                for (int i = 0; i < kShortRow / 2; ++i) xr[i] = (b + h + 2 * i < e) ? __ldg(p.x + (uint32_t)cs[i]) : 0.0;
+#pragma unroll
+                for (int i = 0; i < kShortRow / 2; ++i)
+                    if (b + h + 2 * i < e) acc = fma(vs[i], xr[i], acc);
+            }
+            unsigned longs = __ballot_sync(FULL, lane < 16 && !is_short);
+            while (longs) {
+                const int rr = __ffs(longs) - 1;
+                longs &= longs - 1;
+                const int bb = __shfl_sync(FULL, b, rr), ee = __shfl_sync(FULL, e, rr);
+                double s = 0.0;
+                for (int k0 = bb; k0 < ee; k0 += 128) {
+                    int cs[4];
+                    double vs[4], xv[4];
+#pragma unroll
+                    for (int i = 0; i < 4; ++i) {
+                        const int kq = k0 + lane + 32 * i;
+                        cs[i] = kq < ee ? lds_s32(colS + 4 * kq) : 0;
+                        vs[i] = kq < ee ? lds_f64(valS + 8 * kq) : 0.0;
+                    }
+#pragma unroll
+                    for (int i = 0; i < 4; ++i) xv[i] = (k0 + lane + 32 * i < ee) ? __ldg(p.x + (uint32_t)cs[i]) : 0.0;
+#pragma unroll
+                    for (int i = 0; i < 4; ++i)
+                        if (k0 + lane + 32 * i < ee) s = fma(vs[i], xv[i], s);
+                }
+#pragma unroll
+                for (int o = 16; o >= 1; o >>= 1) s += __shfl_xor_sync(FULL, s, o);
+                if (lane == rr) acc += s;
+            }
+        }
+        __syncwarp();
+        const int npairs = it.ndsc >> 1;
+#pragma unroll 1
+        for (int q = 0; q < npairs; ++q) run_pair(lds_v2u32(dsc + 16 * q + 8 * h), slot, xs, r, acc);
+        acc += __shfl_xor_sync(FULL, acc, 16);
+        write_rows(p, it, lane, acc);
+        __syncwarp();  // slot, x and J scratch free for the next item
+    }
+}
+
+template <int WARPS, int SLOT, int MINB>
+KernelChoice warp_choice(const char *name) {
+    using Cfg = WarpCfg<WARPS, SLOT>;
+    return {name, tilespmv_fp64_warp<WARPS, SLOT, MINB>, Cfg::kThreads, (int)Cfg::kSmem, 0, false, SLOT};
+}
+
+}  // namespace
+
+KernelChoice kernel_warp(int variant) {
+    switch (variant) {
+    case 21: return warp_choice<8, 4608, 4>("warp_w8x4_4.5k");
+    case 22: return warp_choice<8, 5120, 3>("warp_w8x3_5k");
+    case 23: return warp_choice<4, 4608, 8>("warp_w4x8_4.5k");
+    case 24: return warp_choice<8, 4096, 4>("warp_w8x4_4k");
+    default: return warp_choice<8, 4608, 4>("warp_w8x4_4.5k");
+    }
+}
+
+}  // namespace tsp
