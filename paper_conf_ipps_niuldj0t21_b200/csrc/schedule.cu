@@ -3,7 +3,8 @@
 //     by one thread per tile row in two passes (count, scan, write);
 //   * 8-byte tile descriptors derived from the canonical level-1 arrays;
 //   * contiguous, cost-balanced item chunks per CTA for the ring kernels;
-//   * kernel choice (TILESPMV_KERNEL env: 1 = v1 baseline, else ring variant).
+//   * kernel choice (TILESPMV_KERNEL env: 1 = v1 baseline, 20-29 = warp kernel
+//     (default 20), else a ring-kernel variant).
 #include <cub/cub.cuh>
 
 #include <algorithm>
@@ -265,7 +266,7 @@ int build_tdesc(Matrix &M, cudaStream_t st) {
 }
 
 int choose_kernel(Matrix &M) {
-    int version = 0;
+    int version = 20;  // default: high-occupancy warp kernel (spmv_warp.cu)
     if (const char *e = getenv("TILESPMV_KERNEL")) version = atoi(e);
     M.kernel_version = version;
     M.item_bytes = choose(version).slot_bytes;
