@@ -39,9 +39,10 @@ struct __align__(16) Item {
     uint32_t offe;    // payload offset one past the last tile
     int32_t split;    // split-row index, or -1 if the item covers its whole tile row
     int32_t part_nt;  // (part index within the split row) | (number of tiles << 24)
-    int32_t dbeg;     // first entry of the item's tile-descriptor list (dlist)
-    int32_t ndsc;     // entries: the item's tiles grouped by format, groups padded to even length
-    int32_t pad0, pad1;
+    int32_t dbeg;      // first entry of the item's tile-descriptor list (dlist)
+    int32_t ndsc;      // entries: the item's tiles grouped by format, groups padded to even length
+    uint32_t blob16;   // start of the item's execution blob (16-byte units)
+    uint32_t blob_len; // bytes of the blob (blob_parts)
 };
 
 struct Matrix {
@@ -73,8 +74,10 @@ struct Matrix {
     int64_t device_bytes = 0;
     double create_ms = 0;
     // v2 kernel inputs derived from the canonical arrays
-    uint2 *tdesc = nullptr;        // per-item tile-descriptor lists (dlist)
+    uint2 *tdesc = nullptr;        // per-item tile-descriptor lists (dlist), create-time only
     int64_t num_dsc = 0;
+    uint8_t *blob = nullptr;       // per-item execution blobs (blob_parts), read by the kernels
+    int64_t blob_bytes = 0;
     int64_t *cta_begin = nullptr;  // contiguous item chunk per CTA
     // launch shape
     int kernel_version = 2;

@@ -2,9 +2,8 @@
 //   * work items: byte-bounded pieces of one tile row (internal.cuh), built
 //     by one thread per tile row in two passes (count, scan, write);
 //   * 8-byte tile descriptors derived from the canonical level-1 arrays;
-//   * contiguous, cost-balanced item chunks per CTA for the ring kernels;
 //   * kernel choice (TILESPMV_KERNEL env: 1 = v1 baseline, 20-29 = warp kernel
-//     (default 20), else a ring-kernel variant).
+//     variants, default 20).
 #include <cub/cub.cuh>
 
 #include <algorithm>
@@ -42,8 +41,8 @@ __device__ int items_for_row(int64_t I, const int32_t *tilePtr, const uint32_t *
         uint32_t used = 0;
         while (t < tp1 && t - tb < kItemTiles) {
             const uint32_t pay = (tileOff[t + 1] - tileOff[tb]) * 16u;
-            // descriptor list: <= ntiles + 7 pad entries, 8 B each, + 8 B skew
-            const uint32_t dsc = up16(8u + 8u * (uint32_t)(t - tb + 1 + 7));
+            // blob: descriptor list (<= ntiles + 7 pads) + J array (blob_parts)
+            const uint32_t dsc = up16(8u * (uint32_t)(t - tb + 1 + 7)) + up16(4u * (uint32_t)(t - tb + 1));
             if (pay + dsc > (uint32_t)budget) break;
             used = pay + dsc;
             t++;
@@ -73,7 +72,8 @@ __device__ int items_for_row(int64_t I, const int32_t *tilePtr, const uint32_t *
             it.part_nt = (split >= 0 ? cnt : 0) | ((t - tb) << 24);
             it.dbeg = 0;
             it.ndsc = 0;
-            it.pad0 = it.pad1 = 0;
+            it.blob16 = 0;
+            it.blob_len = 0;
             out[cnt] = it;
         }
         cnt++;
@@ -148,6 +148,55 @@ __global__ void k_dsc_write(Item *items, int64_t n, const int32_t *dbeg, const i
     }
 }
 
+__global__ void k_blob_len(const Item *items, int64_t n, int64_t m, int64_t *len16) {
+    int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (k >= n) return;
+    len16[k] = blob_parts(items[k], m).total / 16;
+}
+
+// one warp per item: copy descriptors, J, payload and the rebased remainder
+__global__ void k_blob_fill(Item *items, int64_t n, int64_t m, const int64_t *start16, const uint2 *dlist,
+                            const int32_t *tileColIdx, const uint8_t *payload, const int32_t *remRowPtr,
+                            const int32_t *remCol, const double *remVal, uint8_t *blob) {
+    const int64_t k = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+    const int lane = threadIdx.x & 31;
+    if (k >= n) return;
+    Item it = items[k];
+    const BlobParts b = blob_parts(it, m);
+    uint8_t *dst = blob + start16[k] * 16;
+    if (lane == 0) {
+        it.blob16 = (uint32_t)start16[k];
+        it.blob_len = b.total;
+        items[k] = it;
+    }
+    for (uint32_t o = 4 * lane; o < b.total; o += 128) *reinterpret_cast<uint32_t *>(dst + o) = 0u;  // padding
+    __syncwarp();
+    uint2 *dd = reinterpret_cast<uint2 *>(dst);
+    for (int i = lane; i < it.ndsc; i += 32) dd[i] = dlist[it.dbeg + i];
+    const int nt = it.part_nt >> 24;
+    int32_t *jt = reinterpret_cast<int32_t *>(dst + b.jt);
+    for (int t = lane; t < nt; t += 32) jt[t] = tileColIdx[it.tb + t];
+    const uint4 *ps = reinterpret_cast<const uint4 *>(payload + (size_t)it.offb * 16);
+    uint4 *pd = reinterpret_cast<uint4 *>(dst + b.pay);
+    for (uint32_t i = lane; i < it.offe - it.offb; i += 32) pd[i] = ps[i];
+    if (it.ke > it.kb) {
+        const int rows = (int)imin64(16, m - 16 * (int64_t)it.I);
+        int32_t *rp = reinterpret_cast<int32_t *>(dst + b.rp);
+        if (lane <= rows) {
+            int v = remRowPtr[16 * (int64_t)it.I + lane];
+            v = v < it.kb ? it.kb : (v > it.ke ? it.ke : v);
+            rp[lane] = v - it.kb;
+        }
+        int32_t *cd = reinterpret_cast<int32_t *>(dst + b.col);
+        unsigned long long *vd = reinterpret_cast<unsigned long long *>(dst + b.val);
+        const unsigned long long *vs = reinterpret_cast<const unsigned long long *>(remVal);
+        for (int i = lane; i < it.ke - it.kb; i += 32) {
+            cd[i] = remCol[it.kb + i];
+            vd[i] = vs[it.kb + i];
+        }
+    }
+}
+
 // item cost for the CTA chunking: bytes staged + a fixed per-item overhead
 __global__ void k_item_cost(const Item *items, int64_t n, int64_t m, int64_t *cost) {
     int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
@@ -189,8 +238,7 @@ int scan(F &&f) {
 
 KernelChoice choose(int version) {
     if (version == 1) return kernel_v1();
-    if (version >= 20 && version < 30) return kernel_warp(version);
-    return kernel_ring(version);
+    return kernel_warp(version);
 }
 
 }  // namespace
@@ -240,6 +288,7 @@ int build_tdesc(Matrix &M, cudaStream_t st) {
     const int64_t n = M.num_items;
     if (n == 0) {
         TSP_CK(cudaMalloc(&M.tdesc, 4 * sizeof(uint2)));
+        TSP_CK(cudaMalloc(&M.blob, 256));
         return 0;
     }
     int32_t *cnt = nullptr;
@@ -259,7 +308,25 @@ int build_tdesc(Matrix &M, cudaStream_t st) {
         M.device_bytes += (total + 4) * 8;
         k_dsc_write<<<nb, 256, 0, st>>>(M.items, n, beg, cnt, M.tileColIdx, M.tileFmt, M.tileAux, M.tileNnz, M.tileOff,
                                          M.tdesc);
-        if (cudaStreamSynchronize(st) != cudaSuccess) rc = cuda_status(cudaGetLastError(), "k_dsc_write");
+        if (cudaStreamSynchronize(st) != cudaSuccess) { rc = cuda_status(cudaGetLastError(), "k_dsc_write"); break; }
+        // execution blobs
+        int64_t *len16 = nullptr;
+        if (cudaMalloc(&len16, 2 * (n + 1) * sizeof(int64_t)) != cudaSuccess) { rc = cuda_status(cudaGetLastError(), "cudaMalloc(blob sizes)"); break; }
+        int64_t *start16 = len16 + (n + 1);
+        cudaMemsetAsync(len16 + n, 0, sizeof(int64_t), st);
+        k_blob_len<<<nb, 256, 0, st>>>(M.items, n, M.m, len16);
+        if ((rc = scan([&](void *t, size_t &b) { return cub::DeviceScan::ExclusiveSum(t, b, len16, start16, (int)(n + 1), st); }))) { cudaFree(len16); break; }
+        int64_t total16 = 0;
+        cudaMemcpyAsync(&total16, start16 + n, 8, cudaMemcpyDeviceToHost, st);
+        if (cudaStreamSynchronize(st) != cudaSuccess) { rc = cuda_status(cudaGetLastError(), "blob size"); cudaFree(len16); break; }
+        if (total16 >= (int64_t(1) << 32)) { rc = set_error(TILESPMV_OVERFLOW, "execution blob >= 64 GiB"); cudaFree(len16); break; }
+        M.blob_bytes = total16 * 16;
+        if (cudaMalloc(&M.blob, M.blob_bytes + 256) != cudaSuccess) { rc = cuda_status(cudaGetLastError(), "cudaMalloc(blob)"); cudaFree(len16); break; }
+        M.device_bytes += M.blob_bytes + 256;
+        k_blob_fill<<<(unsigned)((n * 32 + 255) / 256), 256, 0, st>>>(M.items, n, M.m, start16, M.tdesc, M.tileColIdx,
+                                                                     M.payload, M.remRowPtr, M.remCol, M.remVal, M.blob);
+        if (cudaStreamSynchronize(st) != cudaSuccess) rc = cuda_status(cudaGetLastError(), "k_blob_fill");
+        cudaFree(len16);
     } while (0);
     cudaFree(cnt);
     return rc;
@@ -337,6 +404,7 @@ int launch_spmv(const Matrix &M, const double *d_x, double *d_y, cudaStream_t st
     p.m = M.m;
     p.n = M.n;
     p.tdesc = M.tdesc;
+    p.blob = M.blob;
     p.cta_begin = M.cta_begin;
     const KernelChoice kc = choose(M.kernel_version);
     kc.fn<<<M.grid, M.block, M.smem, st>>>(p);

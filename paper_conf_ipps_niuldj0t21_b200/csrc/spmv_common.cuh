@@ -1,5 +1,5 @@
 // spmv_common.cuh -- pieces shared by the SpMV kernels (spmv_v1.cu,
-// spmv_ring.cu) and the schedule builder (schedule.cu).
+// spmv_warp.cu) and the schedule builder (schedule.cu).
 #pragma once
 
 #include "internal.cuh"
@@ -28,7 +28,8 @@ struct Params {
     double *y;
     int64_t m, n;
     const uint2 *tdesc;        // per-item tile-descriptor lists (schedule.cu)
-    const int64_t *cta_begin;  // contiguous item chunk per CTA (ring kernels)
+    const uint8_t *blob;       // per-item execution blobs (schedule.cu)
+    const int64_t *cta_begin;  // unused (reserved)
 };
 
 // ------------------------------------------------------------------ PTX ----
@@ -110,6 +111,68 @@ __host__ __device__ __forceinline__ ItemParts item_parts(const Item &it, int64_t
     return r;
 }
 
+// ---------------------------------------------- one item's execution blob --
+// A create-time copy of everything one work item reads, contiguous and
+// 16-byte aligned part by part, so a single TMA bulk copy stages it:
+//   dsc : the descriptor list (k_dsc_write), ndsc x 8 B
+//   jt  : tile column index J of tiles 0..nt-1, 4 B each
+//   pay : the tiles' canonical payload bytes
+//   rp  : remainder row pointers of the item's rows, rebased to the item's
+//         entry range and clamped to it (rows + 1 ints)
+//   col, val : the item's remainder entries
+struct BlobParts {
+    uint32_t jt, pay, rp, col, val, total;
+};
+
+__host__ __device__ __forceinline__ BlobParts blob_parts(const Item &it, int64_t m) {
+    BlobParts b;
+    const uint32_t nt = (uint32_t)(it.part_nt >> 24);
+    b.jt = up16(8u * (uint32_t)it.ndsc);
+    b.pay = b.jt + up16(4u * nt);
+    b.rp = b.pay + (it.offe - it.offb) * 16u;
+    if (it.ke > it.kb) {
+        const uint32_t rows = (uint32_t)imin64(16, m - 16 * (int64_t)it.I);
+        const uint32_t e = (uint32_t)(it.ke - it.kb);
+        b.col = b.rp + up16(4u * (rows + 1));
+        b.val = b.col + up16(4u * e);
+        b.total = b.val + up16(8u * e);
+    } else {
+        b.col = b.val = b.total = b.rp;
+    }
+    return b;
+}
+
+// L2 cache policies: the streamed blobs are read once (evict first), x is
+// reused by neighbouring tile rows (evict last)
+__device__ __forceinline__ uint64_t policy_evict_first() {
+    uint64_t p;
+    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+__device__ __forceinline__ uint64_t policy_evict_last() {
+    uint64_t p;
+    asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+__device__ __forceinline__ void bulk_g2s_hint(uint32_t dst, const void *src, uint32_t bytes, uint32_t bar,
+                                              uint64_t policy) {
+    asm volatile(
+        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], %4;" ::"r"(dst),
+        "l"(src), "r"(bytes), "r"(bar), "l"(policy)
+        : "memory");
+}
+__device__ __forceinline__ double ldg_hint(const double *p, uint64_t policy) {
+    double v;
+    asm volatile("ld.global.nc.L2::cache_hint.f64 %0, [%1], %2;" : "=d"(v) : "l"(p), "l"(policy));
+    return v;
+}
+// acc += a * b only where pred holds (one predicated DFMA, no select)
+__device__ __forceinline__ void fma_if(bool pred, double a, double b, double &acc) {
+    asm("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %3, 0;\n\t@q fma.rn.f64 %0, %1, %2, %0;\n\t}"
+        : "+d"(acc)
+        : "d"(a), "d"(b), "r"((unsigned)pred));
+}
+
 // ----------------------------------------------------------- y output ------
 // Lanes 0..15 hold the 16 row sums of the item.  A whole tile row writes y
 // directly (one 128-byte store); a split tile row writes its partial and the
@@ -139,16 +202,15 @@ __device__ __forceinline__ void write_rows(const Params &p, const Item &item, in
     }
 }
 
-// kernels (spmv_v1.cu, spmv_ring.cu)
+// kernels (spmv_v1.cu, spmv_warp.cu)
 struct KernelChoice {
     const char *name;
     void (*fn)(Params);
     int threads, smem, ctas_per_sm;
-    bool ring;
+    bool ring;       // one CTA per SM with cta_begin chunks (no current kernel)
     int slot_bytes;  // item budget the schedule must respect
 };
 KernelChoice kernel_v1();
-KernelChoice kernel_ring(int variant);
 KernelChoice kernel_warp(int variant);
 
 }  // namespace tsp

@@ -1,8 +1,7 @@
 // spmv_tiles.cuh -- the per-format tile routines of the tiled SpMV
 // (§III.C) in their B200 form: one tile per half-warp,
 // one lane per tile row, shared-memory operands addressed with 32-bit shared
-// addresses.  Used by the ring kernel (spmv_ring.cu) and the warp kernel
-// (spmv_warp.cu).
+// addresses.  Used by the warp kernel (spmv_warp.cu).
 #pragma once
 
 #include "spmv_common.cuh"
@@ -69,10 +68,10 @@ __device__ __forceinline__ void half_csr(uint32_t P, int nz, uint32_t X, int r, 
         const double v2 = lds_f64(V + 8 * i + 16), v3 = lds_f64(V + 8 * i + 24);
         const double x0 = lds_f64(X + 8 * c0), x1 = lds_f64(X + 8 * c1);
         const double x2 = lds_f64(X + 8 * c2), x3 = lds_f64(X + 8 * c3);
-        if (i < len) acc = fma(v0, x0, acc);
-        if (i + 1 < len) a1 = fma(v1, x1, a1);
-        if (i + 2 < len) acc = fma(v2, x2, acc);
-        if (i + 3 < len) a1 = fma(v3, x3, a1);
+        fma_if(i < len, v0, x0, acc);
+        fma_if(i + 1 < len, v1, x1, a1);
+        fma_if(i + 2 < len, v2, x2, acc);
+        fma_if(i + 3 < len, v3, x3, a1);
     }
     acc += a1;
 }
@@ -90,7 +89,7 @@ __device__ __forceinline__ void half_ell(uint32_t P, int w, uint32_t X, int r, b
         const uint32_t c = (lds_u8(ci + 8 * k) >> sh) & 15u;
         const double v = lds_f64(V + 128 * k);
         const double xv = lds_f64(X + 8 * c);
-        if (k < wq && (k == 0 || c != 0)) acc = fma(v, xv, acc);
+        fma_if(k < wq && (k == 0 || c != 0), v, xv, acc);
     }
 }
 
@@ -114,7 +113,7 @@ __device__ __forceinline__ void half_dnscol(uint32_t P, int nc, uint32_t X, int 
     for (int q = 0; q < trips; ++q) {
         const double v = lds_f64(P + 8 * (16 * q + r));
         const double xv = lds_f64(X + 8 * (lds_u8(cid + q) & 15u));
-        if (q < nq) acc = fma(v, xv, acc);
+        fma_if(q < nq, v, xv, acc);
     }
 }
 
@@ -149,7 +148,7 @@ __device__ __forceinline__ void half_coo(uint32_t V, uint32_t rc, int n, uint32_
         const uint32_t b = lds_u8(rc + j);
         const double v = lds_f64(V + 8 * j);
         const double xv = lds_f64(X + 8 * (b & 15u));
-        if (j < nq && (int)(b >> 4) == r) acc = fma(v, xv, acc);
+        fma_if(j < nq && (int)(b >> 4) == r, v, xv, acc);
     }
 }
 
@@ -163,7 +162,7 @@ __device__ __forceinline__ void half_hyb(uint32_t P, int w, int nz, uint32_t X, 
     for (int k = 0; k < trips; ++k) {
         const double v = lds_f64(P + 8 * (16 * k + r));
         const double xv = lds_f64(X + 8 * ((lds_u8(ei + 8 * k + (r >> 1)) >> sh) & 15u));
-        if (k < wq) acc = fma(v, xv, acc);
+        fma_if(k < wq, v, xv, acc);
     }
     half_coo(P + 128 * w, ei + 8 * w, kc, X, r, ok, acc);
 }

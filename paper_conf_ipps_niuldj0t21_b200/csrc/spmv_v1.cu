@@ -2,8 +2,8 @@
 // non-pipelined.  Each warp stages its item's tile payloads with one
 // cp.async.bulk (TMA, 1-D) into its own shared-memory slot, gathers the x
 // segments, processes the CSR remainder from global memory and then runs the
-// full-warp format routines.  Kept for A/B comparison with the ring kernels
-// (spmv_ring.cu); select with TILESPMV_KERNEL=1.
+// full-warp format routines.  Kept for A/B comparison with the default warp
+// kernel (spmv_warp.cu); select with TILESPMV_KERNEL=1.
 #include "spmv_common.cuh"
 
 namespace tsp {

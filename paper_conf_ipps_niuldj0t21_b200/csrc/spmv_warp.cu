@@ -1,11 +1,16 @@
-// spmv_warp.cu -- high-occupancy variant of the tiled SpMV (TILESPMV_KERNEL
-// 20+): every warp is its own producer and consumer.  Per work item, lane 0
-// stages the item (tile payloads, descriptor list, remainder rowptr/col/val)
-// into the warp's shared-memory slot with TMA bulk copies on the warp's
-// mbarrier; the warp then gathers the x segments, runs the half-warp tile
-// routines of spmv_tiles.cuh and writes y.  Latency is hidden by warp count
-// (~32 warps/SM with small slots) instead of by a deep per-CTA ring; the next
-// item's descriptor is prefetched into registers.
+// spmv_warp.cu -- the default SpMV kernel (TILESPMV_KERNEL 20-29): y =
+// A_tiles*x + A_rem*x in fp64 on sm_100a (§III.C P:118-173 warp-level
+// tile SpMV, P:199 load balancing, P:201 DeferredCOO remainder).
+//
+// High occupancy (32 warps/SM): every warp is its own producer and consumer.
+// Per work item, lane 0 stages the item's execution blob (descriptor list,
+// tile columns, tile payloads, remainder rowptr/col/val; blob_parts) into the
+// warp's shared-memory slot with ONE TMA bulk copy (cp.async.bulk, L2
+// evict-first) completing on the warp's mbarrier; the warp then gathers the
+// x segment of every tile (one 128-byte line, L2 evict-last), runs the
+// half-warp tile routines of spmv_tiles.cuh two tiles at a time and writes
+// y once per row.  Latency is hidden by warp count; the next item's
+// descriptor is prefetched into registers.  No floating-point atomics.
 #include "spmv_tiles.cuh"
 
 namespace tsp {
@@ -15,7 +20,7 @@ template <int WARPS, int SLOT>
 struct WarpCfg {
     static_assert(SLOT % 16 == 0 && SLOT <= kItemBytesMax, "slot size");
     static constexpr uint32_t kX = kItemTiles * 16 * 8;
-    static constexpr uint32_t kPer = SLOT + kX + 64 + 16;  // slot | x | J scratch | mbarrier
+    static constexpr uint32_t kPer = SLOT + kX + 64 + 16;  // slot | x | (spare) | mbarrier
     static constexpr uint32_t kSmem = WARPS * kPer + 256;   // +256: loads may overrun a slot
     static constexpr int kThreads = 32 * WARPS;
 };
@@ -26,7 +31,7 @@ __device__ __forceinline__ Item load_item(const Item *items, int k) {
     Item it;
     it.I = a.x; it.tb = a.y; it.kb = a.z; it.ke = a.w;
     it.offb = (uint32_t)b.x; it.offe = (uint32_t)b.y; it.split = b.z; it.part_nt = b.w;
-    it.dbeg = e.x; it.ndsc = e.y; it.pad0 = e.z; it.pad1 = e.w;
+    it.dbeg = e.x; it.ndsc = e.y; it.blob16 = (uint32_t)e.z; it.blob_len = (uint32_t)e.w;
     return it;
 }
 
@@ -37,7 +42,7 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, MINB) tilespmv
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int h = lane >> 4, r = lane & 15;
     const uint32_t base = smem_u32(smem) + (uint32_t)warp * Cfg::kPer;
-    const uint32_t slot = base, xs = base + SLOT, jt = xs + Cfg::kX, bar = jt + 64;
+    const uint32_t slot = base, xs = base + SLOT, bar = xs + Cfg::kX + 64;
     if (lane == 0) {
         mbar_init(bar, 1);
         fence_mbar_init();
@@ -48,40 +53,26 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, MINB) tilespmv
     const int64_t gw = (int64_t)blockIdx.x * WARPS + warp, nw = (int64_t)gridDim.x * WARPS;
     const int kbeg = (int)(p.num_items * gw / nw), kend = (int)(p.num_items * (gw + 1) / nw);
     uint32_t phase = 0;
+    const uint64_t stream_policy = policy_evict_first(), x_policy = policy_evict_last();
     Item nxt;
     if (kbeg < kend) nxt = load_item(p.items, kbeg);
     for (int k = kbeg; k < kend; ++k) {
         const Item it = nxt;
         if (k + 1 < kend) nxt = load_item(p.items, k + 1);  // in flight during this item
-        const ItemParts pt = item_parts(it, p.m);
-        if (lane == 0 && pt.total) {
+        const BlobParts bp = blob_parts(it, p.m);
+        // the whole item (descriptors, J, payload, remainder) in ONE TMA bulk copy
+        if (lane == 0 && bp.total) {
             fence_proxy_async();
-            mbar_expect_tx(bar, pt.total);
-            uint32_t d = slot;
-            if (pt.pay) bulk_g2s(d, p.payload + (size_t)it.offb * 16, pt.pay, bar);
-            d += pt.pay;
-            if (pt.dsc) bulk_g2s(d, reinterpret_cast<const uint8_t *>(p.tdesc + it.dbeg) - pt.dsc_skew, pt.dsc, bar);
-            d += pt.dsc;
-            if (pt.rp) {
-                bulk_g2s(d, p.remRowPtr + 16 * (int64_t)it.I, pt.rp, bar);
-                d += pt.rp;
-                bulk_g2s(d, reinterpret_cast<const uint8_t *>(p.remCol + it.kb) - pt.col_skew, pt.col, bar);
-                d += pt.col;
-                bulk_g2s(d, reinterpret_cast<const uint8_t *>(p.remVal + it.kb) - pt.val_skew, pt.val, bar);
-            }
+            mbar_expect_tx(bar, bp.total);
+            bulk_g2s_hint(slot, p.blob + (size_t)it.blob16 * 16, bp.total, bar, stream_policy);
         }
-        if (pt.total) {
+        if (bp.total) {
             mbar_wait(bar, phase);
             phase ^= 1u;
         }
         const int nt = it.part_nt >> 24;
-        const uint32_t dsc = slot + pt.pay + pt.dsc_skew;
-        // J of every tile by tile index, then the x segments (lane: tile 2k+h, element r)
-        if (lane < it.ndsc) {
-            const uint2 d = lds_v2u32(dsc + 8 * lane);
-            if (!((d.y >> 27) & 1u)) sts_u32(jt + 4 * ((d.y >> 23) & 15u), d.x & 0x7FFFFFFu);
-        }
-        __syncwarp();
+        const uint32_t dsc = slot, pay = slot + bp.pay;
+        // x segments (lane: tile 2k+h, element r), J from the blob
         {
             double xv[kItemTiles / 2];
 #pragma unroll
@@ -89,21 +80,18 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, MINB) tilespmv
                 const int t = 2 * kk + h;
                 xv[kk] = 0.0;
                 if (t < nt) {
-                    const uint32_t col = 16u * (uint32_t)lds_s32(jt + 4 * t) + (uint32_t)r;
-                    if (col < n32) xv[kk] = __ldg(p.x + col);
+                    const uint32_t col = 16u * (uint32_t)lds_s32(slot + bp.jt + 4 * t) + (uint32_t)r;
+                    if (col < n32) xv[kk] = ldg_hint(p.x + col, x_policy);
                 }
             }
 #pragma unroll
             for (int kk = 0; kk < kItemTiles / 2; ++kk) sts_f64(xs + 8 * ((2 * kk + h) * 16 + r), xv[kk]);
         }
         double acc = 0.0;
-        if (pt.rp) {  // fused CSR remainder: two lanes per short row, warp per long row
-            const uint32_t rb = slot + pt.pay + pt.dsc;
+        if (bp.total > bp.rp) {  // fused CSR remainder: two lanes per short row, warp per long row
             const int rows = (int)imin64(16, p.m - 16 * (int64_t)it.I);
-            int b = lds_s32(rb + 4 * min(r, rows)), e = lds_s32(rb + 4 * min(r + 1, rows));
-            b = max(b, it.kb) - it.kb;
-            e = min(e, it.ke) - it.kb;
-            const uint32_t colS = rb + pt.rp + pt.col_skew, valS = rb + pt.rp + pt.col + pt.val_skew;
+            const int b = lds_s32(slot + bp.rp + 4 * min(r, rows)), e = lds_s32(slot + bp.rp + 4 * min(r + 1, rows));
+            const uint32_t colS = slot + bp.col, valS = slot + bp.val;
             const bool is_short = e - b <= kShortRow;
             if (is_short) {
                 int cs[kShortRow / 2];
@@ -115,10 +103,10 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, MINB) tilespmv
                     vs[i] = kq < e ? lds_f64(valS + 8 * kq) : 0.0;
                 }
 #pragma unroll
-                for (int i = 0; i < kShortRow / 2; ++i) xr[i] = (b + h + 2 * i < e) ? __ldg(p.x + (uint32_t)cs[i]) : 0.0;
-#pragma unroll
                 for (int i = 0; i < kShortRow / 2; ++i)
-                    if (b + h + 2 * i < e) acc = fma(vs[i], xr[i], acc);
+                    xr[i] = (b + h + 2 * i < e) ? ldg_hint(p.x + (uint32_t)cs[i], x_policy) : 0.0;
+#pragma unroll
+                for (int i = 0; i < kShortRow / 2; ++i) fma_if(b + h + 2 * i < e, vs[i], xr[i], acc);
             }
             unsigned longs = __ballot_sync(FULL, lane < 16 && !is_short);
             while (longs) {
@@ -136,10 +124,10 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, MINB) tilespmv
                         vs[i] = kq < ee ? lds_f64(valS + 8 * kq) : 0.0;
                     }
 #pragma unroll
-                    for (int i = 0; i < 4; ++i) xv[i] = (k0 + lane + 32 * i < ee) ? __ldg(p.x + (uint32_t)cs[i]) : 0.0;
-#pragma unroll
                     for (int i = 0; i < 4; ++i)
-                        if (k0 + lane + 32 * i < ee) s = fma(vs[i], xv[i], s);
+                        xv[i] = (k0 + lane + 32 * i < ee) ? ldg_hint(p.x + (uint32_t)cs[i], x_policy) : 0.0;
+#pragma unroll
+                    for (int i = 0; i < 4; ++i) fma_if(k0 + lane + 32 * i < ee, vs[i], xv[i], s);
                 }
 #pragma unroll
                 for (int o = 16; o >= 1; o >>= 1) s += __shfl_xor_sync(FULL, s, o);
@@ -149,7 +137,7 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, MINB) tilespmv
         __syncwarp();
         const int npairs = it.ndsc >> 1;
 #pragma unroll 1
-        for (int q = 0; q < npairs; ++q) run_pair(lds_v2u32(dsc + 16 * q + 8 * h), slot, xs, r, acc);
+        for (int q = 0; q < npairs; ++q) run_pair(lds_v2u32(dsc + 16 * q + 8 * h), pay, xs, r, acc);
         acc += __shfl_xor_sync(FULL, acc, 16);
         write_rows(p, it, lane, acc);
         __syncwarp();  // slot, x and J scratch free for the next item
