@@ -105,8 +105,9 @@ __global__ void k_items_write(const int32_t *tilePtr, const uint32_t *tileOff, c
 // Per-item tile-descriptor list: the item's tiles grouped by format (format
 // order, tile order inside a group), every odd group padded with a copy of
 // its last entry marked invalid, so a half-warp pair never mixes formats.
-// Entry: x = J | fmt << 27 ; y = aux | nnz << 5 | off16 << 14 | t << 23 | invalid << 27
-// (off16: payload offset inside the item in 16-byte units, t: tile index in the item).
+// Entry: x = payload byte offset inside the item | (t * 128) << 14 | fmt << 29
+//        y = aux | nnz << 8 | invalid << 31          (t: tile index in the item;
+// t * 128 is the byte offset of the tile's x segment in the warp's x scratch)
 __global__ void k_dsc_count(Item *items, int64_t n, const uint8_t *tileFmt, int32_t *ndsc) {
     int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     if (k >= n) return;
@@ -137,14 +138,13 @@ __global__ void k_dsc_write(Item *items, int64_t n, const int32_t *dbeg, const i
             const int g = it.tb + t;
             if (tileFmt[g] != f) continue;
             uint2 d;
-            d.x = (uint32_t)tileColIdx[g] | ((uint32_t)f << 27);
-            d.y = (uint32_t)tileAux[g] | ((uint32_t)(tileNnz[g + 1] - tileNnz[g]) << 5) |
-                  ((tileOff[g] - it.offb) << 14) | ((uint32_t)t << 23);
+            d.x = ((tileOff[g] - it.offb) * 16u) | ((uint32_t)t << 21) | ((uint32_t)f << 29);
+            d.y = (uint32_t)tileAux[g] | ((uint32_t)(tileNnz[g + 1] - tileNnz[g]) << 8);
             dlist[pos++] = d;
             last = d;
             c++;
         }
-        if (c & 1) dlist[pos++] = make_uint2(last.x, last.y | (1u << 27));
+        if (c & 1) dlist[pos++] = make_uint2(last.x, last.y | (1u << 31));
     }
 }
 
@@ -406,6 +406,7 @@ int launch_spmv(const Matrix &M, const double *d_x, double *d_y, cudaStream_t st
     p.tdesc = M.tdesc;
     p.blob = M.blob;
     p.cta_begin = M.cta_begin;
+    p.x_vec = (reinterpret_cast<uintptr_t>(d_x) & 15u) == 0;
     const KernelChoice kc = choose(M.kernel_version);
     kc.fn<<<M.grid, M.block, M.smem, st>>>(p);
     TSP_CK(cudaGetLastError());

@@ -30,6 +30,7 @@ struct Params {
     const uint2 *tdesc;        // per-item tile-descriptor lists (schedule.cu)
     const uint8_t *blob;       // per-item execution blobs (schedule.cu)
     const int64_t *cta_begin;  // unused (reserved)
+    int x_vec;                 // x is 16-byte aligned: x segments load as double2
 };
 
 // ------------------------------------------------------------------ PTX ----
@@ -165,6 +166,14 @@ __device__ __forceinline__ double ldg_hint(const double *p, uint64_t policy) {
     double v;
     asm volatile("ld.global.nc.L2::cache_hint.f64 %0, [%1], %2;" : "=d"(v) : "l"(p), "l"(policy));
     return v;
+}
+__device__ __forceinline__ double2 ldg2_hint(const double *p, uint64_t policy) {
+    double2 v;
+    asm volatile("ld.global.nc.L2::cache_hint.v2.f64 {%0, %1}, [%2], %3;" : "=d"(v.x), "=d"(v.y) : "l"(p), "l"(policy));
+    return v;
+}
+__device__ __forceinline__ void sts_v2f64(uint32_t a, double2 v) {
+    asm volatile("st.shared.v2.f64 [%0], {%1, %2};" ::"r"(a), "d"(v.x), "d"(v.y) : "memory");
 }
 // acc += a * b only where pred holds (one predicated DFMA, no select)
 __device__ __forceinline__ void fma_if(bool pred, double a, double b, double &acc) {

@@ -56,10 +56,24 @@ __device__ __forceinline__ void half_csr(uint32_t P, int nz, uint32_t X, int r, 
     const uint32_t b_odd = cb + odd;
     const uint32_t s_even = 4 * odd, s_odd = 4 - 4 * odd;
     const uint32_t V = P + 8 * beg;
-    // four entries per iteration: independent load chains, two FMA chains
+    // four entries per step (independent load chains, two FMA chains); the
+    // first step is straight-line, longer rows (trips > 4) loop
     double a1 = 0.0;
+    {
+        const uint32_t c0 = (lds_u8(cb) >> s_even) & 15u;
+        const uint32_t c1 = (lds_u8(b_odd) >> s_odd) & 15u;
+        const uint32_t c2 = (lds_u8(cb + 1) >> s_even) & 15u;
+        const uint32_t c3 = (lds_u8(b_odd + 1) >> s_odd) & 15u;
+        const double v0 = lds_f64(V), v1 = lds_f64(V + 8), v2 = lds_f64(V + 16), v3 = lds_f64(V + 24);
+        const double x0 = lds_f64(X + 8 * c0), x1 = lds_f64(X + 8 * c1);
+        const double x2 = lds_f64(X + 8 * c2), x3 = lds_f64(X + 8 * c3);
+        fma_if(0 < len, v0, x0, acc);
+        fma_if(1 < len, v1, x1, a1);
+        fma_if(2 < len, v2, x2, acc);
+        fma_if(3 < len, v3, x3, a1);
+    }
 #pragma unroll 1
-    for (int i = 0; i < trips; i += 4) {
+    for (int i = 4; i < trips; i += 4) {
         const uint32_t c0 = (lds_u8(cb + (i >> 1)) >> s_even) & 15u;
         const uint32_t c1 = (lds_u8(b_odd + (i >> 1)) >> s_odd) & 15u;
         const uint32_t c2 = (lds_u8(cb + (i >> 1) + 1) >> s_even) & 15u;
@@ -169,20 +183,22 @@ __device__ __forceinline__ void half_hyb(uint32_t P, int w, int nz, uint32_t X, 
 
 // dispatch one descriptor-list entry pair (see k_dsc_write): half h runs entry 2q + h
 __device__ __forceinline__ void run_pair(uint2 e, uint32_t pay, uint32_t xs, int r, double &acc) {
-    const int f = (int)(e.x >> 27);  // same for both halves by construction
-    const bool ok = !((e.y >> 27) & 1u);
-    const int a = (int)(e.y & 31u);
-    const int nz = (int)((e.y >> 5) & 511u);
-    const uint32_t P = pay + 16 * ((e.y >> 14) & 511u);
-    const uint32_t X = xs + 128 * ((e.y >> 23) & 15u);
+    const int f = (int)(e.x >> 29);  // same for both halves by construction
+    const bool ok = (int)e.y >= 0;
+    const uint32_t P = pay + (e.x & 0x3FFFu);
+    const uint32_t X = xs + ((e.x >> 14) & 0x7FFu);
     switch (f) {
-    case F_CSR: half_csr(P, nz, X, r, ok, acc); break;
-    case F_ELL: half_ell(P, a, X, r, ok, acc); break;
+    case F_CSR: half_csr(P, (int)(e.y >> 8) & 511, X, r, ok, acc); break;
+    case F_ELL: half_ell(P, (int)(e.y & 31u), X, r, ok, acc); break;
     case F_DNS: half_dns(P, X, r, ok, acc); break;
-    case F_DNSCOL: half_dnscol(P, a, X, r, ok, acc); break;
-    case F_DNSROW: half_dnsrow(P, a, X, r, ok, acc); break;
-    case F_COO: half_coo(P, P + 8 * nz, nz, X, r, ok, acc); break;
-    case F_HYB: half_hyb(P, a, nz, X, r, ok, acc); break;
+    case F_DNSCOL: half_dnscol(P, (int)(e.y & 31u), X, r, ok, acc); break;
+    case F_DNSROW: half_dnsrow(P, (int)(e.y & 31u), X, r, ok, acc); break;
+    case F_COO: {
+        const int nz = (int)(e.y >> 8) & 511;
+        half_coo(P, P + 8 * nz, nz, X, r, ok, acc);
+        break;
+    }
+    case F_HYB: half_hyb(P, (int)(e.y & 31u), (int)(e.y >> 8) & 511, X, r, ok, acc); break;
     default: break;
     }
 }

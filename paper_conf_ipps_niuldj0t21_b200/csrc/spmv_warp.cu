@@ -72,20 +72,33 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, MINB) tilespmv
         }
         const int nt = it.part_nt >> 24;
         const uint32_t dsc = slot, pay = slot + bp.pay;
-        // x segments (lane: tile 2k+h, element r), J from the blob
-        {
-            double xv[kItemTiles / 2];
+        // x segments, J from the blob
+        if (p.x_vec) {  // lane l: tile 4k + (l >> 3), elements 2(l & 7) .. +1, one 16-byte load
+            const int q = lane & 7;
+#pragma unroll
+            for (int kk = 0; kk < kItemTiles / 4; ++kk) {
+                const int t = 4 * kk + (lane >> 3);
+                if (t < nt) {
+                    const uint32_t c0 = 16u * (uint32_t)lds_s32(slot + bp.jt + 4 * t) + 2u * q;
+                    double2 v;
+                    if (c0 + 2 <= n32) {
+                        v = ldg2_hint(p.x + c0, x_policy);
+                    } else {
+                        v.x = c0 < n32 ? ldg_hint(p.x + c0, x_policy) : 0.0;
+                        v.y = 0.0;
+                    }
+                    sts_v2f64(xs + 128 * t + 16 * q, v);
+                }
+            }
+        } else {  // lane l: tile 2k + h, element r
 #pragma unroll
             for (int kk = 0; kk < kItemTiles / 2; ++kk) {
                 const int t = 2 * kk + h;
-                xv[kk] = 0.0;
                 if (t < nt) {
                     const uint32_t col = 16u * (uint32_t)lds_s32(slot + bp.jt + 4 * t) + (uint32_t)r;
-                    if (col < n32) xv[kk] = ldg_hint(p.x + col, x_policy);
+                    sts_f64(xs + 8 * (16 * t + r), col < n32 ? ldg_hint(p.x + col, x_policy) : 0.0);
                 }
             }
-#pragma unroll
-            for (int kk = 0; kk < kItemTiles / 2; ++kk) sts_f64(xs + 8 * ((2 * kk + h) * 16 + r), xv[kk]);
         }
         double acc = 0.0;
         if (bp.total > bp.rp) {  // fused CSR remainder: two lanes per short row, warp per long row
@@ -93,21 +106,23 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, MINB) tilespmv
             const int b = lds_s32(slot + bp.rp + 4 * min(r, rows)), e = lds_s32(slot + bp.rp + 4 * min(r + 1, rows));
             const uint32_t colS = slot + bp.col, valS = slot + bp.val;
             const bool is_short = e - b <= kShortRow;
-            if (is_short) {
-                int cs[kShortRow / 2];
-                double vs[kShortRow / 2], xr[kShortRow / 2];
+            // two lanes per short row; warp-uniform trip count, loads first
+            const int trips = (int)__reduce_max_sync(FULL, is_short ? (unsigned)((e - b + 1 - h) >> 1) : 0u);
+            double vs[kShortRow / 2], xr[kShortRow / 2];
+            bool oks[kShortRow / 2];
 #pragma unroll
-                for (int i = 0; i < kShortRow / 2; ++i) {
-                    const int kq = b + h + 2 * i;
-                    cs[i] = kq < e ? lds_s32(colS + 4 * kq) : 0;
-                    vs[i] = kq < e ? lds_f64(valS + 8 * kq) : 0.0;
+            for (int i = 0; i < kShortRow / 2; ++i) {
+                const int kq = b + h + 2 * i;
+                oks[i] = is_short && kq < e;
+                vs[i] = xr[i] = 0.0;
+                if (i < trips) {
+                    const int c = oks[i] ? lds_s32(colS + 4 * kq) : 0;
+                    vs[i] = lds_f64(valS + 8 * (oks[i] ? kq : 0));
+                    if (oks[i]) xr[i] = ldg_hint(p.x + (uint32_t)c, x_policy);
                 }
-#pragma unroll
-                for (int i = 0; i < kShortRow / 2; ++i)
-                    xr[i] = (b + h + 2 * i < e) ? ldg_hint(p.x + (uint32_t)cs[i], x_policy) : 0.0;
-#pragma unroll
-                for (int i = 0; i < kShortRow / 2; ++i) fma_if(b + h + 2 * i < e, vs[i], xr[i], acc);
             }
+#pragma unroll
+            for (int i = 0; i < kShortRow / 2; ++i) fma_if(oks[i], vs[i], xr[i], acc);
             unsigned longs = __ballot_sync(FULL, lane < 16 && !is_short);
             while (longs) {
                 const int rr = __ffs(longs) - 1;
