@@ -38,12 +38,22 @@ struct __align__(16) Item {
     uint32_t offb;    // payload offset of tile tb (16-byte units)
     uint32_t offe;    // payload offset one past the last tile
     int32_t split;    // split-row index, or -1 if the item covers its whole tile row
-    int32_t part_nt;  // (part index within the split row) | (number of tiles << 24)
+    int32_t part_nt;  // part index (bits 0-23) | tiles << 24 (5 bits) | local << 29 | last << 30
     int32_t dbeg;      // first entry of the item's tile-descriptor list (dlist)
     int32_t ndsc;      // entries: the item's tiles grouped by format, groups padded to even length
     uint32_t blob16;   // start of the item's execution blob (16-byte units)
     uint32_t blob_len; // bytes of the blob (blob_parts)
 };
+
+// A split tile row with at most kLocalParts items is "local": one warp runs
+// all of its parts in order, carrying the partial row sums in registers, and
+// writes y once.  Larger (hub) rows combine per-part partials in global
+// memory.  The choice depends only on the row's own content.
+constexpr int kLocalParts = 64;
+__host__ __device__ __forceinline__ int item_nt(const Item &it) { return (it.part_nt >> 24) & 31; }
+__host__ __device__ __forceinline__ int item_part(const Item &it) { return it.part_nt & 0xFFFFFF; }
+__host__ __device__ __forceinline__ bool item_local(const Item &it) { return (it.part_nt >> 29) & 1; }
+__host__ __device__ __forceinline__ bool item_last(const Item &it) { return (it.part_nt >> 30) & 1; }
 
 struct Matrix {
     int device = 0;
@@ -78,7 +88,7 @@ struct Matrix {
     int64_t num_dsc = 0;
     uint8_t *blob = nullptr;       // per-item execution blobs (blob_parts), read by the kernels
     int64_t blob_bytes = 0;
-    int64_t *cta_begin = nullptr;  // contiguous item chunk per CTA
+    int64_t *cta_begin = nullptr;  // contiguous item chunk per warp (row-aligned, cost-balanced)
     // launch shape
     int kernel_version = 2;
     int item_bytes = kItemBytesMax;  // slot size the schedule was built for

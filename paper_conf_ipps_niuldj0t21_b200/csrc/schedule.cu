@@ -26,7 +26,7 @@ namespace {
 // row's remainder entries.  Depends only on the tile row's own content.
 template <bool WRITE>
 __device__ int items_for_row(int64_t I, const int32_t *tilePtr, const uint32_t *tileOff, const int32_t *remRowPtr,
-                             int64_t m, int budget, Item *out, int split) {
+                             int64_t m, int budget, Item *out, int split, int nparts = 0) {
     const int tp0 = tilePtr[I], tp1 = tilePtr[I + 1];
     int k0 = 0, k1 = 0;
     if (remRowPtr) {
@@ -69,7 +69,9 @@ __device__ int items_for_row(int64_t I, const int32_t *tilePtr, const uint32_t *
             it.offb = tileOff[tb];
             it.offe = tileOff[t];
             it.split = split;
-            it.part_nt = (split >= 0 ? cnt : 0) | ((t - tb) << 24);
+            const bool local = split >= 0 && nparts <= kLocalParts;
+            const bool last = split >= 0 && cnt == nparts - 1;
+            it.part_nt = (split >= 0 ? cnt : 0) | ((t - tb) << 24) | ((int)local << 29) | ((int)last << 30);
             it.dbeg = 0;
             it.ndsc = 0;
             it.blob16 = 0;
@@ -98,7 +100,7 @@ __global__ void k_items_write(const int32_t *tilePtr, const uint32_t *tileOff, c
     if (I >= tilem) return;
     const bool split = nitems[I] > 1;
     const int sid = split ? splitId[I] : -1;
-    items_for_row<true>(I, tilePtr, tileOff, remRowPtr, m, budget, items + itemBase[I], sid);
+    items_for_row<true>(I, tilePtr, tileOff, remRowPtr, m, budget, items + itemBase[I], sid, nitems[I]);
     if (split) split_info[sid] = make_int2(partBase[I], nitems[I]);
 }
 
@@ -112,7 +114,7 @@ __global__ void k_dsc_count(Item *items, int64_t n, const uint8_t *tileFmt, int3
     int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     if (k >= n) return;
     const Item it = items[k];
-    const int nt = it.part_nt >> 24;
+    const int nt = item_nt(it);
     int cnt[8] = {0, 0, 0, 0, 0, 0, 0, 0};
     for (int t = 0; t < nt; ++t) cnt[tileFmt[it.tb + t] & 7]++;
     int total = 0;
@@ -126,7 +128,7 @@ __global__ void k_dsc_write(Item *items, int64_t n, const int32_t *dbeg, const i
     int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     if (k >= n) return;
     Item it = items[k];
-    const int nt = it.part_nt >> 24;
+    const int nt = item_nt(it);
     int pos = dbeg[k];
     it.dbeg = pos;
     it.ndsc = ndsc[k];
@@ -173,7 +175,7 @@ __global__ void k_blob_fill(Item *items, int64_t n, int64_t m, const int64_t *st
     __syncwarp();
     uint2 *dd = reinterpret_cast<uint2 *>(dst);
     for (int i = lane; i < it.ndsc; i += 32) dd[i] = dlist[it.dbeg + i];
-    const int nt = it.part_nt >> 24;
+    const int nt = item_nt(it);
     int32_t *jt = reinterpret_cast<int32_t *>(dst + b.jt);
     for (int t = lane; t < nt; t += 32) jt[t] = tileColIdx[it.tb + t];
     const uint4 *ps = reinterpret_cast<const uint4 *>(payload + (size_t)it.offb * 16);
@@ -202,10 +204,10 @@ __global__ void k_item_cost(const Item *items, int64_t n, int64_t m, int64_t *co
     int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     if (k >= n) return;
     const Item it = items[k];
-    cost[k] = (int64_t)item_parts(it, m).total + 40 * (it.part_nt >> 24) + 512;
+    cost[k] = (int64_t)item_parts(it, m).total + 40 * (item_nt(it)) + 512;
 }
 
-__global__ void k_cta_begin(const int64_t *incl, int64_t n, int G, int64_t *cta_begin) {
+__global__ void k_cta_begin(const int64_t *incl, const Item *items, int64_t n, int G, int64_t *cta_begin) {
     const int b = blockIdx.x * blockDim.x + threadIdx.x;
     if (b > G) return;
     if (b == G) {
@@ -221,6 +223,8 @@ __global__ void k_cta_begin(const int64_t *incl, int64_t n, int G, int64_t *cta_
         if (before < target) lo = mid + 1;
         else hi = mid;
     }
+    // never start inside a local split row (its parts run in one warp)
+    while (lo < n && item_local(items[lo]) && item_part(items[lo]) > 0) lo++;
     cta_begin[b] = lo;
 }
 
@@ -350,19 +354,22 @@ int configure_launch(Matrix &M) {
     if (per_sm < 1) return set_error(TILESPMV_CUDA, "SpMV kernel does not fit on an SM");
     M.block = kc.threads;
     M.smem = kc.smem;
-    if (!kc.ring) {
-        const int64_t warps = kc.threads / 32;
+    if (kc.ring) return set_error(TILESPMV_CUDA, "no ring kernel in this build");
+    const int64_t warps = kc.threads / 32;
+    if (version == 1) {  // v1: grid-stride over items
         const int64_t need = (M.num_items + warps - 1) / warps;
         M.grid = (int)std::max<int64_t>(1, std::min<int64_t>(need, (int64_t)sms * per_sm));
         return 0;
     }
-    // ring kernels: one CTA per SM, each owning a contiguous cost-balanced chunk
-    const int G = (int)std::max<int64_t>(1, std::min<int64_t>((int64_t)sms * kc.ctas_per_sm, M.num_items));
-    M.grid = G;
+    // warp kernel: persistent grid, one contiguous, cost-balanced, row-aligned
+    // item chunk per warp
+    const int64_t need = (M.num_items + warps - 1) / warps;
+    M.grid = (int)std::max<int64_t>(1, std::min<int64_t>(need, (int64_t)sms * per_sm));
+    const int W = (int)(M.grid * warps);
     if (M.cta_begin) cudaFree(M.cta_begin);
     M.cta_begin = nullptr;
-    TSP_CK(cudaMalloc(&M.cta_begin, (G + 1) * sizeof(int64_t)));
-    M.device_bytes += (G + 1) * 8;
+    TSP_CK(cudaMalloc(&M.cta_begin, (W + 1) * sizeof(int64_t)));
+    M.device_bytes += (W + 1) * 8;
     if (M.num_items > 0) {
         int64_t *cost = nullptr;
         TSP_CK(cudaMalloc(&cost, 2 * M.num_items * sizeof(int64_t)));
@@ -370,14 +377,14 @@ int configure_launch(Matrix &M) {
         k_item_cost<<<(unsigned)((M.num_items + 255) / 256), 256>>>(M.items, M.num_items, M.m, cost);
         int rc = scan([&](void *t, size_t &b) { return cub::DeviceScan::InclusiveSum(t, b, cost, incl, (int)M.num_items); });
         if (!rc) {
-            k_cta_begin<<<(G + 1 + 255) / 256, 256>>>(incl, M.num_items, G, M.cta_begin);
+            k_cta_begin<<<(W + 1 + 255) / 256, 256>>>(incl, M.items, M.num_items, W, M.cta_begin);
             cudaError_t e = cudaDeviceSynchronize();
             if (e != cudaSuccess) rc = cuda_status(e, "k_cta_begin");
         }
         cudaFree(cost);
         if (rc) return rc;
     } else {
-        TSP_CK(cudaMemset(M.cta_begin, 0, (G + 1) * sizeof(int64_t)));
+        TSP_CK(cudaMemset(M.cta_begin, 0, (W + 1) * sizeof(int64_t)));
     }
     return 0;
 }

@@ -29,7 +29,7 @@ struct Params {
     int64_t m, n;
     const uint2 *tdesc;        // per-item tile-descriptor lists (schedule.cu)
     const uint8_t *blob;       // per-item execution blobs (schedule.cu)
-    const int64_t *cta_begin;  // unused (reserved)
+    const int64_t *cta_begin;  // warp kernel: item chunk of each warp
     int x_vec;                 // x is 16-byte aligned: x segments load as double2
 };
 
@@ -127,7 +127,7 @@ struct BlobParts {
 
 __host__ __device__ __forceinline__ BlobParts blob_parts(const Item &it, int64_t m) {
     BlobParts b;
-    const uint32_t nt = (uint32_t)(it.part_nt >> 24);
+    const uint32_t nt = (uint32_t)item_nt(it);
     b.jt = up16(8u * (uint32_t)it.ndsc);
     b.pay = b.jt + up16(4u * nt);
     b.rp = b.pay + (it.offe - it.offb) * 16u;
@@ -193,7 +193,7 @@ __device__ __forceinline__ void write_rows(const Params &p, const Item &item, in
         return;
     }
     const int2 si = p.split_info[item.split];
-    const int part = item.part_nt & 0xFFFFFF;
+    const int part = item_part(item);
     if (lane < 16) __stcg(p.partials + (int64_t)(si.x + part) * 16 + lane, acc);
     __threadfence();
     __syncwarp();

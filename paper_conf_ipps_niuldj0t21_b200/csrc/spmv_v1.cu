@@ -192,7 +192,7 @@ __global__ void __launch_bounds__(kWarps * 32) tilespmv_fp64_kernel(const Params
     const int64_t stride = (int64_t)gridDim.x * kWarps;
     for (int64_t it = (int64_t)blockIdx.x * kWarps + warp; it < p.num_items; it += stride) {
         const Item item = p.items[it];
-        const int nt = item.part_nt >> 24;
+        const int nt = item_nt(item);
         const uint32_t bytes = (item.offe - item.offb) * 16u;
         // 1. one bulk copy of the item's tile payloads into shared memory
         if (lane == 0 && bytes) {
@@ -246,7 +246,7 @@ __global__ void __launch_bounds__(kWarps * 32) tilespmv_fp64_kernel(const Params
             if (lane < 16 && row < p.m) p.y[row] = acc;
         } else {
             const int2 si = p.split_info[item.split];
-            const int part = item.part_nt & 0xFFFFFF;
+            const int part = item_part(item);
             if (lane < 16) __stcg(p.partials + (int64_t)(si.x + part) * 16 + lane, acc);
             __threadfence();
             __syncwarp();

@@ -49,9 +49,11 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, MINB) tilespmv
     }
     __syncwarp();
     const uint32_t n32 = (uint32_t)p.n;
-    // contiguous item chunk per warp (x segments of neighbouring tile rows are shared)
-    const int64_t gw = (int64_t)blockIdx.x * WARPS + warp, nw = (int64_t)gridDim.x * WARPS;
-    const int kbeg = (int)(p.num_items * gw / nw), kend = (int)(p.num_items * (gw + 1) / nw);
+    // contiguous, cost-balanced, row-aligned item chunk per warp (schedule.cu);
+    // neighbouring tile rows share x segments
+    const int64_t gw = (int64_t)blockIdx.x * WARPS + warp;
+    const int kbeg = (int)p.cta_begin[gw], kend = (int)p.cta_begin[gw + 1];
+    double carry = 0.0;  // partial row sums of a local split tile row
     uint32_t phase = 0;
     const uint64_t stream_policy = policy_evict_first(), x_policy = policy_evict_last();
     Item nxt;
@@ -70,7 +72,7 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, MINB) tilespmv
             mbar_wait(bar, phase);
             phase ^= 1u;
         }
-        const int nt = it.part_nt >> 24;
+        const int nt = item_nt(it);
         const uint32_t dsc = slot, pay = slot + bp.pay;
         // x segments, J from the blob
         if (p.x_vec) {  // lane l: tile 4k + (l >> 3), elements 2(l & 7) .. +1, one 16-byte load
@@ -154,7 +156,17 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, MINB) tilespmv
 #pragma unroll 1
         for (int q = 0; q < npairs; ++q) run_pair(lds_v2u32(dsc + 16 * q + 8 * h), pay, xs, r, acc);
         acc += __shfl_xor_sync(FULL, acc, 16);
-        write_rows(p, it, lane, acc);
+        if (item_local(it)) {  // all parts of this tile row run here, in part order
+            if (!item_last(it)) {
+                carry += acc;
+            } else {
+                const int64_t row = 16 * (int64_t)it.I + lane;
+                if (lane < 16 && row < p.m) p.y[row] = carry + acc;
+                carry = 0.0;
+            }
+        } else {
+            write_rows(p, it, lane, acc);
+        }
         __syncwarp();  // slot, x and J scratch free for the next item
     }
 }
