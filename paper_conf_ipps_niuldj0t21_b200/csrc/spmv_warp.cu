@@ -108,23 +108,27 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, MINB) tilespmv
             const int b = lds_s32(slot + bp.rp + 4 * min(r, rows)), e = lds_s32(slot + bp.rp + 4 * min(r + 1, rows));
             const uint32_t colS = slot + bp.col, valS = slot + bp.val;
             const bool is_short = e - b <= kShortRow;
-            // two lanes per short row; warp-uniform trip count, loads first
+            // two lanes per short row; warp-uniform trip count, batches of four
+            // (loads of a batch first, then its FMAs)
             const int trips = (int)__reduce_max_sync(FULL, is_short ? (unsigned)((e - b + 1 - h) >> 1) : 0u);
-            double vs[kShortRow / 2], xr[kShortRow / 2];
-            bool oks[kShortRow / 2];
+#pragma unroll 1
+            for (int i0 = 0; i0 < trips; i0 += 4) {
+                double vs[4], xr[4];
+                bool oks[4];
 #pragma unroll
-            for (int i = 0; i < kShortRow / 2; ++i) {
-                const int kq = b + h + 2 * i;
-                oks[i] = is_short && kq < e;
-                vs[i] = xr[i] = 0.0;
-                if (i < trips) {
-                    const int c = oks[i] ? lds_s32(colS + 4 * kq) : 0;
-                    vs[i] = lds_f64(valS + 8 * (oks[i] ? kq : 0));
-                    if (oks[i]) xr[i] = ldg_hint(p.x + (uint32_t)c, x_policy);
+                for (int i = 0; i < 4; ++i) {
+                    const int kq = b + h + 2 * (i0 + i);
+                    oks[i] = is_short && kq < e;
+                    vs[i] = xr[i] = 0.0;
+                    if (i0 + i < trips) {
+                        const int c = oks[i] ? lds_s32(colS + 4 * kq) : 0;
+                        vs[i] = lds_f64(valS + 8 * (oks[i] ? kq : 0));
+                        if (oks[i]) xr[i] = ldg_hint(p.x + (uint32_t)c, x_policy);
+                    }
                 }
-            }
 #pragma unroll
-            for (int i = 0; i < kShortRow / 2; ++i) fma_if(oks[i], vs[i], xr[i], acc);
+                for (int i = 0; i < 4; ++i) fma_if(oks[i], vs[i], xr[i], acc);
+            }
             unsigned longs = __ballot_sync(FULL, lane < 16 && !is_short);
             while (longs) {
                 const int rr = __ffs(longs) - 1;
