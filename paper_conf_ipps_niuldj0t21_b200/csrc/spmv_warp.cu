@@ -20,7 +20,7 @@ template <int WARPS, int SLOT>
 struct WarpCfg {
     static_assert(SLOT % 16 == 0 && SLOT <= kItemBytesMax, "slot size");
     static constexpr uint32_t kX = kItemTiles * 16 * 8;
-    static constexpr uint32_t kPer = SLOT + kX + 64 + 16;  // slot | x | (spare) | mbarrier
+    static constexpr uint32_t kPer = SLOT + kX + 128 + 16;  // slot | x | row sums | mbarrier
     static constexpr uint32_t kSmem = WARPS * kPer + 256;   // +256: loads may overrun a slot
     static constexpr int kThreads = 32 * WARPS;
 };
@@ -42,7 +42,7 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, MINB) tilespmv
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int h = lane >> 4, r = lane & 15;
     const uint32_t base = smem_u32(smem) + (uint32_t)warp * Cfg::kPer;
-    const uint32_t slot = base, xs = base + SLOT, bar = xs + Cfg::kX + 64;
+    const uint32_t slot = base, xs = base + SLOT, racc = xs + Cfg::kX, bar = racc + 128;
     if (lane == 0) {
         mbar_init(bar, 1);
         fence_mbar_init();
@@ -103,56 +103,89 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, MINB) tilespmv
             }
         }
         double acc = 0.0;
-        if (bp.total > bp.rp) {  // fused CSR remainder: two lanes per short row, warp per long row
+        if (bp.total > bp.rp) {  // fused CSR remainder: two lanes per short row, or a flat pass
             const int rows = (int)imin64(16, p.m - 16 * (int64_t)it.I);
             const int b = lds_s32(slot + bp.rp + 4 * min(r, rows)), e = lds_s32(slot + bp.rp + 4 * min(r + 1, rows));
             const uint32_t colS = slot + bp.col, valS = slot + bp.val;
             const bool is_short = e - b <= kShortRow;
-            // two lanes per short row; warp-uniform trip count, batches of four
-            // (loads of a batch first, then its FMAs)
-            const int trips = (int)__reduce_max_sync(FULL, is_short ? (unsigned)((e - b + 1 - h) >> 1) : 0u);
+            if (!__any_sync(FULL, !is_short)) {
+                // two lanes per short row; warp-uniform trip count, batches of four
+                // (loads of a batch first, then its FMAs)
+                const int trips = (int)__reduce_max_sync(FULL, is_short ? (unsigned)((e - b + 1 - h) >> 1) : 0u);
 #pragma unroll 1
-            for (int i0 = 0; i0 < trips; i0 += 4) {
-                double vs[4], xr[4];
-                bool oks[4];
-#pragma unroll
-                for (int i = 0; i < 4; ++i) {
-                    const int kq = b + h + 2 * (i0 + i);
-                    oks[i] = is_short && kq < e;
-                    vs[i] = xr[i] = 0.0;
-                    if (i0 + i < trips) {
-                        const int c = oks[i] ? lds_s32(colS + 4 * kq) : 0;
-                        vs[i] = lds_f64(valS + 8 * (oks[i] ? kq : 0));
-                        if (oks[i]) xr[i] = ldg_hint(p.x + (uint32_t)c, x_policy);
-                    }
-                }
-#pragma unroll
-                for (int i = 0; i < 4; ++i) fma_if(oks[i], vs[i], xr[i], acc);
-            }
-            unsigned longs = __ballot_sync(FULL, lane < 16 && !is_short);
-            while (longs) {
-                const int rr = __ffs(longs) - 1;
-                longs &= longs - 1;
-                const int bb = __shfl_sync(FULL, b, rr), ee = __shfl_sync(FULL, e, rr);
-                double s = 0.0;
-                for (int k0 = bb; k0 < ee; k0 += 128) {
-                    int cs[4];
-                    double vs[4], xv[4];
+                for (int i0 = 0; i0 < trips; i0 += 4) {
+                    double vs[4], xr[4];
+                    bool oks[4];
 #pragma unroll
                     for (int i = 0; i < 4; ++i) {
-                        const int kq = k0 + lane + 32 * i;
-                        cs[i] = kq < ee ? lds_s32(colS + 4 * kq) : 0;
-                        vs[i] = kq < ee ? lds_f64(valS + 8 * kq) : 0.0;
+                        const int kq = b + h + 2 * (i0 + i);
+                        oks[i] = is_short && kq < e;
+                        vs[i] = xr[i] = 0.0;
+                        if (i0 + i < trips) {
+                            const int c = oks[i] ? lds_s32(colS + 4 * kq) : 0;
+                            vs[i] = lds_f64(valS + 8 * (oks[i] ? kq : 0));
+                            if (oks[i]) xr[i] = ldg_hint(p.x + (uint32_t)c, x_policy);
+                        }
                     }
 #pragma unroll
-                    for (int i = 0; i < 4; ++i)
-                        xv[i] = (k0 + lane + 32 * i < ee) ? ldg_hint(p.x + (uint32_t)cs[i], x_policy) : 0.0;
-#pragma unroll
-                    for (int i = 0; i < 4; ++i) fma_if(k0 + lane + 32 * i < ee, vs[i], xv[i], s);
+                    for (int i = 0; i < 4; ++i) fma_if(oks[i], vs[i], xr[i], acc);
                 }
+            } else {
+                // a long row: every remainder entry of the item in one flat pass,
+                // one lane per entry, x gathers batched four chunks deep, rows
+                // summed by a segmented shuffle scan (fixed order)
+                const uint32_t rpS = slot + bp.rp;
+                const int etot = lds_s32(rpS + 4 * rows);
+                if (lane < 16) sts_f64(racc + 8 * lane, 0.0);
+                __syncwarp();
+#pragma unroll 1
+                for (int k0 = 0; k0 < etot; k0 += 128) {
+                    double pv[4];
+                    int rw[4];
+                    bool okv[4];
 #pragma unroll
-                for (int o = 16; o >= 1; o >>= 1) s += __shfl_xor_sync(FULL, s, o);
-                if (lane == rr) acc += s;
+                    for (int i = 0; i < 4; ++i) {
+                        const int kq = k0 + 32 * i + lane;
+                        okv[i] = kq < etot;
+                        const int c = okv[i] ? lds_s32(colS + 4 * kq) : 0;
+                        pv[i] = lds_f64(valS + 8 * (okv[i] ? kq : 0));
+                        pv[i] = okv[i] ? pv[i] * ldg_hint(p.x + (uint32_t)c, x_policy) : 0.0;
+                    }
+#pragma unroll
+                    for (int i = 0; i < 4; ++i) {  // row of entry kq: rp[row] <= kq < rp[row+1]
+                        const int kq = k0 + 32 * i + lane;
+                        int lo = 0, hi = rows;
+#pragma unroll
+                        for (int st = 0; st < 5; ++st) {
+                            const int mid = (lo + hi) >> 1;
+                            if (hi - lo > 1) {
+                                if (lds_s32(rpS + 4 * mid) <= kq) lo = mid;
+                                else hi = mid;
+                            }
+                        }
+                        rw[i] = lo;
+                    }
+#pragma unroll
+                    for (int d = 1; d < 32; d <<= 1) {
+#pragma unroll
+                        for (int i = 0; i < 4; ++i) {
+                            const double t = __shfl_up_sync(FULL, pv[i], d);
+                            const int rr = __shfl_up_sync(FULL, rw[i], d);
+                            if (lane >= d && rr == rw[i]) pv[i] += t;
+                        }
+                    }
+#pragma unroll
+                    for (int i = 0; i < 4; ++i) {  // segment tails add to their row, chunk by chunk
+                        const int nr = __shfl_down_sync(FULL, rw[i], 1);
+                        const int kq = k0 + 32 * i + lane;
+                        if (okv[i] && (lane == 31 || nr != rw[i] || kq + 1 >= etot)) {
+                            const uint32_t a = racc + 8 * rw[i];
+                            sts_f64(a, lds_f64(a) + pv[i]);
+                        }
+                        __syncwarp();
+                    }
+                }
+                if (lane < 16) acc += lds_f64(racc + 8 * lane);
             }
         }
         __syncwarp();
