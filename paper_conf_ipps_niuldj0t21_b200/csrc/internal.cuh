@@ -38,17 +38,19 @@ struct __align__(16) Item {
     uint32_t offb;    // payload offset of tile tb (16-byte units)
     uint32_t offe;    // payload offset one past the last tile
     int32_t split;    // split-row index, or -1 if the item covers its whole tile row
-    int32_t part_nt;  // part index (bits 0-23) | tiles << 24 (5 bits) | local << 29 | last << 30
+    int32_t part_nt;  // part index (bits 0-23) | tiles << 24 (5 bits) | local << 29 | last-of-group << 30
     int32_t dbeg;      // first entry of the item's tile-descriptor list (dlist)
     int32_t ndsc;      // entries: the item's tiles grouped by format, groups padded to even length
     uint32_t blob16;   // start of the item's execution blob (16-byte units)
     uint32_t blob_len; // bytes of the blob (blob_parts)
 };
 
-// A split tile row with at most kLocalParts items is "local": one warp runs
-// all of its parts in order, carrying the partial row sums in registers, and
-// writes y once.  Larger (hub) rows combine per-part partials in global
-// memory.  The choice depends only on the row's own content.
+// The parts of a split tile row form groups of kLocalParts consecutive parts.
+// One warp runs a whole group in order, carrying the partial row sums in
+// registers.  A row of one group ("local") writes y directly; a hub row of
+// several groups writes one partial per group and the last group to finish
+// sums the group partials in group order.  Everything depends only on the
+// row's own content (deterministic, shard-invariant).
 constexpr int kLocalParts = 64;
 __host__ __device__ __forceinline__ int item_nt(const Item &it) { return (it.part_nt >> 24) & 31; }
 __host__ __device__ __forceinline__ int item_part(const Item &it) { return it.part_nt & 0xFFFFFF; }

@@ -70,7 +70,7 @@ __device__ int items_for_row(int64_t I, const int32_t *tilePtr, const uint32_t *
             it.offe = tileOff[t];
             it.split = split;
             const bool local = split >= 0 && nparts <= kLocalParts;
-            const bool last = split >= 0 && cnt == nparts - 1;
+            const bool last = split >= 0 && (cnt == nparts - 1 || cnt % kLocalParts == kLocalParts - 1);
             it.part_nt = (split >= 0 ? cnt : 0) | ((t - tb) << 24) | ((int)local << 29) | ((int)last << 30);
             it.dbeg = 0;
             it.ndsc = 0;
@@ -223,8 +223,8 @@ __global__ void k_cta_begin(const int64_t *incl, const Item *items, int64_t n, i
         if (before < target) lo = mid + 1;
         else hi = mid;
     }
-    // never start inside a local split row (its parts run in one warp)
-    while (lo < n && item_local(items[lo]) && item_part(items[lo]) > 0) lo++;
+    // never start inside a group of parts of a split row (a group runs in one warp)
+    while (lo < n && items[lo].split >= 0 && item_part(items[lo]) % kLocalParts != 0) lo++;
     cta_begin[b] = lo;
 }
 

@@ -193,16 +193,35 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, MINB) tilespmv
 #pragma unroll 1
         for (int q = 0; q < npairs; ++q) run_pair(lds_v2u32(dsc + 16 * q + 8 * h), pay, xs, r, acc);
         acc += __shfl_xor_sync(FULL, acc, 16);
-        if (item_local(it)) {  // all parts of this tile row run here, in part order
-            if (!item_last(it)) {
-                carry += acc;
-            } else {
-                const int64_t row = 16 * (int64_t)it.I + lane;
-                if (lane < 16 && row < p.m) p.y[row] = carry + acc;
-                carry = 0.0;
-            }
+        if (it.split < 0) {
+            const int64_t row = 16 * (int64_t)it.I + lane;
+            if (lane < 16 && row < p.m) p.y[row] = acc;
+        } else if (!item_last(it)) {  // a group of parts runs here, in part order
+            carry += acc;
         } else {
-            write_rows(p, it, lane, acc);
+            const double total = carry + acc;
+            carry = 0.0;
+            const int64_t row = 16 * (int64_t)it.I + lane;
+            if (item_local(it)) {  // the row's only group
+                if (lane < 16 && row < p.m) p.y[row] = total;
+            } else {  // hub row: one partial per group, the last group sums them in order
+                const int2 si = p.split_info[it.split];
+                const int ngroups = (si.y + kLocalParts - 1) / kLocalParts;
+                const int g = item_part(it) / kLocalParts;
+                if (lane < 16) __stcg(p.partials + (int64_t)(si.x + g) * 16 + lane, total);
+                __threadfence();
+                __syncwarp();
+                int old = 0;
+                if (lane == 0) old = atomicAdd(p.counters + it.split, 1);
+                old = __shfl_sync(FULL, old, 0);
+                if (old == ngroups - 1) {
+                    __threadfence();
+                    double s = 0.0;
+                    for (int q = 0; q < ngroups; ++q) s += __ldcg(p.partials + (int64_t)(si.x + q) * 16 + r);
+                    if (lane < 16 && row < p.m) p.y[row] = s;
+                    if (lane == 0) p.counters[it.split] = 0;  // ready for the next run
+                }
+            }
         }
         __syncwarp();  // slot, x and J scratch free for the next item
     }
