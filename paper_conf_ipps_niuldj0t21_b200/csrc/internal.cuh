@@ -51,7 +51,7 @@ struct __align__(16) Item {
 // several groups writes one partial per group and the last group to finish
 // sums the group partials in group order.  Everything depends only on the
 // row's own content (deterministic, shard-invariant).
-constexpr int kLocalParts = 64;
+constexpr int kLocalParts = 8;
 __host__ __device__ __forceinline__ int item_nt(const Item &it) { return (it.part_nt >> 24) & 31; }
 __host__ __device__ __forceinline__ int item_part(const Item &it) { return it.part_nt & 0xFFFFFF; }
 __host__ __device__ __forceinline__ bool item_local(const Item &it) { return (it.part_nt >> 29) & 1; }

@@ -214,10 +214,20 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, MINB) tilespmv
                 int old = 0;
                 if (lane == 0) old = atomicAdd(p.counters + it.split, 1);
                 old = __shfl_sync(FULL, old, 0);
-                if (old == ngroups - 1) {
+                if (old == ngroups - 1) {  // half hh sums groups hh, hh+2, ... in order, 4 loads in flight
                     __threadfence();
                     double s = 0.0;
-                    for (int q = 0; q < ngroups; ++q) s += __ldcg(p.partials + (int64_t)(si.x + q) * 16 + r);
+                    for (int q0 = h; q0 < ngroups; q0 += 8) {
+                        double v[4];
+#pragma unroll
+                        for (int i = 0; i < 4; ++i) {
+                            const int q = q0 + 2 * i;
+                            v[i] = q < ngroups ? __ldcg(p.partials + (int64_t)(si.x + q) * 16 + r) : 0.0;
+                        }
+#pragma unroll
+                        for (int i = 0; i < 4; ++i) s += v[i];
+                    }
+                    s += __shfl_xor_sync(FULL, s, 16);
                     if (lane < 16 && row < p.m) p.y[row] = s;
                     if (lane == 0) p.counters[it.split] = 0;  // ready for the next run
                 }
