@@ -178,11 +178,17 @@ def oracle_sample(A, x, seconds: float, rng, max_rows=None):
             break
     rows = np.unique(np.concatenate(blocks)) if blocks else np.arange(min(A.m, 1))
     nnz = int(rowlen[rows].sum())
-    t = time.perf_counter()
-    yref, absy = O.spmv(A, x, rows)
-    dt = time.perf_counter() - t
+    # repeat the sample until about `seconds` of CPU work (at most 3x that)
+    passes, t = 0, time.perf_counter()
+    while True:
+        yref, absy = O.spmv(A, x, rows)
+        passes += 1
+        dt = time.perf_counter() - t
+        if dt >= seconds or dt * (passes + 1) / passes > 3 * seconds:
+            break
     desc = (f"{rows.size} rows ({nnz} nnz, {100.0 * nnz / max(A.nnz, 1):.2f}% of the matrix) "
-            f"in 4096-row blocks at seeded random offsets; one pass, {dt:.2f} s")
+            f"in 4096-row blocks at seeded random offsets; {passes} pass(es), {dt:.2f} s")
+    nnz *= passes
     return 2.0 * nnz / dt / 1e9, rows, yref, absy, desc, dt
 
 
@@ -332,7 +338,9 @@ def measure_workload(workload, mode, steps, warmup, dev, rank, P, group, cpu_sec
     value = 2.0 * nnz_total / (ms_per_step * 1e-3) / 1e9
     peak, peak_src = hbm_peak()
     achieved = info["alg_bytes"] / (float(np.mean(kern_ms)) * 1e-3) / 1e9
+    grid, block, smem = M0.launch_shape()
     res = {"value": value, "ms_per_step": ms_per_step, "info": info, "reps": reps,
+           "launch": {"grid": grid, "block": block, "smem_bytes": smem},
            "kernel_ms_mean": float(np.mean(kern_ms)), "kernel_ms_median": float(np.median(kern_ms)),
            "kernel_ms_max_over_ranks": kern_max, "create_s": create_s,
            "clocks": sampler.summary(), "nnz": nnz_total, "m": m, "n": n,
@@ -340,7 +348,7 @@ def measure_workload(workload, mode, steps, warmup, dev, rank, P, group, cpu_sec
                         "frac": achieved / peak, "traffic": profile_traffic(workload, mode),
                         "peak_source": peak_src,
                         "alg_bytes_per_launch": info["alg_bytes"],
-                        "kernel": "tilespmv_fp64_kernel"}}
+                        "kernel": M0.kernel_name()}}
     # ---- correctness on the oracle's sample + CPU baseline (rank 0, N = 1)
     if want_cpu and rank == 0 and P == 1:
         rng = np.random.default_rng(4321)
@@ -421,6 +429,7 @@ def run_ours(args):
                "kernel_ms": {"mean": res["kernel_ms_mean"], "median": res["kernel_ms_median"],
                              "max_over_ranks": res["kernel_ms_max_over_ranks"]},
                "clocks": res["clocks"],
+               "launch": res["launch"],
                "parity": res.get("parity")}
         if secondary:
             out["secondary"] = secondary

@@ -140,9 +140,13 @@ const char *tilespmv_status_string(int status);
 /* Message of the last failing call on this thread ("" if none). */
 const char *tilespmv_last_error(void);
 
-/* Name of the SpMV kernel symbol (for profiler filters) and its launch shape
- * for this handle: grid CTAs, threads per CTA, dynamic shared memory bytes. */
+/* Launch shape of the SpMV kernel for this handle: grid CTAs, threads per
+ * CTA, dynamic shared memory bytes. */
 int tilespmv_launch_shape(tilespmv_handle_t h, int32_t *grid, int32_t *block, int32_t *smem_bytes);
+
+/* Name of the SpMV kernel variant this handle launches (static string; ""
+ * for a NULL handle). */
+const char *tilespmv_kernel_name(tilespmv_handle_t h);
 
 #ifdef __cplusplus
 }

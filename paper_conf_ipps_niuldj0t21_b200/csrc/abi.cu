@@ -251,4 +251,6 @@ int tilespmv_launch_shape(tilespmv_handle_t h, int32_t *grid, int32_t *block, in
     return TILESPMV_OK;
 }
 
+const char *tilespmv_kernel_name(tilespmv_handle_t h) { return h ? h->kernel_name : ""; }
+
 }  // extern "C"

@@ -92,7 +92,8 @@ struct Matrix {
     int64_t blob_bytes = 0;
     int64_t *cta_begin = nullptr;  // contiguous item chunk per warp (row-aligned, cost-balanced)
     // launch shape
-    int kernel_version = 2;
+    int kernel_version = 20;
+    const char *kernel_name = "";
     int item_bytes = kItemBytesMax;  // slot size the schedule was built for
     int grid = 0, block = 0, smem = 0;
 };

@@ -352,6 +352,7 @@ int configure_launch(Matrix &M) {
     TSP_CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, M.device));
     TSP_CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kc.fn, kc.threads, kc.smem));
     if (per_sm < 1) return set_error(TILESPMV_CUDA, "SpMV kernel does not fit on an SM");
+    M.kernel_name = kc.name;
     M.block = kc.threads;
     M.smem = kc.smem;
     if (kc.ring) return set_error(TILESPMV_CUDA, "no ring kernel in this build");

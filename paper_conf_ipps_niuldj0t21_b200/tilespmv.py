@@ -23,7 +23,7 @@ ARRAYS = {"tilePtr": (0, np.int32), "tileColIdx": (1, np.int32), "tileNnz": (2, 
 EXPORTED_SYMBOLS = ["tilespmv_create_from_csr", "tilespmv_run", "tilespmv_run_host",
                     "tilespmv_destroy", "tilespmv_get_info", "tilespmv_export_size",
                     "tilespmv_export", "tilespmv_status_string", "tilespmv_last_error",
-                    "tilespmv_launch_shape"]
+                    "tilespmv_launch_shape", "tilespmv_kernel_name"]
 
 
 class TileSpMVError(RuntimeError):
@@ -86,6 +86,8 @@ def load(build_if_missing: bool = True):
     L.tilespmv_last_error.restype = ctypes.c_char_p
     L.tilespmv_launch_shape.argtypes = [p, ctypes.POINTER(i32), ctypes.POINTER(i32),
                                         ctypes.POINTER(i32)]
+    L.tilespmv_kernel_name.argtypes = [p]
+    L.tilespmv_kernel_name.restype = ctypes.c_char_p
     for name in ("tilespmv_create_from_csr", "tilespmv_run", "tilespmv_run_host",
                  "tilespmv_destroy", "tilespmv_get_info", "tilespmv_export",
                  "tilespmv_launch_shape"):
@@ -204,6 +206,9 @@ class TiledMatrix:
         _check(load().tilespmv_launch_shape(self._h, ctypes.byref(g), ctypes.byref(b),
                                             ctypes.byref(s)), "tilespmv_launch_shape")
         return g.value, b.value, s.value
+
+    def kernel_name(self) -> str:
+        return load().tilespmv_kernel_name(self._h).decode()
 
     # --------------------------------------------------------------- cleanup
     def close(self):
