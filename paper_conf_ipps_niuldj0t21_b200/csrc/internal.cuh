@@ -45,6 +45,19 @@ struct __align__(16) Item {
     uint32_t blob_len; // bytes of the blob (blob_parts)
 };
 
+// Compact per-item record read by the warp kernel (built with the blobs):
+// blob start, tile row, split bookkeeping, and the blob's part offsets.
+struct __align__(16) WItem {
+    uint32_t blob16;    // blob start (16-byte units)
+    uint32_t I;         // tile row
+    int32_t split;      // split-row index or -1
+    int32_t part_nt;    // as Item::part_nt
+    uint32_t jt_rows_pay;  // jt offset (8 bits) | rows in the tile row (5 bits) << 8 | payload offset << 16
+    uint32_t rp_col;       // rp offset | col offset << 16
+    uint32_t val_tot;      // val offset | total bytes << 16
+    uint32_t groups;       // tile pairs per format f, 4 bits at 4f (descriptor list order)
+};
+
 // The parts of a split tile row form groups of kLocalParts consecutive parts.
 // One warp runs a whole group in order, carrying the partial row sums in
 // registers.  A row of one group ("local") writes y directly; a hub row of
@@ -89,6 +102,7 @@ struct Matrix {
     uint2 *tdesc = nullptr;        // per-item tile-descriptor lists (dlist), create-time only
     int64_t num_dsc = 0;
     uint8_t *blob = nullptr;       // per-item execution blobs (blob_parts), read by the kernels
+    WItem *witems = nullptr;       // compact per-item records for the warp kernel
     int64_t blob_bytes = 0;
     int64_t *cta_begin = nullptr;  // contiguous item chunk per warp (row-aligned, cost-balanced)
     // launch shape

@@ -158,8 +158,9 @@ __global__ void k_blob_len(const Item *items, int64_t n, int64_t m, int64_t *len
 
 // one warp per item: copy descriptors, J, payload and the rebased remainder
 __global__ void k_blob_fill(Item *items, int64_t n, int64_t m, const int64_t *start16, const uint2 *dlist,
-                            const int32_t *tileColIdx, const uint8_t *payload, const int32_t *remRowPtr,
-                            const int32_t *remCol, const double *remVal, uint8_t *blob) {
+                            const int32_t *tileColIdx, const uint8_t *tileFmt, const uint8_t *payload,
+                            const int32_t *remRowPtr, const int32_t *remCol, const double *remVal, uint8_t *blob,
+                            WItem *witems) {
     const int64_t k = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
     const int lane = threadIdx.x & 31;
     if (k >= n) return;
@@ -170,6 +171,21 @@ __global__ void k_blob_fill(Item *items, int64_t n, int64_t m, const int64_t *st
         it.blob16 = (uint32_t)start16[k];
         it.blob_len = b.total;
         items[k] = it;
+        WItem w;
+        w.blob16 = it.blob16;
+        w.I = (uint32_t)it.I;
+        w.split = it.split;
+        w.part_nt = it.part_nt;
+        const uint32_t rows = (uint32_t)imin64(16, m - 16 * (int64_t)it.I);
+        w.jt_rows_pay = b.jt | (rows << 8) | (b.pay << 16);
+        w.rp_col = b.rp | (b.col << 16);
+        w.val_tot = b.val | (b.total << 16);
+        int cnt[7] = {0, 0, 0, 0, 0, 0, 0};
+        for (int t = 0; t < item_nt(it); ++t) cnt[tileFmt[it.tb + t]]++;
+        uint32_t g = 0;
+        for (int f = 0; f < 7; ++f) g |= (uint32_t)((cnt[f] + 1) >> 1) << (4 * f);
+        w.groups = g;
+        witems[k] = w;
     }
     for (uint32_t o = 4 * lane; o < b.total; o += 128) *reinterpret_cast<uint32_t *>(dst + o) = 0u;  // padding
     __syncwarp();
@@ -293,6 +309,7 @@ int build_tdesc(Matrix &M, cudaStream_t st) {
     if (n == 0) {
         TSP_CK(cudaMalloc(&M.tdesc, 4 * sizeof(uint2)));
         TSP_CK(cudaMalloc(&M.blob, 256));
+        TSP_CK(cudaMalloc(&M.witems, sizeof(WItem)));
         return 0;
     }
     int32_t *cnt = nullptr;
@@ -327,8 +344,11 @@ int build_tdesc(Matrix &M, cudaStream_t st) {
         M.blob_bytes = total16 * 16;
         if (cudaMalloc(&M.blob, M.blob_bytes + 256) != cudaSuccess) { rc = cuda_status(cudaGetLastError(), "cudaMalloc(blob)"); cudaFree(len16); break; }
         M.device_bytes += M.blob_bytes + 256;
+        if (cudaMalloc(&M.witems, n * sizeof(WItem)) != cudaSuccess) { rc = cuda_status(cudaGetLastError(), "cudaMalloc(witems)"); cudaFree(len16); break; }
+        M.device_bytes += n * (int64_t)sizeof(WItem);
         k_blob_fill<<<(unsigned)((n * 32 + 255) / 256), 256, 0, st>>>(M.items, n, M.m, start16, M.tdesc, M.tileColIdx,
-                                                                     M.payload, M.remRowPtr, M.remCol, M.remVal, M.blob);
+                                                                     M.tileFmt, M.payload, M.remRowPtr, M.remCol,
+                                                                     M.remVal, M.blob, M.witems);
         if (cudaStreamSynchronize(st) != cudaSuccess) rc = cuda_status(cudaGetLastError(), "k_blob_fill");
         cudaFree(len16);
     } while (0);
@@ -413,6 +433,7 @@ int launch_spmv(const Matrix &M, const double *d_x, double *d_y, cudaStream_t st
     p.n = M.n;
     p.tdesc = M.tdesc;
     p.blob = M.blob;
+    p.witems = M.witems;
     p.cta_begin = M.cta_begin;
     p.x_vec = (reinterpret_cast<uintptr_t>(d_x) & 15u) == 0;
     const KernelChoice kc = choose(M.kernel_version);

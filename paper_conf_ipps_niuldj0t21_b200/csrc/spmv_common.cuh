@@ -29,6 +29,7 @@ struct Params {
     int64_t m, n;
     const uint2 *tdesc;        // per-item tile-descriptor lists (schedule.cu)
     const uint8_t *blob;       // per-item execution blobs (schedule.cu)
+    const WItem *witems;       // compact per-item records (schedule.cu)
     const int64_t *cta_begin;  // warp kernel: item chunk of each warp
     int x_vec;                 // x is 16-byte aligned: x segments load as double2
 };
@@ -175,6 +176,16 @@ __device__ __forceinline__ double2 ldg2_hint(const double *p, uint64_t policy) {
 __device__ __forceinline__ void sts_v2f64(uint32_t a, double2 v) {
     asm volatile("st.shared.v2.f64 [%0], {%1, %2};" ::"r"(a), "d"(v.x), "d"(v.y) : "memory");
 }
+// 16-byte async copy global -> shared; bytes beyond src_bytes (0..16) are zero-filled
+__device__ __forceinline__ void cp_async16(uint32_t dst, const void *src, uint32_t src_bytes, uint64_t policy) {
+    asm volatile("cp.async.cg.shared.global.L2::cache_hint [%0], [%1], 16, %2, %3;" ::"r"(dst), "l"(src),
+                 "r"(src_bytes), "l"(policy)
+                 : "memory");
+}
+__device__ __forceinline__ void cp_async_wait_all() {
+    asm volatile("cp.async.commit_group;\n\tcp.async.wait_group 0;" ::: "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
 // acc += a * b only where pred holds (one predicated DFMA, no select)
 __device__ __forceinline__ void fma_if(bool pred, double a, double b, double &acc) {
     asm("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %3, 0;\n\t@q fma.rn.f64 %0, %1, %2, %0;\n\t}"
