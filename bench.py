@@ -376,6 +376,34 @@ def measure_workload(workload, mode, steps, warmup, dev, rank, P, group, cpu_sec
                       "h2d_bytes_per_step": 8 * n, "d2h_bytes_per_step": 8 * A.m,
                       "ms_per_step": e2e_s * 1e3, "steps": e2e_steps,
                       "call": "tilespmv_run_host (pinned host x -> H2D -> kernel -> D2H y -> sync)"}
+    if want_e2e and P > 1:
+        # per step on every rank: H2D of x (replicated), the local SpMV, the NCCL
+        # all-gather of y, D2H of the gathered y; max over ranks
+        hx = torch.from_numpy(x_h).pin_memory()
+        hy = torch.empty(P * maxrows, dtype=torch.float64).pin_memory()
+        xd = torch.empty(n, dtype=torch.float64, device=dev)
+
+        def e2e_step():
+            xd.copy_(hx, non_blocking=True)
+            y = gathered[rank * maxrows: rank * maxrows + rows_local]
+            M0.run(xd, y)
+            dist.all_gather_into_tensor(gathered, gathered[rank * maxrows:(rank + 1) * maxrows], group=group)
+            hy.copy_(gathered, non_blocking=True)
+            torch.cuda.current_stream(dev).synchronize()
+
+        for _ in range(2):
+            e2e_step()
+        dist.barrier(group=group)
+        t = time.perf_counter()
+        for _ in range(e2e_steps):
+            e2e_step()
+        e2e_s = torch.tensor([(time.perf_counter() - t) / e2e_steps], dtype=torch.float64, device=dev)
+        dist.all_reduce(e2e_s, op=dist.ReduceOp.MAX, group=group)
+        e2e_s = float(e2e_s[0])
+        res["e2e"] = {"value": 2.0 * nnz_total / e2e_s / 1e9, "unit": UNIT,
+                      "h2d_bytes_per_step": 8 * n, "d2h_bytes_per_step": 8 * P * maxrows,
+                      "ms_per_step": e2e_s * 1e3, "steps": e2e_steps,
+                      "call": "per rank: H2D x -> TiledMatrix.run -> NCCL all-gather y -> D2H y (max over ranks)"}
     for M in mats:
         M.close()
     return res

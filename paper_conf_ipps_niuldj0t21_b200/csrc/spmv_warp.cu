@@ -8,7 +8,7 @@
 // warp's shared-memory slot with ONE TMA bulk copy (cp.async.bulk, L2
 // evict-first) completing on the warp's mbarrier.  The warp then
 //   1. starts the x segment of every tile (one 128-byte line) with cp.async
-//      (L2 evict-last, zero-filled past n),
+//      (L2 evict-last; the tail of x past n reads as 0),
 //   2. runs the fused CSR remainder rows of the tile row,
 //   3. runs the tiles two at a time, format group by format group, with the
 //      half-warp routines of spmv_tiles.cuh (one lane per tile row),
@@ -194,8 +194,12 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, MINB) tilespmv
                 const int t = 4 * kk + (lane >> 3);
                 if (t < nt) {
                     const uint32_t c0 = 16u * (uint32_t)lds_s32(jt + 4 * t) + 2u * qq;
-                    const uint32_t nb = c0 < n32 ? min(16u, 8u * (n32 - c0)) : 0u;
-                    cp_async16(xs + 128 * t + 16 * qq, p.x + (nb ? c0 : 0u), nb, x_policy);
+                    if (c0 + 2 <= n32) {
+                        cp_async16(xs + 128 * t + 16 * qq, p.x + c0, 16u, x_policy);
+                    } else {  // the tail of x: never read past x[n-1]
+                        const double v0 = c0 < n32 ? ldg_hint(p.x + c0, x_policy) : 0.0;
+                        sts_v2f64(xs + 128 * t + 16 * qq, make_double2(v0, 0.0));
+                    }
                 }
             }
             cp_async_commit();
