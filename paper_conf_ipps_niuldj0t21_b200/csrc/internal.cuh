@@ -28,7 +28,7 @@ enum : uint8_t { F_CSR = 0, F_COO = 1, F_ELL = 2, F_HYB = 3, F_DNS = 4, F_DNSROW
 // run reproduces the 1-GPU y bitwise.
 // ---------------------------------------------------------------------------
 constexpr int kItemTiles = 16;
-constexpr int kItemBytesMax = 8192;  // largest shared-memory slot of any kernel
+constexpr int kItemBytesMax = 12288;  // largest shared-memory slot of any kernel
 constexpr int kShortRow = 16;     // remainder rows up to this length: 2 lanes per row
 
 struct __align__(16) Item {

@@ -357,7 +357,11 @@ int build_tdesc(Matrix &M, cudaStream_t st) {
 }
 
 int choose_kernel(Matrix &M) {
-    int version = 20;  // default: high-occupancy warp kernel (spmv_warp.cu)
+    // default: the warp kernel with 4.5 KB slots (32 warps/SM); matrices whose
+    // tile rows average more than 6 KB of payload (dense, FEM-like) use 10.5 KB
+    // slots (16 warps/SM) so a tile row stays one item
+    const double row_bytes = M.tilem ? (double)M.payload_bytes / (double)M.tilem : 0.0;
+    int version = row_bytes > 6144.0 ? 25 : 20;
     if (const char *e = getenv("TILESPMV_KERNEL")) version = atoi(e);
     M.kernel_version = version;
     M.item_bytes = choose(version).slot_bytes;

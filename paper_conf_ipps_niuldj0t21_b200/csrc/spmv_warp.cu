@@ -292,6 +292,8 @@ KernelChoice kernel_warp(int variant) {
     case 22: return warp_choice<8, 5120, 3>("tilespmv_fp64_warp<8,5120>");
     case 23: return warp_choice<4, 4608, 8>("tilespmv_fp64_warp<4,4608>");
     case 24: return warp_choice<8, 4096, 4>("tilespmv_fp64_warp<8,4096>");
+    case 25: return warp_choice<4, 10752, 4>("tilespmv_fp64_warp<4,10752>");  // dense tile rows
+    case 26: return warp_choice<4, 8704, 5>("tilespmv_fp64_warp<4,8704>");
     default: return warp_choice<8, 4608, 4>("tilespmv_fp64_warp<8,4608>");
     }
 }
