@@ -52,10 +52,18 @@ struct __align__(16) WItem {
     uint32_t I;         // tile row
     int32_t split;      // split-row index or -1
     int32_t part_nt;    // as Item::part_nt
-    uint32_t jt_rows_pay;  // jt offset (8 bits) | rows in the tile row (5 bits) << 8 | payload offset << 16
+    uint32_t jt_rows_pay;  // (unused, 8 bits) | rows in the tile row (5 bits) << 8 | payload offset << 16
     uint32_t rp_col;       // rp offset | col offset << 16
     uint32_t val_tot;      // val offset | total bytes << 16
     uint32_t groups;       // tile pairs per format f, 4 bits at 4f (descriptor list order)
+};
+
+// Per-warp start record of the warp kernel: the warp's item chunk and a copy
+// of its first item, so the prologue needs one round trip before the blob.
+struct __align__(16) WFirst {
+    int32_t kbeg, kend, pad0, pad1;
+    WItem w;
+    int32_t J[16];
 };
 
 // The parts of a split tile row form groups of kLocalParts consecutive parts.
@@ -103,6 +111,8 @@ struct Matrix {
     int64_t num_dsc = 0;
     uint8_t *blob = nullptr;       // per-item execution blobs (blob_parts), read by the kernels
     WItem *witems = nullptr;       // compact per-item records for the warp kernel
+    int32_t *jcols = nullptr;      // 16 tile columns per item (warp kernel)
+    WFirst *wfirst = nullptr;      // per-warp chunk + first item (warp kernel)
     int64_t blob_bytes = 0;
     int64_t *cta_begin = nullptr;  // contiguous item chunk per warp (row-aligned, cost-balanced)
     // launch shape

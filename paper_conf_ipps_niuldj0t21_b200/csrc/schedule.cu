@@ -160,7 +160,7 @@ __global__ void k_blob_len(const Item *items, int64_t n, int64_t m, int64_t *len
 __global__ void k_blob_fill(Item *items, int64_t n, int64_t m, const int64_t *start16, const uint2 *dlist,
                             const int32_t *tileColIdx, const uint8_t *tileFmt, const uint8_t *payload,
                             const int32_t *remRowPtr, const int32_t *remCol, const double *remVal, uint8_t *blob,
-                            WItem *witems) {
+                            WItem *witems, int32_t *jcols) {
     const int64_t k = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
     const int lane = threadIdx.x & 31;
     if (k >= n) return;
@@ -177,7 +177,7 @@ __global__ void k_blob_fill(Item *items, int64_t n, int64_t m, const int64_t *st
         w.split = it.split;
         w.part_nt = it.part_nt;
         const uint32_t rows = (uint32_t)imin64(16, m - 16 * (int64_t)it.I);
-        w.jt_rows_pay = b.jt | (rows << 8) | (b.pay << 16);
+        w.jt_rows_pay = (rows << 8) | (b.pay << 16);
         w.rp_col = b.rp | (b.col << 16);
         w.val_tot = b.val | (b.total << 16);
         int cnt[7] = {0, 0, 0, 0, 0, 0, 0};
@@ -192,8 +192,7 @@ __global__ void k_blob_fill(Item *items, int64_t n, int64_t m, const int64_t *st
     uint2 *dd = reinterpret_cast<uint2 *>(dst);
     for (int i = lane; i < it.ndsc; i += 32) dd[i] = dlist[it.dbeg + i];
     const int nt = item_nt(it);
-    int32_t *jt = reinterpret_cast<int32_t *>(dst + b.jt);
-    for (int t = lane; t < nt; t += 32) jt[t] = tileColIdx[it.tb + t];
+    if (lane < 16) jcols[k * 16 + lane] = lane < nt ? tileColIdx[it.tb + lane] : 0;
     const uint4 *ps = reinterpret_cast<const uint4 *>(payload + (size_t)it.offb * 16);
     uint4 *pd = reinterpret_cast<uint4 *>(dst + b.pay);
     for (uint32_t i = lane; i < it.offe - it.offb; i += 32) pd[i] = ps[i];
@@ -221,6 +220,23 @@ __global__ void k_item_cost(const Item *items, int64_t n, int64_t m, int64_t *co
     if (k >= n) return;
     const Item it = items[k];
     cost[k] = (int64_t)item_parts(it, m).total + 40 * (item_nt(it)) + 512;
+}
+
+__global__ void k_warp_first(const int64_t *begin, const WItem *witems, const int32_t *jcols, int W, WFirst *wf) {
+    const int b = blockIdx.x * blockDim.x + threadIdx.x;
+    if (b >= W) return;
+    WFirst f;
+    f.kbeg = (int32_t)begin[b];
+    f.kend = (int32_t)begin[b + 1];
+    f.pad0 = f.pad1 = 0;
+    if (f.kbeg < f.kend) {
+        f.w = witems[f.kbeg];
+        for (int i = 0; i < 16; ++i) f.J[i] = jcols[(int64_t)f.kbeg * 16 + i];
+    } else {
+        f.w = WItem{};
+        for (int i = 0; i < 16; ++i) f.J[i] = 0;
+    }
+    wf[b] = f;
 }
 
 __global__ void k_cta_begin(const int64_t *incl, const Item *items, int64_t n, int G, int64_t *cta_begin) {
@@ -310,6 +326,7 @@ int build_tdesc(Matrix &M, cudaStream_t st) {
         TSP_CK(cudaMalloc(&M.tdesc, 4 * sizeof(uint2)));
         TSP_CK(cudaMalloc(&M.blob, 256));
         TSP_CK(cudaMalloc(&M.witems, sizeof(WItem)));
+        TSP_CK(cudaMalloc(&M.jcols, 16 * sizeof(int32_t)));
         return 0;
     }
     int32_t *cnt = nullptr;
@@ -344,11 +361,16 @@ int build_tdesc(Matrix &M, cudaStream_t st) {
         M.blob_bytes = total16 * 16;
         if (cudaMalloc(&M.blob, M.blob_bytes + 256) != cudaSuccess) { rc = cuda_status(cudaGetLastError(), "cudaMalloc(blob)"); cudaFree(len16); break; }
         M.device_bytes += M.blob_bytes + 256;
-        if (cudaMalloc(&M.witems, n * sizeof(WItem)) != cudaSuccess) { rc = cuda_status(cudaGetLastError(), "cudaMalloc(witems)"); cudaFree(len16); break; }
-        M.device_bytes += n * (int64_t)sizeof(WItem);
+        if (cudaMalloc(&M.witems, n * sizeof(WItem)) != cudaSuccess ||
+            cudaMalloc(&M.jcols, n * 16 * sizeof(int32_t)) != cudaSuccess) {
+            rc = cuda_status(cudaGetLastError(), "cudaMalloc(witems)");
+            cudaFree(len16);
+            break;
+        }
+        M.device_bytes += n * (int64_t)(sizeof(WItem) + 64);
         k_blob_fill<<<(unsigned)((n * 32 + 255) / 256), 256, 0, st>>>(M.items, n, M.m, start16, M.tdesc, M.tileColIdx,
                                                                      M.tileFmt, M.payload, M.remRowPtr, M.remCol,
-                                                                     M.remVal, M.blob, M.witems);
+                                                                     M.remVal, M.blob, M.witems, M.jcols);
         if (cudaStreamSynchronize(st) != cudaSuccess) rc = cuda_status(cudaGetLastError(), "k_blob_fill");
         cudaFree(len16);
     } while (0);
@@ -411,6 +433,12 @@ int configure_launch(Matrix &M) {
     } else {
         TSP_CK(cudaMemset(M.cta_begin, 0, (W + 1) * sizeof(int64_t)));
     }
+    if (M.wfirst) cudaFree(M.wfirst);
+    M.wfirst = nullptr;
+    TSP_CK(cudaMalloc(&M.wfirst, W * sizeof(WFirst)));
+    M.device_bytes += W * (int64_t)sizeof(WFirst);
+    k_warp_first<<<(W + 255) / 256, 256>>>(M.cta_begin, M.witems, M.jcols, W, M.wfirst);
+    TSP_CK(cudaDeviceSynchronize());
     return 0;
 }
 
@@ -438,6 +466,8 @@ int launch_spmv(const Matrix &M, const double *d_x, double *d_y, cudaStream_t st
     p.tdesc = M.tdesc;
     p.blob = M.blob;
     p.witems = M.witems;
+    p.jcols = M.jcols;
+    p.wfirst = M.wfirst;
     p.cta_begin = M.cta_begin;
     p.x_vec = (reinterpret_cast<uintptr_t>(d_x) & 15u) == 0;
     const KernelChoice kc = choose(M.kernel_version);

@@ -30,6 +30,8 @@ struct Params {
     const uint2 *tdesc;        // per-item tile-descriptor lists (schedule.cu)
     const uint8_t *blob;       // per-item execution blobs (schedule.cu)
     const WItem *witems;       // compact per-item records (schedule.cu)
+    const int32_t *jcols;      // tile column J of each item's tiles, 16 per item
+    const WFirst *wfirst;      // per-warp chunk and first item (warp kernel)
     const int64_t *cta_begin;  // warp kernel: item chunk of each warp
     int x_vec;                 // x is 16-byte aligned: x segments load as double2
 };
@@ -117,20 +119,17 @@ __host__ __device__ __forceinline__ ItemParts item_parts(const Item &it, int64_t
 // A create-time copy of everything one work item reads, contiguous and
 // 16-byte aligned part by part, so a single TMA bulk copy stages it:
 //   dsc : the descriptor list (k_dsc_write), ndsc x 8 B
-//   jt  : tile column index J of tiles 0..nt-1, 4 B each
 //   pay : the tiles' canonical payload bytes
 //   rp  : remainder row pointers of the item's rows, rebased to the item's
 //         entry range and clamped to it (rows + 1 ints)
 //   col, val : the item's remainder entries
 struct BlobParts {
-    uint32_t jt, pay, rp, col, val, total;
+    uint32_t pay, rp, col, val, total;
 };
 
 __host__ __device__ __forceinline__ BlobParts blob_parts(const Item &it, int64_t m) {
     BlobParts b;
-    const uint32_t nt = (uint32_t)item_nt(it);
-    b.jt = up16(8u * (uint32_t)it.ndsc);
-    b.pay = b.jt + up16(4u * nt);
+    b.pay = up16(8u * (uint32_t)it.ndsc);
     b.rp = b.pay + (it.offe - it.offb) * 16u;
     if (it.ke > it.kb) {
         const uint32_t rows = (uint32_t)imin64(16, m - 16 * (int64_t)it.I);

@@ -162,38 +162,37 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, MINB) tilespmv
     __syncwarp();
     const uint32_t n32 = (uint32_t)p.n;
     // contiguous, cost-balanced, row-aligned item chunk per warp (schedule.cu);
-    // neighbouring tile rows share x segments
+    // neighbouring tile rows share x segments.  The warp's start record holds
+    // the chunk and a copy of the first item (one round trip).
     const int64_t gw = (int64_t)blockIdx.x * WARPS + warp;
-    const int kbeg = (int)p.cta_begin[gw], kend = (int)p.cta_begin[gw + 1];
+    const WFirst *wf = p.wfirst + gw;
+    const int4 wb = __ldg(reinterpret_cast<const int4 *>(wf));
+    const int kbeg = wb.x, kend = wb.y;
     double carry = 0.0;  // partial row sums inside a group of parts of a split tile row
     uint32_t phase = 0;
     const uint64_t stream_policy = policy_evict_first(), x_policy = policy_evict_last();
-    WItem nxt;
-    if (kbeg < kend) nxt = load_witem(p.witems, kbeg);
+    WItem nxt = load_witem(&wf->w, 0);
+    int Jn = lane < 16 ? __ldg(wf->J + lane) : 0;
     for (int k = kbeg; k < kend; ++k) {
         const WItem it = nxt;
-        if (k + 1 < kend) nxt = load_witem(p.witems, k + 1);  // in flight during this item
+        const int J = Jn;
         const uint32_t total = it.val_tot >> 16;
-        // the whole item (descriptors, J, payload, remainder) in ONE TMA bulk copy
+        // the whole item (descriptors, payload, remainder) in ONE TMA bulk copy
         if (lane == 0 && total) {
             fence_proxy_async();
             mbar_expect_tx(bar, total);
             bulk_g2s_hint(slot, p.blob + (size_t)it.blob16 * 16, total, bar, stream_policy);
         }
-        if (total) {
-            mbar_wait(bar, phase);
-            phase ^= 1u;
-        }
         const int nt = (it.part_nt >> 24) & 31;
-        const uint32_t jt = slot + (it.jt_rows_pay & 255u), pay = slot + (it.jt_rows_pay >> 16);
-        // 1. x segments (asynchronous; consumed by the tiles below)
+        const uint32_t pay = slot + (it.jt_rows_pay >> 16);
+        // 1. x segments, issued before the blob lands (J came with the record)
         if (p.x_vec) {  // lane l: tile 4k + (l >> 3), 16 bytes at elements 2(l & 7)
             const uint32_t qq = lane & 7;
 #pragma unroll
             for (int kk = 0; kk < kItemTiles / 4; ++kk) {
                 const int t = 4 * kk + (lane >> 3);
+                const uint32_t c0 = 16u * (uint32_t)__shfl_sync(FULL, J, t) + 2u * qq;
                 if (t < nt) {
-                    const uint32_t c0 = 16u * (uint32_t)lds_s32(jt + 4 * t) + 2u * qq;
                     if (c0 + 2 <= n32) {
                         cp_async16(xs + 128 * t + 16 * qq, p.x + c0, 16u, x_policy);
                     } else {  // the tail of x: never read past x[n-1]
@@ -207,11 +206,17 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, MINB) tilespmv
 #pragma unroll
             for (int kk = 0; kk < kItemTiles / 2; ++kk) {
                 const int t = 2 * kk + h;
-                if (t < nt) {
-                    const uint32_t col = 16u * (uint32_t)lds_s32(jt + 4 * t) + (uint32_t)r;
-                    sts_f64(xs + 8 * (16 * t + r), col < n32 ? ldg_hint(p.x + col, x_policy) : 0.0);
-                }
+                const uint32_t col = 16u * (uint32_t)__shfl_sync(FULL, J, t) + (uint32_t)r;
+                if (t < nt) sts_f64(xs + 8 * (16 * t + r), col < n32 ? ldg_hint(p.x + col, x_policy) : 0.0);
             }
+        }
+        if (k + 1 < kend) {  // the next record and its columns, in flight during this item
+            nxt = load_witem(p.witems, k + 1);
+            Jn = lane < 16 ? __ldg(p.jcols + (int64_t)(k + 1) * 16 + lane) : 0;
+        }
+        if (total) {
+            mbar_wait(bar, phase);
+            phase ^= 1u;
         }
         // 2. fused CSR remainder
         double acc = 0.0;
