@@ -259,3 +259,37 @@ def test_full_size_tiler_and_spmv(cuda_device, name):
         y3 = M.run(xd * 2).cpu().numpy()
         assert np.array_equal(y3, 2 * yh)
         M.close()
+
+
+@pytest.mark.parametrize("variant", ["1", "20", "21", "22", "23", "24", "25", "26"])
+def test_kernel_variants_parity(cuda_device, variant, monkeypatch):
+    """Every SpMV kernel variant (TILESPMV_KERNEL, read at create time) meets
+    the oracle tolerance; each is run-to-run bitwise deterministic."""
+    import torch
+    monkeypatch.setenv("TILESPMV_KERNEL", variant)
+    TM = tm()
+    for name in ("mixed_small", "rmat12", "stencil27_21", "fem_small", "lap2d_37x29"):
+        A, x = gen.make(name)
+        yref, absy = O.spmv(A, x)
+        for mode in ("ADPT", "DEFERRED"):
+            M = TM.from_host_csr(A, mode=mode, device=cuda_device)
+            xd = torch.from_numpy(x).to(cuda_device)
+            y1 = M.run(xd).cpu().numpy()
+            y2 = M.run(xd).cpu().numpy()
+            assert_spmv_close(y1, yref, absy, f"{name}/{mode}/v{variant}")
+            assert np.array_equal(y1.view(np.uint64), y2.view(np.uint64))
+            M.close()
+
+
+def test_misaligned_x_uses_scalar_path(cuda_device):
+    """x not 16-byte aligned (a view at an odd element offset) takes the
+    scalar x-staging path and gives the same y."""
+    import torch
+    TM = tm()
+    A, x = gen.make("stencil27_21")
+    M = TM.from_host_csr(A, device=cuda_device)
+    buf = torch.zeros(A.n + 1, dtype=torch.float64, device=cuda_device)
+    buf[1:].copy_(torch.from_numpy(x))
+    y_mis = M.run(buf[1:]).cpu().numpy()
+    y_al = M.run(torch.from_numpy(x).to(cuda_device)).cpu().numpy()
+    assert np.array_equal(y_mis.view(np.uint64), y_al.view(np.uint64))
