@@ -296,18 +296,21 @@ def measure_workload(workload, mode, steps, warmup, dev, rank, P, group, cpu_sec
     if P > 1:
         dist.barrier(group=group)
     torch.cuda.synchronize(dev)
-    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
-          for _ in range(steps)]
+    # N = 1: a step is exactly one kernel launch; the K launches go back to back
+    # (programmatic dependent launch overlaps one kernel's prologue with the
+    # previous one's tail) between two events, so the kernel's average launch
+    # duration is the timed region / K.  N > 1: per-launch events bracket each
+    # SpMV kernel so its duration is separated from the all-gather.
     kev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
-           for _ in range(steps)]
+           for _ in range(steps if P > 1 else 0)]
     start, end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     sampler = ClockSampler(dev.index if dev.index is not None else 0)
     with sampler:
         start.record(stream)
         for i in range(steps):
             j = i % reps
-            kev[i][0].record(stream)
             if P > 1:
+                kev[i][0].record(stream)
                 y = gathered[rank * maxrows: rank * maxrows + rows_local]
                 mats[j].run(xs[j], y)
                 kev[i][1].record(stream)
@@ -315,14 +318,14 @@ def measure_workload(workload, mode, steps, warmup, dev, rank, P, group, cpu_sec
                                             group=group)
             else:
                 mats[j].run(xs[j], ys[j])
-                kev[i][1].record(stream)
         end.record(stream)
         torch.cuda.synchronize(dev)
     if P > 1:
         dist.barrier(group=group)
     torch.cuda.synchronize(dev)
     total_ms = start.elapsed_time(end)
-    kern_ms = np.array([a.elapsed_time(b) for a, b in kev])
+    kern_ms = (np.array([a.elapsed_time(b) for a, b in kev]) if P > 1
+               else np.array([total_ms / steps]))
     if P > 1:
         t_ = torch.tensor([total_ms, float(np.mean(kern_ms))], dtype=torch.float64, device=dev)
         dist.all_reduce(t_, op=dist.ReduceOp.MAX, group=group)

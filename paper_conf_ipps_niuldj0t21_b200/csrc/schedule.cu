@@ -471,8 +471,17 @@ int launch_spmv(const Matrix &M, const double *d_x, double *d_y, cudaStream_t st
     p.cta_begin = M.cta_begin;
     p.x_vec = (reinterpret_cast<uintptr_t>(d_x) & 15u) == 0;
     const KernelChoice kc = choose(M.kernel_version);
-    kc.fn<<<M.grid, M.block, M.smem, st>>>(p);
-    TSP_CK(cudaGetLastError());
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(M.grid);
+    cfg.blockDim = dim3(M.block);
+    cfg.dynamicSmemBytes = M.smem;
+    cfg.stream = st;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = kc.pdl ? 1 : 0;
+    TSP_CK(cudaLaunchKernelEx(&cfg, kc.fn, p));
     return 0;
 }
 

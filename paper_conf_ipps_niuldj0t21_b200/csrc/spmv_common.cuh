@@ -185,6 +185,12 @@ __device__ __forceinline__ void cp_async_wait_all() {
     asm volatile("cp.async.commit_group;\n\tcp.async.wait_group 0;" ::: "memory");
 }
 __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+// Programmatic dependent launch: let the next kernel in the stream start its
+// prologue early / wait until the previous kernel's writes are visible
+__device__ __forceinline__ void griddep_launch_dependents() {
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+}
+__device__ __forceinline__ void griddep_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
 // acc += a * b only where pred holds (one predicated DFMA, no select)
 __device__ __forceinline__ void fma_if(bool pred, double a, double b, double &acc) {
     asm("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %3, 0;\n\t@q fma.rn.f64 %0, %1, %2, %0;\n\t}"
@@ -228,6 +234,7 @@ struct KernelChoice {
     int threads, smem, ctas_per_sm;
     bool ring;       // one CTA per SM with cta_begin chunks (no current kernel)
     int slot_bytes;  // item budget the schedule must respect
+    bool pdl;        // launched with programmatic dependent launch (kernel waits on griddepcontrol)
 };
 KernelChoice kernel_v1();
 KernelChoice kernel_warp(int variant);

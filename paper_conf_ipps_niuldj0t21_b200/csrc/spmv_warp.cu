@@ -160,6 +160,9 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, MINB) tilespmv
         fence_mbar_init();
     }
     __syncwarp();
+    // PDL: the next SpMV in the stream may start its prologue now; it waits
+    // (griddep_wait) before touching x or y, and so do we
+    griddep_launch_dependents();
     const uint32_t n32 = (uint32_t)p.n;
     // contiguous, cost-balanced, row-aligned item chunk per warp (schedule.cu);
     // neighbouring tile rows share x segments.  The warp's start record holds
@@ -185,6 +188,8 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, MINB) tilespmv
         }
         const int nt = (it.part_nt >> 24) & 31;
         const uint32_t pay = slot + (it.jt_rows_pay >> 16);
+        // the matrix is immutable; x and y may belong to the previous kernel
+        if (k == kbeg) griddep_wait();
         // 1. x segments, issued before the blob lands (J came with the record)
         if (p.x_vec) {  // lane l: tile 4k + (l >> 3), 16 bytes at elements 2(l & 7)
             const uint32_t qq = lane & 7;
@@ -286,7 +291,7 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, MINB) tilespmv
 template <int WARPS, int SLOT, int MINB>
 KernelChoice warp_choice(const char *name) {
     using Cfg = WarpCfg<WARPS, SLOT>;
-    return {name, tilespmv_fp64_warp<WARPS, SLOT, MINB>, Cfg::kThreads, (int)Cfg::kSmem, 0, false, SLOT};
+    return {name, tilespmv_fp64_warp<WARPS, SLOT, MINB>, Cfg::kThreads, (int)Cfg::kSmem, 0, false, SLOT, true};
 }
 
 }  // namespace
