@@ -190,7 +190,18 @@ __global__ void k_blob_fill(Item *items, int64_t n, int64_t m, const int64_t *st
     for (uint32_t o = 4 * lane; o < b.total; o += 128) *reinterpret_cast<uint32_t *>(dst + o) = 0u;  // padding
     __syncwarp();
     uint2 *dd = reinterpret_cast<uint2 *>(dst);
-    for (int i = lane; i < it.ndsc; i += 32) dd[i] = dlist[it.dbeg + i];
+    // kernel-native descriptors: x = distance from the descriptor itself to
+    // the tile's payload (CSR: to its csrRowPtr, after the 8*nnz value bytes),
+    // y = aux | t*128 | nnz << 11 | invalid << 31
+    for (int i = lane; i < it.ndsc; i += 32) {
+        const uint2 d = dlist[it.dbeg + i];
+        const uint32_t off = d.x & 0x1FFFFFu, t = (d.x >> 21) & 0xFFu, f = d.x >> 29;
+        const uint32_t nz = (d.y >> 8) & 0x1FFu;
+        uint2 e;
+        e.x = b.pay + off + (f == F_CSR ? 8u * nz : 0u) - 8u * (uint32_t)i;
+        e.y = (d.y & 0x1Fu) | (t << 7) | (nz << 11) | (d.y & 0x80000000u);
+        dd[i] = e;
+    }
     const int nt = item_nt(it);
     if (lane < 16) jcols[k * 16 + lane] = lane < nt ? tileColIdx[it.tb + lane] : 0;
     const uint4 *ps = reinterpret_cast<const uint4 *>(payload + (size_t)it.offb * 16);
@@ -380,10 +391,11 @@ int build_tdesc(Matrix &M, cudaStream_t st) {
 
 int choose_kernel(Matrix &M) {
     // default: the warp kernel with 4.5 KB slots (32 warps/SM); matrices whose
-    // tile rows average more than 6 KB of payload (dense, FEM-like) use 10.5 KB
-    // slots (16 warps/SM) so a tile row stays one item
+    // tile rows average more than 6 KB of payload (dense, FEM-like) use the
+    // double-buffered kernel with two 5.9 KB slots per warp (16 warps/SM), so
+    // a warp streams the next piece of its tile row while it computes one
     const double row_bytes = M.tilem ? (double)M.payload_bytes / (double)M.tilem : 0.0;
-    int version = row_bytes > 6144.0 ? 25 : 20;
+    int version = row_bytes > 6144.0 ? 30 : 20;
     if (const char *e = getenv("TILESPMV_KERNEL")) version = atoi(e);
     M.kernel_version = version;
     M.item_bytes = choose(version).slot_bytes;

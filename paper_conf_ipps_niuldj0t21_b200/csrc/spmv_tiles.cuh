@@ -29,6 +29,26 @@ __device__ __forceinline__ uint2 lds_v2u32(uint32_t a) {
     asm volatile("ld.shared.v2.u32 {%0, %1}, [%2];" : "=r"(v.x), "=r"(v.y) : "r"(a));
     return v;
 }
+__device__ __forceinline__ uint32_t lds_u32(uint32_t a) {
+    uint32_t v;
+    asm("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(a));
+    return v;
+}
+// v = (i < len) ? [a] : 0.0 -- a predicated load instead of a masked FMA:
+// 0.0 * x adds nothing to the row sum because x is finite (reading R19)
+__device__ __forceinline__ double lds_f64_lt(int i, int len, uint32_t a) {
+    double v;
+    asm("{\n\t.reg .pred q;\n\tsetp.lt.s32 q, %1, %2;\n\tmov.b64 %0, 0;\n\t@q ld.shared.f64 %0, [%3];\n\t}"
+        : "=d"(v)
+        : "r"(i), "r"(len), "r"(a));
+    return v;
+}
+// shared address of x[col] in a tile's 128-byte aligned x segment X, from a
+// column nibble already shifted to bits 3..6 (w's other bits are masked off)
+__device__ __forceinline__ uint32_t xaddr(uint32_t w8, uint32_t X) { return (w8 & 0x78u) | X; }
+__device__ __forceinline__ uint32_t funnel_r(uint32_t lo, uint32_t hi, uint32_t sh) {
+    return __funnelshift_r(lo, hi, sh);
+}
 __device__ __forceinline__ void sts_u32(uint32_t a, uint32_t v) {
     asm volatile("st.shared.u32 [%0], %1;" ::"r"(a), "r"(v) : "memory");
 }
@@ -37,73 +57,67 @@ __device__ __forceinline__ void sts_f64(uint32_t a, double v) {
 }
 
 // --------------------------------------------- half-warp tile routines -----
-// Lane r of a half owns row r of its tile.  P: shared address of the tile's
-// payload, X: of its 16 x values; ok: the half has a tile (else it runs the
+// Lane r of a half owns row r of its tile.  X: shared address of the tile's
+// 16 x values (128-byte aligned); ok: the half has a tile (else it runs the
 // other half's tile with its FMAs masked).  Loads past a tile's end stay
-// inside the CTA's shared memory and are masked out of the FMA.
+// inside the CTA's shared memory and are masked out of the sum; x addresses
+// always stay inside the tile's x segment.
 
-// CSR: csrVal row-major | csrRowPtr[16] u8 | 4-bit columns (Alg. 2)
-__device__ __forceinline__ void half_csr(uint32_t P, int nz, uint32_t X, int r, bool ok, double &acc) {
-    const uint32_t rp = P + 8 * nz;
-    const int beg = (int)lds_u8(rp + r);
-    const int end = r < 15 ? (int)lds_u8(rp + r + 1) : nz;
+// CSR: csrVal row-major | csrRowPtr[16] u8 | 4-bit columns (Alg. 2).
+// RP: shared address of csrRowPtr.  The 8 column nibbles from entry beg on
+// come from two 32-bit words and one funnel shift.
+__device__ __forceinline__ void half_csr(uint32_t RP, int nz, uint32_t X, int r, bool ok, double &acc) {
+    const int beg = (int)lds_u8(RP + r);
+    const int end = r < 15 ? (int)lds_u8(RP + r + 1) : nz;
     const int len = ok ? end - beg : 0;
     const int trips = (int)__reduce_max_sync(FULL, (unsigned)len);
-    // nibble of entry beg+i: byte (beg+i)>>1 = b_even + i/2 (i even) or
-    // b_odd + i/2 (i odd), shifted by s_even / s_odd
-    const uint32_t cb = rp + 16 + (beg >> 1);
-    const uint32_t odd = beg & 1;
-    const uint32_t b_odd = cb + odd;
-    const uint32_t s_even = 4 * odd, s_odd = 4 - 4 * odd;
-    const uint32_t V = P + 8 * beg;
-    // four entries per step (independent load chains, two FMA chains); the
-    // first step is straight-line, longer rows (trips > 4) loop
-    double a1 = 0.0;
+    const uint32_t V = RP + 8 * (beg - nz);
     {
-        const uint32_t c0 = (lds_u8(cb) >> s_even) & 15u;
-        const uint32_t c1 = (lds_u8(b_odd) >> s_odd) & 15u;
-        const uint32_t c2 = (lds_u8(cb + 1) >> s_even) & 15u;
-        const uint32_t c3 = (lds_u8(b_odd + 1) >> s_odd) & 15u;
-        const double v0 = lds_f64(V), v1 = lds_f64(V + 8), v2 = lds_f64(V + 16), v3 = lds_f64(V + 24);
-        const double x0 = lds_f64(X + 8 * c0), x1 = lds_f64(X + 8 * c1);
-        const double x2 = lds_f64(X + 8 * c2), x3 = lds_f64(X + 8 * c3);
-        fma_if(0 < len, v0, x0, acc);
-        fma_if(1 < len, v1, x1, a1);
-        fma_if(2 < len, v2, x2, acc);
-        fma_if(3 < len, v3, x3, a1);
+        const uint32_t wa = RP + 16 + 4 * (beg >> 3);
+        const uint32_t u = funnel_r(lds_u32(wa), lds_u32(wa + 4), 4u * beg);
+        const double x0 = lds_f64(xaddr(u << 3, X)), x1 = lds_f64(xaddr(u >> 1, X));
+        const double x2 = lds_f64(xaddr(u >> 5, X)), x3 = lds_f64(xaddr(u >> 9, X));
+        const double v0 = lds_f64_lt(0, len, V), v1 = lds_f64_lt(1, len, V + 8);
+        const double v2 = lds_f64_lt(2, len, V + 16), v3 = lds_f64_lt(3, len, V + 24);
+        acc = fma(v0, x0, acc);
+        acc = fma(v1, x1, acc);
+        acc = fma(v2, x2, acc);
+        acc = fma(v3, x3, acc);
     }
 #pragma unroll 1
     for (int i = 4; i < trips; i += 4) {
-        const uint32_t c0 = (lds_u8(cb + (i >> 1)) >> s_even) & 15u;
-        const uint32_t c1 = (lds_u8(b_odd + (i >> 1)) >> s_odd) & 15u;
-        const uint32_t c2 = (lds_u8(cb + (i >> 1) + 1) >> s_even) & 15u;
-        const uint32_t c3 = (lds_u8(b_odd + (i >> 1) + 1) >> s_odd) & 15u;
-        const double v0 = lds_f64(V + 8 * i), v1 = lds_f64(V + 8 * i + 8);
-        const double v2 = lds_f64(V + 8 * i + 16), v3 = lds_f64(V + 8 * i + 24);
-        const double x0 = lds_f64(X + 8 * c0), x1 = lds_f64(X + 8 * c1);
-        const double x2 = lds_f64(X + 8 * c2), x3 = lds_f64(X + 8 * c3);
-        fma_if(i < len, v0, x0, acc);
-        fma_if(i + 1 < len, v1, x1, a1);
-        fma_if(i + 2 < len, v2, x2, acc);
-        fma_if(i + 3 < len, v3, x3, a1);
+        const uint32_t wa = RP + 16 + 4 * ((beg + i) >> 3);
+        const uint32_t u = funnel_r(lds_u32(wa), lds_u32(wa + 4), 4u * (beg + i));
+        const double x0 = lds_f64(xaddr(u << 3, X)), x1 = lds_f64(xaddr(u >> 1, X));
+        const double x2 = lds_f64(xaddr(u >> 5, X)), x3 = lds_f64(xaddr(u >> 9, X));
+        const double v0 = lds_f64_lt(i, len, V + 8 * i), v1 = lds_f64_lt(i + 1, len, V + 8 * i + 8);
+        const double v2 = lds_f64_lt(i + 2, len, V + 8 * i + 16), v3 = lds_f64_lt(i + 3, len, V + 8 * i + 24);
+        acc = fma(v0, x0, acc);
+        acc = fma(v1, x1, acc);
+        acc = fma(v2, x2, acc);
+        acc = fma(v3, x3, acc);
     }
-    acc += a1;
 }
 
 // ELL: slots k*16 + r column-major | 4-bit columns (Alg. 4).
-// Pads (k >= 1 with column 0, reading R26) are skipped.
+// Pads hold +0.0 at column 0 (reading R10) and are multiplied like entries:
+// +0.0 * x adds nothing (x finite, R19).
 __device__ __forceinline__ void half_ell(uint32_t P, int w, uint32_t X, int r, bool ok, double &acc) {
     const int wq = ok ? w : 0;
     const int trips = (int)__reduce_max_sync(FULL, (unsigned)wq);
     const uint32_t ci = P + 128 * w + (r >> 1);
     const uint32_t sh = 4 * (r & 1);
     const uint32_t V = P + 8 * r;
-#pragma unroll 4
-    for (int k = 0; k < trips; ++k) {
-        const uint32_t c = (lds_u8(ci + 8 * k) >> sh) & 15u;
-        const double v = lds_f64(V + 128 * k);
-        const double xv = lds_f64(X + 8 * c);
-        fma_if(k < wq && (k == 0 || c != 0), v, xv, acc);
+#pragma unroll 1
+    for (int k = 0; k < trips; k += 4) {
+        double xv[4], v[4];
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+            xv[j] = lds_f64(X + 8 * ((lds_u8(ci + 8 * (k + j)) >> sh) & 15u));
+            v[j] = lds_f64_lt(k + j, wq, V + 128 * (k + j));
+        }
+#pragma unroll
+        for (int j = 0; j < 4; ++j) acc = fma(v[j], xv[j], acc);
     }
 }
 
@@ -125,9 +139,9 @@ __device__ __forceinline__ void half_dnscol(uint32_t P, int nc, uint32_t X, int 
     const int trips = (int)__reduce_max_sync(FULL, (unsigned)nq);
     const uint32_t cid = P + 128 * nc;
     for (int q = 0; q < trips; ++q) {
-        const double v = lds_f64(P + 8 * (16 * q + r));
+        const double v = lds_f64_lt(q, nq, P + 8 * (16 * q + r));
         const double xv = lds_f64(X + 8 * (lds_u8(cid + q) & 15u));
-        fma_if(q < nq, v, xv, acc);
+        acc = fma(v, xv, acc);
     }
 }
 
@@ -174,33 +188,11 @@ __device__ __forceinline__ void half_hyb(uint32_t P, int w, int nz, uint32_t X, 
     const int trips = (int)__reduce_max_sync(FULL, (unsigned)wq);
     const uint32_t sh = 4 * (r & 1);
     for (int k = 0; k < trips; ++k) {
-        const double v = lds_f64(P + 8 * (16 * k + r));
+        const double v = lds_f64_lt(k, wq, P + 8 * (16 * k + r));
         const double xv = lds_f64(X + 8 * ((lds_u8(ei + 8 * k + (r >> 1)) >> sh) & 15u));
-        fma_if(k < wq, v, xv, acc);
+        acc = fma(v, xv, acc);
     }
     half_coo(P + 128 * w, ei + 8 * w, kc, X, r, ok, acc);
-}
-
-// dispatch one descriptor-list entry pair (see k_dsc_write): half h runs entry 2q + h
-__device__ __forceinline__ void run_pair(uint2 e, uint32_t pay, uint32_t xs, int r, double &acc) {
-    const int f = (int)(e.x >> 29);  // same for both halves by construction
-    const bool ok = (int)e.y >= 0;
-    const uint32_t P = pay + (e.x & 0x3FFFu);
-    const uint32_t X = xs + ((e.x >> 14) & 0x7FFu);
-    switch (f) {
-    case F_CSR: half_csr(P, (int)(e.y >> 8) & 511, X, r, ok, acc); break;
-    case F_ELL: half_ell(P, (int)(e.y & 31u), X, r, ok, acc); break;
-    case F_DNS: half_dns(P, X, r, ok, acc); break;
-    case F_DNSCOL: half_dnscol(P, (int)(e.y & 31u), X, r, ok, acc); break;
-    case F_DNSROW: half_dnsrow(P, (int)(e.y & 31u), X, r, ok, acc); break;
-    case F_COO: {
-        const int nz = (int)(e.y >> 8) & 511;
-        half_coo(P, P + 8 * nz, nz, X, r, ok, acc);
-        break;
-    }
-    case F_HYB: half_hyb(P, (int)(e.y & 31u), (int)(e.y >> 8) & 511, X, r, ok, acc); break;
-    default: break;
-    }
 }
 
 }  // namespace tsp

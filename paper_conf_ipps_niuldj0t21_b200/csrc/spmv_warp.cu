@@ -21,12 +21,14 @@
 namespace tsp {
 namespace {
 
-template <int WARPS, int SLOT>
+template <int WARPS, int SLOT, int NBUF = 1>
 struct WarpCfg {
     static_assert(SLOT % 16 == 0 && SLOT <= kItemBytesMax, "slot size");
+    // [x stage of every warp, 2 KB each, 128-byte aligned] [per warp: NBUF
+    // slots | row sums | mbarriers]
     static constexpr uint32_t kX = kItemTiles * 16 * 8;
-    static constexpr uint32_t kPer = SLOT + kX + 128 + 16;  // slot | x | row sums | mbarrier
-    static constexpr uint32_t kSmem = WARPS * kPer + 256;   // +256: loads may overrun a slot
+    static constexpr uint32_t kPer = NBUF * SLOT + 128 + 16;
+    static constexpr uint32_t kSmem = WARPS * (kX + kPer) + 256;  // +256: loads may overrun a slot
     static constexpr int kThreads = 32 * WARPS;
 };
 
@@ -124,37 +126,148 @@ __device__ __forceinline__ void remainder(const Params &p, uint32_t rpS, uint32_
     if (lane < 16) acc += lds_f64(racc + 8 * lane);
 }
 
-// the tiles of one format group, two per step (half-warp each)
+// the tiles of one format group, two per step.  d: shared address of this
+// half's descriptor (see k_blob_fill): x = distance from the descriptor to the
+// tile's payload (CSR: to its csrRowPtr), y = aux | t*128 | nz << 11 | invalid << 31
 template <int F>
-__device__ __forceinline__ void run_group(int np, uint32_t &q, uint32_t dsc, uint32_t pay, uint32_t xs, int r, int h,
-                                          double &acc) {
+__device__ __forceinline__ void run_group(int np, uint32_t &d, uint32_t xs, int r, double &acc) {
 #pragma unroll 1
-    for (int i = 0; i < np; ++i, ++q) {
-        const uint2 e = lds_v2u32(dsc + 16 * q + 8 * h);
+    for (int i = 0; i < np; ++i, d += 16) {
+        const uint2 e = lds_v2u32(d);
         const bool ok = (int)e.y >= 0;
-        const uint32_t P = pay + (e.x & 0x3FFFu);
-        const uint32_t X = xs + ((e.x >> 14) & 0x7FFu);
-        if (F == F_CSR) half_csr(P, (int)(e.y >> 8) & 511, X, r, ok, acc);
-        if (F == F_ELL) half_ell(P, (int)(e.y & 31u), X, r, ok, acc);
+        const uint32_t P = d + e.x;
+        const uint32_t X = xs + (e.y & 0x780u);
+        const int aux = (int)(e.y & 31u), nz = (int)(e.y >> 11) & 511;
+        if (F == F_CSR) half_csr(P, nz, X, r, ok, acc);
+        if (F == F_ELL) half_ell(P, aux, X, r, ok, acc);
         if (F == F_DNS) half_dns(P, X, r, ok, acc);
-        if (F == F_DNSCOL) half_dnscol(P, (int)(e.y & 31u), X, r, ok, acc);
-        if (F == F_DNSROW) half_dnsrow(P, (int)(e.y & 31u), X, r, ok, acc);
-        if (F == F_COO) {
-            const int nz = (int)(e.y >> 8) & 511;
-            half_coo(P, P + 8 * nz, nz, X, r, ok, acc);
-        }
-        if (F == F_HYB) half_hyb(P, (int)(e.y & 31u), (int)(e.y >> 8) & 511, X, r, ok, acc);
+        if (F == F_DNSCOL) half_dnscol(P, aux, X, r, ok, acc);
+        if (F == F_DNSROW) half_dnsrow(P, aux, X, r, ok, acc);
+        if (F == F_COO) half_coo(P, P + 8 * nz, nz, X, r, ok, acc);
+        if (F == F_HYB) half_hyb(P, aux, nz, X, r, ok, acc);
     }
 }
 
+// lane 0: the whole item (descriptors, payload, remainder) in ONE TMA bulk copy
+__device__ __forceinline__ void issue_blob(const Params &p, const WItem &it, uint32_t slot, uint32_t bar,
+                                           uint64_t policy, int lane) {
+    const uint32_t total = it.val_tot >> 16;
+    if (lane == 0 && total) {
+        fence_proxy_async();
+        mbar_expect_tx(bar, total);
+        bulk_g2s_hint(slot, p.blob + (size_t)it.blob16 * 16, total, bar, policy);
+    }
+}
+
+// the x segment of every tile of the item (J: tile column of tile `lane`),
+// issued before the blob lands
+__device__ __forceinline__ void issue_x(const Params &p, int J, int nt, uint32_t xs, uint64_t x_policy, int lane) {
+    const uint32_t n32 = (uint32_t)p.n;
+    if (p.x_vec) {  // lane l: tile 4k + (l >> 3), 16 bytes at elements 2(l & 7)
+        const uint32_t qq = lane & 7;
+#pragma unroll
+        for (int kk = 0; kk < kItemTiles / 4; ++kk) {
+            const int t = 4 * kk + (lane >> 3);
+            const uint32_t c0 = 16u * (uint32_t)__shfl_sync(FULL, J, t) + 2u * qq;
+            if (t < nt) {
+                if (c0 + 2 <= n32) {
+                    cp_async16(xs + 128 * t + 16 * qq, p.x + c0, 16u, x_policy);
+                } else {  // the tail of x: never read past x[n-1]
+                    const double v0 = c0 < n32 ? ldg_hint(p.x + c0, x_policy) : 0.0;
+                    sts_v2f64(xs + 128 * t + 16 * qq, make_double2(v0, 0.0));
+                }
+            }
+        }
+        cp_async_commit();
+    } else {  // lane l: tile 2k + h, element r
+        const int h = lane >> 4, r = lane & 15;
+#pragma unroll
+        for (int kk = 0; kk < kItemTiles / 2; ++kk) {
+            const int t = 2 * kk + h;
+            const uint32_t col = 16u * (uint32_t)__shfl_sync(FULL, J, t) + (uint32_t)r;
+            if (t < nt) sts_f64(xs + 8 * (16 * t + r), col < n32 ? ldg_hint(p.x + col, x_policy) : 0.0);
+        }
+    }
+}
+
+// steps 2-4 of an item whose blob is in `slot` and whose x segments are in
+// flight into `xs`: remainder, tiles, y (or the split-row carry)
+__device__ __forceinline__ void compute_item(const Params &p, const WItem &it, uint32_t slot, uint32_t xs,
+                                             uint32_t racc, uint64_t x_policy, int lane, double &carry) {
+    const int h = lane >> 4, r = lane & 15;
+    const uint32_t total = it.val_tot >> 16;
+    // 2. fused CSR remainder
+    double acc = 0.0;
+    const uint32_t rp = it.rp_col & 0xFFFFu;
+    if (total > rp)
+        remainder(p, slot + rp, slot + (it.rp_col >> 16), slot + (it.val_tot & 0xFFFFu),
+                  (int)((it.jt_rows_pay >> 8) & 31u), racc, x_policy, lane, acc);
+    if (p.x_vec) cp_async_wait_all();
+    __syncwarp();
+    // 3. tiles: format group by format group, two tiles per step
+    {
+        const uint32_t g = it.groups;
+        uint32_t d = slot + 8 * h;
+        run_group<F_CSR>((int)(g & 15u), d, xs, r, acc);
+        run_group<F_COO>((int)((g >> 4) & 15u), d, xs, r, acc);
+        run_group<F_ELL>((int)((g >> 8) & 15u), d, xs, r, acc);
+        run_group<F_HYB>((int)((g >> 12) & 15u), d, xs, r, acc);
+        run_group<F_DNS>((int)((g >> 16) & 15u), d, xs, r, acc);
+        run_group<F_DNSROW>((int)((g >> 20) & 15u), d, xs, r, acc);
+        run_group<F_DNSCOL>((int)((g >> 24) & 15u), d, xs, r, acc);
+    }
+    acc += __shfl_xor_sync(FULL, acc, 16);
+    // 4. y, once per row
+    const int64_t row = 16 * (int64_t)it.I + lane;
+    if (it.split < 0) {
+        if (lane < 16 && row < p.m) p.y[row] = acc;
+    } else if (!((it.part_nt >> 30) & 1)) {  // a group of parts runs here, in part order
+        carry += acc;
+    } else {
+        const double sum = carry + acc;
+        carry = 0.0;
+        if ((it.part_nt >> 29) & 1) {  // the row's only group
+            if (lane < 16 && row < p.m) p.y[row] = sum;
+        } else {  // hub row: one partial per group, the last group sums them in order
+            const int2 si = p.split_info[it.split];
+            const int ngroups = (si.y + kLocalParts - 1) / kLocalParts;
+            const int gidx = (it.part_nt & 0xFFFFFF) / kLocalParts;
+            if (lane < 16) __stcg(p.partials + (int64_t)(si.x + gidx) * 16 + lane, sum);
+            __threadfence();
+            __syncwarp();
+            int old = 0;
+            if (lane == 0) old = atomicAdd(p.counters + it.split, 1);
+            old = __shfl_sync(FULL, old, 0);
+            if (old == ngroups - 1) {  // half h sums groups h, h+2, ... in order, 4 loads in flight
+                __threadfence();
+                double s = 0.0;
+                for (int q0 = h; q0 < ngroups; q0 += 8) {
+                    double v[4];
+#pragma unroll
+                    for (int i = 0; i < 4; ++i) {
+                        const int qg = q0 + 2 * i;
+                        v[i] = qg < ngroups ? __ldcg(p.partials + (int64_t)(si.x + qg) * 16 + r) : 0.0;
+                    }
+#pragma unroll
+                    for (int i = 0; i < 4; ++i) s += v[i];
+                }
+                s += __shfl_xor_sync(FULL, s, 16);
+                if (lane < 16 && row < p.m) p.y[row] = s;
+                if (lane == 0) p.counters[it.split] = 0;  // ready for the next run
+            }
+        }
+    }
+}
+
+// one blob in flight per warp: latency hidden by warp count (32 warps/SM)
 template <int WARPS, int SLOT, int MINB>
 __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, MINB) tilespmv_fp64_warp(const Params p) {
     using Cfg = WarpCfg<WARPS, SLOT>;
     extern __shared__ __align__(128) uint8_t smem[];
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    const int h = lane >> 4, r = lane & 15;
-    const uint32_t base = smem_u32(smem) + (uint32_t)warp * Cfg::kPer;
-    const uint32_t slot = base, xs = base + SLOT, racc = xs + Cfg::kX, bar = racc + 128;
+    const uint32_t xs = smem_u32(smem) + (uint32_t)warp * Cfg::kX;
+    const uint32_t slot = smem_u32(smem) + WARPS * Cfg::kX + (uint32_t)warp * Cfg::kPer;
+    const uint32_t racc = slot + SLOT, bar = racc + 128;
     if (lane == 0) {
         mbar_init(bar, 1);
         fence_mbar_init();
@@ -163,7 +276,6 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, MINB) tilespmv
     // PDL: the next SpMV in the stream may start its prologue now; it waits
     // (griddep_wait) before touching x or y, and so do we
     griddep_launch_dependents();
-    const uint32_t n32 = (uint32_t)p.n;
     // contiguous, cost-balanced, row-aligned item chunk per warp (schedule.cu);
     // neighbouring tile rows share x segments.  The warp's start record holds
     // the chunk and a copy of the first item (one round trip).
@@ -179,112 +291,81 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, MINB) tilespmv
     for (int k = kbeg; k < kend; ++k) {
         const WItem it = nxt;
         const int J = Jn;
-        const uint32_t total = it.val_tot >> 16;
-        // the whole item (descriptors, payload, remainder) in ONE TMA bulk copy
-        if (lane == 0 && total) {
-            fence_proxy_async();
-            mbar_expect_tx(bar, total);
-            bulk_g2s_hint(slot, p.blob + (size_t)it.blob16 * 16, total, bar, stream_policy);
-        }
-        const int nt = (it.part_nt >> 24) & 31;
-        const uint32_t pay = slot + (it.jt_rows_pay >> 16);
+        issue_blob(p, it, slot, bar, stream_policy, lane);
         // the matrix is immutable; x and y may belong to the previous kernel
         if (k == kbeg) griddep_wait();
         // 1. x segments, issued before the blob lands (J came with the record)
-        if (p.x_vec) {  // lane l: tile 4k + (l >> 3), 16 bytes at elements 2(l & 7)
-            const uint32_t qq = lane & 7;
-#pragma unroll
-            for (int kk = 0; kk < kItemTiles / 4; ++kk) {
-                const int t = 4 * kk + (lane >> 3);
-                const uint32_t c0 = 16u * (uint32_t)__shfl_sync(FULL, J, t) + 2u * qq;
-                if (t < nt) {
-                    if (c0 + 2 <= n32) {
-                        cp_async16(xs + 128 * t + 16 * qq, p.x + c0, 16u, x_policy);
-                    } else {  // the tail of x: never read past x[n-1]
-                        const double v0 = c0 < n32 ? ldg_hint(p.x + c0, x_policy) : 0.0;
-                        sts_v2f64(xs + 128 * t + 16 * qq, make_double2(v0, 0.0));
-                    }
-                }
-            }
-            cp_async_commit();
-        } else {  // lane l: tile 2k + h, element r
-#pragma unroll
-            for (int kk = 0; kk < kItemTiles / 2; ++kk) {
-                const int t = 2 * kk + h;
-                const uint32_t col = 16u * (uint32_t)__shfl_sync(FULL, J, t) + (uint32_t)r;
-                if (t < nt) sts_f64(xs + 8 * (16 * t + r), col < n32 ? ldg_hint(p.x + col, x_policy) : 0.0);
-            }
-        }
+        issue_x(p, J, (it.part_nt >> 24) & 31, xs, x_policy, lane);
         if (k + 1 < kend) {  // the next record and its columns, in flight during this item
             nxt = load_witem(p.witems, k + 1);
             Jn = lane < 16 ? __ldg(p.jcols + (int64_t)(k + 1) * 16 + lane) : 0;
         }
-        if (total) {
+        if (it.val_tot >> 16) {
             mbar_wait(bar, phase);
             phase ^= 1u;
         }
-        // 2. fused CSR remainder
-        double acc = 0.0;
-        const uint32_t rp = it.rp_col & 0xFFFFu;
-        if (total > rp)
-            remainder(p, slot + rp, slot + (it.rp_col >> 16), slot + (it.val_tot & 0xFFFFu),
-                      (int)((it.jt_rows_pay >> 8) & 31u), racc, x_policy, lane, acc);
-        if (p.x_vec) cp_async_wait_all();
-        __syncwarp();
-        // 3. tiles: format group by format group, two tiles per step
-        {
-            const uint32_t g = it.groups;
-            uint32_t q = 0;
-            run_group<F_CSR>((int)(g & 15u), q, slot, pay, xs, r, h, acc);
-            run_group<F_COO>((int)((g >> 4) & 15u), q, slot, pay, xs, r, h, acc);
-            run_group<F_ELL>((int)((g >> 8) & 15u), q, slot, pay, xs, r, h, acc);
-            run_group<F_HYB>((int)((g >> 12) & 15u), q, slot, pay, xs, r, h, acc);
-            run_group<F_DNS>((int)((g >> 16) & 15u), q, slot, pay, xs, r, h, acc);
-            run_group<F_DNSROW>((int)((g >> 20) & 15u), q, slot, pay, xs, r, h, acc);
-            run_group<F_DNSCOL>((int)((g >> 24) & 15u), q, slot, pay, xs, r, h, acc);
-        }
-        acc += __shfl_xor_sync(FULL, acc, 16);
-        // 4. y, once per row
-        const int64_t row = 16 * (int64_t)it.I + lane;
-        if (it.split < 0) {
-            if (lane < 16 && row < p.m) p.y[row] = acc;
-        } else if (!((it.part_nt >> 30) & 1)) {  // a group of parts runs here, in part order
-            carry += acc;
-        } else {
-            const double sum = carry + acc;
-            carry = 0.0;
-            if ((it.part_nt >> 29) & 1) {  // the row's only group
-                if (lane < 16 && row < p.m) p.y[row] = sum;
-            } else {  // hub row: one partial per group, the last group sums them in order
-                const int2 si = p.split_info[it.split];
-                const int ngroups = (si.y + kLocalParts - 1) / kLocalParts;
-                const int gidx = (it.part_nt & 0xFFFFFF) / kLocalParts;
-                if (lane < 16) __stcg(p.partials + (int64_t)(si.x + gidx) * 16 + lane, sum);
-                __threadfence();
-                __syncwarp();
-                int old = 0;
-                if (lane == 0) old = atomicAdd(p.counters + it.split, 1);
-                old = __shfl_sync(FULL, old, 0);
-                if (old == ngroups - 1) {  // half h sums groups h, h+2, ... in order, 4 loads in flight
-                    __threadfence();
-                    double s = 0.0;
-                    for (int q0 = h; q0 < ngroups; q0 += 8) {
-                        double v[4];
-#pragma unroll
-                        for (int i = 0; i < 4; ++i) {
-                            const int qg = q0 + 2 * i;
-                            v[i] = qg < ngroups ? __ldcg(p.partials + (int64_t)(si.x + qg) * 16 + r) : 0.0;
-                        }
-#pragma unroll
-                        for (int i = 0; i < 4; ++i) s += v[i];
-                    }
-                    s += __shfl_xor_sync(FULL, s, 16);
-                    if (lane < 16 && row < p.m) p.y[row] = s;
-                    if (lane == 0) p.counters[it.split] = 0;  // ready for the next run
-                }
+        compute_item(p, it, slot, xs, racc, x_policy, lane, carry);
+        __syncwarp();  // slot and x scratch free for the next item
+    }
+}
+
+// two blobs in flight per warp: item k+1 streams in while item k computes
+// (dense tile rows, where few large slots fit per SM)
+template <int WARPS, int SLOT, int MINB>
+__global__ void __launch_bounds__(WarpCfg<WARPS, SLOT, 2>::kThreads, MINB) tilespmv_fp64_warp2(const Params p) {
+    using Cfg = WarpCfg<WARPS, SLOT, 2>;
+    extern __shared__ __align__(128) uint8_t smem[];
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const uint32_t xs = smem_u32(smem) + (uint32_t)warp * Cfg::kX;
+    const uint32_t base = smem_u32(smem) + WARPS * Cfg::kX + (uint32_t)warp * Cfg::kPer;
+    const uint32_t racc = base + 2 * SLOT, bar0 = racc + 128;
+    if (lane == 0) {
+        mbar_init(bar0, 1);
+        mbar_init(bar0 + 8, 1);
+        fence_mbar_init();
+    }
+    __syncwarp();
+    griddep_launch_dependents();
+    const int64_t gw = (int64_t)blockIdx.x * WARPS + warp;
+    const WFirst *wf = p.wfirst + gw;
+    const int4 wb = __ldg(reinterpret_cast<const int4 *>(wf));
+    const int kbeg = wb.x, kend = wb.y;
+    double carry = 0.0;
+    uint32_t phases = 0;  // bit s: parity of slot s's barrier
+    const uint64_t stream_policy = policy_evict_first(), x_policy = policy_evict_last();
+    WItem cur = load_witem(&wf->w, 0), nx{};
+    int Jc = lane < 16 ? __ldg(wf->J + lane) : 0, Jx = 0;
+    if (kbeg < kend) issue_blob(p, cur, base, bar0, stream_policy, lane);
+    if (kbeg + 1 < kend) {
+        nx = load_witem(p.witems, kbeg + 1);
+        Jx = lane < 16 ? __ldg(p.jcols + (int64_t)(kbeg + 1) * 16 + lane) : 0;
+    }
+    for (int k = kbeg; k < kend; ++k) {
+        const uint32_t s = (uint32_t)(k - kbeg) & 1u;
+        const uint32_t slot = base + s * SLOT, bar = bar0 + 8 * s;
+        if (k == kbeg) griddep_wait();
+        issue_x(p, Jc, (cur.part_nt >> 24) & 31, xs, x_policy, lane);
+        // item k+1 into the other slot (free: item k-1 finished before the
+        // __syncwarp that ended the last iteration)
+        WItem n2{};
+        int J2 = 0;
+        if (k + 1 < kend) {
+            issue_blob(p, nx, base + (s ^ 1u) * SLOT, bar0 + 8 * (s ^ 1u), stream_policy, lane);
+            if (k + 2 < kend) {
+                n2 = load_witem(p.witems, k + 2);
+                J2 = lane < 16 ? __ldg(p.jcols + (int64_t)(k + 2) * 16 + lane) : 0;
             }
         }
-        __syncwarp();  // slot and x scratch free for the next item
+        if (cur.val_tot >> 16) {
+            mbar_wait(bar, (phases >> s) & 1u);
+            phases ^= 1u << s;
+        }
+        compute_item(p, cur, slot, xs, racc, x_policy, lane, carry);
+        __syncwarp();
+        cur = nx;
+        Jc = Jx;
+        nx = n2;
+        Jx = J2;
     }
 }
 
@@ -292,6 +373,12 @@ template <int WARPS, int SLOT, int MINB>
 KernelChoice warp_choice(const char *name) {
     using Cfg = WarpCfg<WARPS, SLOT>;
     return {name, tilespmv_fp64_warp<WARPS, SLOT, MINB>, Cfg::kThreads, (int)Cfg::kSmem, 0, false, SLOT, true};
+}
+
+template <int WARPS, int SLOT, int MINB>
+KernelChoice warp2_choice(const char *name) {
+    using Cfg = WarpCfg<WARPS, SLOT, 2>;
+    return {name, tilespmv_fp64_warp2<WARPS, SLOT, MINB>, Cfg::kThreads, (int)Cfg::kSmem, 0, false, SLOT, true};
 }
 
 }  // namespace
@@ -304,6 +391,11 @@ KernelChoice kernel_warp(int variant) {
     case 24: return warp_choice<8, 4096, 4>("tilespmv_fp64_warp<8,4096>");
     case 25: return warp_choice<4, 10752, 4>("tilespmv_fp64_warp<4,10752>");  // dense tile rows
     case 26: return warp_choice<4, 8704, 5>("tilespmv_fp64_warp<4,8704>");
+    // double-buffered
+    case 30: return warp2_choice<4, 6016, 4>("tilespmv_fp64_warp2<4,6016>");
+    case 31: return warp2_choice<6, 4608, 3>("tilespmv_fp64_warp2<6,4608>");
+    case 32: return warp2_choice<4, 8448, 3>("tilespmv_fp64_warp2<4,8448>");
+    case 33: return warp2_choice<4, 10752, 2>("tilespmv_fp64_warp2<4,10752>");
     default: return warp_choice<8, 4608, 4>("tilespmv_fp64_warp<8,4608>");
     }
 }
