@@ -43,6 +43,13 @@ __device__ __forceinline__ double lds_f64_lt(int i, int len, uint32_t a) {
         : "r"(i), "r"(len), "r"(a));
     return v;
 }
+// a remainder entry k (column, value) if k < e, else (0, 0.0)
+__device__ __forceinline__ void lds_entry_lt(int k, int e, uint32_t ca, uint32_t va, int &c, double &v) {
+    asm("{\n\t.reg .pred q;\n\tsetp.lt.s32 q, %2, %3;\n\tmov.b32 %0, 0;\n\tmov.b64 %1, 0;\n\t"
+        "@q ld.shared.s32 %0, [%4];\n\t@q ld.shared.f64 %1, [%5];\n\t}"
+        : "=r"(c), "=d"(v)
+        : "r"(k), "r"(e), "r"(ca), "r"(va));
+}
 // shared address of x[col] in a tile's 128-byte aligned x segment X, from a
 // column nibble already shifted to bits 3..6 (w's other bits are masked off)
 __device__ __forceinline__ uint32_t xaddr(uint32_t w8, uint32_t X) { return (w8 & 0x78u) | X; }

@@ -49,25 +49,21 @@ __device__ __forceinline__ void remainder(const Params &p, uint32_t rpS, uint32_
     const int b = lds_s32(rpS + 4 * min(r, rows)), e = lds_s32(rpS + 4 * min(r + 1, rows));
     const bool is_short = e - b <= kShortRow;
     if (!__any_sync(FULL, !is_short)) {
-        // two lanes per row; warp-uniform trip count, batches of four (loads first)
+        // two lanes per row, entries b + h, b + h + 2, ...; warp-uniform trip
+        // count, two entries per step.  A masked entry reads column 0 and
+        // value 0.0 (x[0] exists whenever the item has remainder entries).
         const int trips = (int)__reduce_max_sync(FULL, (unsigned)((e - b + 1 - h) >> 1));
+        const double *x = p.x;
 #pragma unroll 1
-        for (int i0 = 0; i0 < trips; i0 += 4) {
-            double vs[4], xr[4];
-            bool oks[4];
-#pragma unroll
-            for (int i = 0; i < 4; ++i) {
-                const int kq = b + h + 2 * (i0 + i);
-                oks[i] = kq < e;
-                vs[i] = xr[i] = 0.0;
-                if (i0 + i < trips) {
-                    const int c = oks[i] ? lds_s32(colS + 4 * kq) : 0;
-                    vs[i] = lds_f64(valS + 8 * (oks[i] ? kq : 0));
-                    if (oks[i]) xr[i] = ldg_hint(p.x + (uint32_t)c, x_policy);
-                }
-            }
-#pragma unroll
-            for (int i = 0; i < 4; ++i) fma_if(oks[i], vs[i], xr[i], acc);
+        for (int i = 0; i < trips; i += 2) {
+            const int k0 = b + h + 2 * i, k1 = k0 + 2;
+            int c0, c1;
+            double v0, v1;
+            lds_entry_lt(k0, e, colS + 4 * k0, valS + 8 * k0, c0, v0);
+            lds_entry_lt(k1, e, colS + 4 * k1, valS + 8 * k1, c1, v1);
+            const double x0 = ldg_hint(x + (uint32_t)c0, x_policy), x1 = ldg_hint(x + (uint32_t)c1, x_policy);
+            acc = fma(v0, x0, acc);
+            acc = fma(v1, x1, acc);
         }
         return;
     }
@@ -163,7 +159,20 @@ __device__ __forceinline__ void issue_blob(const Params &p, const WItem &it, uin
 // issued before the blob lands
 __device__ __forceinline__ void issue_x(const Params &p, int J, int nt, uint32_t xs, uint64_t x_policy, int lane) {
     const uint32_t n32 = (uint32_t)p.n;
-    if (p.x_vec) {  // lane l: tile 4k + (l >> 3), 16 bytes at elements 2(l & 7)
+    // tile columns ascend within an item: only the last one can reach the
+    // ragged end of x
+    const uint32_t jlast = (uint32_t)__shfl_sync(FULL, J, max(nt - 1, 0));
+    if (p.x_vec && 16u * jlast + 16u <= n32) {  // lane l: tile 4k + (l >> 3), 16 bytes at elements 2(l & 7)
+        const double *xq = p.x + 2 * (lane & 7);
+        const uint32_t xs_l = xs + 16 * (lane & 7);
+#pragma unroll
+        for (int kk = 0; kk < kItemTiles / 4; ++kk) {
+            const int t = 4 * kk + (lane >> 3);
+            const uint32_t Jt = (uint32_t)__shfl_sync(FULL, J, t);
+            if (t < nt) cp_async16(xs_l + 128 * t, xq + 16u * Jt, 16u, x_policy);
+        }
+        cp_async_commit();
+    } else if (p.x_vec) {
         const uint32_t qq = lane & 7;
 #pragma unroll
         for (int kk = 0; kk < kItemTiles / 4; ++kk) {
