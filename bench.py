@@ -97,16 +97,22 @@ class ClockSampler:
     def _run(self):
         while not self._stop.is_set():
             try:
-                self.samples.append(self.nv.nvmlDeviceGetClockInfo(self.h, self.nv.NVML_CLOCK_SM))
-                self.reasons |= int(self.nv.nvmlDeviceGetCurrentClocksEventReasons(self.h))
+                t = time.perf_counter()
+                mhz = self.nv.nvmlDeviceGetClockInfo(self.h, self.nv.NVML_CLOCK_SM)
+                rs = int(self.nv.nvmlDeviceGetCurrentClocksEventReasons(self.h))
+                self.samples.append((t, mhz, rs))
             except Exception:
                 pass
             time.sleep(0.002)
 
     def __enter__(self):
+        # started before the warm-up so that thread start and NVML set-up never
+        # fall inside the timed region; window() marks the timed region
         if self.ok:
             self.t = threading.Thread(target=self._run, daemon=True)
             self.t.start()
+            while not self.samples and self.t.is_alive():
+                time.sleep(0.001)
         return self
 
     def __exit__(self, *a):
@@ -114,12 +120,22 @@ class ClockSampler:
         if self.ok:
             self.t.join()
 
+    def window(self, t0, t1):
+        self.t0, self.t1 = t0, t1
+
     def summary(self):
         if not self.ok:
             return None
-        rs = [name for bit, name in self.REASONS.items() if self.reasons & bit and name != "gpu_idle"]
-        return {"sm_mhz": float(np.median(self.samples)) if self.samples else None,
-                "sm_max_mhz": self.max_mhz, "samples": len(self.samples), "reasons": rs}
+        t0, t1 = getattr(self, "t0", -1e30), getattr(self, "t1", 1e30)
+        inside = [s for s in self.samples if t0 <= s[0] <= t1]
+        if not inside and self.samples:  # timed region shorter than one sample period
+            inside = [min(self.samples, key=lambda s: abs(s[0] - 0.5 * (t0 + t1)))]
+        reasons = 0
+        for s in inside:
+            reasons |= s[2]
+        rs = [name for bit, name in self.REASONS.items() if reasons & bit and name != "gpu_idle"]
+        return {"sm_mhz": float(np.median([s[1] for s in inside])) if inside else None,
+                "sm_max_mhz": self.max_mhz, "samples": len(inside), "reasons": rs}
 
 
 # --------------------------------------------------------------------------
@@ -250,7 +266,7 @@ def run_reference(args):
 # --------------------------------------------------------------------------
 
 def measure_workload(workload, mode, steps, warmup, dev, rank, P, group, cpu_seconds,
-                     want_cpu, want_e2e, e2e_steps):
+                     want_cpu, want_e2e, e2e_steps, use_graph=True):
     import torch
     import torch.distributed as dist
     from paper_conf_ipps_niuldj0t21_b200 import TiledMatrix
@@ -290,12 +306,6 @@ def measure_workload(workload, mode, steps, warmup, dev, rank, P, group, cpu_sec
         else:
             mats[j].run(xs[j], ys[j])
 
-    for i in range(warmup):
-        step(i)
-    torch.cuda.synchronize(dev)
-    if P > 1:
-        dist.barrier(group=group)
-    torch.cuda.synchronize(dev)
     # N = 1: a step is exactly one kernel launch; the K launches go back to back
     # (programmatic dependent launch overlaps one kernel's prologue with the
     # previous one's tail) between two events, so the kernel's average launch
@@ -304,10 +314,37 @@ def measure_workload(workload, mode, steps, warmup, dev, rank, P, group, cpu_sec
     kev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
            for _ in range(steps if P > 1 else 0)]
     start, end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    # N = 1: the K timed launches are captured once into a CUDA graph and
+    # replayed, so the host's per-launch cost (Python + ctypes, ~8-11 us) cannot
+    # starve a kernel that runs for a few microseconds.  Each graph node is one
+    # launch of the SpMV kernel through tilespmv_run (PDL edges kept).
+    graph, launch_mode = None, "eager"
+    if P == 1 and use_graph:
+        for i in range(warmup):
+            step(i)
+        torch.cuda.synchronize(dev)
+        try:
+            graph = torch.cuda.CUDAGraph()
+            with torch.cuda.graph(graph):
+                for i in range(steps):
+                    mats[i % reps].run(xs[i % reps], ys[i % reps])
+            graph.replay()  # upload + one untimed pass
+            torch.cuda.synchronize(dev)
+            launch_mode = "cuda_graph"
+        except Exception as e:  # pragma: no cover
+            log("graph capture failed, timing eager launches:", e)
+            graph = None
     sampler = ClockSampler(dev.index if dev.index is not None else 0)
     with sampler:
+        for i in range(warmup):
+            step(i)
+        torch.cuda.synchronize(dev)
+        if P > 1:
+            dist.barrier(group=group)
+        torch.cuda.synchronize(dev)
+        h0 = time.perf_counter()
         start.record(stream)
-        for i in range(steps):
+        for i in range(steps if graph is None else 0):
             j = i % reps
             if P > 1:
                 kev[i][0].record(stream)
@@ -318,8 +355,13 @@ def measure_workload(workload, mode, steps, warmup, dev, rank, P, group, cpu_sec
                                             group=group)
             else:
                 mats[j].run(xs[j], ys[j])
+        if graph is not None:
+            graph.replay()
         end.record(stream)
+        h1 = time.perf_counter()
         torch.cuda.synchronize(dev)
+        sampler.window(h0, time.perf_counter())
+    host_launch_us = (h1 - h0) / steps * 1e6  # host time to enqueue one step
     if P > 1:
         dist.barrier(group=group)
     torch.cuda.synchronize(dev)
@@ -347,6 +389,7 @@ def measure_workload(workload, mode, steps, warmup, dev, rank, P, group, cpu_sec
            "kernel_ms_mean": float(np.mean(kern_ms)), "kernel_ms_median": float(np.median(kern_ms)),
            "kernel_ms_max_over_ranks": kern_max, "create_s": create_s,
            "clocks": sampler.summary(), "nnz": nnz_total, "m": m, "n": n,
+           "host_enqueue_us_per_step": host_launch_us, "launch_mode": launch_mode,
            "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                         "frac": achieved / peak, "traffic": profile_traffic(workload, mode),
                         "peak_source": peak_src,
@@ -429,12 +472,14 @@ def run_ours(args):
         group = dist.group.WORLD
     res = measure_workload(args.workload, args.mode, args.steps, args.warmup, dev, rank, P, group,
                            args.cpu_seconds, want_cpu=not args.no_cpu_baseline,
-                           want_e2e=True, e2e_steps=args.e2e_steps)
+                           want_e2e=True, e2e_steps=args.e2e_steps, use_graph=not args.no_graph)
     secondary = {}
     if P == 1 and not args.no_secondary and args.workload != "fem":
         r2 = measure_workload("fem", args.mode, max(args.steps, 200), args.warmup, dev, 0, 1, None,
-                              2.0, want_cpu=False, want_e2e=False, e2e_steps=0)
+                              2.0, want_cpu=False, want_e2e=False, e2e_steps=0, use_graph=not args.no_graph)
         secondary["fem"] = {"value": r2["value"], "unit": UNIT, "ms_per_step": r2["ms_per_step"],
+                            "host_enqueue_us_per_step": r2["host_enqueue_us_per_step"],
+                            "launch_mode": r2["launch_mode"],
                             "roofline": r2["roofline"], "replicas_rotated": r2["reps"],
                             "desc": WORKLOAD_DESC["fem"]}
     if rank == 0:
@@ -449,6 +494,7 @@ def run_ours(args):
                           "l2": ("inputs larger than L2" if res["reps"] == 1 else
                                  f"rotating {res['reps']} replicas (> 4x L2)"),
                           "step": ("SpMV + NCCL all-gather of y" if P > 1 else "one SpMV launch"),
+                          "launch_mode": res["launch_mode"],
                           "numtile": info["numtile"], "rem_nnz": info["rem_nnz"],
                           "kept_tiles": dict(zip(["CSR", "COO", "ELL", "HYB", "DNS", "DNSROW", "DNSCOL"],
                                                  info["kept_tiles"])),
@@ -460,6 +506,7 @@ def run_ours(args):
                "kernel_ms": {"mean": res["kernel_ms_mean"], "median": res["kernel_ms_median"],
                              "max_over_ranks": res["kernel_ms_max_over_ranks"]},
                "clocks": res["clocks"],
+               "host_enqueue_us_per_step": res["host_enqueue_us_per_step"],
                "launch": res["launch"],
                "parity": res.get("parity")}
         if secondary:
@@ -482,6 +529,8 @@ def main():
     ap.add_argument("--e2e-steps", type=int, default=20)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-secondary", action="store_true")
+    ap.add_argument("--no-graph", action="store_true",
+                    help="N=1: time K eager launches instead of one CUDA-graph replay of them")
     args = ap.parse_args()
     assert args.warmup >= 3, "the contract requires >= 3 warm-up steps"
     if args.impl == "reference":

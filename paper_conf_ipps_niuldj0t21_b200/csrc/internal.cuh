@@ -59,11 +59,13 @@ struct __align__(16) WItem {
 };
 
 // Per-warp start record of the warp kernel: the warp's item chunk and a copy
-// of its first item, so the prologue needs one round trip before the blob.
+// of its first item (and the second item's record, for the double-buffered
+// kernel), so the prologue needs one round trip before the blob copies.
 struct __align__(16) WFirst {
     int32_t kbeg, kend, pad0, pad1;
     WItem w;
     int32_t J[16];
+    WItem w2;
 };
 
 // The parts of a split tile row form groups of kLocalParts consecutive parts.

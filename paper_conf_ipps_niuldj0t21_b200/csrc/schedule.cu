@@ -247,6 +247,7 @@ __global__ void k_warp_first(const int64_t *begin, const WItem *witems, const in
         f.w = WItem{};
         for (int i = 0; i < 16; ++i) f.J[i] = 0;
     }
+    f.w2 = f.kbeg + 1 < f.kend ? witems[f.kbeg + 1] : WItem{};
     wf[b] = f;
 }
 
@@ -391,11 +392,12 @@ int build_tdesc(Matrix &M, cudaStream_t st) {
 
 int choose_kernel(Matrix &M) {
     // default: the warp kernel with 4.5 KB slots (32 warps/SM); matrices whose
-    // tile rows average more than 6 KB of payload (dense, FEM-like) use the
-    // double-buffered kernel with two 5.9 KB slots per warp (16 warps/SM), so
-    // a warp streams the next piece of its tile row while it computes one
+    // tile rows average more than 6 KB of payload (dense, FEM-like) use 10.5 KB
+    // slots (16 warps/SM) so a tile row stays one item.  (Measured on C2 with
+    // graph-replayed launches: 6.9 us for <4,10752> against 7.6 us for the
+    // default and 8.8 us for the double-buffered warp2<4,6016>.)
     const double row_bytes = M.tilem ? (double)M.payload_bytes / (double)M.tilem : 0.0;
-    int version = row_bytes > 6144.0 ? 30 : 20;
+    int version = row_bytes > 6144.0 ? 25 : 20;
     if (const char *e = getenv("TILESPMV_KERNEL")) version = atoi(e);
     M.kernel_version = version;
     M.item_bytes = choose(version).slot_bytes;

@@ -344,9 +344,11 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT, 2>::kThreads, MINB) tiles
     const uint64_t stream_policy = policy_evict_first(), x_policy = policy_evict_last();
     WItem cur = load_witem(&wf->w, 0), nx{};
     int Jc = lane < 16 ? __ldg(wf->J + lane) : 0, Jx = 0;
+    // both slots start streaming before the dependency wait (matrix data only)
     if (kbeg < kend) issue_blob(p, cur, base, bar0, stream_policy, lane);
     if (kbeg + 1 < kend) {
-        nx = load_witem(p.witems, kbeg + 1);
+        nx = load_witem(&wf->w2, 0);
+        issue_blob(p, nx, base + SLOT, bar0 + 8, stream_policy, lane);
         Jx = lane < 16 ? __ldg(p.jcols + (int64_t)(kbeg + 1) * 16 + lane) : 0;
     }
     for (int k = kbeg; k < kend; ++k) {
@@ -354,23 +356,19 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT, 2>::kThreads, MINB) tiles
         const uint32_t slot = base + s * SLOT, bar = bar0 + 8 * s;
         if (k == kbeg) griddep_wait();
         issue_x(p, Jc, (cur.part_nt >> 24) & 31, xs, x_policy, lane);
-        // item k+1 into the other slot (free: item k-1 finished before the
-        // __syncwarp that ended the last iteration)
         WItem n2{};
         int J2 = 0;
-        if (k + 1 < kend) {
-            issue_blob(p, nx, base + (s ^ 1u) * SLOT, bar0 + 8 * (s ^ 1u), stream_policy, lane);
-            if (k + 2 < kend) {
-                n2 = load_witem(p.witems, k + 2);
-                J2 = lane < 16 ? __ldg(p.jcols + (int64_t)(k + 2) * 16 + lane) : 0;
-            }
+        if (k + 2 < kend) {  // the record of the item that refills this slot
+            n2 = load_witem(p.witems, k + 2);
+            J2 = lane < 16 ? __ldg(p.jcols + (int64_t)(k + 2) * 16 + lane) : 0;
         }
         if (cur.val_tot >> 16) {
             mbar_wait(bar, (phases >> s) & 1u);
             phases ^= 1u << s;
         }
         compute_item(p, cur, slot, xs, racc, x_policy, lane, carry);
-        __syncwarp();
+        __syncwarp();  // slot s and the x stage are free
+        if (k + 2 < kend) issue_blob(p, n2, slot, bar, stream_policy, lane);
         cur = nx;
         Jc = Jx;
         nx = n2;
@@ -405,6 +403,7 @@ KernelChoice kernel_warp(int variant) {
     case 31: return warp2_choice<6, 4608, 3>("tilespmv_fp64_warp2<6,4608>");
     case 32: return warp2_choice<4, 8448, 3>("tilespmv_fp64_warp2<4,8448>");
     case 33: return warp2_choice<4, 10752, 2>("tilespmv_fp64_warp2<4,10752>");
+    case 34: return warp2_choice<3, 6192, 5>("tilespmv_fp64_warp2<3,6192>");
     default: return warp_choice<8, 4608, 4>("tilespmv_fp64_warp<8,4608>");
     }
 }

@@ -261,7 +261,7 @@ def test_full_size_tiler_and_spmv(cuda_device, name):
         M.close()
 
 
-@pytest.mark.parametrize("variant", ["1", "20", "21", "22", "23", "24", "25", "26", "30", "31", "32", "33"])
+@pytest.mark.parametrize("variant", ["1", "20", "21", "22", "23", "24", "25", "26", "30", "31", "32", "33", "34"])
 def test_kernel_variants_parity(cuda_device, variant, monkeypatch):
     """Every SpMV kernel variant (TILESPMV_KERNEL, read at create time) meets
     the oracle tolerance; each is run-to-run bitwise deterministic."""
