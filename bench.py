@@ -268,11 +268,11 @@ def run_reference(args):
 def measure_workload(workload, mode, steps, warmup, dev, rank, P, group, cpu_seconds,
                      want_cpu, want_e2e, e2e_steps, use_graph=True):
     import torch
-    import torch.distributed as dist
     from paper_conf_ipps_niuldj0t21_b200 import TiledMatrix
     from synthetic import gen
 
     t0 = time.perf_counter()
+    assert P == 1, "measure_workload is the N = 1 path"
     A, m, n, bounds = build_local(workload, rank, P)
     log(f"[rank {rank}] {workload}: local {A.m}x{A.n} nnz {A.nnz} generated in "
         f"{time.perf_counter() - t0:.1f}s")
@@ -287,39 +287,26 @@ def measure_workload(workload, mode, steps, warmup, dev, rank, P, group, cpu_sec
     create_s = time.perf_counter() - t
     info = M0.info()
     L2 = torch.cuda.get_device_properties(dev).L2_cache_size
-    reps = 1 if P > 1 else max(1, -(-4 * L2 // max(info["alg_bytes"], 1)))
+    reps = max(1, -(-4 * L2 // max(info["alg_bytes"], 1)))
     mats = [M0] + [TiledMatrix.from_csr(rp, ci, va, A.m, A.n, mode=mode) for _ in range(reps - 1)]
     del rp, ci, va
     xs = [torch.from_numpy(x_h).to(dev) for _ in range(reps)]
     ys = [torch.empty(A.m, dtype=torch.float64, device=dev) for _ in range(reps)]
-    rows_local = A.m
-    maxrows = max(bounds[i + 1] - bounds[i] for i in range(P))
-    gathered = torch.empty(P * maxrows, dtype=torch.float64, device=dev) if P > 1 else None
-
     def step(i):
         j = i % reps
-        if P > 1:
-            y = gathered[rank * maxrows: rank * maxrows + rows_local]
-            mats[j].run(xs[j], y)
-            dist.all_gather_into_tensor(gathered, gathered[rank * maxrows:(rank + 1) * maxrows],
-                                        group=group)
-        else:
-            mats[j].run(xs[j], ys[j])
+        mats[j].run(xs[j], ys[j])
 
-    # N = 1: a step is exactly one kernel launch; the K launches go back to back
+    # a step is exactly one kernel launch; the K launches go back to back
     # (programmatic dependent launch overlaps one kernel's prologue with the
     # previous one's tail) between two events, so the kernel's average launch
-    # duration is the timed region / K.  N > 1: per-launch events bracket each
-    # SpMV kernel so its duration is separated from the all-gather.
-    kev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
-           for _ in range(steps if P > 1 else 0)]
+    # duration is the timed region / K.
     start, end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     # N = 1: the K timed launches are captured once into a CUDA graph and
     # replayed, so the host's per-launch cost (Python + ctypes, ~8-11 us) cannot
     # starve a kernel that runs for a few microseconds.  Each graph node is one
     # launch of the SpMV kernel through tilespmv_run (PDL edges kept).
     graph, launch_mode = None, "eager"
-    if P == 1 and use_graph:
+    if use_graph:
         for i in range(warmup):
             step(i)
         torch.cuda.synchronize(dev)
@@ -339,22 +326,10 @@ def measure_workload(workload, mode, steps, warmup, dev, rank, P, group, cpu_sec
         for i in range(warmup):
             step(i)
         torch.cuda.synchronize(dev)
-        if P > 1:
-            dist.barrier(group=group)
-        torch.cuda.synchronize(dev)
         h0 = time.perf_counter()
         start.record(stream)
         for i in range(steps if graph is None else 0):
-            j = i % reps
-            if P > 1:
-                kev[i][0].record(stream)
-                y = gathered[rank * maxrows: rank * maxrows + rows_local]
-                mats[j].run(xs[j], y)
-                kev[i][1].record(stream)
-                dist.all_gather_into_tensor(gathered, gathered[rank * maxrows:(rank + 1) * maxrows],
-                                            group=group)
-            else:
-                mats[j].run(xs[j], ys[j])
+            step(i)
         if graph is not None:
             graph.replay()
         end.record(stream)
@@ -362,23 +337,11 @@ def measure_workload(workload, mode, steps, warmup, dev, rank, P, group, cpu_sec
         torch.cuda.synchronize(dev)
         sampler.window(h0, time.perf_counter())
     host_launch_us = (h1 - h0) / steps * 1e6  # host time to enqueue one step
-    if P > 1:
-        dist.barrier(group=group)
     torch.cuda.synchronize(dev)
     total_ms = start.elapsed_time(end)
-    kern_ms = (np.array([a.elapsed_time(b) for a, b in kev]) if P > 1
-               else np.array([total_ms / steps]))
-    if P > 1:
-        t_ = torch.tensor([total_ms, float(np.mean(kern_ms))], dtype=torch.float64, device=dev)
-        dist.all_reduce(t_, op=dist.ReduceOp.MAX, group=group)
-        total_ms, kern_max = float(t_[0]), float(t_[1])
-    else:
-        kern_max = float(np.mean(kern_ms))
+    kern_ms = np.array([total_ms / steps])
+    kern_max = float(np.mean(kern_ms))
     nnz_total = A.nnz
-    if P > 1:
-        t_ = torch.tensor([A.nnz], dtype=torch.int64, device=dev)
-        dist.all_reduce(t_, group=group)
-        nnz_total = int(t_[0])
     ms_per_step = total_ms / steps
     value = 2.0 * nnz_total / (ms_per_step * 1e-3) / 1e9
     peak, peak_src = hbm_peak()
@@ -396,7 +359,7 @@ def measure_workload(workload, mode, steps, warmup, dev, rank, P, group, cpu_sec
                         "alg_bytes_per_launch": info["alg_bytes"],
                         "kernel": M0.kernel_name()}}
     # ---- correctness on the oracle's sample + CPU baseline (rank 0, N = 1)
-    if want_cpu and rank == 0 and P == 1:
+    if want_cpu and rank == 0:
         rng = np.random.default_rng(4321)
         val, rows, yref, absy, desc, dt = oracle_sample(A, x_h, cpu_seconds, rng)
         y = ys[0].cpu().numpy()
@@ -408,7 +371,7 @@ def measure_workload(workload, mode, steps, warmup, dev, rank, P, group, cpu_sec
                          "max_err_over_absy": float(np.max(err / (absy + 1e-300))) if rows.size else 0.0,
                          "tolerance": "1e-12*sum|a_ij x_j| + 1e-300"}
     # ---- end to end through the host-buffer C-ABI call
-    if want_e2e and P == 1:
+    if want_e2e:
         hx = torch.from_numpy(x_h).pin_memory()
         hy = torch.empty(A.m, dtype=torch.float64).pin_memory()
         for _ in range(2):
@@ -422,20 +385,140 @@ def measure_workload(workload, mode, steps, warmup, dev, rank, P, group, cpu_sec
                       "h2d_bytes_per_step": 8 * n, "d2h_bytes_per_step": 8 * A.m,
                       "ms_per_step": e2e_s * 1e3, "steps": e2e_steps,
                       "call": "tilespmv_run_host (pinned host x -> H2D -> kernel -> D2H y -> sync)"}
-    if want_e2e and P > 1:
-        # per step on every rank: H2D of x (replicated), the local SpMV, the NCCL
-        # all-gather of y, D2H of the gathered y; max over ranks
-        hx = torch.from_numpy(x_h).pin_memory()
-        hy = torch.empty(P * maxrows, dtype=torch.float64).pin_memory()
-        xd = torch.empty(n, dtype=torch.float64, device=dev)
+    for M in mats:
+        M.close()
+    return res
+
+
+def measure_sharded(workload, mode, steps, warmup, dev, rank, P, group, exchange, e2e_steps):
+    """N > 1: tile-row shards (x replicated at start), one step = the rank's
+    SpMV plus the exchange that makes x_{k+1} available where it is needed:
+      halo      -- neighbour-only NCCL send/recv of the x rows each peer's
+                   columns touch, overlapped with the interior SpMV; the
+                   boundary SpMVs run after it lands (SURVEY 8(f) f1);
+      allgather -- the SpMV of all local rows, then an NCCL all-gather of y
+                   (SURVEY 8(e)).
+    x stays fixed across steps (the exchanged rows equal what is there), so
+    the timed work is exactly one iteration's and values stay finite.  Times
+    are device events on the compute stream, max over ranks."""
+    import torch
+    import torch.distributed as dist
+    from paper_conf_ipps_niuldj0t21_b200 import TiledMatrix
+    from paper_conf_ipps_niuldj0t21_b200.sharded import HaloSpMV, plan_halo
+    from synthetic import gen
+
+    t0 = time.perf_counter()
+    A, m, n, bounds = build_local(workload, rank, P)
+    a, b = bounds[rank], bounds[rank + 1]
+    log(f"[rank {rank}] {workload}: rows [{a},{b}) nnz {A.nnz} generated in {time.perf_counter() - t0:.1f}s")
+    x_h = gen.dense_x(n, 101)
+    stream = torch.cuda.current_stream(dev)
+    x = torch.from_numpy(x_h).to(dev)
+    torch.cuda.synchronize(dev)
+    t = time.perf_counter()
+    if exchange == "halo":
+        plan = plan_halo(A.rowptr, A.colidx, bounds, rank, P, group)
+        parts = plan.parts
+    else:
+        plan, parts = None, [(a, b, True)]
+    mats = []
+    for r0, r1, _ in parts:
+        S = A.row_slice(r0 - a, r1 - a)
+        mats.append(TiledMatrix.from_csr(torch.from_numpy(S.rowptr).to(dev), torch.from_numpy(S.colidx).to(dev),
+                                         torch.from_numpy(S.val).to(dev), S.m, S.n, mode=mode))
+    torch.cuda.synchronize(dev)
+    create_s = time.perf_counter() - t
+    infos = [M.info() for M in mats]
+    dom = max(range(len(mats)), key=lambda i: infos[i]["alg_bytes"])  # dominant kernel
+    maxrows = max(bounds[i + 1] - bounds[i] for i in range(P))
+    y = torch.empty(n if exchange == "halo" else P * maxrows, dtype=torch.float64, device=dev)
+    kev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(steps)]
+
+    if exchange == "halo":
+        def mk(M):
+            return lambda xf, yo: M.run(xf, yo)
+        H = HaloSpMV(plan, [mk(M) for M in mats], group=group)
+        ev_slot = [None]
+
+        def timed(xf, yo, M=mats[dom]):
+            e = ev_slot[0]
+            if e is not None:
+                e[0].record(stream)
+            M.run(xf, yo)
+            if e is not None:
+                e[1].record(stream)
+        H.spmvs[dom] = timed
+
+        def step(i, ev=None):
+            ev_slot[0] = ev
+            H.step(x, y)
+    else:
+        def step(i, ev=None):
+            yl = y[rank * maxrows: rank * maxrows + (b - a)]
+            if ev is not None:
+                ev[0].record(stream)
+            mats[0].run(x, yl)
+            if ev is not None:
+                ev[1].record(stream)
+            dist.all_gather_into_tensor(y, y[rank * maxrows:(rank + 1) * maxrows], group=group)
+
+    start, end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    sampler = ClockSampler(dev.index if dev.index is not None else 0)
+    with sampler:
+        for i in range(warmup):
+            step(i)
+        torch.cuda.synchronize(dev)
+        dist.barrier(group=group)
+        torch.cuda.synchronize(dev)
+        h0 = time.perf_counter()
+        start.record(stream)
+        for i in range(steps):
+            step(i, kev[i])
+        end.record(stream)
+        torch.cuda.synchronize(dev)
+        sampler.window(h0, time.perf_counter())
+    dist.barrier(group=group)
+    total_ms = start.elapsed_time(end)
+    kern_ms = np.array([e0.elapsed_time(e1) for e0, e1 in kev])
+    t_ = torch.tensor([total_ms, float(np.mean(kern_ms))], dtype=torch.float64, device=dev)
+    dist.all_reduce(t_, op=dist.ReduceOp.MAX, group=group)
+    total_ms, kern_max = float(t_[0]), float(t_[1])
+    t_ = torch.tensor([A.nnz], dtype=torch.int64, device=dev)
+    dist.all_reduce(t_, group=group)
+    nnz_total = int(t_[0])
+    ms_per_step = total_ms / steps
+    peak, peak_src = hbm_peak()
+    achieved = infos[dom]["alg_bytes"] / (float(np.mean(kern_ms)) * 1e-3) / 1e9
+    grid, block, smem = mats[dom].launch_shape()
+    res = {"value": 2.0 * nnz_total / (ms_per_step * 1e-3) / 1e9, "ms_per_step": ms_per_step,
+           "info": infos[dom], "reps": 1, "nnz": nnz_total, "m": m, "n": n, "create_s": create_s,
+           "launch": {"grid": grid, "block": block, "smem_bytes": smem},
+           "kernel_ms_mean": float(np.mean(kern_ms)), "kernel_ms_median": float(np.median(kern_ms)),
+           "kernel_ms_max_over_ranks": kern_max, "clocks": sampler.summary(),
+           "host_enqueue_us_per_step": None, "launch_mode": "eager",
+           "launches_per_step": len(mats),
+           "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                        "frac": achieved / peak, "traffic": None, "peak_source": peak_src,
+                        "alg_bytes_per_launch": infos[dom]["alg_bytes"],
+                        "kernel": mats[dom].kernel_name() + (" (interior part)" if exchange == "halo" else "")}}
+    if exchange == "halo":
+        res["exchange"] = {"kind": "halo (NCCL send/recv, overlapped with the interior SpMV)",
+                           "recv_bytes_rank0": 8 * plan.recv_elems, "send_bytes_rank0": 8 * plan.send_elems,
+                           "parts_rank0": [[r0, r1, bool(it)] for r0, r1, it in parts]}
+    else:
+        res["exchange"] = {"kind": "NCCL all-gather of y", "bytes_per_rank": 8 * P * maxrows}
+    # ---- end to end: per step every rank copies its own x rows in (pinned
+    # host -> device), runs the step, and reads its own y rows back
+    if e2e_steps > 0:
+        hx = torch.from_numpy(x_h[a:b].copy()).pin_memory()
+        hy = torch.empty(b - a, dtype=torch.float64).pin_memory()
 
         def e2e_step():
-            xd.copy_(hx, non_blocking=True)
-            y = gathered[rank * maxrows: rank * maxrows + rows_local]
-            M0.run(xd, y)
-            dist.all_gather_into_tensor(gathered, gathered[rank * maxrows:(rank + 1) * maxrows], group=group)
-            hy.copy_(gathered, non_blocking=True)
-            torch.cuda.current_stream(dev).synchronize()
+            x[a:b].copy_(hx, non_blocking=True)
+            step(0)
+            hy.copy_(y[a:b] if exchange == "halo" else y[rank * maxrows: rank * maxrows + (b - a)],
+                     non_blocking=True)
+            stream.synchronize()
 
         for _ in range(2):
             e2e_step()
@@ -447,9 +530,10 @@ def measure_workload(workload, mode, steps, warmup, dev, rank, P, group, cpu_sec
         dist.all_reduce(e2e_s, op=dist.ReduceOp.MAX, group=group)
         e2e_s = float(e2e_s[0])
         res["e2e"] = {"value": 2.0 * nnz_total / e2e_s / 1e9, "unit": UNIT,
-                      "h2d_bytes_per_step": 8 * n, "d2h_bytes_per_step": 8 * P * maxrows,
+                      "h2d_bytes_per_step": 8 * n, "d2h_bytes_per_step": 8 * m,
                       "ms_per_step": e2e_s * 1e3, "steps": e2e_steps,
-                      "call": "per rank: H2D x -> TiledMatrix.run -> NCCL all-gather y -> D2H y (max over ranks)"}
+                      "call": "per rank: H2D own x rows -> step (exchange + SpMV) -> D2H own y rows; "
+                              "bytes summed over ranks, time max over ranks"}
     for M in mats:
         M.close()
     return res
@@ -470,9 +554,13 @@ def run_ours(args):
     if P > 1:
         dist.init_process_group("nccl", device_id=dev)
         group = dist.group.WORLD
-    res = measure_workload(args.workload, args.mode, args.steps, args.warmup, dev, rank, P, group,
-                           args.cpu_seconds, want_cpu=not args.no_cpu_baseline,
-                           want_e2e=True, e2e_steps=args.e2e_steps, use_graph=not args.no_graph)
+    if P > 1:
+        res = measure_sharded(args.workload, args.mode, args.steps, args.warmup, dev, rank, P, group,
+                              args.exchange, args.e2e_steps)
+    else:
+        res = measure_workload(args.workload, args.mode, args.steps, args.warmup, dev, rank, P, group,
+                               args.cpu_seconds, want_cpu=not args.no_cpu_baseline,
+                               want_e2e=True, e2e_steps=args.e2e_steps, use_graph=not args.no_graph)
     secondary = {}
     if P == 1 and not args.no_secondary and args.workload != "fem":
         r2 = measure_workload("fem", args.mode, max(args.steps, 200), args.warmup, dev, 0, 1, None,
@@ -493,7 +581,9 @@ def run_ours(args):
                           "parallelism": f"tile-row shards x{P}" if P > 1 else "1 GPU",
                           "l2": ("inputs larger than L2" if res["reps"] == 1 else
                                  f"rotating {res['reps']} replicas (> 4x L2)"),
-                          "step": ("SpMV + NCCL all-gather of y" if P > 1 else "one SpMV launch"),
+                          "step": (("halo exchange overlapped with the interior SpMV + boundary SpMVs"
+                                    if args.exchange == "halo" else "SpMV + NCCL all-gather of y")
+                                   if P > 1 else "one SpMV launch"),
                           "launch_mode": res["launch_mode"],
                           "numtile": info["numtile"], "rem_nnz": info["rem_nnz"],
                           "kept_tiles": dict(zip(["CSR", "COO", "ELL", "HYB", "DNS", "DNSROW", "DNSCOL"],
@@ -509,6 +599,9 @@ def run_ours(args):
                "host_enqueue_us_per_step": res["host_enqueue_us_per_step"],
                "launch": res["launch"],
                "parity": res.get("parity")}
+        if "exchange" in res:
+            out["exchange"] = res["exchange"]
+            out["gpu_launches"] = args.steps * res["launches_per_step"]
         if secondary:
             out["secondary"] = secondary
         print(json.dumps(out), flush=True)
@@ -526,6 +619,8 @@ def main():
     ap.add_argument("--workload", default=DEFAULT_WORKLOAD)
     ap.add_argument("--mode", default="DEFERRED", choices=["ADPT", "DEFERRED", "AUTO", "FORCE_CSR"])
     ap.add_argument("--cpu-seconds", type=float, default=10.0)
+    ap.add_argument("--exchange", default="halo", choices=["halo", "allgather"],
+                    help="N>1: neighbour-only x exchange (default) or all-gather of y")
     ap.add_argument("--e2e-steps", type=int, default=20)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-secondary", action="store_true")

@@ -98,3 +98,107 @@ def test_partition_properties():
     b = partition_tile_rows(1600, 4, w)
     loads = [w[b[i] // 16:b[i + 1] // 16].sum() for i in range(4)]
     assert max(loads) <= 1.5 * (w.sum() / 4) + 50
+
+
+# ---------------------------------------------------------------------------
+# halo exchange: neighbour-only x exchange + overlap
+# ---------------------------------------------------------------------------
+
+def _halo_worker(rank, world, port, name, iters, q):
+    try:
+        from oracle import oracle as O
+        from paper_conf_ipps_niuldj0t21_b200.sharded import HaloSpMV, plan_halo
+        from synthetic import gen
+        os.environ["MASTER_ADDR"] = "127.0.0.1"
+        os.environ["MASTER_PORT"] = str(port)
+        dist.init_process_group("gloo", rank=rank, world_size=world)
+        A, x = gen.make(name)
+        b = partition_tile_rows(A.m, world)
+        S = A.row_slice(b[rank], b[rank + 1])
+        plan = plan_halo(S.rowptr, S.colidx, b, rank, world)
+
+        def part_spmv(r0, r1):
+            P = A.row_slice(r0, r1)
+
+            def f(xf, yout):
+                y, _ = O.spmv(P, xf.numpy())
+                yout.copy_(torch.from_numpy(y))
+            return f
+
+        h = HaloSpMV(plan, [part_spmv(r0, r1) for r0, r1, _ in plan.parts])
+        # x_0 is replicated; afterwards only own rows + halo are valid: poison
+        # the rest so that a missing halo entry shows up as NaN
+        xa = torch.from_numpy(x.copy())
+        xb = torch.full((A.n,), float("nan"), dtype=torch.float64)
+        outs = []
+        for k in range(iters):
+            h.step(xa, xb)
+            outs.append(xb[b[rank]:b[rank + 1]].numpy().copy())
+            xa, xb = xb, xa
+            xb.fill_(float("nan"))
+        q.put((rank, b, plan.as_dict(), outs))
+        dist.destroy_process_group()
+    except Exception as e:  # pragma: no cover
+        import traceback
+        q.put((rank, None, traceback.format_exc(), None))
+
+
+@pytest.mark.parametrize("name,world", [("stencil27_40", 2), ("stencil27_21", 3), ("lap2d_37x29", 2),
+                                        ("rmat12", 2)])
+def test_halo_exchange_equals_unsharded(name, world):
+    """Each rank's rows of x_k equal the unsharded oracle iterate bitwise,
+    although only the halo (not the whole x) crossed ranks."""
+    from oracle import oracle as O
+    from synthetic import gen
+    iters = 3
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _port()
+    procs = [ctx.Process(target=_halo_worker, args=(r, world, port, name, iters, q))
+             for r in range(world)]
+    for p in procs:
+        p.start()
+    res = [q.get(timeout=300) for _ in range(world)]
+    for p in procs:
+        p.join(timeout=60)
+    for r, b, plan, outs in res:
+        assert b is not None, plan
+    A, x = gen.make(name)
+    ref, xk = [], x.copy()
+    for _ in range(iters):
+        xk, _ = O.spmv(A, xk)
+        ref.append(xk.copy())
+    for r, b, plan, outs in res:
+        for k in range(iters):
+            assert np.array_equal(outs[k].view(np.uint64), ref[k][b[r]:b[r + 1]].view(np.uint64)), (name, r, k)
+        # parts tile the rank's rows on tile-row boundaries
+        parts = plan["parts"]
+        assert parts[0][0] == b[r] and parts[-1][1] == b[r + 1]
+        assert all(parts[i][1] == parts[i + 1][0] for i in range(len(parts) - 1))
+        assert all(p0 % 16 == 0 for p0, _, _ in parts)
+    # send lists mirror recv lists
+    sends = {(r, q, lo, hi) for r, b, plan, _ in res for q, lo, hi in plan["send"]}
+    recvs = {(q, r, lo, hi) for r, b, plan, _ in res for q, lo, hi in plan["recv"]}
+    assert sends == recvs
+
+
+def test_halo_needs_stencil_closed_form():
+    """27-point stencil nx^3 (nx = 40, so a rank boundary falls on a z-plane
+    boundary), 2 ranks: each rank needs exactly the neighbouring z-plane
+    (nx^2 rows) of the other, and exactly its own plane next to the boundary
+    is boundary rows; everything else is interior."""
+    from paper_conf_ipps_niuldj0t21_b200.sharded import halo_needs
+    from synthetic import gen
+    nx = 40
+    A = gen.stencil27(nx)
+    b = partition_tile_rows(A.m, 2)
+    pl = nx * nx
+    assert b[1] % pl == 0
+    S0 = A.row_slice(b[0], b[1])
+    recv0, parts0 = halo_needs(S0.rowptr, S0.colidx, b, 0)
+    assert recv0 == [(1, b[1], b[1] + pl)]
+    assert parts0 == [(0, b[1] - pl, True), (b[1] - pl, b[1], False)]
+    S1 = A.row_slice(b[1], b[2])
+    recv1, parts1 = halo_needs(S1.rowptr, S1.colidx, b, 1)
+    assert recv1 == [(0, b[1] - pl, b[1])]
+    assert parts1 == [(b[1], b[1] + pl, False), (b[1] + pl, b[2], True)]
