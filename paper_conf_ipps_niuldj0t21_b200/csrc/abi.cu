@@ -36,7 +36,7 @@ static void free_matrix(tilespmv_matrix *M) {
     if (cur != M->device) cudaSetDevice(M->device);
     void *ptrs[] = {M->tilePtr, M->tileColIdx, M->tileNnz, M->tileFmt, M->tileAux, M->tileOff,
                     M->payload, M->remRowPtr, M->remCol, M->remVal, M->items, M->split_info,
-                    M->partials, M->counters, M->xstage, M->ystage, M->tdesc, M->cta_begin, M->blob, M->witems, M->jcols, M->wfirst};
+                    M->partials, M->counters, M->xstage, M->ystage, M->tdesc, M->cta_begin, M->blob, M->witems, M->jcols, M->wfirst, M->units};
     for (void *p : ptrs)
         if (p) cudaFree(p);
     if (cur >= 0 && cur != M->device) cudaSetDevice(cur);

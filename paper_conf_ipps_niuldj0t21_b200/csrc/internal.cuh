@@ -43,7 +43,18 @@ struct __align__(16) Item {
     int32_t ndsc;      // entries: the item's tiles grouped by format, groups padded to even length
     uint32_t blob16;   // start of the item's execution blob (16-byte units)
     uint32_t blob_len; // bytes of the blob (blob_parts)
+    int32_t ntr;       // row-group item: consecutive tile rows I..I+ntr-1 (0: ordinary item)
 };
+
+// Row-group items (warp kernel): consecutive tile rows that hold no stored
+// tile and whose remainder rows fit one slot together (power-law matrices:
+// most R-MAT tile rows hold a few dozen remainder entries, or none) share one
+// item of up to kGroupTileRows tile rows, formed inside windows of
+// kGroupWindow tile rows.  Every tile row of a group item is summed by the
+// same flat pass whether it is grouped with its neighbours or alone, so the
+// grouping never changes a bit of y (shard invariance).
+constexpr int kGroupTileRows = 16;
+constexpr int kGroupWindow = 64;
 
 // Compact per-item record read by the warp kernel (built with the blobs):
 // blob start, tile row, split bookkeeping, and the blob's part offsets.
@@ -52,7 +63,7 @@ struct __align__(16) WItem {
     uint32_t I;         // tile row
     int32_t split;      // split-row index or -1
     int32_t part_nt;    // as Item::part_nt
-    uint32_t jt_rows_pay;  // (unused, 8 bits) | rows in the tile row (5 bits) << 8 | payload offset << 16
+    uint32_t jt_rows_pay;  // tile rows of a row-group item (8 bits, 0: ordinary) | rows in the (last) tile row (5 bits) << 8 | payload offset << 16
     uint32_t rp_col;       // rp offset | col offset << 16
     uint32_t val_tot;      // val offset | total bytes << 16
     uint32_t groups;       // tile pairs per format f, 4 bits at 4f (descriptor list order)
@@ -75,6 +86,11 @@ struct __align__(16) WFirst {
 // sums the group partials in group order.  Everything depends only on the
 // row's own content (deterministic, shard-invariant).
 constexpr int kLocalParts = 8;
+// per-item fixed cost (bytes-equivalent of an item's latency chain: record,
+// blob, x gathers) used to balance the warps' item chunks; measured on R-MAT
+// (power-law, many small items): 2048 gives 174 us against 188 us for 512,
+// neutral on the stencil and mixed matrices
+constexpr int64_t kItemFixedCost = 2048;
 __host__ __device__ __forceinline__ int item_nt(const Item &it) { return (it.part_nt >> 24) & 31; }
 __host__ __device__ __forceinline__ int item_part(const Item &it) { return it.part_nt & 0xFFFFFF; }
 __host__ __device__ __forceinline__ bool item_local(const Item &it) { return (it.part_nt >> 29) & 1; }
@@ -116,7 +132,10 @@ struct Matrix {
     int32_t *jcols = nullptr;      // 16 tile columns per item (warp kernel)
     WFirst *wfirst = nullptr;      // per-warp chunk + first item (warp kernel)
     int64_t blob_bytes = 0;
-    int64_t *cta_begin = nullptr;  // contiguous item chunk per warp (row-aligned, cost-balanced)
+    int64_t *cta_begin = nullptr;  // contiguous item chunk per warp (row-aligned, cost-balanced),
+                                   // or unit range per CTA (SM-queue kernel)
+    int32_t *units = nullptr;      // SM-queue kernel: first item of each unit, num_units + 1
+    int64_t num_units = 0;
     // launch shape
     int kernel_version = 20;
     const char *kernel_name = "";

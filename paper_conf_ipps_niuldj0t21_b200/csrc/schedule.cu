@@ -76,6 +76,7 @@ __device__ int items_for_row(int64_t I, const int32_t *tilePtr, const uint32_t *
             it.ndsc = 0;
             it.blob16 = 0;
             it.blob_len = 0;
+            it.ntr = 0;
             out[cnt] = it;
         }
         cnt++;
@@ -93,15 +94,80 @@ __global__ void k_items_count(const int32_t *tilePtr, const uint32_t *tileOff, c
     parts[I] = c > 1 ? c : 0;
 }
 
-__global__ void k_items_write(const int32_t *tilePtr, const uint32_t *tileOff, const int32_t *remRowPtr, int64_t m,
-                              int budget, int64_t tilem, const int32_t *itemBase, const int32_t *splitId, const int32_t *nitems,
-                              const int32_t *partBase, Item *items, int2 *split_info) {
-    int64_t I = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
-    if (I >= tilem) return;
-    const bool split = nitems[I] > 1;
-    const int sid = split ? splitId[I] : -1;
-    items_for_row<true>(I, tilePtr, tileOff, remRowPtr, m, budget, items + itemBase[I], sid, nitems[I]);
-    if (split) split_info[sid] = make_int2(partBase[I], nitems[I]);
+// a tile row that may join a row-group item: no stored tile, one item
+__device__ __forceinline__ bool groupable(int64_t I, const int32_t *tilePtr, const int32_t *nitems) {
+    return tilePtr[I + 1] == tilePtr[I] && nitems[I] == 1;
+}
+
+// The items of window w (kGroupWindow tile rows) in tile-row order: ordinary
+// tile rows give their items_for_row items; runs of groupable tile rows are
+// packed greedily into row-group items (<= kGroupTileRows tile rows, blob
+// within budget).  group = false: no row-group items (kernels without them).
+template <bool WRITE>
+__device__ int window_items(int64_t w, const int32_t *tilePtr, const uint32_t *tileOff, const int32_t *remRowPtr,
+                            int64_t m, int budget, int64_t tilem, bool group, const int32_t *nitems,
+                            const int32_t *splitId, Item *out) {
+    const int64_t I0 = w * kGroupWindow, I1 = imin64(I0 + kGroupWindow, tilem);
+    int cnt = 0;
+    int64_t I = I0;
+    while (I < I1) {
+        if (!group || !groupable(I, tilePtr, nitems)) {
+            if (WRITE) items_for_row<true>(I, tilePtr, tileOff, remRowPtr, m, budget, out + cnt,
+                                           nitems[I] > 1 ? splitId[I] : -1, nitems[I]);
+            cnt += nitems[I];
+            ++I;
+            continue;
+        }
+        int64_t J = I;
+        int R = 0;
+        while (J < I1 && R < kGroupTileRows && groupable(J, tilePtr, nitems)) {
+            const int64_t rows = imin64(16 * (int64_t)(R + 1), m - 16 * I);
+            const uint32_t e = remRowPtr ? (uint32_t)(remRowPtr[imin64(16 * (J + 1), m)] - remRowPtr[16 * I]) : 0u;
+            const uint32_t bytes = e ? up16(4u * (uint32_t)(rows + 1)) + up16(4u * e) + up16(8u * e) : 0u;
+            if (R > 0 && bytes + 64u > (uint32_t)budget) break;
+            ++R;
+            ++J;
+        }
+        if (WRITE) {
+            Item it;
+            it.I = (int32_t)I;
+            it.tb = tilePtr[I];
+            it.kb = remRowPtr ? remRowPtr[16 * I] : 0;
+            it.ke = remRowPtr ? remRowPtr[imin64(16 * J, m)] : 0;
+            it.offb = it.offe = tileOff[it.tb];
+            it.split = -1;
+            it.part_nt = 0;
+            it.dbeg = it.ndsc = 0;
+            it.blob16 = it.blob_len = 0;
+            it.ntr = R;
+            out[cnt] = it;
+        }
+        ++cnt;
+        I = J;
+    }
+    return cnt;
+}
+
+__global__ void k_window_count(const int32_t *tilePtr, const uint32_t *tileOff, const int32_t *remRowPtr, int64_t m,
+                               int budget, int64_t tilem, int group, const int32_t *nitems, int64_t nwin,
+                               int32_t *wcount) {
+    const int64_t w = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (w >= nwin) return;
+    wcount[w] = window_items<false>(w, tilePtr, tileOff, remRowPtr, m, budget, tilem, group != 0, nitems, nullptr,
+                                    nullptr);
+}
+
+__global__ void k_window_write(const int32_t *tilePtr, const uint32_t *tileOff, const int32_t *remRowPtr, int64_t m,
+                               int budget, int64_t tilem, int group, const int32_t *nitems, int64_t nwin,
+                               const int32_t *wbase, const int32_t *splitId, const int32_t *partBase, Item *items,
+                               int2 *split_info) {
+    const int64_t w = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (w >= nwin) return;
+    window_items<true>(w, tilePtr, tileOff, remRowPtr, m, budget, tilem, group != 0, nitems, splitId,
+                       items + wbase[w]);
+    const int64_t I1 = imin64((w + 1) * kGroupWindow, tilem);
+    for (int64_t I = w * kGroupWindow; I < I1; ++I)
+        if (nitems[I] > 1) split_info[splitId[I]] = make_int2(partBase[I], nitems[I]);
 }
 
 // Per-item tile-descriptor list: the item's tiles grouped by format (format
@@ -176,8 +242,9 @@ __global__ void k_blob_fill(Item *items, int64_t n, int64_t m, const int64_t *st
         w.I = (uint32_t)it.I;
         w.split = it.split;
         w.part_nt = it.part_nt;
-        const uint32_t rows = (uint32_t)imin64(16, m - 16 * (int64_t)it.I);
-        w.jt_rows_pay = (rows << 8) | (b.pay << 16);
+        const uint32_t rows = (uint32_t)item_rows(it, m);
+        const uint32_t last = it.ntr > 0 ? rows - 16u * (uint32_t)(it.ntr - 1) : rows;
+        w.jt_rows_pay = (uint32_t)it.ntr | (last << 8) | (b.pay << 16);
         w.rp_col = b.rp | (b.col << 16);
         w.val_tot = b.val | (b.total << 16);
         int cnt[7] = {0, 0, 0, 0, 0, 0, 0};
@@ -208,12 +275,12 @@ __global__ void k_blob_fill(Item *items, int64_t n, int64_t m, const int64_t *st
     uint4 *pd = reinterpret_cast<uint4 *>(dst + b.pay);
     for (uint32_t i = lane; i < it.offe - it.offb; i += 32) pd[i] = ps[i];
     if (it.ke > it.kb) {
-        const int rows = (int)imin64(16, m - 16 * (int64_t)it.I);
+        const int rows = (int)item_rows(it, m);
         int32_t *rp = reinterpret_cast<int32_t *>(dst + b.rp);
-        if (lane <= rows) {
-            int v = remRowPtr[16 * (int64_t)it.I + lane];
+        for (int i = lane; i <= rows; i += 32) {
+            int v = remRowPtr[16 * (int64_t)it.I + i];
             v = v < it.kb ? it.kb : (v > it.ke ? it.ke : v);
-            rp[lane] = v - it.kb;
+            rp[i] = v - it.kb;
         }
         int32_t *cd = reinterpret_cast<int32_t *>(dst + b.col);
         unsigned long long *vd = reinterpret_cast<unsigned long long *>(dst + b.val);
@@ -226,11 +293,11 @@ __global__ void k_blob_fill(Item *items, int64_t n, int64_t m, const int64_t *st
 }
 
 // item cost for the CTA chunking: bytes staged + a fixed per-item overhead
-__global__ void k_item_cost(const Item *items, int64_t n, int64_t m, int64_t *cost) {
+__global__ void k_item_cost(const Item *items, int64_t n, int64_t m, int64_t fixed, int64_t *cost) {
     int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     if (k >= n) return;
     const Item it = items[k];
-    cost[k] = (int64_t)item_parts(it, m).total + 40 * (item_nt(it)) + 512;
+    cost[k] = (int64_t)item_parts(it, m).total + 40 * (item_nt(it)) + fixed;
 }
 
 __global__ void k_warp_first(const int64_t *begin, const WItem *witems, const int32_t *jcols, int W, WFirst *wf) {
@@ -272,6 +339,47 @@ __global__ void k_cta_begin(const int64_t *incl, const Item *items, int64_t n, i
     cta_begin[b] = lo;
 }
 
+// units of the SM-queue kernel: an item that is not an inner part of a group
+// of parts starts a unit
+__global__ void k_unit_flags(const Item *items, int64_t n, int32_t *flag) {
+    const int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (k >= n) return;
+    const Item it = items[k];
+    flag[k] = (it.split < 0 || item_part(it) % kLocalParts == 0) ? 1 : 0;
+}
+
+__global__ void k_unit_write(const int32_t *flag, const int32_t *pos, int64_t n, int32_t *units) {
+    const int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (k > n) return;
+    if (k == n) {
+        units[pos[n]] = (int32_t)n;
+        return;
+    }
+    if (flag[k]) units[pos[k]] = (int32_t)k;
+}
+
+// per-CTA unit ranges balanced by the inclusive item-cost prefix: CTA b
+// starts at the first unit whose cost-before reaches total * b / G
+__global__ void k_cta_units(const int64_t *incl, const int32_t *units, int64_t nu, int64_t n, int G,
+                            int64_t *cta_begin) {
+    const int b = blockIdx.x * blockDim.x + threadIdx.x;
+    if (b > G) return;
+    if (b == G) {
+        cta_begin[b] = nu;
+        return;
+    }
+    const int64_t total = n ? incl[n - 1] : 0;
+    const int64_t target = total * b / G;
+    int64_t lo = 0, hi = nu;
+    while (lo < hi) {
+        const int64_t mid = (lo + hi) / 2;
+        const int64_t before = units[mid] ? incl[units[mid] - 1] : 0;
+        if (before < target) lo = mid + 1;
+        else hi = mid;
+    }
+    cta_begin[b] = lo;
+}
+
 template <class F>
 int scan(F &&f) {
     size_t bytes = 0;
@@ -296,19 +404,25 @@ int build_schedule(Matrix &M, cudaStream_t st) {
     const int64_t T = M.tilem;
     if (T == 0) return 0;
     auto blocks = [&](int64_t n) { return (unsigned)std::max<int64_t>(1, (n + TB - 1) / TB); };
+    const int64_t NW = (T + kGroupWindow - 1) / kGroupWindow;
+    // row-group items only for the kernels that run them (compute_item)
+    const int group = M.kernel_version != 1 && !getenv("TILESPMV_NO_GROUPS");
     int32_t *buf = nullptr;
-    TSP_CK(cudaMalloc(&buf, 6 * (T + 1) * sizeof(int32_t)));
-    int32_t *nitems = buf, *nsplit = buf + (T + 1), *parts = buf + 2 * (T + 1), *itemBase = buf + 3 * (T + 1),
-            *splitId = buf + 4 * (T + 1), *partBase = buf + 5 * (T + 1);
+    TSP_CK(cudaMalloc(&buf, (5 * (T + 1) + 2 * (NW + 1)) * sizeof(int32_t)));
+    int32_t *nitems = buf, *nsplit = buf + (T + 1), *parts = buf + 2 * (T + 1), *splitId = buf + 3 * (T + 1),
+            *partBase = buf + 4 * (T + 1), *wcount = buf + 5 * (T + 1), *wbase = wcount + (NW + 1);
     int rc = 0;
     do {
-        if (cudaMemsetAsync(buf, 0, 3 * (T + 1) * sizeof(int32_t), st) != cudaSuccess) { rc = cuda_status(cudaGetLastError(), "memset"); break; }
+        if (cudaMemsetAsync(buf, 0, 3 * (T + 1) * sizeof(int32_t), st) != cudaSuccess ||
+            cudaMemsetAsync(wcount, 0, (NW + 1) * sizeof(int32_t), st) != cudaSuccess) { rc = cuda_status(cudaGetLastError(), "memset"); break; }
         k_items_count<<<blocks(T), TB, 0, st>>>(M.tilePtr, M.tileOff, M.remRowPtr, M.m, M.item_bytes, T, nitems, nsplit, parts);
-        if ((rc = scan([&](void *t, size_t &b) { return cub::DeviceScan::ExclusiveSum(t, b, nitems, itemBase, (int)(T + 1), st); }))) break;
+        k_window_count<<<blocks(NW), TB, 0, st>>>(M.tilePtr, M.tileOff, M.remRowPtr, M.m, M.item_bytes, T, group, nitems,
+                                                   NW, wcount);
+        if ((rc = scan([&](void *t, size_t &b) { return cub::DeviceScan::ExclusiveSum(t, b, wcount, wbase, (int)(NW + 1), st); }))) break;
         if ((rc = scan([&](void *t, size_t &b) { return cub::DeviceScan::ExclusiveSum(t, b, nsplit, splitId, (int)(T + 1), st); }))) break;
         if ((rc = scan([&](void *t, size_t &b) { return cub::DeviceScan::ExclusiveSum(t, b, parts, partBase, (int)(T + 1), st); }))) break;
         int32_t h[3];
-        cudaMemcpyAsync(&h[0], itemBase + T, 4, cudaMemcpyDeviceToHost, st);
+        cudaMemcpyAsync(&h[0], wbase + NW, 4, cudaMemcpyDeviceToHost, st);
         cudaMemcpyAsync(&h[1], splitId + T, 4, cudaMemcpyDeviceToHost, st);
         cudaMemcpyAsync(&h[2], partBase + T, 4, cudaMemcpyDeviceToHost, st);
         if (cudaStreamSynchronize(st) != cudaSuccess) { rc = cuda_status(cudaGetLastError(), "schedule sizes"); break; }
@@ -324,9 +438,9 @@ int build_schedule(Matrix &M, cudaStream_t st) {
         }
         M.device_bytes += M.num_items * (int64_t)sizeof(Item) + M.num_split * 12 + nparts * 128;
         cudaMemsetAsync(M.counters, 0, std::max<int64_t>(M.num_split, 1) * sizeof(int32_t), st);
-        k_items_write<<<blocks(T), TB, 0, st>>>(M.tilePtr, M.tileOff, M.remRowPtr, M.m, M.item_bytes, T, itemBase, splitId, nitems,
-                                                partBase, M.items, M.split_info);
-        if (cudaStreamSynchronize(st) != cudaSuccess) rc = cuda_status(cudaGetLastError(), "k_items_write");
+        k_window_write<<<blocks(NW), TB, 0, st>>>(M.tilePtr, M.tileOff, M.remRowPtr, M.m, M.item_bytes, T, group, nitems,
+                                                   NW, wbase, splitId, partBase, M.items, M.split_info);
+        if (cudaStreamSynchronize(st) != cudaSuccess) rc = cuda_status(cudaGetLastError(), "k_window_write");
     } while (0);
     cudaFree(buf);
     return rc;
@@ -391,17 +505,69 @@ int build_tdesc(Matrix &M, cudaStream_t st) {
 }
 
 int choose_kernel(Matrix &M) {
-    // default: the warp kernel with 4.5 KB slots (32 warps/SM); matrices whose
-    // tile rows average more than 6 KB of payload (dense, FEM-like) use 10.5 KB
-    // slots (16 warps/SM) so a tile row stays one item.  (Measured on C2 with
-    // graph-replayed launches: 6.9 us for <4,10752> against 7.6 us for the
-    // default and 8.8 us for the double-buffered warp2<4,6016>.)
+    // default: the SM-queue kernel (one CTA of 32 warps per SM, 4.5 KB slots,
+    // warps claim units from a shared-memory counter); matrices whose tile
+    // rows average more than 6 KB of payload (dense, FEM-like) use the warp
+    // kernel with 10.5 KB slots (16 warps/SM) so a tile row stays one item.
+    // Measured (graph-replayed launches, profiles/): C5 498 us (sm<32,4608>)
+    // vs 512 us (warp<8,4608>); R-MAT 145 vs 163 us; mixed 113 vs 116 us;
+    // C2 6.9 us for warp<4,10752> vs 7.5 us for sm<16,10752>.
     const double row_bytes = M.tilem ? (double)M.payload_bytes / (double)M.tilem : 0.0;
-    int version = row_bytes > 6144.0 ? 25 : 20;
+    int version = row_bytes > 6144.0 ? 25 : 40;
     if (const char *e = getenv("TILESPMV_KERNEL")) version = atoi(e);
     M.kernel_version = version;
     M.item_bytes = choose(version).slot_bytes;
     return 0;
+}
+
+// SM-queue kernel: units (items, or whole groups of parts) and a
+// contiguous, cost-balanced unit range per CTA
+static int configure_sm_queue(Matrix &M, int G) {
+    M.grid = G;
+    const int64_t n = M.num_items;
+    if (M.cta_begin) cudaFree(M.cta_begin);
+    if (M.units) cudaFree(M.units);
+    M.cta_begin = nullptr;
+    M.units = nullptr;
+    TSP_CK(cudaMalloc(&M.cta_begin, (G + 1) * sizeof(int64_t)));
+    TSP_CK(cudaMalloc(&M.units, (n + 1) * sizeof(int32_t)));
+    M.device_bytes += (G + 1) * 8 + (n + 1) * 4;
+    if (n == 0) {
+        TSP_CK(cudaMemset(M.cta_begin, 0, (G + 1) * sizeof(int64_t)));
+        TSP_CK(cudaMemset(M.units, 0, sizeof(int32_t)));
+        M.num_units = 0;
+        return 0;
+    }
+    int64_t *cost = nullptr;
+    int32_t *flag = nullptr;
+    TSP_CK(cudaMalloc(&cost, 2 * n * sizeof(int64_t)));
+    if (cudaMalloc(&flag, 2 * (n + 1) * sizeof(int32_t)) != cudaSuccess) {
+        cudaFree(cost);
+        return cuda_status(cudaGetLastError(), "cudaMalloc(unit flags)");
+    }
+    int32_t *pos = flag + (n + 1);
+    int64_t *incl = cost + n;
+    int rc = 0;
+    do {
+        int64_t fixed = kItemFixedCost;
+        if (const char *e = getenv("TILESPMV_ITEM_COST")) fixed = atoll(e);
+        const unsigned nb = (unsigned)((n + 1 + 255) / 256);
+        k_item_cost<<<nb, 256>>>(M.items, n, M.m, fixed, cost);
+        if ((rc = scan([&](void *t, size_t &b) { return cub::DeviceScan::InclusiveSum(t, b, cost, incl, (int)n); }))) break;
+        cudaMemset(flag + n, 0, sizeof(int32_t));
+        k_unit_flags<<<nb, 256>>>(M.items, n, flag);
+        if ((rc = scan([&](void *t, size_t &b) { return cub::DeviceScan::ExclusiveSum(t, b, flag, pos, (int)(n + 1)); }))) break;
+        int32_t nu = 0;
+        cudaMemcpy(&nu, pos + n, 4, cudaMemcpyDeviceToHost);
+        M.num_units = nu;
+        k_unit_write<<<nb, 256>>>(flag, pos, n, M.units);
+        k_cta_units<<<(G + 1 + 255) / 256, 256>>>(incl, M.units, nu, n, G, M.cta_begin);
+        cudaError_t e = cudaDeviceSynchronize();
+        if (e != cudaSuccess) rc = cuda_status(e, "k_cta_units");
+    } while (0);
+    cudaFree(cost);
+    cudaFree(flag);
+    return rc;
 }
 
 int configure_launch(Matrix &M) {
@@ -422,6 +588,7 @@ int configure_launch(Matrix &M) {
         M.grid = (int)std::max<int64_t>(1, std::min<int64_t>(need, (int64_t)sms * per_sm));
         return 0;
     }
+    if (kc.sm_queue) return configure_sm_queue(M, sms * per_sm);
     // warp kernel: persistent grid, one contiguous, cost-balanced, row-aligned
     // item chunk per warp
     const int64_t need = (M.num_items + warps - 1) / warps;
@@ -435,7 +602,10 @@ int configure_launch(Matrix &M) {
         int64_t *cost = nullptr;
         TSP_CK(cudaMalloc(&cost, 2 * M.num_items * sizeof(int64_t)));
         int64_t *incl = cost + M.num_items;
-        k_item_cost<<<(unsigned)((M.num_items + 255) / 256), 256>>>(M.items, M.num_items, M.m, cost);
+        // TILESPMV_ITEM_COST overrides the per-item fixed cost for sweeps
+        int64_t fixed = kItemFixedCost;
+        if (const char *e = getenv("TILESPMV_ITEM_COST")) fixed = atoll(e);
+        k_item_cost<<<(unsigned)((M.num_items + 255) / 256), 256>>>(M.items, M.num_items, M.m, fixed, cost);
         int rc = scan([&](void *t, size_t &b) { return cub::DeviceScan::InclusiveSum(t, b, cost, incl, (int)M.num_items); });
         if (!rc) {
             k_cta_begin<<<(W + 1 + 255) / 256, 256>>>(incl, M.items, M.num_items, W, M.cta_begin);
@@ -484,6 +654,7 @@ int launch_spmv(const Matrix &M, const double *d_x, double *d_y, cudaStream_t st
     p.wfirst = M.wfirst;
     p.cta_begin = M.cta_begin;
     p.x_vec = (reinterpret_cast<uintptr_t>(d_x) & 15u) == 0;
+    p.units = M.units;
     const KernelChoice kc = choose(M.kernel_version);
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3(M.grid);

@@ -34,6 +34,7 @@ struct Params {
     const WFirst *wfirst;      // per-warp chunk and first item (warp kernel)
     const int64_t *cta_begin;  // warp kernel: item chunk of each warp
     int x_vec;                 // x is 16-byte aligned: x segments load as double2
+    const int32_t *units;      // SM-queue kernel: first item of each unit (+ end), see schedule.cu
 };
 
 // ------------------------------------------------------------------ PTX ----
@@ -96,13 +97,18 @@ struct ItemParts {
     uint32_t dsc_skew, col_skew, val_skew;
 };
 
+// rows the item's remainder row pointers cover
+__host__ __device__ __forceinline__ int64_t item_rows(const Item &it, int64_t m) {
+    return imin64(it.ntr > 0 ? 16 * (int64_t)it.ntr : 16, m - 16 * (int64_t)it.I);
+}
+
 __host__ __device__ __forceinline__ ItemParts item_parts(const Item &it, int64_t m) {
     ItemParts r;
     r.pay = (it.offe - it.offb) * 16u;
     r.dsc_skew = (uint32_t)(it.dbeg & 1) * 8u;
     r.dsc = it.ndsc ? up16(r.dsc_skew + 8u * (uint32_t)it.ndsc) : 0u;
     if (it.ke > it.kb) {
-        const int64_t rows = imin64(16, m - 16 * (int64_t)it.I);
+        const int64_t rows = item_rows(it, m);
         r.rp = up16((uint32_t)(rows + 1) * 4u);
         r.col_skew = ((uint32_t)it.kb * 4u) & 15u;
         r.col = up16(r.col_skew + 4u * (uint32_t)(it.ke - it.kb));
@@ -132,7 +138,7 @@ __host__ __device__ __forceinline__ BlobParts blob_parts(const Item &it, int64_t
     b.pay = up16(8u * (uint32_t)it.ndsc);
     b.rp = b.pay + (it.offe - it.offb) * 16u;
     if (it.ke > it.kb) {
-        const uint32_t rows = (uint32_t)imin64(16, m - 16 * (int64_t)it.I);
+        const uint32_t rows = (uint32_t)item_rows(it, m);
         const uint32_t e = (uint32_t)(it.ke - it.kb);
         b.col = b.rp + up16(4u * (rows + 1));
         b.val = b.col + up16(4u * e);
@@ -235,6 +241,7 @@ struct KernelChoice {
     bool ring;       // one CTA per SM with cta_begin chunks (no current kernel)
     int slot_bytes;  // item budget the schedule must respect
     bool pdl;        // launched with programmatic dependent launch (kernel waits on griddepcontrol)
+    bool sm_queue;   // one CTA per SM; its warps claim units from a shared-memory counter
 };
 KernelChoice kernel_v1();
 KernelChoice kernel_warp(int variant);

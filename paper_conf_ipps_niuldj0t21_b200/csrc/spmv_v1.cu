@@ -272,7 +272,7 @@ __global__ void __launch_bounds__(kWarps * 32) tilespmv_fp64_kernel(const Params
 }  // namespace
 
 KernelChoice kernel_v1() {
-    return {"v1_warp_staged", tilespmv_fp64_kernel, kWarps * 32, kSmemBytes, 0, false, kItemBytesMax, false};
+    return {"v1_warp_staged", tilespmv_fp64_kernel, kWarps * 32, kSmemBytes, 0, false, kItemBytesMax, false, false};
 }
 
 }  // namespace tsp

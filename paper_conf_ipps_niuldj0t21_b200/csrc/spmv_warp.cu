@@ -19,6 +19,33 @@
 #include "spmv_tiles.cuh"
 
 namespace tsp {
+
+#ifdef TSP_TRACE
+// development build only (scripts/trace_items.py): %globaltimer stamps of the
+// first kTraceItems items of every warp: start, blob landed, item info, end
+constexpr int kTraceItems = 192;
+__device__ unsigned long long *g_trace = nullptr;
+__device__ __forceinline__ unsigned long long gtimer() {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+    return t;
+}
+#define TSP_STAMP(gw, j, slot) \
+    do { if (g_trace && lane == 0 && (j) < kTraceItems) g_trace[((size_t)(gw) * kTraceItems + (j)) * 4 + (slot)] = gtimer(); } while (0)
+// item k, blob bytes, row-group tile rows, tiles
+#define TSP_INFO(gw, j, k, it) \
+    do { if (g_trace && lane == 0 && (j) < kTraceItems) g_trace[((size_t)(gw) * kTraceItems + (j)) * 4 + 2] = \
+        ((unsigned long long)(k) << 32) | ((it).val_tot & 0xFFFF0000u) | (((it).jt_rows_pay & 0xFFu) << 8) | (((it).part_nt >> 24) & 31u); } while (0)
+// the warp's SM, after the item stamps
+#define TSP_SMID(gw, nw) \
+    do { if (g_trace && lane == 0) { unsigned sm; asm volatile("mov.u32 %0, %smid;" : "=r"(sm)); \
+         g_trace[(size_t)(nw) * kTraceItems * 4 + (gw)] = sm; } } while (0)
+#else
+#define TSP_STAMP(gw, j, slot) do { } while (0)
+#define TSP_INFO(gw, j, k, it) do { } while (0)
+#define TSP_SMID(gw, nw) do { } while (0)
+#endif
+
 namespace {
 
 template <int WARPS, int SLOT, int NBUF = 1>
@@ -42,84 +69,177 @@ __device__ __forceinline__ WItem load_witem(const WItem *w, int k) {
 }
 
 // fused CSR remainder of the item's rows; adds row sums into acc of
-// lane r (and r + 16).  rpS: rebased row pointers (rows + 1), colS/valS: entries
+// lane r (and r + 16).  rpS: rebased row pointers (rows + 1), colS/valS: entries.
+//  * every row <= 4 entries (stencil-like): two lanes per row, two entries
+//    each, one round trip of gathers;
+//  * otherwise rows of <= kShortRow entries run two lanes per row, all at
+//    once, and the longer rows (power-law hubs) a half-warp per row, two rows
+//    at a time (the whole warp when one is left), four entries per lane in
+//    flight, summed by an xor-shuffle tree.
+// The order of every sum depends only on the item's content: y stays bitwise
+// deterministic.
 __device__ __forceinline__ void remainder(const Params &p, uint32_t rpS, uint32_t colS, uint32_t valS, int rows,
-                                          uint32_t racc, uint64_t x_policy, int lane, double &acc) {
+                                          uint64_t x_policy, int lane, double &acc) {
     const int r = lane & 15, h = lane >> 4;
     const int b = lds_s32(rpS + 4 * min(r, rows)), e = lds_s32(rpS + 4 * min(r + 1, rows));
-    const bool is_short = e - b <= kShortRow;
-    if (!__any_sync(FULL, !is_short)) {
-        // two lanes per row, entries b + h, b + h + 2, ...; warp-uniform trip
-        // count, two entries per step.  A masked entry reads column 0 and
-        // value 0.0 (x[0] exists whenever the item has remainder entries).
-        const int trips = (int)__reduce_max_sync(FULL, (unsigned)((e - b + 1 - h) >> 1));
-        const double *x = p.x;
+    const double *x = p.x;
+    const int maxlen = (int)__reduce_max_sync(FULL, (unsigned)(e - b));
+    if (maxlen <= 4) {
+        // entries b + h and b + h + 2 of row r; a masked entry reads column 0
+        // and value 0.0 (x[0] exists whenever the item has remainder entries)
+        const int k0 = b + h, k1 = k0 + 2;
+        int c0, c1;
+        double v0, v1;
+        lds_entry_lt(k0, e, colS + 4 * k0, valS + 8 * k0, c0, v0);
+        lds_entry_lt(k1, e, colS + 4 * k1, valS + 8 * k1, c1, v1);
+        const double x0 = ldg_hint(x + (uint32_t)c0, x_policy), x1 = ldg_hint(x + (uint32_t)c1, x_policy);
+        acc = fma(v0, x0, acc);
+        acc = fma(v1, x1, acc);
+        return;
+    }
+    const bool lng = e - b > kShortRow;
+    {
+        const int ee = lng ? b : e;
+        const int trips = (int)__reduce_max_sync(FULL, (unsigned)((ee - b + 1 - h) >> 1));
 #pragma unroll 1
         for (int i = 0; i < trips; i += 2) {
             const int k0 = b + h + 2 * i, k1 = k0 + 2;
             int c0, c1;
             double v0, v1;
-            lds_entry_lt(k0, e, colS + 4 * k0, valS + 8 * k0, c0, v0);
-            lds_entry_lt(k1, e, colS + 4 * k1, valS + 8 * k1, c1, v1);
+            lds_entry_lt(k0, ee, colS + 4 * k0, valS + 8 * k0, c0, v0);
+            lds_entry_lt(k1, ee, colS + 4 * k1, valS + 8 * k1, c1, v1);
             const double x0 = ldg_hint(x + (uint32_t)c0, x_policy), x1 = ldg_hint(x + (uint32_t)c1, x_policy);
             acc = fma(v0, x0, acc);
             acc = fma(v1, x1, acc);
         }
-        return;
     }
-    // a long row: every entry in one flat pass, one lane per entry, gathers
-    // batched four chunks deep, rows summed by a segmented shuffle scan
-    const int etot = lds_s32(rpS + 4 * rows);
-    if (lane < 16) sts_f64(racc + 8 * lane, 0.0);
-    __syncwarp();
+    // long rows: lanes 0-15 of the ballot = rows 0-15
+    uint32_t lm = __ballot_sync(FULL, lng && h == 0 && r < rows);
 #pragma unroll 1
-    for (int k0 = 0; k0 < etot; k0 += 128) {
-        double pv[4];
-        int rw[4];
-        bool okv[4];
-#pragma unroll
-        for (int i = 0; i < 4; ++i) {
-            const int kq = k0 + 32 * i + lane;
-            okv[i] = kq < etot;
-            const int c = okv[i] ? lds_s32(colS + 4 * kq) : 0;
-            const double v = lds_f64(valS + 8 * (okv[i] ? kq : 0));
-            pv[i] = okv[i] ? v * ldg_hint(p.x + (uint32_t)c, x_policy) : 0.0;
+    while (lm) {
+        const int r0 = __ffs(lm) - 1;
+        lm &= lm - 1;
+        const int r1 = lm ? __ffs(lm) - 1 : -1;
+        if (lm) lm &= lm - 1;
+        const bool pair = r1 >= 0;  // warp-uniform
+        const int myrow = (pair && h) ? r1 : r0;
+        const int off = pair ? r : lane, stride = pair ? 16 : 32;
+        const int bb = lds_s32(rpS + 4 * myrow), e2 = lds_s32(rpS + 4 * myrow + 4);
+        const int t2 = (int)__reduce_max_sync(FULL, (unsigned)((e2 - bb + 4 * stride - 1) / (4 * stride)));
+        double s0 = 0.0, s1 = 0.0, s2 = 0.0, s3 = 0.0;
+#pragma unroll 1
+        for (int t = 0; t < t2; ++t) {
+            const int k = bb + off + 4 * stride * t;
+            int c0, c1, c2, c3;
+            double v0, v1, v2, v3;
+            lds_entry_lt(k, e2, colS + 4 * k, valS + 8 * k, c0, v0);
+            lds_entry_lt(k + stride, e2, colS + 4 * (k + stride), valS + 8 * (k + stride), c1, v1);
+            lds_entry_lt(k + 2 * stride, e2, colS + 4 * (k + 2 * stride), valS + 8 * (k + 2 * stride), c2, v2);
+            lds_entry_lt(k + 3 * stride, e2, colS + 4 * (k + 3 * stride), valS + 8 * (k + 3 * stride), c3, v3);
+            s0 = fma(v0, ldg_hint(x + (uint32_t)c0, x_policy), s0);
+            s1 = fma(v1, ldg_hint(x + (uint32_t)c1, x_policy), s1);
+            s2 = fma(v2, ldg_hint(x + (uint32_t)c2, x_policy), s2);
+            s3 = fma(v3, ldg_hint(x + (uint32_t)c3, x_policy), s3);
         }
-#pragma unroll
-        for (int i = 0; i < 4; ++i) {  // row of entry kq: rp[row] <= kq < rp[row + 1]
-            const int kq = k0 + 32 * i + lane;
-            int lo = 0, hi = rows;
-#pragma unroll
-            for (int st = 0; st < 5; ++st) {
-                const int mid = (lo + hi) >> 1;
-                if (hi - lo > 1) {
-                    if (lds_s32(rpS + 4 * mid) <= kq) lo = mid;
-                    else hi = mid;
-                }
-            }
-            rw[i] = lo;
-        }
-#pragma unroll
-        for (int d = 1; d < 32; d <<= 1) {
-#pragma unroll
-            for (int i = 0; i < 4; ++i) {
-                const double t = __shfl_up_sync(FULL, pv[i], d);
-                const int rr = __shfl_up_sync(FULL, rw[i], d);
-                if (lane >= d && rr == rw[i]) pv[i] += t;
-            }
-        }
-#pragma unroll
-        for (int i = 0; i < 4; ++i) {  // segment tails add to their row, chunk by chunk
-            const int nr = __shfl_down_sync(FULL, rw[i], 1);
-            const int kq = k0 + 32 * i + lane;
-            if (okv[i] && (lane == 31 || nr != rw[i] || kq + 1 >= etot)) {
-                const uint32_t a = racc + 8 * rw[i];
-                sts_f64(a, lds_f64(a) + pv[i]);
-            }
-            __syncwarp();
-        }
+        double s = (s0 + s1) + (s2 + s3);
+        if (!pair) s += __shfl_xor_sync(FULL, s, 16);
+        s += __shfl_xor_sync(FULL, s, 8);
+        s += __shfl_xor_sync(FULL, s, 4);
+        s += __shfl_xor_sync(FULL, s, 2);
+        s += __shfl_xor_sync(FULL, s, 1);
+        if (pair ? r == myrow : lane == r0) acc += s;
     }
-    if (lane < 16) acc += lds_f64(racc + 8 * lane);
+}
+
+// Row-group item (internal.cuh): ntr consecutive tile rows without stored
+// tiles, only remainder rows.  1. one lane per entry, the x gathers of
+// 256 entries in flight at once, each value in the slot overwritten by its
+// product; 2. per tile row, the rows are summed from shared memory -- rows of
+// <= kShortRow products two lanes per row, longer rows a half-warp per row
+// (two rows at a time, the whole warp for the last one) with an xor tree --
+// and y is written once per row.  The order of every row's sum depends only on
+// its own tile row, so grouping never changes a bit of y.
+__device__ __forceinline__ void group_item(const Params &p, const WItem &it, uint32_t slot, uint64_t x_policy,
+                                           int lane) {
+    const int r = lane & 15, h = lane >> 4;
+    const int ntr = (int)(it.jt_rows_pay & 0xFFu);
+    const int rows_last = (int)((it.jt_rows_pay >> 8) & 31u);
+    const uint32_t total = it.val_tot >> 16, rp = it.rp_col & 0xFFFFu;
+    const bool has_rem = total > rp;
+    const uint32_t rpS = slot + rp, colS = slot + (it.rp_col >> 16), valS = slot + (it.val_tot & 0xFFFFu);
+    if (has_rem) {
+        const int E = lds_s32(rpS + 4 * (16 * (ntr - 1) + rows_last));
+#pragma unroll 1
+        for (int k0 = 0; k0 < E; k0 += 256) {
+            double pv[8];
+#pragma unroll
+            for (int j = 0; j < 8; ++j) {
+                const int k = k0 + 32 * j + lane;
+                int c;
+                double v;
+                lds_entry_lt(k, E, colS + 4 * k, valS + 8 * k, c, v);
+                pv[j] = __dmul_rn(v, ldg_hint(p.x + (uint32_t)c, x_policy));
+            }
+#pragma unroll
+            for (int j = 0; j < 8; ++j) {
+                const int k = k0 + 32 * j + lane;
+                if (k < E) sts_f64(valS + 8 * k, pv[j]);
+            }
+        }
+        __syncwarp();
+    }
+#pragma unroll 1
+    for (int g = 0; g < ntr; ++g) {
+        const int rows = g + 1 < ntr ? 16 : rows_last;
+        double acc = 0.0;
+        if (has_rem) {
+            const uint32_t rq = rpS + 64u * (uint32_t)g;
+            const int b = lds_s32(rq + 4 * min(r, rows)), e = lds_s32(rq + 4 * min(r + 1, rows));
+            const bool lng = e - b > kShortRow;
+            const int ee = lng ? b : e;
+            const int trips = (int)__reduce_max_sync(FULL, (unsigned)((ee - b + 1 - h) >> 1));
+            double s0 = 0.0, s1 = 0.0;
+#pragma unroll 1
+            for (int i = 0; i < trips; i += 2) {
+                const int k0 = b + h + 2 * i;
+                s0 += lds_f64_lt(k0, ee, valS + 8 * k0);
+                s1 += lds_f64_lt(k0 + 2, ee, valS + 8 * k0 + 16);
+            }
+            acc = s0 + s1;
+            uint32_t lm = __ballot_sync(FULL, lng && h == 0 && r < rows);
+#pragma unroll 1
+            while (lm) {
+                const int r0 = __ffs(lm) - 1;
+                lm &= lm - 1;
+                const int r1 = lm ? __ffs(lm) - 1 : -1;
+                if (lm) lm &= lm - 1;
+                const bool pair = r1 >= 0;  // warp-uniform
+                const int myrow = (pair && h) ? r1 : r0;
+                const int off = pair ? r : lane, stride = pair ? 16 : 32;
+                const int bb = lds_s32(rq + 4 * myrow), e2 = lds_s32(rq + 4 * myrow + 4);
+                const int t2 = (int)__reduce_max_sync(FULL, (unsigned)((e2 - bb + 4 * stride - 1) / (4 * stride)));
+                double q0 = 0.0, q1 = 0.0, q2 = 0.0, q3 = 0.0;
+#pragma unroll 1
+                for (int t = 0; t < t2; ++t) {
+                    const int k = bb + off + 4 * stride * t;
+                    q0 += lds_f64_lt(k, e2, valS + 8 * k);
+                    q1 += lds_f64_lt(k + stride, e2, valS + 8 * (k + stride));
+                    q2 += lds_f64_lt(k + 2 * stride, e2, valS + 8 * (k + 2 * stride));
+                    q3 += lds_f64_lt(k + 3 * stride, e2, valS + 8 * (k + 3 * stride));
+                }
+                double sq = (q0 + q1) + (q2 + q3);
+                if (!pair) sq += __shfl_xor_sync(FULL, sq, 16);
+                sq += __shfl_xor_sync(FULL, sq, 8);
+                sq += __shfl_xor_sync(FULL, sq, 4);
+                sq += __shfl_xor_sync(FULL, sq, 2);
+                sq += __shfl_xor_sync(FULL, sq, 1);
+                if (pair ? r == myrow : lane == r0) acc += sq;
+            }
+        }
+        acc += __shfl_xor_sync(FULL, acc, 16);
+        const int64_t row = 16 * ((int64_t)it.I + g) + lane;
+        if (lane < 16 && row < p.m) p.y[row] = acc;
+    }
 }
 
 // the tiles of one format group, two per step.  d: shared address of this
@@ -203,6 +323,11 @@ __device__ __forceinline__ void issue_x(const Params &p, int J, int nt, uint32_t
 // flight into `xs`: remainder, tiles, y (or the split-row carry)
 __device__ __forceinline__ void compute_item(const Params &p, const WItem &it, uint32_t slot, uint32_t xs,
                                              uint32_t racc, uint64_t x_policy, int lane, double &carry) {
+    if (it.jt_rows_pay & 0xFFu) {  // row-group item
+        if (p.x_vec) cp_async_wait_all();
+        group_item(p, it, slot, x_policy, lane);
+        return;
+    }
     const int h = lane >> 4, r = lane & 15;
     const uint32_t total = it.val_tot >> 16;
     // 2. fused CSR remainder
@@ -210,7 +335,7 @@ __device__ __forceinline__ void compute_item(const Params &p, const WItem &it, u
     const uint32_t rp = it.rp_col & 0xFFFFu;
     if (total > rp)
         remainder(p, slot + rp, slot + (it.rp_col >> 16), slot + (it.val_tot & 0xFFFFu),
-                  (int)((it.jt_rows_pay >> 8) & 31u), racc, x_policy, lane, acc);
+                  (int)((it.jt_rows_pay >> 8) & 31u), x_policy, lane, acc);
     if (p.x_vec) cp_async_wait_all();
     __syncwarp();
     // 3. tiles: format group by format group, two tiles per step
@@ -289,6 +414,7 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, MINB) tilespmv
     // neighbouring tile rows share x segments.  The warp's start record holds
     // the chunk and a copy of the first item (one round trip).
     const int64_t gw = (int64_t)blockIdx.x * WARPS + warp;
+    TSP_SMID(gw, (int64_t)gridDim.x * WARPS);
     const WFirst *wf = p.wfirst + gw;
     const int4 wb = __ldg(reinterpret_cast<const int4 *>(wf));
     const int kbeg = wb.x, kend = wb.y;
@@ -300,6 +426,7 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, MINB) tilespmv
     for (int k = kbeg; k < kend; ++k) {
         const WItem it = nxt;
         const int J = Jn;
+        TSP_STAMP(gw, k - kbeg, 0);
         issue_blob(p, it, slot, bar, stream_policy, lane);
         // the matrix is immutable; x and y may belong to the previous kernel
         if (k == kbeg) griddep_wait();
@@ -313,8 +440,101 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, MINB) tilespmv
             mbar_wait(bar, phase);
             phase ^= 1u;
         }
+        TSP_STAMP(gw, k - kbeg, 1);
+        TSP_INFO(gw, k - kbeg, k, it);
         compute_item(p, it, slot, xs, racc, x_policy, lane, carry);
         __syncwarp();  // slot and x scratch free for the next item
+        TSP_STAMP(gw, k - kbeg, 3);
+    }
+}
+
+// One CTA per SM (WARPS warps, one blob in flight each).  The CTA owns a
+// contiguous, cost-balanced range of units (schedule.cu: a unit is one item,
+// or the items of a group of parts of a split tile row, which must run in
+// order in one warp); its warps claim units from a shared-memory counter, so
+// warps that draw slow units take fewer and all warps of the SM finish
+// together (with several CTAs per SM the hardware's oldest-first issue
+// priority leaves the youngest CTAs as a serial tail).  Each warp claims its
+// next unit when it starts one, so the claim and the unit's bounds are in
+// flight while the current unit runs.
+template <int WARPS, int SLOT>
+__global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, 1) tilespmv_fp64_sm(const Params p) {
+    using Cfg = WarpCfg<WARPS, SLOT>;
+    extern __shared__ __align__(128) uint8_t smem[];
+    __shared__ int s_next;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const uint32_t xs = smem_u32(smem) + (uint32_t)warp * Cfg::kX;
+    const uint32_t slot = smem_u32(smem) + WARPS * Cfg::kX + (uint32_t)warp * Cfg::kPer;
+    const uint32_t racc = slot + SLOT, bar = racc + 128;
+    const int ub = (int)__ldg(p.cta_begin + blockIdx.x), ue = (int)__ldg(p.cta_begin + blockIdx.x + 1);
+    if (lane == 0) {
+        mbar_init(bar, 1);
+        fence_mbar_init();
+    }
+    if (threadIdx.x == 0) s_next = ub + WARPS;  // units ub .. ub+WARPS-1 are the warps' first
+    __syncthreads();
+    griddep_launch_dependents();
+    const int64_t gw = (int64_t)blockIdx.x * WARPS + warp;
+    TSP_SMID(gw, (int64_t)gridDim.x * WARPS);
+    double carry = 0.0;  // partial row sums inside a group of parts of a split tile row
+    uint32_t phase = 0;
+    const uint64_t stream_policy = policy_evict_first(), x_policy = policy_evict_last();
+    int k = -1, ke = 0, nb = -1, ne = 0;
+    if (ub + warp < ue) {
+        k = __ldg(p.units + ub + warp);
+        ke = __ldg(p.units + ub + warp + 1);
+    }
+    int kb = k;
+    WItem nxt{};
+    int Jn = 0;
+    if (k >= 0) {
+        nxt = load_witem(p.witems, k);
+        Jn = lane < 16 ? __ldg(p.jcols + (int64_t)k * 16 + lane) : 0;
+    }
+    bool waited = false;
+    int j = 0;
+    while (k >= 0) {
+        const WItem it = nxt;
+        const int J = Jn;
+        TSP_STAMP(gw, j, 0);
+        issue_blob(p, it, slot, bar, stream_policy, lane);
+        // the matrix is immutable; x and y may belong to the previous kernel
+        if (!waited) {
+            griddep_wait();
+            waited = true;
+        }
+        if (k == kb) {  // a unit starts: claim the next one and fetch its bounds
+            int c = 0;
+            if (lane == 0) c = atomicAdd(&s_next, 1);
+            c = __shfl_sync(FULL, c, 0);
+            nb = -1;
+            if (c < ue) {
+                nb = __ldg(p.units + c);
+                ne = __ldg(p.units + c + 1);
+            }
+        }
+        // 1. x segments, issued before the blob lands (J came with the record)
+        issue_x(p, J, (it.part_nt >> 24) & 31, xs, x_policy, lane);
+        const int kn = k + 1 < ke ? k + 1 : nb;
+        if (kn >= 0) {  // the next record and its columns, in flight during this item
+            nxt = load_witem(p.witems, kn);
+            Jn = lane < 16 ? __ldg(p.jcols + (int64_t)kn * 16 + lane) : 0;
+        }
+        if (it.val_tot >> 16) {
+            mbar_wait(bar, phase);
+            phase ^= 1u;
+        }
+        TSP_STAMP(gw, j, 1);
+        TSP_INFO(gw, j, k, it);
+        compute_item(p, it, slot, xs, racc, x_policy, lane, carry);
+        __syncwarp();  // slot and x scratch free for the next item
+        TSP_STAMP(gw, j, 3);
+        ++j;
+        if (k + 1 >= ke) {
+            kb = nb;
+            ke = ne;
+        }
+        k = kn;
     }
 }
 
@@ -379,13 +599,19 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT, 2>::kThreads, MINB) tiles
 template <int WARPS, int SLOT, int MINB>
 KernelChoice warp_choice(const char *name) {
     using Cfg = WarpCfg<WARPS, SLOT>;
-    return {name, tilespmv_fp64_warp<WARPS, SLOT, MINB>, Cfg::kThreads, (int)Cfg::kSmem, 0, false, SLOT, true};
+    return {name, tilespmv_fp64_warp<WARPS, SLOT, MINB>, Cfg::kThreads, (int)Cfg::kSmem, 0, false, SLOT, true, false};
+}
+
+template <int WARPS, int SLOT>
+KernelChoice sm_choice(const char *name) {
+    using Cfg = WarpCfg<WARPS, SLOT>;
+    return {name, tilespmv_fp64_sm<WARPS, SLOT>, Cfg::kThreads, (int)Cfg::kSmem, 1, false, SLOT, true, true};
 }
 
 template <int WARPS, int SLOT, int MINB>
 KernelChoice warp2_choice(const char *name) {
     using Cfg = WarpCfg<WARPS, SLOT, 2>;
-    return {name, tilespmv_fp64_warp2<WARPS, SLOT, MINB>, Cfg::kThreads, (int)Cfg::kSmem, 0, false, SLOT, true};
+    return {name, tilespmv_fp64_warp2<WARPS, SLOT, MINB>, Cfg::kThreads, (int)Cfg::kSmem, 0, false, SLOT, true, false};
 }
 
 }  // namespace
@@ -404,8 +630,21 @@ KernelChoice kernel_warp(int variant) {
     case 32: return warp2_choice<4, 8448, 3>("tilespmv_fp64_warp2<4,8448>");
     case 33: return warp2_choice<4, 10752, 2>("tilespmv_fp64_warp2<4,10752>");
     case 34: return warp2_choice<3, 6192, 5>("tilespmv_fp64_warp2<3,6192>");
+    // one CTA per SM, shared-memory unit queue
+    case 40: return sm_choice<32, 4608>("tilespmv_fp64_sm<32,4608>");
+    case 41: return sm_choice<16, 10752>("tilespmv_fp64_sm<16,10752>");
+    case 42: return sm_choice<24, 6144>("tilespmv_fp64_sm<24,6144>");
     default: return warp_choice<8, 4608, 4>("tilespmv_fp64_warp<8,4608>");
     }
 }
 
 }  // namespace tsp
+
+#ifdef TSP_TRACE
+// development build only: point the item trace at a device buffer of
+// (warps x kTraceItems x 4) uint64 (NULL disables it)
+extern "C" int tilespmv_debug_set_trace(void *d_buf) {
+    unsigned long long *p = reinterpret_cast<unsigned long long *>(d_buf);
+    return cudaMemcpyToSymbol(tsp::g_trace, &p, sizeof(p)) == cudaSuccess ? 0 : -1;
+}
+#endif

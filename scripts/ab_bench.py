@@ -36,7 +36,12 @@ def main():
     l2 = torch.cuda.get_device_properties(0).L2_cache_size
     hs = {}
     for v in a.variants.split(","):
-        os.environ["TILESPMV_KERNEL"] = v
+        # VARIANT[@NAME=VALUE...]: kernel variant plus TILESPMV_<NAME> settings
+        kv, *envs = v.split("@")
+        os.environ["TILESPMV_KERNEL"] = kv
+        for e in envs:
+            k_, v_ = e.split("=")
+            os.environ["TILESPMV_" + k_] = v_
         M0 = T.TiledMatrix.from_host_csr(A, mode=a.mode, device=dev)
         alg = M0.info()["alg_bytes"]
         reps = max(1, int(np.ceil(4 * l2 / max(alg, 1))))
@@ -44,6 +49,8 @@ def main():
         xs = [torch.from_numpy(x).to(dev) for _ in range(reps)]
         ys = [torch.empty(A.m, dtype=torch.float64, device=dev) for _ in range(reps)]
         hs[v] = (Ms, xs, ys, alg, M0.kernel_name())
+        for e in envs:
+            os.environ.pop("TILESPMV_" + e.split("=")[0], None)
     os.environ.pop("TILESPMV_KERNEL", None)
     res = {v: [] for v in hs}
     graphs = {}

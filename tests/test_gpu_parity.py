@@ -261,7 +261,7 @@ def test_full_size_tiler_and_spmv(cuda_device, name):
         M.close()
 
 
-@pytest.mark.parametrize("variant", ["1", "20", "21", "22", "23", "24", "25", "26", "30", "31", "32", "33", "34"])
+@pytest.mark.parametrize("variant", ["1", "20", "21", "22", "23", "24", "25", "26", "30", "31", "32", "33", "34", "40", "41", "42"])
 def test_kernel_variants_parity(cuda_device, variant, monkeypatch):
     """Every SpMV kernel variant (TILESPMV_KERNEL, read at create time) meets
     the oracle tolerance; each is run-to-run bitwise deterministic."""
@@ -293,3 +293,32 @@ def test_misaligned_x_uses_scalar_path(cuda_device):
     y_mis = M.run(buf[1:]).cpu().numpy()
     y_al = M.run(torch.from_numpy(x).to(cuda_device)).cpu().numpy()
     assert np.array_equal(y_mis.view(np.uint64), y_al.view(np.uint64))
+
+
+@pytest.mark.parametrize("name", ["rmat12", "mixed_small", "stencil27_40", "lap2d_37x29", "heavy_row"])
+@pytest.mark.parametrize("mode", ["DEFERRED", "ADPT"])
+@pytest.mark.parametrize("variant", ["20", "25", "40", "41"])
+def test_row_slices_bitwise_equal_full(cuda_device, name, mode, variant, monkeypatch):
+    """Tile-row sharding relies on every row's summation order
+    depending only on its own tile row (for a given kernel variant, i.e. slot
+    size): handles built from row slices cut at arbitrary 16-row boundaries
+    (not aligned to the schedule's grouping windows) must reproduce the full
+    handle's y bit for bit."""
+    import torch
+    monkeypatch.setenv("TILESPMV_KERNEL", variant)
+    TM = tm()
+    if name == "heavy_row":
+        A = [a for a in _special() if a.name == "heavy_row"][0]
+        x = gen.dense_x(A.n, 101)
+    else:
+        A, x = gen.make(name)
+    xd = torch.from_numpy(x).to(cuda_device)
+    with TM.from_host_csr(A, mode=mode, device=cuda_device) as M:
+        yfull = M.run(xd).cpu().numpy()
+    T = (A.m + 15) // 16
+    cuts = sorted({0, A.m} | {min(A.m, 16 * t) for t in (1, 37, T // 3, T // 2 + 5, T - 3) if 0 < t < T})
+    for r0, r1 in zip(cuts[:-1], cuts[1:]):
+        S = A.row_slice(r0, r1)
+        with TM.from_host_csr(S, mode=mode, device=cuda_device) as M:
+            ys = M.run(xd).cpu().numpy()
+        assert np.array_equal(ys.view(np.uint64), yfull[r0:r1].view(np.uint64)), (name, mode, r0, r1)
