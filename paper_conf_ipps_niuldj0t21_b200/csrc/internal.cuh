@@ -85,7 +85,7 @@ struct __align__(16) WFirst {
 // several groups writes one partial per group and the last group to finish
 // sums the group partials in group order.  Everything depends only on the
 // row's own content (deterministic, shard-invariant).
-constexpr int kLocalParts = 8;
+constexpr int kLocalParts = 4;
 // per-item fixed cost (bytes-equivalent of an item's latency chain: record,
 // blob, x gathers) used to balance the warps' item chunks; measured on R-MAT
 // (power-law, many small items): 2048 gives 174 us against 188 us for 512,
@@ -136,6 +136,7 @@ struct Matrix {
                                    // or unit range per CTA (SM-queue kernel)
     int32_t *units = nullptr;      // SM-queue kernel: first item of each unit, num_units + 1
     int64_t num_units = 0;
+    int local_parts = kLocalParts;  // parts per group of a split tile row (TILESPMV_LOCAL_PARTS)
     // launch shape
     int kernel_version = 20;
     const char *kernel_name = "";

@@ -26,7 +26,7 @@ namespace {
 // row's remainder entries.  Depends only on the tile row's own content.
 template <bool WRITE>
 __device__ int items_for_row(int64_t I, const int32_t *tilePtr, const uint32_t *tileOff, const int32_t *remRowPtr,
-                             int64_t m, int budget, Item *out, int split, int nparts = 0) {
+                             int64_t m, int budget, Item *out, int split, int nparts = 0, int lp = kLocalParts) {
     const int tp0 = tilePtr[I], tp1 = tilePtr[I + 1];
     int k0 = 0, k1 = 0;
     if (remRowPtr) {
@@ -69,8 +69,8 @@ __device__ int items_for_row(int64_t I, const int32_t *tilePtr, const uint32_t *
             it.offb = tileOff[tb];
             it.offe = tileOff[t];
             it.split = split;
-            const bool local = split >= 0 && nparts <= kLocalParts;
-            const bool last = split >= 0 && (cnt == nparts - 1 || cnt % kLocalParts == kLocalParts - 1);
+            const bool local = split >= 0 && nparts <= lp;
+            const bool last = split >= 0 && (cnt == nparts - 1 || cnt % lp == lp - 1);
             it.part_nt = (split >= 0 ? cnt : 0) | ((t - tb) << 24) | ((int)local << 29) | ((int)last << 30);
             it.dbeg = 0;
             it.ndsc = 0;
@@ -106,14 +106,14 @@ __device__ __forceinline__ bool groupable(int64_t I, const int32_t *tilePtr, con
 template <bool WRITE>
 __device__ int window_items(int64_t w, const int32_t *tilePtr, const uint32_t *tileOff, const int32_t *remRowPtr,
                             int64_t m, int budget, int64_t tilem, bool group, const int32_t *nitems,
-                            const int32_t *splitId, Item *out) {
+                            const int32_t *splitId, Item *out, int lp) {
     const int64_t I0 = w * kGroupWindow, I1 = imin64(I0 + kGroupWindow, tilem);
     int cnt = 0;
     int64_t I = I0;
     while (I < I1) {
         if (!group || !groupable(I, tilePtr, nitems)) {
             if (WRITE) items_for_row<true>(I, tilePtr, tileOff, remRowPtr, m, budget, out + cnt,
-                                           nitems[I] > 1 ? splitId[I] : -1, nitems[I]);
+                                           nitems[I] > 1 ? splitId[I] : -1, nitems[I], lp);
             cnt += nitems[I];
             ++I;
             continue;
@@ -154,17 +154,17 @@ __global__ void k_window_count(const int32_t *tilePtr, const uint32_t *tileOff, 
     const int64_t w = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     if (w >= nwin) return;
     wcount[w] = window_items<false>(w, tilePtr, tileOff, remRowPtr, m, budget, tilem, group != 0, nitems, nullptr,
-                                    nullptr);
+                                    nullptr, kLocalParts);
 }
 
 __global__ void k_window_write(const int32_t *tilePtr, const uint32_t *tileOff, const int32_t *remRowPtr, int64_t m,
                                int budget, int64_t tilem, int group, const int32_t *nitems, int64_t nwin,
                                const int32_t *wbase, const int32_t *splitId, const int32_t *partBase, Item *items,
-                               int2 *split_info) {
+                               int2 *split_info, int lp) {
     const int64_t w = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     if (w >= nwin) return;
     window_items<true>(w, tilePtr, tileOff, remRowPtr, m, budget, tilem, group != 0, nitems, splitId,
-                       items + wbase[w]);
+                       items + wbase[w], lp);
     const int64_t I1 = imin64((w + 1) * kGroupWindow, tilem);
     for (int64_t I = w * kGroupWindow; I < I1; ++I)
         if (nitems[I] > 1) split_info[splitId[I]] = make_int2(partBase[I], nitems[I]);
@@ -318,7 +318,7 @@ __global__ void k_warp_first(const int64_t *begin, const WItem *witems, const in
     wf[b] = f;
 }
 
-__global__ void k_cta_begin(const int64_t *incl, const Item *items, int64_t n, int G, int64_t *cta_begin) {
+__global__ void k_cta_begin(const int64_t *incl, const Item *items, int64_t n, int G, int lp, int64_t *cta_begin) {
     const int b = blockIdx.x * blockDim.x + threadIdx.x;
     if (b > G) return;
     if (b == G) {
@@ -335,17 +335,17 @@ __global__ void k_cta_begin(const int64_t *incl, const Item *items, int64_t n, i
         else hi = mid;
     }
     // never start inside a group of parts of a split row (a group runs in one warp)
-    while (lo < n && items[lo].split >= 0 && item_part(items[lo]) % kLocalParts != 0) lo++;
+    while (lo < n && items[lo].split >= 0 && item_part(items[lo]) % lp != 0) lo++;
     cta_begin[b] = lo;
 }
 
 // units of the SM-queue kernel: an item that is not an inner part of a group
 // of parts starts a unit
-__global__ void k_unit_flags(const Item *items, int64_t n, int32_t *flag) {
+__global__ void k_unit_flags(const Item *items, int64_t n, int lp, int32_t *flag) {
     const int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     if (k >= n) return;
     const Item it = items[k];
-    flag[k] = (it.split < 0 || item_part(it) % kLocalParts == 0) ? 1 : 0;
+    flag[k] = (it.split < 0 || item_part(it) % lp == 0) ? 1 : 0;
 }
 
 __global__ void k_unit_write(const int32_t *flag, const int32_t *pos, int64_t n, int32_t *units) {
@@ -439,7 +439,7 @@ int build_schedule(Matrix &M, cudaStream_t st) {
         M.device_bytes += M.num_items * (int64_t)sizeof(Item) + M.num_split * 12 + nparts * 128;
         cudaMemsetAsync(M.counters, 0, std::max<int64_t>(M.num_split, 1) * sizeof(int32_t), st);
         k_window_write<<<blocks(NW), TB, 0, st>>>(M.tilePtr, M.tileOff, M.remRowPtr, M.m, M.item_bytes, T, group, nitems,
-                                                   NW, wbase, splitId, partBase, M.items, M.split_info);
+                                                   NW, wbase, splitId, partBase, M.items, M.split_info, M.local_parts);
         if (cudaStreamSynchronize(st) != cudaSuccess) rc = cuda_status(cudaGetLastError(), "k_window_write");
     } while (0);
     cudaFree(buf);
@@ -515,6 +515,7 @@ int choose_kernel(Matrix &M) {
     const double row_bytes = M.tilem ? (double)M.payload_bytes / (double)M.tilem : 0.0;
     int version = row_bytes > 6144.0 ? 25 : 40;
     if (const char *e = getenv("TILESPMV_KERNEL")) version = atoi(e);
+    if (const char *e = getenv("TILESPMV_LOCAL_PARTS")) M.local_parts = std::max(1, atoi(e));
     M.kernel_version = version;
     M.item_bytes = choose(version).slot_bytes;
     return 0;
@@ -555,7 +556,7 @@ static int configure_sm_queue(Matrix &M, int G) {
         k_item_cost<<<nb, 256>>>(M.items, n, M.m, fixed, cost);
         if ((rc = scan([&](void *t, size_t &b) { return cub::DeviceScan::InclusiveSum(t, b, cost, incl, (int)n); }))) break;
         cudaMemset(flag + n, 0, sizeof(int32_t));
-        k_unit_flags<<<nb, 256>>>(M.items, n, flag);
+        k_unit_flags<<<nb, 256>>>(M.items, n, M.local_parts, flag);
         if ((rc = scan([&](void *t, size_t &b) { return cub::DeviceScan::ExclusiveSum(t, b, flag, pos, (int)(n + 1)); }))) break;
         int32_t nu = 0;
         cudaMemcpy(&nu, pos + n, 4, cudaMemcpyDeviceToHost);
@@ -608,7 +609,7 @@ int configure_launch(Matrix &M) {
         k_item_cost<<<(unsigned)((M.num_items + 255) / 256), 256>>>(M.items, M.num_items, M.m, fixed, cost);
         int rc = scan([&](void *t, size_t &b) { return cub::DeviceScan::InclusiveSum(t, b, cost, incl, (int)M.num_items); });
         if (!rc) {
-            k_cta_begin<<<(W + 1 + 255) / 256, 256>>>(incl, M.items, M.num_items, W, M.cta_begin);
+            k_cta_begin<<<(W + 1 + 255) / 256, 256>>>(incl, M.items, M.num_items, W, M.local_parts, M.cta_begin);
             cudaError_t e = cudaDeviceSynchronize();
             if (e != cudaSuccess) rc = cuda_status(e, "k_cta_begin");
         }
@@ -655,6 +656,7 @@ int launch_spmv(const Matrix &M, const double *d_x, double *d_y, cudaStream_t st
     p.cta_begin = M.cta_begin;
     p.x_vec = (reinterpret_cast<uintptr_t>(d_x) & 15u) == 0;
     p.units = M.units;
+    p.local_parts = M.local_parts;
     const KernelChoice kc = choose(M.kernel_version);
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3(M.grid);

@@ -35,6 +35,7 @@ struct Params {
     const int64_t *cta_begin;  // warp kernel: item chunk of each warp
     int x_vec;                 // x is 16-byte aligned: x segments load as double2
     const int32_t *units;      // SM-queue kernel: first item of each unit (+ end), see schedule.cu
+    int local_parts;           // parts per group of a split tile row (Matrix::local_parts)
 };
 
 // ------------------------------------------------------------------ PTX ----

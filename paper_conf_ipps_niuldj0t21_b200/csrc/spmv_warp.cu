@@ -72,12 +72,15 @@ __device__ __forceinline__ WItem load_witem(const WItem *w, int k) {
 // lane r (and r + 16).  rpS: rebased row pointers (rows + 1), colS/valS: entries.
 //  * every row <= 4 entries (stencil-like): two lanes per row, two entries
 //    each, one round trip of gathers;
-//  * otherwise rows of <= kShortRow entries run two lanes per row, all at
-//    once, and the longer rows (power-law hubs) a half-warp per row, two rows
-//    at a time (the whole warp when one is left), four entries per lane in
-//    flight, summed by an xor-shuffle tree.
-// The order of every sum depends only on the item's content: y stays bitwise
-// deterministic.
+//  * every row <= kShortRow entries: two lanes per row, all rows at once;
+//  * a longer row (power-law hubs): the flat pass (flat_products, flat_rows),
+//    all gathers of the item in flight together.
+// The path and the order of every sum depend only on the item's content: y
+// stays bitwise deterministic.
+__device__ __forceinline__ void flat_products(const Params &p, uint32_t colS, uint32_t valS, int E,
+                                              uint64_t x_policy, int lane);
+__device__ __forceinline__ double flat_rows(uint32_t rq, uint32_t valS, int rows, int lane);
+
 __device__ __forceinline__ void remainder(const Params &p, uint32_t rpS, uint32_t colS, uint32_t valS, int rows,
                                           uint64_t x_policy, int lane, double &acc) {
     const int r = lane & 15, h = lane >> 4;
@@ -97,23 +100,69 @@ __device__ __forceinline__ void remainder(const Params &p, uint32_t rpS, uint32_
         acc = fma(v1, x1, acc);
         return;
     }
-    const bool lng = e - b > kShortRow;
-    {
-        const int ee = lng ? b : e;
-        const int trips = (int)__reduce_max_sync(FULL, (unsigned)((ee - b + 1 - h) >> 1));
+    if (maxlen > kShortRow) {
+        flat_products(p, colS, valS, lds_s32(rpS + 4 * rows), x_policy, lane);
+        acc += flat_rows(rpS, valS, rows, lane);
+        return;
+    }
+    const int trips = (int)__reduce_max_sync(FULL, (unsigned)((e - b + 1 - h) >> 1));
 #pragma unroll 1
-        for (int i = 0; i < trips; i += 2) {
-            const int k0 = b + h + 2 * i, k1 = k0 + 2;
-            int c0, c1;
-            double v0, v1;
-            lds_entry_lt(k0, ee, colS + 4 * k0, valS + 8 * k0, c0, v0);
-            lds_entry_lt(k1, ee, colS + 4 * k1, valS + 8 * k1, c1, v1);
-            const double x0 = ldg_hint(x + (uint32_t)c0, x_policy), x1 = ldg_hint(x + (uint32_t)c1, x_policy);
-            acc = fma(v0, x0, acc);
-            acc = fma(v1, x1, acc);
+    for (int i = 0; i < trips; i += 2) {
+        const int k0 = b + h + 2 * i, k1 = k0 + 2;
+        int c0, c1;
+        double v0, v1;
+        lds_entry_lt(k0, e, colS + 4 * k0, valS + 8 * k0, c0, v0);
+        lds_entry_lt(k1, e, colS + 4 * k1, valS + 8 * k1, c1, v1);
+        const double x0 = ldg_hint(x + (uint32_t)c0, x_policy), x1 = ldg_hint(x + (uint32_t)c1, x_policy);
+        acc = fma(v0, x0, acc);
+        acc = fma(v1, x1, acc);
+    }
+}
+
+// Flat remainder pass, step 1: one lane per entry, the x gathers of 256
+// entries in flight at once; each value in the slot is overwritten by its
+// product (rounded, so every later order of summation sees the same terms).
+__device__ __forceinline__ void flat_products(const Params &p, uint32_t colS, uint32_t valS, int E,
+                                              uint64_t x_policy, int lane) {
+#pragma unroll 1
+    for (int k0 = 0; k0 < E; k0 += 256) {
+        double pv[8];
+#pragma unroll
+        for (int j = 0; j < 8; ++j) {
+            const int k = k0 + 32 * j + lane;
+            int c;
+            double v;
+            lds_entry_lt(k, E, colS + 4 * k, valS + 8 * k, c, v);
+            pv[j] = __dmul_rn(v, ldg_hint(p.x + (uint32_t)c, x_policy));
+        }
+#pragma unroll
+        for (int j = 0; j < 8; ++j) {
+            const int k = k0 + 32 * j + lane;
+            if (k < E) sts_f64(valS + 8 * k, pv[j]);
         }
     }
-    // long rows: lanes 0-15 of the ballot = rows 0-15
+    __syncwarp();
+}
+
+// Flat remainder pass, step 2, for one tile row (rows <= 16, row pointers at
+// rq): rows of <= kShortRow products two lanes per row, longer rows a
+// half-warp per row (two rows at a time, the whole warp for the last one)
+// with an xor tree.  Returns lane r's (or r + 16's) share of row r.  The order
+// of every sum depends only on this tile row.
+__device__ __forceinline__ double flat_rows(uint32_t rq, uint32_t valS, int rows, int lane) {
+    const int r = lane & 15, h = lane >> 4;
+    const int b = lds_s32(rq + 4 * min(r, rows)), e = lds_s32(rq + 4 * min(r + 1, rows));
+    const bool lng = e - b > kShortRow;
+    const int ee = lng ? b : e;
+    const int trips = (int)__reduce_max_sync(FULL, (unsigned)((ee - b + 1 - h) >> 1));
+    double s0 = 0.0, s1 = 0.0;
+#pragma unroll 1
+    for (int i = 0; i < trips; i += 2) {
+        const int k0 = b + h + 2 * i;
+        s0 += lds_f64_lt(k0, ee, valS + 8 * k0);
+        s1 += lds_f64_lt(k0 + 2, ee, valS + 8 * k0 + 16);
+    }
+    double acc = s0 + s1;
     uint32_t lm = __ballot_sync(FULL, lng && h == 0 && r < rows);
 #pragma unroll 1
     while (lm) {
@@ -124,118 +173,44 @@ __device__ __forceinline__ void remainder(const Params &p, uint32_t rpS, uint32_
         const bool pair = r1 >= 0;  // warp-uniform
         const int myrow = (pair && h) ? r1 : r0;
         const int off = pair ? r : lane, stride = pair ? 16 : 32;
-        const int bb = lds_s32(rpS + 4 * myrow), e2 = lds_s32(rpS + 4 * myrow + 4);
+        const int bb = lds_s32(rq + 4 * myrow), e2 = lds_s32(rq + 4 * myrow + 4);
         const int t2 = (int)__reduce_max_sync(FULL, (unsigned)((e2 - bb + 4 * stride - 1) / (4 * stride)));
-        double s0 = 0.0, s1 = 0.0, s2 = 0.0, s3 = 0.0;
+        double q0 = 0.0, q1 = 0.0, q2 = 0.0, q3 = 0.0;
 #pragma unroll 1
         for (int t = 0; t < t2; ++t) {
             const int k = bb + off + 4 * stride * t;
-            int c0, c1, c2, c3;
-            double v0, v1, v2, v3;
-            lds_entry_lt(k, e2, colS + 4 * k, valS + 8 * k, c0, v0);
-            lds_entry_lt(k + stride, e2, colS + 4 * (k + stride), valS + 8 * (k + stride), c1, v1);
-            lds_entry_lt(k + 2 * stride, e2, colS + 4 * (k + 2 * stride), valS + 8 * (k + 2 * stride), c2, v2);
-            lds_entry_lt(k + 3 * stride, e2, colS + 4 * (k + 3 * stride), valS + 8 * (k + 3 * stride), c3, v3);
-            s0 = fma(v0, ldg_hint(x + (uint32_t)c0, x_policy), s0);
-            s1 = fma(v1, ldg_hint(x + (uint32_t)c1, x_policy), s1);
-            s2 = fma(v2, ldg_hint(x + (uint32_t)c2, x_policy), s2);
-            s3 = fma(v3, ldg_hint(x + (uint32_t)c3, x_policy), s3);
+            q0 += lds_f64_lt(k, e2, valS + 8 * k);
+            q1 += lds_f64_lt(k + stride, e2, valS + 8 * (k + stride));
+            q2 += lds_f64_lt(k + 2 * stride, e2, valS + 8 * (k + 2 * stride));
+            q3 += lds_f64_lt(k + 3 * stride, e2, valS + 8 * (k + 3 * stride));
         }
-        double s = (s0 + s1) + (s2 + s3);
-        if (!pair) s += __shfl_xor_sync(FULL, s, 16);
-        s += __shfl_xor_sync(FULL, s, 8);
-        s += __shfl_xor_sync(FULL, s, 4);
-        s += __shfl_xor_sync(FULL, s, 2);
-        s += __shfl_xor_sync(FULL, s, 1);
-        if (pair ? r == myrow : lane == r0) acc += s;
+        double sq = (q0 + q1) + (q2 + q3);
+        if (!pair) sq += __shfl_xor_sync(FULL, sq, 16);
+        sq += __shfl_xor_sync(FULL, sq, 8);
+        sq += __shfl_xor_sync(FULL, sq, 4);
+        sq += __shfl_xor_sync(FULL, sq, 2);
+        sq += __shfl_xor_sync(FULL, sq, 1);
+        if (pair ? r == myrow : lane == r0) acc += sq;
     }
+    return acc;
 }
 
 // Row-group item (internal.cuh): ntr consecutive tile rows without stored
-// tiles, only remainder rows.  1. one lane per entry, the x gathers of
-// 256 entries in flight at once, each value in the slot overwritten by its
-// product; 2. per tile row, the rows are summed from shared memory -- rows of
-// <= kShortRow products two lanes per row, longer rows a half-warp per row
-// (two rows at a time, the whole warp for the last one) with an xor tree --
-// and y is written once per row.  The order of every row's sum depends only on
-// its own tile row, so grouping never changes a bit of y.
+// tiles, only remainder rows: the flat pass over all their entries,
+// then per tile row the row sums from shared memory and y written once per
+// row.  Every tile row is summed exactly as it would be alone, so grouping
+// never changes a bit of y.
 __device__ __forceinline__ void group_item(const Params &p, const WItem &it, uint32_t slot, uint64_t x_policy,
                                            int lane) {
-    const int r = lane & 15, h = lane >> 4;
     const int ntr = (int)(it.jt_rows_pay & 0xFFu);
     const int rows_last = (int)((it.jt_rows_pay >> 8) & 31u);
     const uint32_t total = it.val_tot >> 16, rp = it.rp_col & 0xFFFFu;
     const bool has_rem = total > rp;
     const uint32_t rpS = slot + rp, colS = slot + (it.rp_col >> 16), valS = slot + (it.val_tot & 0xFFFFu);
-    if (has_rem) {
-        const int E = lds_s32(rpS + 4 * (16 * (ntr - 1) + rows_last));
-#pragma unroll 1
-        for (int k0 = 0; k0 < E; k0 += 256) {
-            double pv[8];
-#pragma unroll
-            for (int j = 0; j < 8; ++j) {
-                const int k = k0 + 32 * j + lane;
-                int c;
-                double v;
-                lds_entry_lt(k, E, colS + 4 * k, valS + 8 * k, c, v);
-                pv[j] = __dmul_rn(v, ldg_hint(p.x + (uint32_t)c, x_policy));
-            }
-#pragma unroll
-            for (int j = 0; j < 8; ++j) {
-                const int k = k0 + 32 * j + lane;
-                if (k < E) sts_f64(valS + 8 * k, pv[j]);
-            }
-        }
-        __syncwarp();
-    }
+    if (has_rem) flat_products(p, colS, valS, lds_s32(rpS + 4 * (16 * (ntr - 1) + rows_last)), x_policy, lane);
 #pragma unroll 1
     for (int g = 0; g < ntr; ++g) {
-        const int rows = g + 1 < ntr ? 16 : rows_last;
-        double acc = 0.0;
-        if (has_rem) {
-            const uint32_t rq = rpS + 64u * (uint32_t)g;
-            const int b = lds_s32(rq + 4 * min(r, rows)), e = lds_s32(rq + 4 * min(r + 1, rows));
-            const bool lng = e - b > kShortRow;
-            const int ee = lng ? b : e;
-            const int trips = (int)__reduce_max_sync(FULL, (unsigned)((ee - b + 1 - h) >> 1));
-            double s0 = 0.0, s1 = 0.0;
-#pragma unroll 1
-            for (int i = 0; i < trips; i += 2) {
-                const int k0 = b + h + 2 * i;
-                s0 += lds_f64_lt(k0, ee, valS + 8 * k0);
-                s1 += lds_f64_lt(k0 + 2, ee, valS + 8 * k0 + 16);
-            }
-            acc = s0 + s1;
-            uint32_t lm = __ballot_sync(FULL, lng && h == 0 && r < rows);
-#pragma unroll 1
-            while (lm) {
-                const int r0 = __ffs(lm) - 1;
-                lm &= lm - 1;
-                const int r1 = lm ? __ffs(lm) - 1 : -1;
-                if (lm) lm &= lm - 1;
-                const bool pair = r1 >= 0;  // warp-uniform
-                const int myrow = (pair && h) ? r1 : r0;
-                const int off = pair ? r : lane, stride = pair ? 16 : 32;
-                const int bb = lds_s32(rq + 4 * myrow), e2 = lds_s32(rq + 4 * myrow + 4);
-                const int t2 = (int)__reduce_max_sync(FULL, (unsigned)((e2 - bb + 4 * stride - 1) / (4 * stride)));
-                double q0 = 0.0, q1 = 0.0, q2 = 0.0, q3 = 0.0;
-#pragma unroll 1
-                for (int t = 0; t < t2; ++t) {
-                    const int k = bb + off + 4 * stride * t;
-                    q0 += lds_f64_lt(k, e2, valS + 8 * k);
-                    q1 += lds_f64_lt(k + stride, e2, valS + 8 * (k + stride));
-                    q2 += lds_f64_lt(k + 2 * stride, e2, valS + 8 * (k + 2 * stride));
-                    q3 += lds_f64_lt(k + 3 * stride, e2, valS + 8 * (k + 3 * stride));
-                }
-                double sq = (q0 + q1) + (q2 + q3);
-                if (!pair) sq += __shfl_xor_sync(FULL, sq, 16);
-                sq += __shfl_xor_sync(FULL, sq, 8);
-                sq += __shfl_xor_sync(FULL, sq, 4);
-                sq += __shfl_xor_sync(FULL, sq, 2);
-                sq += __shfl_xor_sync(FULL, sq, 1);
-                if (pair ? r == myrow : lane == r0) acc += sq;
-            }
-        }
+        double acc = has_rem ? flat_rows(rpS + 64u * (uint32_t)g, valS, g + 1 < ntr ? 16 : rows_last, lane) : 0.0;
         acc += __shfl_xor_sync(FULL, acc, 16);
         const int64_t row = 16 * ((int64_t)it.I + g) + lane;
         if (lane < 16 && row < p.m) p.y[row] = acc;
@@ -364,8 +339,8 @@ __device__ __forceinline__ void compute_item(const Params &p, const WItem &it, u
             if (lane < 16 && row < p.m) p.y[row] = sum;
         } else {  // hub row: one partial per group, the last group sums them in order
             const int2 si = p.split_info[it.split];
-            const int ngroups = (si.y + kLocalParts - 1) / kLocalParts;
-            const int gidx = (it.part_nt & 0xFFFFFF) / kLocalParts;
+            const int ngroups = (si.y + p.local_parts - 1) / p.local_parts;
+            const int gidx = (it.part_nt & 0xFFFFFF) / p.local_parts;
             if (lane < 16) __stcg(p.partials + (int64_t)(si.x + gidx) * 16 + lane, sum);
             __threadfence();
             __syncwarp();
