@@ -120,6 +120,23 @@ int tilespmv_run(tilespmv_handle_t h, const double *d_x, double *d_y, void *stre
  * h_x / h_y should be page-locked for asynchronous copies.                  */
 int tilespmv_run_host(tilespmv_handle_t h, const double *h_x, double *h_y, void *stream);
 
+/* Conjugate-gradient solve of A x = b (the iterative
+ * solver use that motivates SpMV), built on tilespmv_run's kernel.
+ * Hestenes-Stiefel CG in fp64 (cg.cu states the recurrence); A must be
+ * square (m == n) and symmetric positive definite -- symmetry and
+ * definiteness are NOT checked (an indefinite A may stall or diverge).
+ *   d_b     double[n] device, read.
+ *   d_x     double[n] device: the initial guess on entry, the iterate on
+ *           exit; must be finite and must not overlap d_b.
+ *   tol     stop once ||r_k|| <= tol * ||b|| (recursive residual), tol >= 0.
+ *   maxit   at most this many iterations (>= 0).
+ *   iters   (optional) iterations performed; relres (optional) ||r_k||/||b||.
+ * Synchronous: work is queued on `stream`, which is synchronised before the
+ * call returns.  Work memory (3 n doubles) is allocated and freed per call.
+ * Errors: INVALID_ARG (m != n, NULL vectors, bad tol/maxit), OOM, CUDA.      */
+int tilespmv_cg(tilespmv_handle_t h, const double *d_b, double *d_x, double tol, int32_t maxit,
+                int32_t *iters, double *relres, void *stream);
+
 /* Release all device storage; NULL is a no-op returning TILESPMV_OK. */
 int tilespmv_destroy(tilespmv_handle_t h);
 

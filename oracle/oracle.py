@@ -198,3 +198,43 @@ def decode(A, mode: str | int = "DEFERRED"):
 def tile_row_sizes(T: Tiling) -> np.ndarray:
     """Payload bytes per tile (16-byte rounded) from tileOff."""
     return (np.diff(T.tileOff.astype(np.int64)) * 16) if T.numtile else np.zeros(0, np.int64)
+
+
+def cg(A, b: np.ndarray, x0: np.ndarray | None = None, tol: float = 1e-10, maxit: int = 1000):
+    """Conjugate gradients for SPD A (the iterative-solver
+    use of SpMV), written out as the textbook Hestenes-Stiefel
+    recurrence (e.g. Saad, Iterative Methods for Sparse Linear Systems,
+    Alg. 6.18), in the order the GPU path (csrc/cg.cu) states it:
+
+        r0 = b - A x0, p0 = r0
+        q = A p_j;  alpha = (r_j, r_j) / (p_j, q)
+        x_{j+1} = x_j + alpha p_j;  r_{j+1} = r_j - alpha q
+        stop if ||r_{j+1}|| <= tol ||b||
+        beta = (r_{j+1}, r_{j+1}) / (r_j, r_j);  p_{j+1} = r_{j+1} + beta p_j
+
+    The matrix-vector products are this oracle's spmv (Alg. 1, long-double
+    rows); dot products are numpy's.  Returns (x, iterations, ||r||/||b||)."""
+    b = np.asarray(b, dtype=np.float64)
+    x = np.zeros_like(b) if x0 is None else np.array(x0, dtype=np.float64)
+    q, _ = spmv(A, x)
+    r = b - q
+    p = r.copy()
+    rr = float(np.dot(r, r))
+    bb = float(np.dot(b, b))
+    it = 0
+    if rr == 0.0:
+        return x, 0, 0.0
+    for j in range(maxit):
+        q, _ = spmv(A, p)
+        alpha = rr / float(np.dot(p, q))
+        x = x + alpha * p
+        r = r - alpha * q
+        rr_new = float(np.dot(r, r))
+        it = j + 1
+        if rr_new <= tol * tol * bb:
+            rr = rr_new
+            break
+        beta = rr_new / rr
+        p = r + beta * p
+        rr = rr_new
+    return x, it, (np.sqrt(rr / bb) if bb > 0 else 0.0)

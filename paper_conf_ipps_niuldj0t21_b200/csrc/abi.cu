@@ -168,6 +168,23 @@ int tilespmv_run_host(tilespmv_handle_t h, const double *h_x, double *h_y, void 
     return TILESPMV_OK;
 }
 
+int tilespmv_cg(tilespmv_handle_t h, const double *d_b, double *d_x, double tol, int32_t maxit, int32_t *iters,
+                double *relres, void *stream) {
+    if (int rc = check_handle(h)) return rc;
+    if (h->m != h->n) return set_error(TILESPMV_INVALID_ARG, "CG needs a square matrix");
+    if (h->n > 0 && (!d_b || !d_x)) return set_error(TILESPMV_INVALID_ARG, "NULL vector");
+    if (!(tol >= 0.0) || maxit < 0) return set_error(TILESPMV_INVALID_ARG, "tol must be >= 0 and maxit >= 0");
+    if (h->n > 0 && d_b < d_x + h->n && d_x < d_b + h->n) return set_error(TILESPMV_INVALID_ARG, "b and x overlap");
+    int it = 0;
+    double rel = 0.0;
+    if (h->n > 0) {
+        if (int rc = cg_solve(*h, d_b, d_x, tol, maxit, &it, &rel, static_cast<cudaStream_t>(stream))) return rc;
+    }
+    if (iters) *iters = it;
+    if (relres) *relres = rel;
+    return TILESPMV_OK;
+}
+
 int tilespmv_destroy(tilespmv_handle_t h) {
     if (!h) return TILESPMV_OK;
     free_matrix(h);

@@ -157,5 +157,8 @@ int build_schedule(Matrix &M, cudaStream_t stream);
 int build_tdesc(Matrix &M, cudaStream_t stream);
 int configure_launch(Matrix &M);
 int launch_spmv(const Matrix &M, const double *d_x, double *d_y, cudaStream_t stream);
+// cg.cu
+int cg_solve(const Matrix &M, const double *d_b, double *d_x, double tol, int maxit, int *iters, double *relres,
+             cudaStream_t stream);
 
 }  // namespace tsp

@@ -437,6 +437,8 @@ int build_schedule(Matrix &M, cudaStream_t st) {
             break;
         }
         M.device_bytes += M.num_items * (int64_t)sizeof(Item) + M.num_split * 12 + nparts * 128;
+        // whole records (padding included) are copied later: start from zeros
+        cudaMemsetAsync(M.items, 0, std::max<int64_t>(M.num_items, 1) * sizeof(Item), st);
         cudaMemsetAsync(M.counters, 0, std::max<int64_t>(M.num_split, 1) * sizeof(int32_t), st);
         k_window_write<<<blocks(NW), TB, 0, st>>>(M.tilePtr, M.tileOff, M.remRowPtr, M.m, M.item_bytes, T, group, nitems,
                                                    NW, wbase, splitId, partBase, M.items, M.split_info, M.local_parts);

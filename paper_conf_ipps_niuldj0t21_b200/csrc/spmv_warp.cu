@@ -451,6 +451,7 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, 1) tilespmv_fp
     griddep_launch_dependents();
     const int64_t gw = (int64_t)blockIdx.x * WARPS + warp;
     TSP_SMID(gw, (int64_t)gridDim.x * WARPS);
+    (void)gw;
     double carry = 0.0;  // partial row sums inside a group of parts of a split tile row
     uint32_t phase = 0;
     const uint64_t stream_policy = policy_evict_first(), x_policy = policy_evict_last();

@@ -23,7 +23,7 @@ ARRAYS = {"tilePtr": (0, np.int32), "tileColIdx": (1, np.int32), "tileNnz": (2, 
 EXPORTED_SYMBOLS = ["tilespmv_create_from_csr", "tilespmv_run", "tilespmv_run_host",
                     "tilespmv_destroy", "tilespmv_get_info", "tilespmv_export_size",
                     "tilespmv_export", "tilespmv_status_string", "tilespmv_last_error",
-                    "tilespmv_launch_shape", "tilespmv_kernel_name"]
+                    "tilespmv_launch_shape", "tilespmv_kernel_name", "tilespmv_cg"]
 
 
 class TileSpMVError(RuntimeError):
@@ -86,11 +86,12 @@ def load(build_if_missing: bool = True):
     L.tilespmv_last_error.restype = ctypes.c_char_p
     L.tilespmv_launch_shape.argtypes = [p, ctypes.POINTER(i32), ctypes.POINTER(i32),
                                         ctypes.POINTER(i32)]
+    L.tilespmv_cg.argtypes = [p, p, p, ctypes.c_double, i32, ctypes.POINTER(i32), ctypes.POINTER(ctypes.c_double), p]
     L.tilespmv_kernel_name.argtypes = [p]
     L.tilespmv_kernel_name.restype = ctypes.c_char_p
     for name in ("tilespmv_create_from_csr", "tilespmv_run", "tilespmv_run_host",
                  "tilespmv_destroy", "tilespmv_get_info", "tilespmv_export",
-                 "tilespmv_launch_shape"):
+                 "tilespmv_launch_shape", "tilespmv_cg"):
         getattr(L, name).restype = ctypes.c_int
     _lib = L
     return L
@@ -180,6 +181,22 @@ class TiledMatrix:
                                       ptr(hy) if self.m else None, _stream_ptr(stream))
         _check(rc, "tilespmv_run_host")
         return hy
+
+    def cg(self, b, x=None, tol: float = 1e-10, maxit: int = 1000, stream=None):
+        """Solve A x = b by conjugate gradients on the GPU (tilespmv_cg); A
+        must be square SPD.  b (and x, the initial guess, zeros if None) are
+        contiguous float64 CUDA tensors; returns (x, iterations, relres)."""
+        import torch
+        if x is None:
+            x = torch.zeros(self.n, dtype=torch.float64, device=b.device)
+        for t in (b, x):
+            if not (t.is_cuda and t.dtype == torch.float64 and t.is_contiguous() and t.numel() == self.n):
+                raise TileSpMVError("b and x must be contiguous float64 CUDA tensors of length n")
+        it, rel = ctypes.c_int32(), ctypes.c_double()
+        rc = load().tilespmv_cg(self._h, b.data_ptr() if self.n else None, x.data_ptr() if self.n else None,
+                                float(tol), int(maxit), ctypes.byref(it), ctypes.byref(rel), _stream_ptr(stream))
+        _check(rc, "tilespmv_cg")
+        return x, it.value, rel.value
 
     # ------------------------------------------------------------------ info
     def info(self) -> dict:

@@ -20,7 +20,7 @@ timeout 1200 $NCU --set full --clock-control none --import-source on -k regex:ti
 timeout 900 $NCU --set full --clock-control none --import-source on -k regex:tilespmv_fp64 -s 3 -c 1 \
    -o $OUT/full_fem -f python bench.py --workload fem --steps 2 --warmup 3 --no-cpu-baseline --no-secondary --e2e-steps 1 > $OUT/full_fem.log 2>&1
 for tool in memcheck racecheck synccheck initcheck; do
-  timeout 900 /usr/local/cuda/bin/compute-sanitizer --tool $tool --error-exitcode 9 python scripts/sanitize_small.py > $OUT/sanitizer_$tool.log 2>&1
+  timeout 900 /usr/local/cuda/bin/compute-sanitizer --tool $tool --num-cuda-barriers 64 --error-exitcode 9 python scripts/sanitize_small.py > $OUT/sanitizer_$tool.log 2>&1
   echo "rc=$?" >> $OUT/sanitizer_$tool.log
 done
 echo done > $OUT/DONE
