@@ -437,7 +437,8 @@ def measure_sharded(workload, mode, steps, warmup, dev, rank, P, group, exchange
     if exchange == "halo":
         def mk(M):
             return lambda xf, yo: M.run(xf, yo)
-        H = HaloSpMV(plan, [mk(M) for M in mats], group=group)
+        H = HaloSpMV(plan, [mk(M) for M in mats], group=group,
+                     host_staging=os.environ.get("TILESPMV_BENCH_ONE_GPU") == "1")
         ev_slot = [None]
 
         def timed(xf, yo, M=mats[dom]):
@@ -549,10 +550,16 @@ def run_ours(args):
     if P != args.gpus:
         log(f"warning: --gpus {args.gpus} but WORLD_SIZE {P}")
     group = None
-    dev = torch.device("cuda", local)
+    # development hook: TILESPMV_BENCH_ONE_GPU=1 runs every rank on cuda:0 over
+    # gloo (exercises the N > 1 code path on a one-GPU box; not a bench number)
+    one_gpu = os.environ.get("TILESPMV_BENCH_ONE_GPU") == "1"
+    dev = torch.device("cuda", 0 if one_gpu else local)
     torch.cuda.set_device(dev)
     if P > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        if one_gpu:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=dev)
         group = dist.group.WORLD
     if P > 1:
         res = measure_sharded(args.workload, args.mode, args.steps, args.warmup, dev, rank, P, group,

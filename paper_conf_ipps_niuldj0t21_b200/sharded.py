@@ -184,15 +184,26 @@ class HaloSpMV:
     TiledMatrix.run of that row range).  x buffers are full length (n); only
     the rank's own rows and its halo are ever valid."""
 
-    def __init__(self, plan: HaloPlan, spmvs, group=None):
+    def __init__(self, plan: HaloPlan, spmvs, group=None, host_staging: bool = False):
+        """host_staging: move the halo through host buffers (a backend such as
+        gloo that cannot send device tensors; development runs only)."""
         assert len(spmvs) == len(plan.parts)
         self.plan, self.spmvs, self.group = plan, list(spmvs), group
+        self.host_staging = host_staging
+        self._staged = []
 
     def exchange(self, x):
         """Starts the halo exchange of x (own rows out, halo in); returns works."""
         import torch.distributed as dist
-        ops = [dist.P2POp(dist.isend, x[lo:hi], q, group=self.group) for q, lo, hi in self.plan.send]
-        ops += [dist.P2POp(dist.irecv, x[lo:hi], q, group=self.group) for q, lo, hi in self.plan.recv]
+        if self.host_staging:
+            sends = [(q, x[lo:hi].cpu()) for q, lo, hi in self.plan.send]
+            self._staged = [(x[lo:hi], x.new_empty(hi - lo, device="cpu")) for _, lo, hi in self.plan.recv]
+            ops = [dist.P2POp(dist.isend, t, q, group=self.group) for q, t in sends]
+            ops += [dist.P2POp(dist.irecv, h, q, group=self.group)
+                    for (q, _, _), (_, h) in zip(self.plan.recv, self._staged)]
+        else:
+            ops = [dist.P2POp(dist.isend, x[lo:hi], q, group=self.group) for q, lo, hi in self.plan.send]
+            ops += [dist.P2POp(dist.irecv, x[lo:hi], q, group=self.group) for q, lo, hi in self.plan.recv]
         return dist.batch_isend_irecv(ops) if ops else []
 
     def step(self, x_cur, x_next):
@@ -205,6 +216,9 @@ class HaloSpMV:
             f(x_cur, x_next[r0:r1])
         for w in pending:
             w.wait()
+        for dst, h in self._staged:
+            dst.copy_(h)
+        self._staged = []
         for (r0, r1, interior), f in zip(self.plan.parts, self.spmvs):
             if interior:
                 continue
