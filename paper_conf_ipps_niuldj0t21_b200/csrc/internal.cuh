@@ -30,6 +30,8 @@ enum : uint8_t { F_CSR = 0, F_COO = 1, F_ELL = 2, F_HYB = 3, F_DNS = 4, F_DNSROW
 constexpr int kItemTiles = 16;
 constexpr int kItemBytesMax = 12288;  // largest shared-memory slot of any kernel
 constexpr int kShortRow = 16;     // remainder rows up to this length: 2 lanes per row
+constexpr int kMedRow = 32;       // TM kernels: item remainder rows up to this length stay 2 lanes per row
+                                  // (the 27-point stencil's wrap rows hold up to 21; hubs take the flat pass)
 
 struct __align__(16) Item {
     int32_t I;        // tile row

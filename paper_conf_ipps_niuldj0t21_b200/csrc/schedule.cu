@@ -259,15 +259,33 @@ __global__ void k_blob_fill(Item *items, int64_t n, int64_t m, const int64_t *st
     uint2 *dd = reinterpret_cast<uint2 *>(dst);
     // kernel-native descriptors: x = distance from the descriptor itself to
     // the tile's payload (CSR: to its csrRowPtr, after the 8*nnz value bytes),
-    // y = aux | t*128 | nnz << 11 | invalid << 31
-    for (int i = lane; i < it.ndsc; i += 32) {
-        const uint2 d = dlist[it.dbeg + i];
-        const uint32_t off = d.x & 0x1FFFFFu, t = (d.x >> 21) & 0xFFu, f = d.x >> 29;
-        const uint32_t nz = (d.y >> 8) & 0x1FFu;
-        uint2 e;
-        e.x = b.pay + off + (f == F_CSR ? 8u * nz : 0u) - 8u * (uint32_t)i;
-        e.y = (d.y & 0x1Fu) | (t << 7) | (nz << 11) | (d.y & 0x80000000u);
-        dd[i] = e;
+    // y = aux | t*128 | nnz << 11 | tm << 20 | invalid << 31, where tm is the
+    // larger extent of the two tiles of the half-warp pair (2j, 2j+1): CSR the
+    // longest row, ELL the width (ndsc is even; the loop is warp-uniform)
+    const uint8_t *tpay = payload + (size_t)it.offb * 16;
+    for (int i0 = 0; i0 < it.ndsc; i0 += 32) {
+        const int i = i0 + lane;
+        uint2 e = make_uint2(0u, 0u);
+        uint32_t tm = 0;
+        if (i < it.ndsc) {
+            const uint2 d = dlist[it.dbeg + i];
+            const uint32_t off = d.x & 0x1FFFFFu, t = (d.x >> 21) & 0xFFu, f = d.x >> 29;
+            const uint32_t nz = (d.y >> 8) & 0x1FFu;
+            e.x = b.pay + off + (f == F_CSR ? 8u * nz : 0u) - 8u * (uint32_t)i;
+            e.y = (d.y & 0x1Fu) | (t << 7) | (nz << 11) | (d.y & 0x80000000u);
+            if (f == F_CSR) {
+                const uint8_t *rp = tpay + off + 8u * nz;
+                for (int r = 0; r < 16; ++r) {
+                    const uint32_t len = (r < 15 ? rp[r + 1] : nz) - rp[r];
+                    tm = len > tm ? len : tm;
+                }
+            } else if (f == F_ELL) {
+                tm = d.y & 0x1Fu;
+            }
+        }
+        const uint32_t tmo = __shfl_xor_sync(0xFFFFFFFFu, tm, 1);
+        tm = tmo > tm ? tmo : tm;
+        if (i < it.ndsc) dd[i] = make_uint2(e.x, e.y | (tm << 20));
     }
     const int nt = item_nt(it);
     if (lane < 16) jcols[k * 16 + lane] = lane < nt ? tileColIdx[it.tb + lane] : 0;
@@ -511,11 +529,13 @@ int choose_kernel(Matrix &M) {
     // warps claim units from a shared-memory counter); matrices whose tile
     // rows average more than 6 KB of payload (dense, FEM-like) use the warp
     // kernel with 10.5 KB slots (16 warps/SM) so a tile row stays one item.
+    // The SM-queue kernel runs CSR and ELL tiles with the pair extent known
+    // (variant 43, descriptor bits 20-24): C5 -9%, mixed -8% against 40.
     // Measured (graph-replayed launches, profiles/): C5 498 us (sm<32,4608>)
     // vs 512 us (warp<8,4608>); R-MAT 145 vs 163 us; mixed 113 vs 116 us;
     // C2 6.9 us for warp<4,10752> vs 7.5 us for sm<16,10752>.
     const double row_bytes = M.tilem ? (double)M.payload_bytes / (double)M.tilem : 0.0;
-    int version = row_bytes > 6144.0 ? 25 : 40;
+    int version = row_bytes > 6144.0 ? 25 : 43;
     if (const char *e = getenv("TILESPMV_KERNEL")) version = atoi(e);
     if (const char *e = getenv("TILESPMV_LOCAL_PARTS")) M.local_parts = std::max(1, atoi(e));
     M.kernel_version = version;

@@ -187,6 +187,83 @@ __device__ __forceinline__ void half_coo(uint32_t V, uint32_t rc, int n, uint32_
     }
 }
 
+// ------------------------------- routines with the pair's extent known -----
+// The schedule stores in every descriptor the longest row (CSR) or width
+// (ELL) of the two tiles of its half-warp pair (bits 20-24), so the trip count
+// is known without a warp vote and short tiles run straight-line code of
+// exactly that many steps.  A step past a lane's own row loads the value +0.0
+// (predicated load) and a column nibble that stays inside the x segment.
+
+// CSR entries base .. base+N-1 of the lane's row: values at V, their column
+// nibbles in u from bit 0
+template <int N>
+__device__ __forceinline__ void csr_steps(uint32_t V, uint32_t u, uint32_t X, int base, int len, double &acc) {
+    double xv[N], v[N];
+#pragma unroll
+    for (int j = 0; j < N; ++j) {
+        xv[j] = lds_f64(xaddr(j == 0 ? u << 3 : u >> (4 * j - 3), X));
+        v[j] = lds_f64_lt(base + j, len, V + 8 * j);
+    }
+#pragma unroll
+    for (int j = 0; j < N; ++j) acc = fma(v[j], xv[j], acc);
+}
+
+// CSR (Alg. 2), tm = longest row of the pair
+__device__ __forceinline__ void half_csr_tm(uint32_t RP, int nz, int tm, uint32_t X, int r, bool ok, double &acc) {
+    const int beg = (int)lds_u8(RP + r);
+    const int end = r < 15 ? (int)lds_u8(RP + r + 1) : nz;
+    const int len = ok ? end - beg : 0;
+    const uint32_t V = RP + 8 * (beg - nz);
+    const uint32_t wa = RP + 16 + 4 * (beg >> 3);
+    const uint32_t u = funnel_r(lds_u32(wa), lds_u32(wa + 4), 4u * beg);
+    if (tm == 3) {
+        csr_steps<3>(V, u, X, 0, len, acc);
+    } else if (tm <= 2) {
+        if (tm == 2) csr_steps<2>(V, u, X, 0, len, acc);
+        else csr_steps<1>(V, u, X, 0, len, acc);
+    } else {
+        csr_steps<4>(V, u, X, 0, len, acc);
+#pragma unroll 1
+        for (int i = 4; i < tm; i += 4) {
+            const uint32_t wb = RP + 16 + 4 * ((beg + i) >> 3);
+            const uint32_t ui = funnel_r(lds_u32(wb), lds_u32(wb + 4), 4u * (beg + i));
+            csr_steps<4>(V + 8 * i, ui, X, i, len, acc);
+        }
+    }
+}
+
+// ELL slots base .. base+N-1 of row r (column nibble bytes ci + 8k, shift sh)
+template <int N>
+__device__ __forceinline__ void ell_steps(uint32_t V, uint32_t ci, uint32_t sh, uint32_t X, int base, int wq,
+                                          double &acc) {
+    double xv[N], v[N];
+#pragma unroll
+    for (int j = 0; j < N; ++j) {
+        xv[j] = lds_f64(X + 8 * ((lds_u8(ci + 8 * j) >> sh) & 15u));
+        v[j] = lds_f64_lt(base + j, wq, V + 128 * j);
+    }
+#pragma unroll
+    for (int j = 0; j < N; ++j) acc = fma(v[j], xv[j], acc);
+}
+
+// ELL (Alg. 4), tm = larger width of the pair; pads are +0.0
+// at column 0 and are multiplied like entries (x finite, R19)
+__device__ __forceinline__ void half_ell_tm(uint32_t P, int w, int tm, uint32_t X, int r, bool ok, double &acc) {
+    const int wq = ok ? w : 0;
+    const uint32_t ci = P + 128 * w + (r >> 1);
+    const uint32_t sh = 4 * (r & 1);
+    const uint32_t V = P + 8 * r;
+    if (tm == 3) {
+        ell_steps<3>(V, ci, sh, X, 0, wq, acc);
+    } else if (tm <= 2) {
+        if (tm == 2) ell_steps<2>(V, ci, sh, X, 0, wq, acc);
+        else ell_steps<1>(V, ci, sh, X, 0, wq, acc);
+    } else {
+#pragma unroll 1
+        for (int k = 0; k < tm; k += 4) ell_steps<4>(V + 128 * k, ci + 8 * k, sh, X, k, wq, acc);
+    }
+}
+
 // HYB: ELL(w) values | COO values | ELL 4-bit columns | COO (row<<4|col)
 __device__ __forceinline__ void half_hyb(uint32_t P, int w, int nz, uint32_t X, int r, bool ok, double &acc) {
     const int kc = nz - 16 * w;

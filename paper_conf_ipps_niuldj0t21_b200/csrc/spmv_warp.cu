@@ -72,7 +72,8 @@ __device__ __forceinline__ WItem load_witem(const WItem *w, int k) {
 // lane r (and r + 16).  rpS: rebased row pointers (rows + 1), colS/valS: entries.
 //  * every row <= 4 entries (stencil-like): two lanes per row, two entries
 //    each, one round trip of gathers;
-//  * every row <= kShortRow entries: two lanes per row, all rows at once;
+//  * every row <= MED entries (kShortRow, or kMedRow for the TM kernels):
+//    two lanes per row, all rows at once;
 //  * a longer row (power-law hubs): the flat pass (flat_products, flat_rows),
 //    all gathers of the item in flight together.
 // The path and the order of every sum depend only on the item's content: y
@@ -81,6 +82,7 @@ __device__ __forceinline__ void flat_products(const Params &p, uint32_t colS, ui
                                               uint64_t x_policy, int lane);
 __device__ __forceinline__ double flat_rows(uint32_t rq, uint32_t valS, int rows, int lane);
 
+template <int MED>
 __device__ __forceinline__ void remainder(const Params &p, uint32_t rpS, uint32_t colS, uint32_t valS, int rows,
                                           uint64_t x_policy, int lane, double &acc) {
     const int r = lane & 15, h = lane >> 4;
@@ -100,7 +102,7 @@ __device__ __forceinline__ void remainder(const Params &p, uint32_t rpS, uint32_
         acc = fma(v1, x1, acc);
         return;
     }
-    if (maxlen > kShortRow) {
+    if (maxlen > MED) {
         flat_products(p, colS, valS, lds_s32(rpS + 4 * rows), x_policy, lane);
         acc += flat_rows(rpS, valS, rows, lane);
         return;
@@ -174,7 +176,7 @@ __device__ __forceinline__ double flat_rows(uint32_t rq, uint32_t valS, int rows
         const int myrow = (pair && h) ? r1 : r0;
         const int off = pair ? r : lane, stride = pair ? 16 : 32;
         const int bb = lds_s32(rq + 4 * myrow), e2 = lds_s32(rq + 4 * myrow + 4);
-        const int t2 = (int)__reduce_max_sync(FULL, (unsigned)((e2 - bb + 4 * stride - 1) / (4 * stride)));
+        const int t2 = (int)__reduce_max_sync(FULL, (unsigned)((e2 - bb + 4 * stride - 1) >> (pair ? 6 : 7)));
         double q0 = 0.0, q1 = 0.0, q2 = 0.0, q3 = 0.0;
 #pragma unroll 1
         for (int t = 0; t < t2; ++t) {
@@ -219,8 +221,10 @@ __device__ __forceinline__ void group_item(const Params &p, const WItem &it, uin
 
 // the tiles of one format group, two per step.  d: shared address of this
 // half's descriptor (see k_blob_fill): x = distance from the descriptor to the
-// tile's payload (CSR: to its csrRowPtr), y = aux | t*128 | nz << 11 | invalid << 31
-template <int F>
+// tile's payload (CSR: to its csrRowPtr), y = aux | t*128 | nz << 11 | tm << 20 |
+// invalid << 31 (tm: the pair's longest CSR row / larger ELL width).  TM:
+// run CSR and ELL with the tm routines.
+template <int F, bool TM>
 __device__ __forceinline__ void run_group(int np, uint32_t &d, uint32_t xs, int r, double &acc) {
 #pragma unroll 1
     for (int i = 0; i < np; ++i, d += 16) {
@@ -229,8 +233,11 @@ __device__ __forceinline__ void run_group(int np, uint32_t &d, uint32_t xs, int 
         const uint32_t P = d + e.x;
         const uint32_t X = xs + (e.y & 0x780u);
         const int aux = (int)(e.y & 31u), nz = (int)(e.y >> 11) & 511;
-        if (F == F_CSR) half_csr(P, nz, X, r, ok, acc);
-        if (F == F_ELL) half_ell(P, aux, X, r, ok, acc);
+        const int tm = (int)(e.y >> 20) & 31;
+        if (F == F_CSR && TM) half_csr_tm(P, nz, tm, X, r, ok, acc);
+        if (F == F_CSR && !TM) half_csr(P, nz, X, r, ok, acc);
+        if (F == F_ELL && TM) half_ell_tm(P, aux, tm, X, r, ok, acc);
+        if (F == F_ELL && !TM) half_ell(P, aux, X, r, ok, acc);
         if (F == F_DNS) half_dns(P, X, r, ok, acc);
         if (F == F_DNSCOL) half_dnscol(P, aux, X, r, ok, acc);
         if (F == F_DNSROW) half_dnsrow(P, aux, X, r, ok, acc);
@@ -296,6 +303,7 @@ __device__ __forceinline__ void issue_x(const Params &p, int J, int nt, uint32_t
 
 // steps 2-4 of an item whose blob is in `slot` and whose x segments are in
 // flight into `xs`: remainder, tiles, y (or the split-row carry)
+template <bool TM>
 __device__ __forceinline__ void compute_item(const Params &p, const WItem &it, uint32_t slot, uint32_t xs,
                                              uint32_t racc, uint64_t x_policy, int lane, double &carry) {
     if (it.jt_rows_pay & 0xFFu) {  // row-group item
@@ -309,7 +317,7 @@ __device__ __forceinline__ void compute_item(const Params &p, const WItem &it, u
     double acc = 0.0;
     const uint32_t rp = it.rp_col & 0xFFFFu;
     if (total > rp)
-        remainder(p, slot + rp, slot + (it.rp_col >> 16), slot + (it.val_tot & 0xFFFFu),
+        remainder<TM ? kMedRow : kShortRow>(p, slot + rp, slot + (it.rp_col >> 16), slot + (it.val_tot & 0xFFFFu),
                   (int)((it.jt_rows_pay >> 8) & 31u), x_policy, lane, acc);
     if (p.x_vec) cp_async_wait_all();
     __syncwarp();
@@ -317,13 +325,13 @@ __device__ __forceinline__ void compute_item(const Params &p, const WItem &it, u
     {
         const uint32_t g = it.groups;
         uint32_t d = slot + 8 * h;
-        run_group<F_CSR>((int)(g & 15u), d, xs, r, acc);
-        run_group<F_COO>((int)((g >> 4) & 15u), d, xs, r, acc);
-        run_group<F_ELL>((int)((g >> 8) & 15u), d, xs, r, acc);
-        run_group<F_HYB>((int)((g >> 12) & 15u), d, xs, r, acc);
-        run_group<F_DNS>((int)((g >> 16) & 15u), d, xs, r, acc);
-        run_group<F_DNSROW>((int)((g >> 20) & 15u), d, xs, r, acc);
-        run_group<F_DNSCOL>((int)((g >> 24) & 15u), d, xs, r, acc);
+        run_group<F_CSR, TM>((int)(g & 15u), d, xs, r, acc);
+        run_group<F_COO, TM>((int)((g >> 4) & 15u), d, xs, r, acc);
+        run_group<F_ELL, TM>((int)((g >> 8) & 15u), d, xs, r, acc);
+        run_group<F_HYB, TM>((int)((g >> 12) & 15u), d, xs, r, acc);
+        run_group<F_DNS, TM>((int)((g >> 16) & 15u), d, xs, r, acc);
+        run_group<F_DNSROW, TM>((int)((g >> 20) & 15u), d, xs, r, acc);
+        run_group<F_DNSCOL, TM>((int)((g >> 24) & 15u), d, xs, r, acc);
     }
     acc += __shfl_xor_sync(FULL, acc, 16);
     // 4. y, once per row
@@ -417,7 +425,7 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, MINB) tilespmv
         }
         TSP_STAMP(gw, k - kbeg, 1);
         TSP_INFO(gw, k - kbeg, k, it);
-        compute_item(p, it, slot, xs, racc, x_policy, lane, carry);
+        compute_item<false>(p, it, slot, xs, racc, x_policy, lane, carry);
         __syncwarp();  // slot and x scratch free for the next item
         TSP_STAMP(gw, k - kbeg, 3);
     }
@@ -432,7 +440,7 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, MINB) tilespmv
 // priority leaves the youngest CTAs as a serial tail).  Each warp claims its
 // next unit when it starts one, so the claim and the unit's bounds are in
 // flight while the current unit runs.
-template <int WARPS, int SLOT>
+template <int WARPS, int SLOT, bool TM>
 __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, 1) tilespmv_fp64_sm(const Params p) {
     using Cfg = WarpCfg<WARPS, SLOT>;
     extern __shared__ __align__(128) uint8_t smem[];
@@ -502,7 +510,7 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, 1) tilespmv_fp
         }
         TSP_STAMP(gw, j, 1);
         TSP_INFO(gw, j, k, it);
-        compute_item(p, it, slot, xs, racc, x_policy, lane, carry);
+        compute_item<TM>(p, it, slot, xs, racc, x_policy, lane, carry);
         __syncwarp();  // slot and x scratch free for the next item
         TSP_STAMP(gw, j, 3);
         ++j;
@@ -562,7 +570,7 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT, 2>::kThreads, MINB) tiles
             mbar_wait(bar, (phases >> s) & 1u);
             phases ^= 1u << s;
         }
-        compute_item(p, cur, slot, xs, racc, x_policy, lane, carry);
+        compute_item<false>(p, cur, slot, xs, racc, x_policy, lane, carry);
         __syncwarp();  // slot s and the x stage are free
         if (k + 2 < kend) issue_blob(p, n2, slot, bar, stream_policy, lane);
         cur = nx;
@@ -578,10 +586,10 @@ KernelChoice warp_choice(const char *name) {
     return {name, tilespmv_fp64_warp<WARPS, SLOT, MINB>, Cfg::kThreads, (int)Cfg::kSmem, 0, false, SLOT, true, false};
 }
 
-template <int WARPS, int SLOT>
+template <int WARPS, int SLOT, bool TM = false>
 KernelChoice sm_choice(const char *name) {
     using Cfg = WarpCfg<WARPS, SLOT>;
-    return {name, tilespmv_fp64_sm<WARPS, SLOT>, Cfg::kThreads, (int)Cfg::kSmem, 1, false, SLOT, true, true};
+    return {name, tilespmv_fp64_sm<WARPS, SLOT, TM>, Cfg::kThreads, (int)Cfg::kSmem, 1, false, SLOT, true, true};
 }
 
 template <int WARPS, int SLOT, int MINB>
@@ -610,6 +618,7 @@ KernelChoice kernel_warp(int variant) {
     case 40: return sm_choice<32, 4608>("tilespmv_fp64_sm<32,4608>");
     case 41: return sm_choice<16, 10752>("tilespmv_fp64_sm<16,10752>");
     case 42: return sm_choice<24, 6144>("tilespmv_fp64_sm<24,6144>");
+    case 43: return sm_choice<32, 4608, true>("tilespmv_fp64_sm<32,4608,tm>");
     default: return warp_choice<8, 4608, 4>("tilespmv_fp64_warp<8,4608>");
     }
 }

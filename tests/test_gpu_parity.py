@@ -261,7 +261,7 @@ def test_full_size_tiler_and_spmv(cuda_device, name):
         M.close()
 
 
-@pytest.mark.parametrize("variant", ["1", "20", "21", "22", "23", "24", "25", "26", "30", "31", "32", "33", "34", "40", "41", "42"])
+@pytest.mark.parametrize("variant", ["1", "20", "21", "22", "23", "24", "25", "26", "30", "31", "32", "33", "34", "40", "41", "42", "43"])
 def test_kernel_variants_parity(cuda_device, variant, monkeypatch):
     """Every SpMV kernel variant (TILESPMV_KERNEL, read at create time) meets
     the oracle tolerance; each is run-to-run bitwise deterministic."""
@@ -297,7 +297,7 @@ def test_misaligned_x_uses_scalar_path(cuda_device):
 
 @pytest.mark.parametrize("name", ["rmat12", "mixed_small", "stencil27_40", "lap2d_37x29", "heavy_row"])
 @pytest.mark.parametrize("mode", ["DEFERRED", "ADPT"])
-@pytest.mark.parametrize("variant", ["20", "25", "40", "41"])
+@pytest.mark.parametrize("variant", ["20", "25", "40", "41", "43"])
 def test_row_slices_bitwise_equal_full(cuda_device, name, mode, variant, monkeypatch):
     """Tile-row sharding relies on every row's summation order
     depending only on its own tile row (for a given kernel variant, i.e. slot
