@@ -219,6 +219,71 @@ __device__ __forceinline__ void group_item(const Params &p, const WItem &it, uin
     }
 }
 
+// Row-group item, TM kernels: after the flat pass, two tile rows at a time,
+// half-warp h on tile row g + h and lane r on its row r alone (4 running
+// sums over the row's products, in entry order mod 4); rows longer than
+// kShortRow are summed by the whole warp with an xor tree.  A tile row's sums
+// depend only on its own entries (grouping never changes a bit of y).
+__device__ __forceinline__ void group_item2(const Params &p, const WItem &it, uint32_t slot, uint64_t x_policy,
+                                            int lane) {
+    const int ntr = (int)(it.jt_rows_pay & 0xFFu);
+    const int rows_last = (int)((it.jt_rows_pay >> 8) & 31u);
+    const uint32_t total = it.val_tot >> 16, rp = it.rp_col & 0xFFFFu;
+    const bool has_rem = total > rp;
+    const uint32_t rpS = slot + rp, colS = slot + (it.rp_col >> 16), valS = slot + (it.val_tot & 0xFFFFu);
+    if (has_rem) flat_products(p, colS, valS, lds_s32(rpS + 4 * (16 * (ntr - 1) + rows_last)), x_policy, lane);
+    const int h = lane >> 4, r = lane & 15;
+#pragma unroll 1
+    for (int g = 0; g < ntr; g += 2) {
+        const int gg = g + h;
+        const int rows = gg < ntr ? (gg + 1 < ntr ? 16 : rows_last) : 0;
+        double acc = 0.0;
+        if (has_rem) {
+            const uint32_t rq = rpS + 64u * (uint32_t)gg;
+            const int b = lds_s32(rq + 4 * min(r, rows)), e = lds_s32(rq + 4 * min(r + 1, rows));
+            const bool lng = e - b > kShortRow;
+            const int ee = lng ? b : e;
+            const int trips = (int)__reduce_max_sync(FULL, (unsigned)((ee - b + 3) >> 2));
+            double s0 = 0.0, s1 = 0.0, s2 = 0.0, s3 = 0.0;
+#pragma unroll 1
+            for (int t = 0; t < trips; ++t) {
+                const int k = b + 4 * t;
+                s0 += lds_f64_lt(k, ee, valS + 8 * k);
+                s1 += lds_f64_lt(k + 1, ee, valS + 8 * k + 8);
+                s2 += lds_f64_lt(k + 2, ee, valS + 8 * k + 16);
+                s3 += lds_f64_lt(k + 3, ee, valS + 8 * k + 24);
+            }
+            acc = (s0 + s1) + (s2 + s3);
+            uint32_t lm = __ballot_sync(FULL, lng);
+#pragma unroll 1
+            while (lm) {  // one long row at a time, the whole warp
+                const int src = __ffs(lm) - 1;
+                lm &= lm - 1;
+                const int bb = __shfl_sync(FULL, b, src), e2 = __shfl_sync(FULL, e, src);
+                const int t2 = (e2 - bb + 127) >> 7;
+                double q0 = 0.0, q1 = 0.0, q2 = 0.0, q3 = 0.0;
+#pragma unroll 1
+                for (int t = 0; t < t2; ++t) {
+                    const int k = bb + lane + 128 * t;
+                    q0 += lds_f64_lt(k, e2, valS + 8 * k);
+                    q1 += lds_f64_lt(k + 32, e2, valS + 8 * k + 256);
+                    q2 += lds_f64_lt(k + 64, e2, valS + 8 * k + 512);
+                    q3 += lds_f64_lt(k + 96, e2, valS + 8 * k + 768);
+                }
+                double sq = (q0 + q1) + (q2 + q3);
+                sq += __shfl_xor_sync(FULL, sq, 16);
+                sq += __shfl_xor_sync(FULL, sq, 8);
+                sq += __shfl_xor_sync(FULL, sq, 4);
+                sq += __shfl_xor_sync(FULL, sq, 2);
+                sq += __shfl_xor_sync(FULL, sq, 1);
+                if (lane == src) acc += sq;
+            }
+        }
+        const int64_t row = 16 * ((int64_t)it.I + gg) + r;
+        if (gg < ntr && row < p.m) p.y[row] = acc;
+    }
+}
+
 // the tiles of one format group, two per step.  d: shared address of this
 // half's descriptor (see k_blob_fill): x = distance from the descriptor to the
 // tile's payload (CSR: to its csrRowPtr), y = aux | t*128 | nz << 11 | tm << 20 |
@@ -308,7 +373,8 @@ __device__ __forceinline__ void compute_item(const Params &p, const WItem &it, u
                                              uint32_t racc, uint64_t x_policy, int lane, double &carry) {
     if (it.jt_rows_pay & 0xFFu) {  // row-group item
         if (p.x_vec) cp_async_wait_all();
-        group_item(p, it, slot, x_policy, lane);
+        if (TM) group_item2(p, it, slot, x_policy, lane);
+        else group_item(p, it, slot, x_policy, lane);
         return;
     }
     const int h = lane >> 4, r = lane & 15;
