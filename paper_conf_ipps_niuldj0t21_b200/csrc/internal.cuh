@@ -68,7 +68,8 @@ struct __align__(16) WItem {
     uint32_t jt_rows_pay;  // tile rows of a row-group item (8 bits, 0: ordinary) | rows in the (last) tile row (5 bits) << 8 | payload offset << 16
     uint32_t rp_col;       // rp offset | col offset << 16
     uint32_t val_tot;      // val offset | total bytes << 16
-    uint32_t groups;       // tile pairs per format f, 4 bits at 4f (descriptor list order)
+    uint32_t groups;       // tile pairs per format f, 4 bits at 4f (descriptor list order);
+                           // bit 28: every CSR row of the item <= 3 entries, bit 29: every ELL width <= 3
 };
 
 // Per-warp start record of the warp kernel: the warp's item chunk and a copy

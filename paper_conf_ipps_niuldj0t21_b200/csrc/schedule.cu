@@ -263,6 +263,7 @@ __global__ void k_blob_fill(Item *items, int64_t n, int64_t m, const int64_t *st
     // larger extent of the two tiles of the half-warp pair (2j, 2j+1): CSR the
     // longest row, ELL the width (ndsc is even; the loop is warp-uniform)
     const uint8_t *tpay = payload + (size_t)it.offb * 16;
+    uint32_t csr_max = 0, ell_max = 0;
     for (int i0 = 0; i0 < it.ndsc; i0 += 32) {
         const int i = i0 + lane;
         uint2 e = make_uint2(0u, 0u);
@@ -286,7 +287,13 @@ __global__ void k_blob_fill(Item *items, int64_t n, int64_t m, const int64_t *st
         const uint32_t tmo = __shfl_xor_sync(0xFFFFFFFFu, tm, 1);
         tm = tmo > tm ? tmo : tm;
         if (i < it.ndsc) dd[i] = make_uint2(e.x, e.y | (tm << 20));
+        const uint32_t fi = i < it.ndsc ? dlist[it.dbeg + i].x >> 29 : 7u;
+        csr_max = max(csr_max, __reduce_max_sync(0xFFFFFFFFu, fi == F_CSR ? tm : 0u));
+        ell_max = max(ell_max, __reduce_max_sync(0xFFFFFFFFu, fi == F_ELL ? tm : 0u));
     }
+    // item-wide extents: the kernel runs such items' CSR / ELL groups with
+    // straight-line 3-step routines and no per-pair dispatch
+    if (lane == 0) witems[k].groups |= (csr_max <= 3 ? 1u << 28 : 0u) | (ell_max <= 3 ? 1u << 29 : 0u);
     const int nt = item_nt(it);
     if (lane < 16) jcols[k * 16 + lane] = lane < nt ? tileColIdx[it.tb + lane] : 0;
     const uint4 *ps = reinterpret_cast<const uint4 *>(payload + (size_t)it.offb * 16);

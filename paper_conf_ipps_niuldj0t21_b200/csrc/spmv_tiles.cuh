@@ -52,7 +52,11 @@ __device__ __forceinline__ void lds_entry_lt(int k, int e, uint32_t ca, uint32_t
 }
 // shared address of x[col] in a tile's 128-byte aligned x segment X, from a
 // column nibble already shifted to bits 3..6 (w's other bits are masked off)
-__device__ __forceinline__ uint32_t xaddr(uint32_t w8, uint32_t X) { return (w8 & 0x78u) | X; }
+__device__ __forceinline__ uint32_t xaddr(uint32_t w8, uint32_t X) {
+    uint32_t a;  // one LOP3: (w8 & 0x78) | X
+    asm("lop3.b32 %0, %1, 0x78, %2, 0xEA;" : "=r"(a) : "r"(w8), "r"(X));
+    return a;
+}
 __device__ __forceinline__ uint32_t funnel_r(uint32_t lo, uint32_t hi, uint32_t sh) {
     return __funnelshift_r(lo, hi, sh);
 }
@@ -232,14 +236,28 @@ __device__ __forceinline__ void half_csr_tm(uint32_t RP, int nz, int tm, uint32_
     }
 }
 
-// ELL slots base .. base+N-1 of row r (column nibble bytes ci + 8k, shift sh)
+// CSR of an item whose rows all hold <= N entries: N straight-line steps
 template <int N>
-__device__ __forceinline__ void ell_steps(uint32_t V, uint32_t ci, uint32_t sh, uint32_t X, int base, int wq,
+__device__ __forceinline__ void half_csr_n(uint32_t RP, int nz, uint32_t X, int r, bool ok, double &acc) {
+    const int beg = (int)lds_u8(RP + r);
+    const int end = r < 15 ? (int)lds_u8(RP + r + 1) : nz;
+    const int len = ok ? end - beg : 0;
+    const uint32_t wa = RP + 16 + 4 * (beg >> 3);
+    const uint32_t u = funnel_r(lds_u32(wa), lds_u32(wa + 4), 4u * beg);
+    csr_steps<N>(RP + 8 * (beg - nz), u, X, 0, len, acc);
+}
+
+// ELL slots base .. base+N-1 of row r (column nibble bytes ci + 8k, shift sh)
+// rot = 3 (even row: low nibble) or 31 (odd row: high nibble): rotating the
+// nibble byte left by rot puts the row's column at bits 3..6
+template <int N>
+__device__ __forceinline__ void ell_steps(uint32_t V, uint32_t ci, uint32_t rot, uint32_t X, int base, int wq,
                                           double &acc) {
     double xv[N], v[N];
 #pragma unroll
     for (int j = 0; j < N; ++j) {
-        xv[j] = lds_f64(X + 8 * ((lds_u8(ci + 8 * j) >> sh) & 15u));
+        const uint32_t b = lds_u8(ci + 8 * j);
+        xv[j] = lds_f64(xaddr(__funnelshift_l(b, b, rot), X));
         v[j] = lds_f64_lt(base + j, wq, V + 128 * j);
     }
 #pragma unroll
@@ -251,17 +269,23 @@ __device__ __forceinline__ void ell_steps(uint32_t V, uint32_t ci, uint32_t sh, 
 __device__ __forceinline__ void half_ell_tm(uint32_t P, int w, int tm, uint32_t X, int r, bool ok, double &acc) {
     const int wq = ok ? w : 0;
     const uint32_t ci = P + 128 * w + (r >> 1);
-    const uint32_t sh = 4 * (r & 1);
+    const uint32_t rot = (r & 1) ? 31u : 3u;
     const uint32_t V = P + 8 * r;
     if (tm == 3) {
-        ell_steps<3>(V, ci, sh, X, 0, wq, acc);
+        ell_steps<3>(V, ci, rot, X, 0, wq, acc);
     } else if (tm <= 2) {
-        if (tm == 2) ell_steps<2>(V, ci, sh, X, 0, wq, acc);
-        else ell_steps<1>(V, ci, sh, X, 0, wq, acc);
+        if (tm == 2) ell_steps<2>(V, ci, rot, X, 0, wq, acc);
+        else ell_steps<1>(V, ci, rot, X, 0, wq, acc);
     } else {
 #pragma unroll 1
-        for (int k = 0; k < tm; k += 4) ell_steps<4>(V + 128 * k, ci + 8 * k, sh, X, k, wq, acc);
+        for (int k = 0; k < tm; k += 4) ell_steps<4>(V + 128 * k, ci + 8 * k, rot, X, k, wq, acc);
     }
+}
+
+// ELL of an item whose widths are all <= N: N straight-line steps
+template <int N>
+__device__ __forceinline__ void half_ell_n(uint32_t P, int w, uint32_t X, int r, bool ok, double &acc) {
+    ell_steps<N>(P + 8 * r, P + 128 * w + (r >> 1), (r & 1) ? 31u : 3u, X, 0, ok ? w : 0, acc);
 }
 
 // HYB: ELL(w) values | COO values | ELL 4-bit columns | COO (row<<4|col)

@@ -84,7 +84,7 @@ __device__ __forceinline__ double flat_rows(uint32_t rq, uint32_t valS, int rows
 
 template <int MED>
 __device__ __forceinline__ void remainder(const Params &p, uint32_t rpS, uint32_t colS, uint32_t valS, int rows,
-                                          uint64_t x_policy, int lane, double &acc) {
+                                          uint64_t x_policy, int lane, double &acc, bool &dirty) {
     const int r = lane & 15, h = lane >> 4;
     const int b = lds_s32(rpS + 4 * min(r, rows)), e = lds_s32(rpS + 4 * min(r + 1, rows));
     const double *x = p.x;
@@ -103,6 +103,7 @@ __device__ __forceinline__ void remainder(const Params &p, uint32_t rpS, uint32_
         return;
     }
     if (maxlen > MED) {
+        dirty = true;  // the slot now holds products written by the generic proxy
         flat_products(p, colS, valS, lds_s32(rpS + 4 * rows), x_policy, lane);
         acc += flat_rows(rpS, valS, rows, lane);
         return;
@@ -289,7 +290,7 @@ __device__ __forceinline__ void group_item2(const Params &p, const WItem &it, ui
 // tile's payload (CSR: to its csrRowPtr), y = aux | t*128 | nz << 11 | tm << 20 |
 // invalid << 31 (tm: the pair's longest CSR row / larger ELL width).  TM:
 // run CSR and ELL with the tm routines.
-template <int F, bool TM>
+template <int F, bool TM, int N = 0>
 __device__ __forceinline__ void run_group(int np, uint32_t &d, uint32_t xs, int r, double &acc) {
 #pragma unroll 1
     for (int i = 0; i < np; ++i, d += 16) {
@@ -299,9 +300,11 @@ __device__ __forceinline__ void run_group(int np, uint32_t &d, uint32_t xs, int 
         const uint32_t X = xs + (e.y & 0x780u);
         const int aux = (int)(e.y & 31u), nz = (int)(e.y >> 11) & 511;
         const int tm = (int)(e.y >> 20) & 31;
-        if (F == F_CSR && TM) half_csr_tm(P, nz, tm, X, r, ok, acc);
+        if (F == F_CSR && N == 3) half_csr_n<3>(P, nz, X, r, ok, acc);
+        if (F == F_CSR && TM && N == 0) half_csr_tm(P, nz, tm, X, r, ok, acc);
         if (F == F_CSR && !TM) half_csr(P, nz, X, r, ok, acc);
-        if (F == F_ELL && TM) half_ell_tm(P, aux, tm, X, r, ok, acc);
+        if (F == F_ELL && N == 3) half_ell_n<3>(P, aux, X, r, ok, acc);
+        if (F == F_ELL && TM && N == 0) half_ell_tm(P, aux, tm, X, r, ok, acc);
         if (F == F_ELL && !TM) half_ell(P, aux, X, r, ok, acc);
         if (F == F_DNS) half_dns(P, X, r, ok, acc);
         if (F == F_DNSCOL) half_dnscol(P, aux, X, r, ok, acc);
@@ -311,12 +314,14 @@ __device__ __forceinline__ void run_group(int np, uint32_t &d, uint32_t xs, int 
     }
 }
 
-// lane 0: the whole item (descriptors, payload, remainder) in ONE TMA bulk copy
+// lane 0: the whole item (descriptors, payload, remainder) in ONE TMA bulk copy.
+// fence: the previous item wrote the slot with generic-proxy stores (flat
+// pass), which must be ordered before the async-proxy write
 __device__ __forceinline__ void issue_blob(const Params &p, const WItem &it, uint32_t slot, uint32_t bar,
-                                           uint64_t policy, int lane) {
+                                           uint64_t policy, int lane, bool fence = true) {
     const uint32_t total = it.val_tot >> 16;
     if (lane == 0 && total) {
-        fence_proxy_async();
+        if (fence) fence_proxy_async();
         mbar_expect_tx(bar, total);
         bulk_g2s_hint(slot, p.blob + (size_t)it.blob16 * 16, total, bar, policy);
     }
@@ -370,8 +375,10 @@ __device__ __forceinline__ void issue_x(const Params &p, int J, int nt, uint32_t
 // flight into `xs`: remainder, tiles, y (or the split-row carry)
 template <bool TM>
 __device__ __forceinline__ void compute_item(const Params &p, const WItem &it, uint32_t slot, uint32_t xs,
-                                             uint32_t racc, uint64_t x_policy, int lane, double &carry) {
+                                             uint32_t racc, uint64_t x_policy, int lane, double &carry,
+                                             bool &dirty) {
     if (it.jt_rows_pay & 0xFFu) {  // row-group item
+        dirty = true;
         if (p.x_vec) cp_async_wait_all();
         if (TM) group_item2(p, it, slot, x_policy, lane);
         else group_item(p, it, slot, x_policy, lane);
@@ -384,16 +391,20 @@ __device__ __forceinline__ void compute_item(const Params &p, const WItem &it, u
     const uint32_t rp = it.rp_col & 0xFFFFu;
     if (total > rp)
         remainder<TM ? kMedRow : kShortRow>(p, slot + rp, slot + (it.rp_col >> 16), slot + (it.val_tot & 0xFFFFu),
-                  (int)((it.jt_rows_pay >> 8) & 31u), x_policy, lane, acc);
+                  (int)((it.jt_rows_pay >> 8) & 31u), x_policy, lane, acc, dirty);
     if (p.x_vec) cp_async_wait_all();
     __syncwarp();
     // 3. tiles: format group by format group, two tiles per step
     {
         const uint32_t g = it.groups;
         uint32_t d = slot + 8 * h;
-        run_group<F_CSR, TM>((int)(g & 15u), d, xs, r, acc);
+        // TM: items whose CSR rows / ELL widths are all <= 3 (bits 28, 29)
+        // run those groups without per-pair dispatch
+        if (TM && ((g >> 28) & 1u)) run_group<F_CSR, TM, 3>((int)(g & 15u), d, xs, r, acc);
+        else run_group<F_CSR, TM>((int)(g & 15u), d, xs, r, acc);
         run_group<F_COO, TM>((int)((g >> 4) & 15u), d, xs, r, acc);
-        run_group<F_ELL, TM>((int)((g >> 8) & 15u), d, xs, r, acc);
+        if (TM && ((g >> 29) & 1u)) run_group<F_ELL, TM, 3>((int)((g >> 8) & 15u), d, xs, r, acc);
+        else run_group<F_ELL, TM>((int)((g >> 8) & 15u), d, xs, r, acc);
         run_group<F_HYB, TM>((int)((g >> 12) & 15u), d, xs, r, acc);
         run_group<F_DNS, TM>((int)((g >> 16) & 15u), d, xs, r, acc);
         run_group<F_DNSROW, TM>((int)((g >> 20) & 15u), d, xs, r, acc);
@@ -468,6 +479,7 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, MINB) tilespmv
     const int4 wb = __ldg(reinterpret_cast<const int4 *>(wf));
     const int kbeg = wb.x, kend = wb.y;
     double carry = 0.0;  // partial row sums inside a group of parts of a split tile row
+    bool dirty = true;   // the slot may hold generic-proxy writes (TM kernels track it)
     uint32_t phase = 0;
     const uint64_t stream_policy = policy_evict_first(), x_policy = policy_evict_last();
     WItem nxt = load_witem(&wf->w, 0);
@@ -491,7 +503,7 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, MINB) tilespmv
         }
         TSP_STAMP(gw, k - kbeg, 1);
         TSP_INFO(gw, k - kbeg, k, it);
-        compute_item<false>(p, it, slot, xs, racc, x_policy, lane, carry);
+        compute_item<false>(p, it, slot, xs, racc, x_policy, lane, carry, dirty);
         __syncwarp();  // slot and x scratch free for the next item
         TSP_STAMP(gw, k - kbeg, 3);
     }
@@ -527,6 +539,7 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, 1) tilespmv_fp
     TSP_SMID(gw, (int64_t)gridDim.x * WARPS);
     (void)gw;
     double carry = 0.0;  // partial row sums inside a group of parts of a split tile row
+    bool dirty = true;   // the slot may hold generic-proxy writes (TM kernels track it)
     uint32_t phase = 0;
     const uint64_t stream_policy = policy_evict_first(), x_policy = policy_evict_last();
     int k = -1, ke = 0, nb = -1, ne = 0;
@@ -547,7 +560,8 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, 1) tilespmv_fp
         const WItem it = nxt;
         const int J = Jn;
         TSP_STAMP(gw, j, 0);
-        issue_blob(p, it, slot, bar, stream_policy, lane);
+        issue_blob(p, it, slot, bar, stream_policy, lane, !TM || dirty);
+        dirty = false;
         // the matrix is immutable; x and y may belong to the previous kernel
         if (!waited) {
             griddep_wait();
@@ -576,7 +590,7 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, 1) tilespmv_fp
         }
         TSP_STAMP(gw, j, 1);
         TSP_INFO(gw, j, k, it);
-        compute_item<TM>(p, it, slot, xs, racc, x_policy, lane, carry);
+        compute_item<TM>(p, it, slot, xs, racc, x_policy, lane, carry, dirty);
         __syncwarp();  // slot and x scratch free for the next item
         TSP_STAMP(gw, j, 3);
         ++j;
@@ -610,6 +624,7 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT, 2>::kThreads, MINB) tiles
     const int4 wb = __ldg(reinterpret_cast<const int4 *>(wf));
     const int kbeg = wb.x, kend = wb.y;
     double carry = 0.0;
+    bool dirty = true;
     uint32_t phases = 0;  // bit s: parity of slot s's barrier
     const uint64_t stream_policy = policy_evict_first(), x_policy = policy_evict_last();
     WItem cur = load_witem(&wf->w, 0), nx{};
@@ -636,7 +651,7 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT, 2>::kThreads, MINB) tiles
             mbar_wait(bar, (phases >> s) & 1u);
             phases ^= 1u << s;
         }
-        compute_item<false>(p, cur, slot, xs, racc, x_policy, lane, carry);
+        compute_item<false>(p, cur, slot, xs, racc, x_policy, lane, carry, dirty);
         __syncwarp();  // slot s and the x stage are free
         if (k + 2 < kend) issue_blob(p, n2, slot, bar, stream_policy, lane);
         cur = nx;
