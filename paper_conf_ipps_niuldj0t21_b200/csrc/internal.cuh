@@ -69,7 +69,8 @@ struct __align__(16) WItem {
     uint32_t rp_col;       // rp offset | col offset << 16
     uint32_t val_tot;      // val offset | total bytes << 16
     uint32_t groups;       // tile pairs per format f, 4 bits at 4f (descriptor list order);
-                           // bit 28: every CSR row of the item <= 3 entries, bit 29: every ELL width <= 3
+                           // bit 28: every CSR row of the item <= 3 entries, bit 29: every ELL width <= 3,
+                           // bit 30: the last tile column's x segment passes x[n-1] (ragged tail)
 };
 
 // Per-warp start record of the warp kernel: the warp's item chunk and a copy

@@ -223,13 +223,13 @@ __global__ void k_blob_len(const Item *items, int64_t n, int64_t m, int64_t *len
 }
 
 // one warp per item: copy descriptors, J, payload and the rebased remainder
-__global__ void k_blob_fill(Item *items, int64_t n, int64_t m, const int64_t *start16, const uint2 *dlist,
+__global__ void k_blob_fill(Item *items, int64_t nitems, int64_t m, int64_t n, const int64_t *start16, const uint2 *dlist,
                             const int32_t *tileColIdx, const uint8_t *tileFmt, const uint8_t *payload,
                             const int32_t *remRowPtr, const int32_t *remCol, const double *remVal, uint8_t *blob,
                             WItem *witems, int32_t *jcols) {
     const int64_t k = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
     const int lane = threadIdx.x & 31;
-    if (k >= n) return;
+    if (k >= nitems) return;
     Item it = items[k];
     const BlobParts b = blob_parts(it, m);
     uint8_t *dst = blob + start16[k] * 16;
@@ -293,8 +293,10 @@ __global__ void k_blob_fill(Item *items, int64_t n, int64_t m, const int64_t *st
     }
     // item-wide extents: the kernel runs such items' CSR / ELL groups with
     // straight-line 3-step routines and no per-pair dispatch
-    if (lane == 0) witems[k].groups |= (csr_max <= 3 ? 1u << 28 : 0u) | (ell_max <= 3 ? 1u << 29 : 0u);
     const int nt = item_nt(it);
+    const bool xtail = nt > 0 && 16 * (int64_t)tileColIdx[it.tb + nt - 1] + 16 > n;
+    if (lane == 0)
+        witems[k].groups |= (csr_max <= 3 ? 1u << 28 : 0u) | (ell_max <= 3 ? 1u << 29 : 0u) | (xtail ? 1u << 30 : 0u);
     if (lane < 16) jcols[k * 16 + lane] = lane < nt ? tileColIdx[it.tb + lane] : 0;
     const uint4 *ps = reinterpret_cast<const uint4 *>(payload + (size_t)it.offb * 16);
     uint4 *pd = reinterpret_cast<uint4 *>(dst + b.pay);
@@ -521,7 +523,7 @@ int build_tdesc(Matrix &M, cudaStream_t st) {
             break;
         }
         M.device_bytes += n * (int64_t)(sizeof(WItem) + 64);
-        k_blob_fill<<<(unsigned)((n * 32 + 255) / 256), 256, 0, st>>>(M.items, n, M.m, start16, M.tdesc, M.tileColIdx,
+        k_blob_fill<<<(unsigned)((n * 32 + 255) / 256), 256, 0, st>>>(M.items, n, M.m, M.n, start16, M.tdesc, M.tileColIdx,
                                                                      M.tileFmt, M.payload, M.remRowPtr, M.remCol,
                                                                      M.remVal, M.blob, M.witems, M.jcols);
         if (cudaStreamSynchronize(st) != cudaSuccess) rc = cuda_status(cudaGetLastError(), "k_blob_fill");
