@@ -216,10 +216,14 @@ __global__ void k_dsc_write(Item *items, int64_t n, const int32_t *dbeg, const i
     }
 }
 
-__global__ void k_blob_len(const Item *items, int64_t n, int64_t m, int64_t *len16) {
+// blob length per item; *over is set if one exceeds the kernel's slot (a
+// schedule bug: the kernel would stage past its shared-memory slot)
+__global__ void k_blob_len(const Item *items, int64_t n, int64_t m, uint32_t slot, int64_t *len16, int32_t *over) {
     int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     if (k >= n) return;
-    len16[k] = blob_parts(items[k], m).total / 16;
+    const uint32_t total = blob_parts(items[k], m).total;
+    len16[k] = total / 16;
+    if (total > slot) atomicOr(over, 1);
 }
 
 // one warp per item: copy descriptors, J, payload and the rebased remainder
@@ -507,11 +511,15 @@ int build_tdesc(Matrix &M, cudaStream_t st) {
         if (cudaMalloc(&len16, 2 * (n + 1) * sizeof(int64_t)) != cudaSuccess) { rc = cuda_status(cudaGetLastError(), "cudaMalloc(blob sizes)"); break; }
         int64_t *start16 = len16 + (n + 1);
         cudaMemsetAsync(len16 + n, 0, sizeof(int64_t), st);
-        k_blob_len<<<nb, 256, 0, st>>>(M.items, n, M.m, len16);
+        cudaMemsetAsync(cnt + n, 0, sizeof(int32_t), st);  // cnt[n]: slot overflow flag
+        k_blob_len<<<nb, 256, 0, st>>>(M.items, n, M.m, (uint32_t)choose(M.kernel_version).slot_bytes, len16, cnt + n);
         if ((rc = scan([&](void *t, size_t &b) { return cub::DeviceScan::ExclusiveSum(t, b, len16, start16, (int)(n + 1), st); }))) { cudaFree(len16); break; }
         int64_t total16 = 0;
+        int32_t over = 0;
         cudaMemcpyAsync(&total16, start16 + n, 8, cudaMemcpyDeviceToHost, st);
+        cudaMemcpyAsync(&over, cnt + n, 4, cudaMemcpyDeviceToHost, st);
         if (cudaStreamSynchronize(st) != cudaSuccess) { rc = cuda_status(cudaGetLastError(), "blob size"); cudaFree(len16); break; }
+        if (over) { rc = set_error(TILESPMV_CUDA, "schedule: an item's blob exceeds the kernel's slot"); cudaFree(len16); break; }
         if (total16 >= (int64_t(1) << 32)) { rc = set_error(TILESPMV_OVERFLOW, "execution blob >= 64 GiB"); cudaFree(len16); break; }
         M.blob_bytes = total16 * 16;
         if (cudaMalloc(&M.blob, M.blob_bytes + 256) != cudaSuccess) { rc = cuda_status(cudaGetLastError(), "cudaMalloc(blob)"); cudaFree(len16); break; }
