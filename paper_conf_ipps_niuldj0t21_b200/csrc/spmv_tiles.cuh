@@ -29,6 +29,11 @@ __device__ __forceinline__ uint2 lds_v2u32(uint32_t a) {
     asm volatile("ld.shared.v2.u32 {%0, %1}, [%2];" : "=r"(v.x), "=r"(v.y) : "r"(a));
     return v;
 }
+__device__ __forceinline__ double2 lds_v2f64(uint32_t a) {  // a 16-byte aligned
+    double2 v;
+    asm volatile("ld.shared.v2.f64 {%0, %1}, [%2];" : "=d"(v.x), "=d"(v.y) : "r"(a));
+    return v;
+}
 __device__ __forceinline__ uint32_t lds_u32(uint32_t a) {
     uint32_t v;
     asm("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(a));
@@ -132,14 +137,16 @@ __device__ __forceinline__ void half_ell(uint32_t P, int w, uint32_t X, int r, b
     }
 }
 
-// Dns: 256 values column-major
+// Dns: 256 values column-major; x[c], x[c+1] arrive as one
+// 16-byte broadcast load
 __device__ __forceinline__ void half_dns(uint32_t P, uint32_t X, int r, bool ok, double &acc) {
     const uint32_t V = P + 8 * r;
     double a0 = 0.0, a1 = 0.0;
 #pragma unroll
     for (int c = 0; c < 16; c += 2) {
-        a0 = fma(lds_f64(V + 128 * c), lds_f64(X + 8 * c), a0);
-        a1 = fma(lds_f64(V + 128 * c + 128), lds_f64(X + 8 * c + 8), a1);
+        const double2 xc = lds_v2f64(X + 8 * c);
+        a0 = fma(lds_f64(V + 128 * c), xc.x, a0);
+        a1 = fma(lds_f64(V + 128 * c + 128), xc.y, a1);
     }
     if (ok) acc += a0 + a1;
 }
@@ -153,6 +160,25 @@ __device__ __forceinline__ void half_dnscol(uint32_t P, int nc, uint32_t X, int 
         const double v = lds_f64_lt(q, nq, P + 8 * (16 * q + r));
         const double xv = lds_f64(X + 8 * (lds_u8(cid + q) & 15u));
         acc = fma(v, xv, acc);
+    }
+}
+
+// DnsRow, the paper's mapping: lane c of the half multiplies value
+// q*16 + c of every full row q by x[c] (one coalesced 128-byte row per q),
+// a 16-lane xor tree sums the row, and the lane r == rowid[q] adds it.
+__device__ __forceinline__ void half_dnsrow_tree(uint32_t P, int nr, uint32_t X, int r, bool ok, double &acc) {
+    const uint32_t rid = P + 128 * nr;
+    const int nq = ok ? nr : 0;
+    const int trips = (int)__reduce_max_sync(FULL, (unsigned)nq);
+    const double xc = lds_f64(X + 8 * r);
+#pragma unroll 1
+    for (int q = 0; q < trips; ++q) {
+        double s = lds_f64_lt(q, nq, P + 8 * (16 * q + r)) * xc;
+        s += __shfl_xor_sync(FULL, s, 8);
+        s += __shfl_xor_sync(FULL, s, 4);
+        s += __shfl_xor_sync(FULL, s, 2);
+        s += __shfl_xor_sync(FULL, s, 1);
+        if (q < nq && (int)lds_u8(rid + q) == r) acc += s;
     }
 }
 

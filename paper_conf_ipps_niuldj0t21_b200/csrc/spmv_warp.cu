@@ -308,7 +308,8 @@ __device__ __forceinline__ void run_group(int np, uint32_t &d, uint32_t xs, int 
         if (F == F_ELL && !TM) half_ell(P, aux, X, r, ok, acc);
         if (F == F_DNS) half_dns(P, X, r, ok, acc);
         if (F == F_DNSCOL) half_dnscol(P, aux, X, r, ok, acc);
-        if (F == F_DNSROW) half_dnsrow(P, aux, X, r, ok, acc);
+        if (F == F_DNSROW && TM) half_dnsrow_tree(P, aux, X, r, ok, acc);
+        if (F == F_DNSROW && !TM) half_dnsrow(P, aux, X, r, ok, acc);
         if (F == F_COO) half_coo(P, P + 8 * nz, nz, X, r, ok, acc);
         if (F == F_HYB) half_hyb(P, aux, nz, X, r, ok, acc);
     }
