@@ -314,6 +314,48 @@ __device__ __forceinline__ void half_ell_n(uint32_t P, int w, uint32_t X, int r,
     ell_steps<N>(P + 8 * r, P + 128 * w + (r >> 1), (r & 1) ? 31u : 3u, X, 0, ok ? w : 0, acc);
 }
 
+// COO (n <= 11 by the selection rule; Alg. 3) with one lane
+// per entry: lane j of the half multiplies entry j; an inclusive segmented
+// scan over the half (entries are row-major, so a row's entries are adjacent
+// lanes) leaves each row's sum on the row's last entry, which stores it in
+// the warp's row scratch S (16 doubles per half) for the row's lane.
+__device__ __forceinline__ void half_coo_scan(uint32_t V, uint32_t rc, int n, uint32_t X, int r, int h, uint32_t S,
+                                              bool ok, double &acc) {
+    const int nq = ok ? n : 0;
+    const bool have = r < nq;
+    uint32_t b = 0;
+    double p = 0.0;
+    if (have) {
+        b = lds_u8(rc + r);
+        p = lds_f64(V + 8 * r) * lds_f64(X + 8 * (b & 15u));
+    }
+    const int row = have ? (int)(b >> 4) : 16 + r;  // idle lanes: a row of their own
+    {  // (every lane executes every shuffle: no shuffle inside a short-circuit)
+        const double pp = __shfl_up_sync(FULL, p, 1, 16);
+        const int r1 = __shfl_up_sync(FULL, row, 1, 16);
+        if (r >= 1 && r1 == row) p += pp;
+    }
+    // rows of three or more entries are rare in a COO tile (n <= 11): the
+    // longer steps run only when some row needs them
+    const int r2 = __shfl_up_sync(FULL, row, 2, 16);
+    if (__any_sync(FULL, r >= 2 && r2 == row)) {
+#pragma unroll
+        for (int off = 2; off < 16; off <<= 1) {
+            const double pp = __shfl_up_sync(FULL, p, off, 16);
+            const int rr = __shfl_up_sync(FULL, row, off, 16);
+            if (r >= off && rr == row) p += pp;
+        }
+    }
+    const int rnext = __shfl_down_sync(FULL, row, 1, 16);
+    const bool tail = have && (r == nq - 1 || rnext != row);
+    const uint32_t rows = __reduce_or_sync(FULL, tail ? 1u << (16 * h + row) : 0u);
+    const uint32_t Sh = S + 128 * h;
+    __syncwarp();  // the previous pair's reads of S are done
+    if (tail) sts_f64(Sh + 8 * row, p);
+    __syncwarp();
+    if ((rows >> (16 * h + r)) & 1u) acc += lds_f64(Sh + 8 * r);
+}
+
 // HYB: ELL(w) values | COO values | ELL 4-bit columns | COO (row<<4|col)
 __device__ __forceinline__ void half_hyb(uint32_t P, int w, int nz, uint32_t X, int r, bool ok, double &acc) {
     const int kc = nz - 16 * w;

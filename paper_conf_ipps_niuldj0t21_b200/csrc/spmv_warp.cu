@@ -48,13 +48,14 @@ __device__ __forceinline__ unsigned long long gtimer() {
 
 namespace {
 
-template <int WARPS, int SLOT, int NBUF = 1>
+template <int WARPS, int SLOT, int NBUF = 1, int RACC = 128>
 struct WarpCfg {
     static_assert(SLOT % 16 == 0 && SLOT <= kItemBytesMax, "slot size");
     // [x stage of every warp, 2 KB each, 128-byte aligned] [per warp: NBUF
-    // slots | row sums | mbarriers]
+    // slots | row-sum scratch (RACC bytes) | mbarriers]
     static constexpr uint32_t kX = kItemTiles * 16 * 8;
-    static constexpr uint32_t kPer = NBUF * SLOT + 128 + 16;
+    static constexpr uint32_t kRacc = RACC;
+    static constexpr uint32_t kPer = NBUF * SLOT + RACC + 16;
     static constexpr uint32_t kSmem = WARPS * (kX + kPer) + 256;  // +256: loads may overrun a slot
     static constexpr int kThreads = 32 * WARPS;
 };
@@ -291,7 +292,8 @@ __device__ __forceinline__ void group_item2(const Params &p, const WItem &it, ui
 // invalid << 31 (tm: the pair's longest CSR row / larger ELL width).  TM:
 // run CSR and ELL with the tm routines.
 template <int F, bool TM, int N = 0>
-__device__ __forceinline__ void run_group(int np, uint32_t &d, uint32_t xs, int r, double &acc) {
+__device__ __forceinline__ void run_group(int np, uint32_t &d, uint32_t xs, int r, double &acc, uint32_t racc = 0) {
+    const int lane_h = (int)(threadIdx.x >> 4) & 1;
 #pragma unroll 1
     for (int i = 0; i < np; ++i, d += 16) {
         const uint2 e = lds_v2u32(d);
@@ -310,7 +312,8 @@ __device__ __forceinline__ void run_group(int np, uint32_t &d, uint32_t xs, int 
         if (F == F_DNSCOL) half_dnscol(P, aux, X, r, ok, acc);
         if (F == F_DNSROW && TM) half_dnsrow_tree(P, aux, X, r, ok, acc);
         if (F == F_DNSROW && !TM) half_dnsrow(P, aux, X, r, ok, acc);
-        if (F == F_COO) half_coo(P, P + 8 * nz, nz, X, r, ok, acc);
+        if (F == F_COO && TM) half_coo_scan(P, P + 8 * nz, nz, X, r, lane_h, racc, ok, acc);
+        if (F == F_COO && !TM) half_coo(P, P + 8 * nz, nz, X, r, ok, acc);
         if (F == F_HYB) half_hyb(P, aux, nz, X, r, ok, acc);
     }
 }
@@ -406,7 +409,7 @@ __device__ __forceinline__ void compute_item(const Params &p, const WItem &it, u
         // run those groups without per-pair dispatch
         if (TM && ((g >> 28) & 1u)) run_group<F_CSR, TM, 3>((int)(g & 15u), d, xs, r, acc);
         else run_group<F_CSR, TM>((int)(g & 15u), d, xs, r, acc);
-        if (!TM || (g & 0xF0u)) run_group<F_COO, TM>((int)((g >> 4) & 15u), d, xs, r, acc);
+        if (!TM || (g & 0xF0u)) run_group<F_COO, TM>((int)((g >> 4) & 15u), d, xs, r, acc, racc);
         if (TM && ((g >> 29) & 1u)) run_group<F_ELL, TM, 3>((int)((g >> 8) & 15u), d, xs, r, acc);
         else run_group<F_ELL, TM>((int)((g >> 8) & 15u), d, xs, r, acc);
         if (!TM || (g & 0x0FFFF000u)) {  // TM: one test skips the four rarer formats
@@ -526,13 +529,13 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, MINB) tilespmv
 // flight while the current unit runs.
 template <int WARPS, int SLOT, bool TM>
 __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, 1) tilespmv_fp64_sm(const Params p) {
-    using Cfg = WarpCfg<WARPS, SLOT>;
+    using Cfg = WarpCfg<WARPS, SLOT, 1, TM ? 256 : 128>;
     extern __shared__ __align__(128) uint8_t smem[];
     __shared__ int s_next;
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const uint32_t xs = smem_u32(smem) + (uint32_t)warp * Cfg::kX;
     const uint32_t slot = smem_u32(smem) + WARPS * Cfg::kX + (uint32_t)warp * Cfg::kPer;
-    const uint32_t racc = slot + SLOT, bar = racc + 128;
+    const uint32_t racc = slot + SLOT, bar = racc + Cfg::kRacc;
     const int ub = (int)__ldg(p.cta_begin + blockIdx.x), ue = (int)__ldg(p.cta_begin + blockIdx.x + 1);
     if (lane == 0) {
         mbar_init(bar, 1);
@@ -675,7 +678,7 @@ KernelChoice warp_choice(const char *name) {
 
 template <int WARPS, int SLOT, bool TM = false>
 KernelChoice sm_choice(const char *name) {
-    using Cfg = WarpCfg<WARPS, SLOT>;
+    using Cfg = WarpCfg<WARPS, SLOT, 1, TM ? 256 : 128>;
     return {name, tilespmv_fp64_sm<WARPS, SLOT, TM>, Cfg::kThreads, (int)Cfg::kSmem, 1, false, SLOT, true, true};
 }
 
