@@ -83,3 +83,24 @@ def test_no_cpu_fallback():
     with pytest.raises(TileSpMVError, match="no CUDA device"):
         TiledMatrix.from_host_csr(gen.identity(4))
     assert np  # silence
+
+
+def test_default_spmv_kernel_has_no_register_spills(tmp_path):
+    """The default SpMV kernels (SM-queue `tm` variant, dense-row warp
+    variant) are register-capped at 64 per thread by their launch bounds; a
+    spill puts local-memory traffic on the hot path (it cost 10% once).
+    ptxas -v must report zero spill bytes for them."""
+    from paper_conf_ipps_niuldj0t21_b200 import _build
+    src = os.path.join(_build.PKG, "csrc", "spmv_warp.cu")
+    out = subprocess.run([_build.NVCC, "-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-std=c++17",
+                          "-cubin", "-Xptxas", "-v", "-o", str(tmp_path / "k.cubin"), src],
+                         capture_output=True, text=True, check=True).stderr
+    blocks = re.split(r"Compiling entry function", out)
+    checked = 0
+    for b in blocks[1:]:
+        name = b.split("'")[1]
+        if ("tilespmv_fp64_smILi32ELi4608ELb1" in name) or ("tilespmv_fp64_warpILi4ELi10752" in name):
+            m = re.search(r"(\d+) bytes spill stores, (\d+) bytes spill loads", b)
+            assert m and m.group(1) == "0" and m.group(2) == "0", (name, m and m.group(0))
+            checked += 1
+    assert checked == 2
