@@ -18,13 +18,19 @@
 // kCheckEvery iterations.
 #include <algorithm>
 #include <cmath>
+#include <cstdlib>
 
 #include "spmv_common.cuh"
 
 namespace tsp {
 namespace {
 
-constexpr int kBlocks = 296;  // 2 x 148 SMs
+// one wave of 6 blocks of 8 warps per SM (48 warps; the update kernel's 42
+// registers allow 6): the vector kernels are HBM-bound and need many loads
+// in flight, every thread moves double2 pairs.  Measured per CG iteration on
+// C5: 296 blocks 0.609 ms, 888 blocks 0.558 ms, 1184 (1.3 waves) 0.796 ms.
+// TILESPMV_CG_BLOCKS overrides the grid (<= kBlocks partial slots).
+constexpr int kBlocks = 6 * 148;
 constexpr int kThreads = 256;
 constexpr int kCheckEvery = 8;
 
@@ -51,10 +57,10 @@ __device__ __forceinline__ double block_sum(double v, double *sh) {
     return s;  // valid in thread 0
 }
 
-// sum of kBlocks partials in a fixed order (every thread gets the result)
-__device__ __forceinline__ double sum_partials(const double *part, double *sh) {
+// sum of the G partials of a grid in a fixed order (every thread gets the result)
+__device__ __forceinline__ double sum_partials(const double *part, double *sh, int G = (int)gridDim.x) {
     double v = 0.0;
-    for (int i = threadIdx.x; i < kBlocks; i += kThreads) v += part[i];
+    for (int i = threadIdx.x; i < G; i += kThreads) v += part[i];
     const double s = block_sum(v, sh);
     if (threadIdx.x == 0) sh[32] = s;
     __syncthreads();
@@ -63,11 +69,34 @@ __device__ __forceinline__ double sum_partials(const double *part, double *sh) {
     return r;
 }
 
+// Element loops: thread t of block g takes the pairs (2i, 2i+1) for i = g *
+// kThreads + t + k * gridDim.x * kThreads (16-byte loads; vectors come from
+// cudaMalloc or torch, 16-byte aligned), and block 0's thread 0 the last
+// element when n is odd.  The partial sums follow that fixed order.
+#define CG_PAIRS(i2) \
+    for (int64_t i2 = blockIdx.x * (int64_t)kThreads + threadIdx.x; i2 < (n >> 1); i2 += (int64_t)gridDim.x * kThreads)
+#define CG_TAIL(i) \
+    if ((n & 1) && blockIdx.x == 0 && threadIdx.x == 0) \
+        for (int64_t i = n - 1; i < n; ++i)
+
+__device__ __forceinline__ double2 ld2(const double *a, int64_t i2) { return reinterpret_cast<const double2 *>(a)[i2]; }
+__device__ __forceinline__ void st2(double *a, int64_t i2, double2 v) { reinterpret_cast<double2 *>(a)[i2] = v; }
+
 // r = b - q (q = A x0), p = r; partials of (r, r) and (b, b)
 __global__ void k_cg_init(const double *b, const double *q, double *r, double *p, int64_t n, CgState *st) {
     __shared__ double sh[40];
     double rr = 0.0, bb = 0.0;
-    for (int64_t i = blockIdx.x * (int64_t)kThreads + threadIdx.x; i < n; i += (int64_t)kBlocks * kThreads) {
+    CG_PAIRS(i2) {
+        const double2 bi = ld2(b, i2), qi = ld2(q, i2);
+        const double2 ri = make_double2(bi.x - qi.x, bi.y - qi.y);
+        st2(r, i2, ri);
+        st2(p, i2, ri);
+        rr = fma(ri.x, ri.x, rr);
+        rr = fma(ri.y, ri.y, rr);
+        bb = fma(bi.x, bi.x, bb);
+        bb = fma(bi.y, bi.y, bb);
+    }
+    CG_TAIL(i) {
         const double ri = b[i] - q[i];
         r[i] = ri;
         p[i] = ri;
@@ -81,9 +110,9 @@ __global__ void k_cg_init(const double *b, const double *q, double *r, double *p
     }
 }
 
-__global__ void k_cg_init_scalars(CgState *st) {
+__global__ void k_cg_init_scalars(CgState *st, int G) {  // G: k_cg_init's grid
     __shared__ double sh[40];
-    const double rr = sum_partials(st->rrp[0], sh), bb = sum_partials(st->bbp, sh);
+    const double rr = sum_partials(st->rrp[0], sh, G), bb = sum_partials(st->bbp, sh, G);
     if (threadIdx.x == 0) {
         st->rr = rr;
         st->bb = bb;
@@ -97,8 +126,13 @@ __global__ void k_cg_pq(const double *p, const double *q, int64_t n, CgState *st
     if (st->done) return;
     __shared__ double sh[40];
     double s = 0.0;
-    for (int64_t i = blockIdx.x * (int64_t)kThreads + threadIdx.x; i < n; i += (int64_t)kBlocks * kThreads)
-        s = fma(p[i], q[i], s);
+#pragma unroll 2
+    CG_PAIRS(i2) {
+        const double2 pi = ld2(p, i2), qi = ld2(q, i2);
+        s = fma(pi.x, qi.x, s);
+        s = fma(pi.y, qi.y, s);
+    }
+    CG_TAIL(i) s = fma(p[i], q[i], s);
     s = block_sum(s, sh);
     if (threadIdx.x == 0) st->pq[blockIdx.x] = s;
 }
@@ -110,7 +144,16 @@ __global__ void k_cg_update(double *x, double *r, const double *p, const double 
     const double rr = sum_partials(st->rrp[j & 1], sh), pq = sum_partials(st->pq, sh);
     const double alpha = rr / pq;
     double s = 0.0;
-    for (int64_t i = blockIdx.x * (int64_t)kThreads + threadIdx.x; i < n; i += (int64_t)kBlocks * kThreads) {
+#pragma unroll 2
+    CG_PAIRS(i2) {
+        const double2 xi = ld2(x, i2), pi = ld2(p, i2), qi = ld2(q, i2), r0 = ld2(r, i2);
+        st2(x, i2, make_double2(fma(alpha, pi.x, xi.x), fma(alpha, pi.y, xi.y)));
+        const double2 ri = make_double2(fma(-alpha, qi.x, r0.x), fma(-alpha, qi.y, r0.y));
+        st2(r, i2, ri);
+        s = fma(ri.x, ri.x, s);
+        s = fma(ri.y, ri.y, s);
+    }
+    CG_TAIL(i) {
         x[i] = fma(alpha, p[i], x[i]);
         const double ri = fma(-alpha, q[i], r[i]);
         r[i] = ri;
@@ -136,8 +179,12 @@ __global__ void k_cg_direction(double *p, const double *r, int64_t n, int j, dou
         return;
     }
     const double beta = rr1 / rr0;
-    for (int64_t i = blockIdx.x * (int64_t)kThreads + threadIdx.x; i < n; i += (int64_t)kBlocks * kThreads)
-        p[i] = fma(beta, p[i], r[i]);
+#pragma unroll 2
+    CG_PAIRS(i2) {
+        const double2 pi = ld2(p, i2), ri = ld2(r, i2);
+        st2(p, i2, make_double2(fma(beta, pi.x, ri.x), fma(beta, pi.y, ri.y)));
+    }
+    CG_TAIL(i) p[i] = fma(beta, p[i], r[i]);
 }
 
 }  // namespace
@@ -145,16 +192,29 @@ __global__ void k_cg_direction(double *p, const double *r, int64_t n, int j, dou
 int cg_solve(const Matrix &M, const double *d_b, double *d_x, double tol, int maxit, int *iters, double *relres,
              cudaStream_t st) {
     const int64_t n = M.n;
+    // the vector kernels move 16-byte pairs: every vector starts 16-byte
+    // aligned (work vectors at an even stride; b and x staged when the
+    // caller's are not)
+    const int64_t n2 = (std::max<int64_t>(n, 1) + 1) & ~int64_t(1);
+    const bool staged = ((reinterpret_cast<uintptr_t>(d_b) | reinterpret_cast<uintptr_t>(d_x)) & 15u) != 0;
     CgState *S = nullptr;
     double *work = nullptr;
     cudaError_t e = cudaMallocAsync(reinterpret_cast<void **>(&S), sizeof(CgState), st);
     if (e != cudaSuccess) return cuda_status(e, "cudaMallocAsync(cg state)");
-    e = cudaMallocAsync(reinterpret_cast<void **>(&work), 3 * std::max<int64_t>(n, 1) * sizeof(double), st);
+    e = cudaMallocAsync(reinterpret_cast<void **>(&work), (staged ? 5 : 3) * n2 * sizeof(double), st);
     if (e != cudaSuccess) {
         cudaFreeAsync(S, st);
         return cuda_status(e, "cudaMallocAsync(cg vectors)");
     }
-    double *r = work, *p = work + n, *q = work + 2 * n;
+    double *r = work, *p = work + n2, *q = work + 2 * n2;
+    double *const x_user = d_x;
+    if (staged) {
+        double *bs = work + 3 * n2, *xs = work + 4 * n2;
+        cudaMemcpyAsync(bs, d_b, n * sizeof(double), cudaMemcpyDeviceToDevice, st);
+        cudaMemcpyAsync(xs, d_x, n * sizeof(double), cudaMemcpyDeviceToDevice, st);
+        d_b = bs;
+        d_x = xs;
+    }
     int rc = 0;
     struct {
         double bb, rr;
@@ -162,15 +222,17 @@ int cg_solve(const Matrix &M, const double *d_b, double *d_x, double tol, int ma
     } h{};
     do {
         if ((rc = launch_spmv(M, d_x, q, st))) break;  // q = A x0
-        k_cg_init<<<kBlocks, kThreads, 0, st>>>(d_b, q, r, p, n, S);
-        k_cg_init_scalars<<<1, kThreads, 0, st>>>(S);
+        int G = kBlocks;
+        if (const char *ev = getenv("TILESPMV_CG_BLOCKS")) G = std::min(kBlocks, std::max(1, atoi(ev)));
+        k_cg_init<<<G, kThreads, 0, st>>>(d_b, q, r, p, n, S);
+        k_cg_init_scalars<<<1, kThreads, 0, st>>>(S, G);
         const double tol2 = tol * tol;
         int j = 0;
         for (; j < maxit; ++j) {
             if ((rc = launch_spmv(M, p, q, st))) break;
-            k_cg_pq<<<kBlocks, kThreads, 0, st>>>(p, q, n, S);
-            k_cg_update<<<kBlocks, kThreads, 0, st>>>(d_x, r, p, q, n, j, S);
-            k_cg_direction<<<kBlocks, kThreads, 0, st>>>(p, r, n, j, tol2, S);
+            k_cg_pq<<<G, kThreads, 0, st>>>(p, q, n, S);
+            k_cg_update<<<G, kThreads, 0, st>>>(d_x, r, p, q, n, j, S);
+            k_cg_direction<<<G, kThreads, 0, st>>>(p, r, n, j, tol2, S);
             if ((j + 1) % kCheckEvery == 0 || j + 1 == maxit) {
                 if ((e = cudaMemcpyAsync(&h, S, sizeof h, cudaMemcpyDeviceToHost, st)) != cudaSuccess ||
                     (e = cudaStreamSynchronize(st)) != cudaSuccess) {
@@ -188,6 +250,7 @@ int cg_solve(const Matrix &M, const double *d_b, double *d_x, double tol, int ma
         }
         if (iters) *iters = h.iters;
         if (relres) *relres = h.bb > 0.0 ? std::sqrt(h.rr / h.bb) : 0.0;
+        if (staged) cudaMemcpyAsync(x_user, d_x, n * sizeof(double), cudaMemcpyDeviceToDevice, st);
     } while (0);
     cudaFreeAsync(work, st);
     cudaFreeAsync(S, st);

@@ -470,7 +470,7 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, MINB) tilespmv
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const uint32_t xs = smem_u32(smem) + (uint32_t)warp * Cfg::kX;
     const uint32_t slot = smem_u32(smem) + WARPS * Cfg::kX + (uint32_t)warp * Cfg::kPer;
-    const uint32_t racc = slot + SLOT, bar = racc + 128;
+    const uint32_t racc = slot + SLOT, bar = racc + Cfg::kRacc;
     if (lane == 0) {
         mbar_init(bar, 1);
         fence_mbar_init();
@@ -620,7 +620,7 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT, 2>::kThreads, MINB) tiles
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const uint32_t xs = smem_u32(smem) + (uint32_t)warp * Cfg::kX;
     const uint32_t base = smem_u32(smem) + WARPS * Cfg::kX + (uint32_t)warp * Cfg::kPer;
-    const uint32_t racc = base + 2 * SLOT, bar0 = racc + 128;
+    const uint32_t racc = base + 2 * SLOT, bar0 = racc + Cfg::kRacc;
     if (lane == 0) {
         mbar_init(bar0, 1);
         mbar_init(bar0 + 8, 1);

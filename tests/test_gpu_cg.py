@@ -67,3 +67,30 @@ def test_cg_deterministic_and_args(cuda_device):
     with TiledMatrix.from_host_csr(R, device=cuda_device) as M:
         with pytest.raises(TileSpMVError):
             M.cg(torch.zeros(33, dtype=torch.float64, device=cuda_device))
+
+
+def test_cg_odd_n_and_misaligned_vectors(cuda_device):
+    """Odd n (the vector kernels' pair loop plus the tail element) and b, x
+    that are not 16-byte aligned (views at an odd element offset, staged
+    internally): the oracle-matching solve, bitwise equal to the aligned
+    call."""
+    import torch
+    from paper_conf_ipps_niuldj0t21_b200 import TiledMatrix
+    A = gen.lap2d(37, 29)  # n = 1073
+    assert A.n % 2 == 1
+    b = gen.dense_x(A.n, 33)
+    tol = 1e-11
+    xo, ito, _ = O.cg(A, b, tol=tol, maxit=5000)
+    with TiledMatrix.from_host_csr(A, device=cuda_device) as M:
+        bd = torch.from_numpy(b).to(cuda_device)
+        xa, ita, rela = M.cg(bd, tol=tol, maxit=5000)
+        buf_b = torch.zeros(A.n + 1, dtype=torch.float64, device=cuda_device)
+        buf_x = torch.zeros(A.n + 1, dtype=torch.float64, device=cuda_device)
+        buf_b[1:].copy_(bd)
+        xm, itm, relm = M.cg(buf_b[1:], x=buf_x[1:], tol=tol, maxit=5000)
+        assert buf_b[1:].data_ptr() % 16 == 8
+        xa, xm = xa.cpu().numpy(), xm.cpu().numpy()
+    assert abs(ita - ito) <= 2 and relm <= tol
+    assert ita == itm and np.array_equal(xa.view(np.uint64), xm.view(np.uint64))
+    assert np.linalg.norm(xa - xo) <= 1e-7 * np.linalg.norm(xo)
+    assert float(buf_x[0]) == 0.0  # nothing written outside the view
