@@ -251,6 +251,19 @@ __device__ __forceinline__ void half_csr_tm(uint32_t RP, int nz, int tm, uint32_
     } else if (tm <= 2) {
         if (tm == 2) csr_steps<2>(V, u, X, 0, len, acc);
         else csr_steps<1>(V, u, X, 0, len, acc);
+    } else if (tm >= 6 && tm <= 8) {
+        // rows of 6..8 entries: lane r starts at entry r mod 8 of its row and
+        // wraps (8 steps cover entries 0..7 once each; steps past the row's
+        // end are predicated off).  Equal-length rows laid end to end would
+        // otherwise put the lanes' values 8*len bytes apart, on the same
+        // shared-memory banks (4-way conflicts for rows of 8).
+#pragma unroll
+        for (int j = 0; j < 8; ++j) {
+            const int jj = (j + r) & 7;
+            const double v = lds_f64_lt(jj, len, V + 8 * jj);
+            const double xv = lds_f64(xaddr((u >> (4 * jj)) << 3, X));
+            acc = fma(v, xv, acc);
+        }
     } else {
         csr_steps<4>(V, u, X, 0, len, acc);
 #pragma unroll 1
