@@ -171,6 +171,40 @@ def build_local(workload: str, rank: int, P: int):
 # CPU oracle timing (the cpu_baseline leg; rank 0 only)
 # --------------------------------------------------------------------------
 
+def cpu_context(A, x, info, create_s):
+    """SURVEY §8(d) D5 items 2 and 3, context beside the oracle baseline:
+    an OpenMP fp64 CSR SpMV on every core of the process (whole matrix, best
+    of 3; not the oracle), and the oracle's single-threaded tiler on a
+    bounded row slice next to the GPU tiler (create) per million nonzeros
+    (the Fig. 11 analogue)."""
+    from oracle import oracle as O
+    out = {}
+    try:
+        model = next((l.split(":", 1)[1].strip() for l in open("/proc/cpuinfo") if l.startswith("model name")), "")
+    except OSError:
+        model = ""
+    best = float("inf")
+    threads = 0
+    for _ in range(3):
+        t = time.perf_counter()
+        _, threads = O.cpu_csr_omp(A, x)
+        best = min(best, time.perf_counter() - t)
+    out["omp_csr"] = {"value": 2.0 * A.nnz / best / 1e9, "unit": UNIT, "cores": threads,
+                      "affinity_cores": len(os.sched_getaffinity(0)), "cpu": model,
+                      "kind": "openmp row-parallel fp64 CSR (not the oracle)",
+                      "sample": "whole matrix, best of 3 passes"}
+    rowlen = np.diff(A.rowptr.astype(np.int64))
+    r1 = int(min(A.m, max(16, np.searchsorted(np.cumsum(rowlen), 2_000_000) // 16 * 16 + 16)))
+    S = A.row_slice(0, r1)
+    t = time.perf_counter()
+    O.tile(S, {0: "ADPT", 1: "DEFERRED", 3: "FORCE_CSR"}.get(int(info.get("mode", 1)), "DEFERRED"))
+    dt = time.perf_counter() - t
+    out["tiler"] = {"oracle_s_per_Mnnz": dt / max(S.nnz, 1) * 1e6, "oracle_sample_nnz": int(S.nnz),
+                    "gpu_create_s_per_Mnnz": create_s / max(A.nnz, 1) * 1e6,
+                    "note": "oracle tiler: one thread, first rows of the matrix; GPU: tilespmv_create_from_csr"}
+    return out
+
+
 def oracle_sample(A, x, seconds: float, rng, max_rows=None):
     """Times the oracle (oracle/oracle.c, long-double Alg. 1, 1 thread) on a
     bounded sample of rows of A: contiguous blocks at random offsets, sized
@@ -370,6 +404,7 @@ def measure_workload(workload, mode, steps, warmup, dev, rank, P, group, cpu_sec
         res["parity"] = {"rows_checked": int(rows.size), "ok": ok,
                          "max_err_over_absy": float(np.max(err / (absy + 1e-300))) if rows.size else 0.0,
                          "tolerance": "1e-12*sum|a_ij x_j| + 1e-300"}
+        res["cpu_context"] = cpu_context(A, x_h, info, create_s)
     # ---- end to end through the host-buffer C-ABI call
     if want_e2e:
         hx = torch.from_numpy(x_h).pin_memory()
@@ -606,6 +641,8 @@ def run_ours(args):
                "host_enqueue_us_per_step": res["host_enqueue_us_per_step"],
                "launch": res["launch"],
                "parity": res.get("parity")}
+        if res.get("cpu_context"):
+            out["cpu_context"] = res["cpu_context"]
         if "exchange" in res:
             out["exchange"] = res["exchange"]
             out["gpu_launches"] = args.steps * res["launches_per_step"]

@@ -22,12 +22,35 @@ CSR, COO, ELL, HYB, DNS, DNSROW, DNSCOL = range(7)
 MODES = {"ADPT": 0, "DEFERRED": 1, "AUTO": 2, "FORCE_CSR": 3}
 
 
+OMP_SRC = os.path.join(HERE, "cpu_csr_omp.c")
+OMP_LIB = os.path.join(HERE, "libcpu_csr_omp.so")
+
+
 def build(force: bool = False) -> str:
-    """gcc the oracle (plain C, -O2, no fast-math)."""
+    """gcc the oracle (plain C, -O2, no fast-math) and the multi-threaded CPU
+    CSR baseline beside it (not the oracle; bench context only)."""
     if force or not os.path.exists(LIB) or os.path.getmtime(LIB) < os.path.getmtime(SRC):
         subprocess.check_call(["gcc", "-O2", "-std=c11", "-Wall", "-fPIC", "-shared",
                                "-o", LIB, SRC])
+    if force or not os.path.exists(OMP_LIB) or os.path.getmtime(OMP_LIB) < os.path.getmtime(OMP_SRC):
+        subprocess.check_call(["gcc", "-O3", "-std=c11", "-Wall", "-fopenmp", "-fPIC", "-shared",
+                               "-o", OMP_LIB, OMP_SRC])
     return LIB
+
+
+def cpu_csr_omp(A, x: np.ndarray):
+    """y = A x by the OpenMP CSR baseline (all threads of the process);
+    returns (y, threads).  Not the oracle: fp64 running sums."""
+    build()
+    L = ctypes.CDLL(OMP_LIB)
+    p = ctypes.c_void_p
+    L.cpu_csr_omp_spmv.argtypes = [ctypes.c_int64, p, p, p, p, p]
+    L.cpu_csr_omp_threads.restype = ctypes.c_int
+    rp, ci, va = _csr_arrays(A)
+    x = np.ascontiguousarray(x, dtype=np.float64)
+    y = np.empty(A.m, dtype=np.float64)
+    L.cpu_csr_omp_spmv(A.m, _ptr(rp), _ptr(ci), _ptr(va), _ptr(x), _ptr(y))
+    return y, int(L.cpu_csr_omp_threads())
 
 
 _lib = None

@@ -140,3 +140,17 @@ def test_zero_sized():
     A = gen.random_sparse(4, 0, 0.5)
     y, _ = O.spmv(A, np.zeros(0))
     assert np.array_equal(y, np.zeros(4))
+
+
+def test_cpu_csr_omp_baseline_matches_oracle():
+    """The multi-threaded CSR baseline bench.py reports as context (not the
+    oracle) computes y = A x within the north-star tolerance of the oracle."""
+    import numpy as np
+    from oracle import oracle as O
+    from synthetic import gen
+    for name in ("mixed_small", "rmat12", "stencil27_21"):
+        A, x = gen.make(name)
+        y, threads = O.cpu_csr_omp(A, x)
+        yr, absy = O.spmv(A, x)
+        assert threads >= 1
+        assert np.all(np.abs(y - yr) <= 1e-12 * absy + 1e-300), name
