@@ -332,15 +332,18 @@ __device__ __forceinline__ void half_ell_n(uint32_t P, int w, uint32_t X, int r,
 // scan over the half (entries are row-major, so a row's entries are adjacent
 // lanes) leaves each row's sum on the row's last entry, which stores it in
 // the warp's row scratch S (16 doubles per half) for the row's lane.
+// base: first entry of this pass (HYB's COO part may hold more than 16
+// entries and runs in passes of 16; a row that straddles two passes gets two
+// partial sums, added in pass order)
 __device__ __forceinline__ void half_coo_scan(uint32_t V, uint32_t rc, int n, uint32_t X, int r, int h, uint32_t S,
-                                              bool ok, double &acc) {
+                                              bool ok, double &acc, int base = 0) {
     const int nq = ok ? n : 0;
-    const bool have = r < nq;
+    const bool have = base + r < nq;
     uint32_t b = 0;
     double p = 0.0;
     if (have) {
-        b = lds_u8(rc + r);
-        p = lds_f64(V + 8 * r) * lds_f64(X + 8 * (b & 15u));
+        b = lds_u8(rc + base + r);
+        p = lds_f64(V + 8 * (base + r)) * lds_f64(X + 8 * (b & 15u));
     }
     const int row = have ? (int)(b >> 4) : 16 + r;  // idle lanes: a row of their own
     {  // (every lane executes every shuffle: no shuffle inside a short-circuit)
@@ -360,13 +363,32 @@ __device__ __forceinline__ void half_coo_scan(uint32_t V, uint32_t rc, int n, ui
         }
     }
     const int rnext = __shfl_down_sync(FULL, row, 1, 16);
-    const bool tail = have && (r == nq - 1 || rnext != row);
+    const bool tail = have && (base + r == nq - 1 || r == 15 || rnext != row);
     const uint32_t rows = __reduce_or_sync(FULL, tail ? 1u << (16 * h + row) : 0u);
     const uint32_t Sh = S + 128 * h;
     __syncwarp();  // the previous pair's reads of S are done
     if (tail) sts_f64(Sh + 8 * row, p);
     __syncwarp();
     if ((rows >> (16 * h + r)) & 1u) acc += lds_f64(Sh + 8 * r);
+}
+
+// HYB in the TM kernels: the ELL part as ELL, the COO part with the
+// lane-per-entry scan in passes of 16 entries
+__device__ __forceinline__ void half_hyb_scan(uint32_t P, int w, int nz, uint32_t X, int r, int h, uint32_t S, bool ok,
+                                              double &acc) {
+    const int kc = nz - 16 * w;
+    const uint32_t ei = P + 128 * w + 8 * kc;
+    const int wq = ok ? w : 0;
+    const int trips = (int)__reduce_max_sync(FULL, (unsigned)wq);
+    const uint32_t sh = 4 * (r & 1);
+    for (int k = 0; k < trips; ++k) {
+        const double v = lds_f64_lt(k, wq, P + 8 * (16 * k + r));
+        const double xv = lds_f64(X + 8 * ((lds_u8(ei + 8 * k + (r >> 1)) >> sh) & 15u));
+        acc = fma(v, xv, acc);
+    }
+    const int passes = (int)__reduce_max_sync(FULL, (unsigned)(ok ? (kc + 15) >> 4 : 0));
+#pragma unroll 1
+    for (int c = 0; c < passes; ++c) half_coo_scan(P + 128 * w, ei + 8 * w, kc, X, r, h, S, ok, acc, 16 * c);
 }
 
 // HYB: ELL(w) values | COO values | ELL 4-bit columns | COO (row<<4|col)

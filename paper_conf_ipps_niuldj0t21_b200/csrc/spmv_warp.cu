@@ -314,7 +314,8 @@ __device__ __forceinline__ void run_group(int np, uint32_t &d, uint32_t xs, int 
         if (F == F_DNSROW && !TM) half_dnsrow(P, aux, X, r, ok, acc);
         if (F == F_COO && TM) half_coo_scan(P, P + 8 * nz, nz, X, r, lane_h, racc, ok, acc);
         if (F == F_COO && !TM) half_coo(P, P + 8 * nz, nz, X, r, ok, acc);
-        if (F == F_HYB) half_hyb(P, aux, nz, X, r, ok, acc);
+        if (F == F_HYB && TM) half_hyb_scan(P, aux, nz, X, r, lane_h, racc, ok, acc);
+        if (F == F_HYB && !TM) half_hyb(P, aux, nz, X, r, ok, acc);
     }
 }
 
@@ -413,7 +414,7 @@ __device__ __forceinline__ void compute_item(const Params &p, const WItem &it, u
         if (TM && ((g >> 29) & 1u)) run_group<F_ELL, TM, 3>((int)((g >> 8) & 15u), d, xs, r, acc);
         else run_group<F_ELL, TM>((int)((g >> 8) & 15u), d, xs, r, acc);
         if (!TM || (g & 0x0FFFF000u)) {  // TM: one test skips the four rarer formats
-            run_group<F_HYB, TM>((int)((g >> 12) & 15u), d, xs, r, acc);
+            run_group<F_HYB, TM>((int)((g >> 12) & 15u), d, xs, r, acc, racc);
             run_group<F_DNS, TM>((int)((g >> 16) & 15u), d, xs, r, acc);
             run_group<F_DNSROW, TM>((int)((g >> 20) & 15u), d, xs, r, acc);
             run_group<F_DNSCOL, TM>((int)((g >> 24) & 15u), d, xs, r, acc);
