@@ -265,7 +265,8 @@ __global__ void k_blob_fill(Item *items, int64_t nitems, int64_t m, int64_t n, c
     // the tile's payload (CSR: to its csrRowPtr, after the 8*nnz value bytes),
     // y = aux | t*128 | nnz << 11 | tm << 20 | invalid << 31, where tm is the
     // larger extent of the two tiles of the half-warp pair (2j, 2j+1): CSR the
-    // longest row, ELL the width (ndsc is even; the loop is warp-uniform)
+    // longest row, ELL the width, COO the entry count (ndsc is even; the
+    // loop is warp-uniform)
     const uint8_t *tpay = payload + (size_t)it.offb * 16;
     uint32_t csr_max = 0, ell_max = 0;
     for (int i0 = 0; i0 < it.ndsc; i0 += 32) {
@@ -286,6 +287,8 @@ __global__ void k_blob_fill(Item *items, int64_t nitems, int64_t m, int64_t n, c
                 }
             } else if (f == F_ELL) {
                 tm = d.y & 0x1Fu;
+            } else if (f == F_COO) {
+                tm = nz;  // <= 11
             }
         }
         const uint32_t tmo = __shfl_xor_sync(0xFFFFFFFFu, tm, 1);

@@ -203,6 +203,19 @@ __device__ __forceinline__ void half_dnsrow(uint32_t P, int nr, uint32_t X, int 
     }
 }
 
+// COO with at most N entries per tile of the pair (tm <= N): every lane of
+// the half walks the entries, the lane of the entry's row adds it
+template <int N>
+__device__ __forceinline__ void half_coo_n(uint32_t V, uint32_t rc, int n, uint32_t X, int r, bool ok, double &acc) {
+    const int nq = ok ? n : 0;
+#pragma unroll
+    for (int j = 0; j < N; ++j) {
+        const uint32_t b = lds_u8(rc + j);
+        const double v = lds_f64_lt(j, (int)(b >> 4) == r ? nq : 0, V + 8 * j);
+        acc = fma(v, lds_f64(X + 8 * (b & 15u)), acc);
+    }
+}
+
 // COO entries: value j, packed (row << 4 | col) byte (Alg. 3); the lane
 // of the entry's row adds it (no atomics, fixed order)
 __device__ __forceinline__ void half_coo(uint32_t V, uint32_t rc, int n, uint32_t X, int r, bool ok, double &acc) {

@@ -312,7 +312,10 @@ __device__ __forceinline__ void run_group(int np, uint32_t &d, uint32_t xs, int 
         if (F == F_DNSCOL) half_dnscol(P, aux, X, r, ok, acc);
         if (F == F_DNSROW && TM) half_dnsrow_tree(P, aux, X, r, ok, acc);
         if (F == F_DNSROW && !TM) half_dnsrow(P, aux, X, r, ok, acc);
-        if (F == F_COO && TM) half_coo_scan(P, P + 8 * nz, nz, X, r, lane_h, racc, ok, acc);
+        if (F == F_COO && TM) {  // tiny tiles (power-law, stencil corners): walk; else scan
+            if (tm <= 2) half_coo_n<2>(P, P + 8 * nz, nz, X, r, ok, acc);
+            else half_coo_scan(P, P + 8 * nz, nz, X, r, lane_h, racc, ok, acc);
+        }
         if (F == F_COO && !TM) half_coo(P, P + 8 * nz, nz, X, r, ok, acc);
         if (F == F_HYB && TM) half_hyb_scan(P, aux, nz, X, r, lane_h, racc, ok, acc);
         if (F == F_HYB && !TM) half_hyb(P, aux, nz, X, r, ok, acc);
