@@ -277,6 +277,18 @@ __device__ __forceinline__ void half_csr_tm(uint32_t RP, int nz, int tm, uint32_
             const double xv = lds_f64(xaddr((u >> (4 * jj)) << 3, X));
             acc = fma(v, xv, acc);
         }
+    } else if (tm >= 13) {
+        // rows of 13..16 entries (FORCE_CSR on dense tiles): the same lane
+        // rotation over 16 entries, column nibbles from two 8-entry windows
+        const uint32_t wb = RP + 16 + 4 * ((beg + 8) >> 3);
+        const uint64_t u2 = (uint64_t)u | ((uint64_t)funnel_r(lds_u32(wb), lds_u32(wb + 4), 4u * (beg + 8)) << 32);
+#pragma unroll 4
+        for (int j = 0; j < 16; ++j) {
+            const int jj = (j + r) & 15;
+            const double v = lds_f64_lt(jj, len, V + 8 * jj);
+            const double xv = lds_f64(xaddr((uint32_t)(u2 >> (4 * jj)) << 3, X));
+            acc = fma(v, xv, acc);
+        }
     } else {
         csr_steps<4>(V, u, X, 0, len, acc);
 #pragma unroll 1
