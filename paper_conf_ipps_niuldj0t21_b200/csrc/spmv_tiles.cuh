@@ -79,6 +79,34 @@ __device__ __forceinline__ void sts_f64(uint32_t a, double v) {
 // inside the CTA's shared memory and are masked out of the sum; x addresses
 // always stay inside the tile's x segment.
 
+// Lane-rotated CSR rows: lane r starts at entry r mod 8 (mod 16) of its
+// row and wraps, so 8 (16) steps cover every entry once and steps past the
+// row's end are predicated off.  Rows of equal length laid end to end would
+// otherwise put the lanes' values 8*len bytes apart, on the same
+// shared-memory banks (4-way conflicts for rows of 8, 16-way for 16).
+// u: the 8 column nibbles from entry beg on.
+__device__ __forceinline__ void csr_rot8(uint32_t V, uint32_t u, uint32_t X, int r, int len, double &acc) {
+#pragma unroll
+    for (int j = 0; j < 8; ++j) {
+        const int jj = (j + r) & 7;
+        const double v = lds_f64_lt(jj, len, V + 8 * jj);
+        const double xv = lds_f64(xaddr((u >> (4 * jj)) << 3, X));
+        acc = fma(v, xv, acc);
+    }
+}
+__device__ __forceinline__ void csr_rot16(uint32_t RP, int beg, uint32_t V, uint32_t u, uint32_t X, int r, int len,
+                                          double &acc) {
+    const uint32_t wb = RP + 16 + 4 * ((beg + 8) >> 3);
+    const uint64_t u2 = (uint64_t)u | ((uint64_t)funnel_r(lds_u32(wb), lds_u32(wb + 4), 4u * (beg + 8)) << 32);
+#pragma unroll 4
+    for (int j = 0; j < 16; ++j) {
+        const int jj = (j + r) & 15;
+        const double v = lds_f64_lt(jj, len, V + 8 * jj);
+        const double xv = lds_f64(xaddr((uint32_t)(u2 >> (4 * jj)) << 3, X));
+        acc = fma(v, xv, acc);
+    }
+}
+
 // CSR: csrVal row-major | csrRowPtr[16] u8 | 4-bit columns (Alg. 2).
 // RP: shared address of csrRowPtr.  The 8 column nibbles from entry beg on
 // come from two 32-bit words and one funnel shift.
@@ -88,6 +116,13 @@ __device__ __forceinline__ void half_csr(uint32_t RP, int nz, uint32_t X, int r,
     const int len = ok ? end - beg : 0;
     const int trips = (int)__reduce_max_sync(FULL, (unsigned)len);
     const uint32_t V = RP + 8 * (beg - nz);
+    if ((trips >= 6 && trips <= 8) || trips >= 13) {  // long equal rows: lane-rotated
+        const uint32_t wa = RP + 16 + 4 * (beg >> 3);
+        const uint32_t u = funnel_r(lds_u32(wa), lds_u32(wa + 4), 4u * beg);
+        if (trips <= 8) csr_rot8(V, u, X, r, len, acc);
+        else csr_rot16(RP, beg, V, u, X, r, len, acc);
+        return;
+    }
     {
         const uint32_t wa = RP + 16 + 4 * (beg >> 3);
         const uint32_t u = funnel_r(lds_u32(wa), lds_u32(wa + 4), 4u * beg);
@@ -265,30 +300,9 @@ __device__ __forceinline__ void half_csr_tm(uint32_t RP, int nz, int tm, uint32_
         if (tm == 2) csr_steps<2>(V, u, X, 0, len, acc);
         else csr_steps<1>(V, u, X, 0, len, acc);
     } else if (tm >= 6 && tm <= 8) {
-        // rows of 6..8 entries: lane r starts at entry r mod 8 of its row and
-        // wraps (8 steps cover entries 0..7 once each; steps past the row's
-        // end are predicated off).  Equal-length rows laid end to end would
-        // otherwise put the lanes' values 8*len bytes apart, on the same
-        // shared-memory banks (4-way conflicts for rows of 8).
-#pragma unroll
-        for (int j = 0; j < 8; ++j) {
-            const int jj = (j + r) & 7;
-            const double v = lds_f64_lt(jj, len, V + 8 * jj);
-            const double xv = lds_f64(xaddr((u >> (4 * jj)) << 3, X));
-            acc = fma(v, xv, acc);
-        }
+        csr_rot8(V, u, X, r, len, acc);
     } else if (tm >= 13) {
-        // rows of 13..16 entries (FORCE_CSR on dense tiles): the same lane
-        // rotation over 16 entries, column nibbles from two 8-entry windows
-        const uint32_t wb = RP + 16 + 4 * ((beg + 8) >> 3);
-        const uint64_t u2 = (uint64_t)u | ((uint64_t)funnel_r(lds_u32(wb), lds_u32(wb + 4), 4u * (beg + 8)) << 32);
-#pragma unroll 4
-        for (int j = 0; j < 16; ++j) {
-            const int jj = (j + r) & 15;
-            const double v = lds_f64_lt(jj, len, V + 8 * jj);
-            const double xv = lds_f64(xaddr((uint32_t)(u2 >> (4 * jj)) << 3, X));
-            acc = fma(v, xv, acc);
-        }
+        csr_rot16(RP, beg, V, u, X, r, len, acc);
     } else {
         csr_steps<4>(V, u, X, 0, len, acc);
 #pragma unroll 1
