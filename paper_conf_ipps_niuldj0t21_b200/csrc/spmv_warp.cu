@@ -221,11 +221,24 @@ __device__ __forceinline__ void group_item(const Params &p, const WItem &it, uin
     }
 }
 
-// Row-group item, TM kernels: after the flat pass, two tile rows at a time,
-// half-warp h on tile row g + h and lane r on its row r alone (4 running
-// sums over the row's products, in entry order mod 4); rows longer than
-// kShortRow are summed by the whole warp with an xor tree.  A tile row's sums
-// depend only on its own entries (grouping never changes a bit of y).
+// product of remainder entry k (rounded on its own, exactly as flat_products
+// stores it) if k < e, else +0.0 -- the term the row sums would have read
+__device__ __forceinline__ double rem_product(const Params &p, int k, int e, uint32_t colS, uint32_t valS,
+                                              uint64_t x_policy) {
+    int c;
+    double v;
+    lds_entry_lt(k, e, colS + 4 * k, valS + 8 * k, c, v);
+    const double pr = __dmul_rn(v, ldg_hint(p.x + (uint32_t)c, x_policy));
+    return k < e ? pr : 0.0;
+}
+
+// Row-group item, TM kernels: two tile rows at a time, half-warp h on tile
+// row g + h and lane r on its row r alone (4 running sums over the row's
+// products, in entry order mod 4); rows longer than kShortRow are summed by
+// the whole warp with an xor tree.  Each product is formed where it is summed
+// (no shared-memory round trip), rounded on its own, so the terms and their
+// order are those of the flat pass.  A tile row's sums depend only on its own
+// entries (grouping never changes a bit of y).
 __device__ __forceinline__ void group_item2(const Params &p, const WItem &it, uint32_t slot, uint64_t x_policy,
                                             int lane) {
     const int ntr = (int)(it.jt_rows_pay & 0xFFu);
@@ -233,7 +246,6 @@ __device__ __forceinline__ void group_item2(const Params &p, const WItem &it, ui
     const uint32_t total = it.val_tot >> 16, rp = it.rp_col & 0xFFFFu;
     const bool has_rem = total > rp;
     const uint32_t rpS = slot + rp, colS = slot + (it.rp_col >> 16), valS = slot + (it.val_tot & 0xFFFFu);
-    if (has_rem) flat_products(p, colS, valS, lds_s32(rpS + 4 * (16 * (ntr - 1) + rows_last)), x_policy, lane);
     const int h = lane >> 4, r = lane & 15;
 #pragma unroll 1
     for (int g = 0; g < ntr; g += 2) {
@@ -250,10 +262,10 @@ __device__ __forceinline__ void group_item2(const Params &p, const WItem &it, ui
 #pragma unroll 1
             for (int t = 0; t < trips; ++t) {
                 const int k = b + 4 * t;
-                s0 += lds_f64_lt(k, ee, valS + 8 * k);
-                s1 += lds_f64_lt(k + 1, ee, valS + 8 * k + 8);
-                s2 += lds_f64_lt(k + 2, ee, valS + 8 * k + 16);
-                s3 += lds_f64_lt(k + 3, ee, valS + 8 * k + 24);
+                s0 += rem_product(p, k, ee, colS, valS, x_policy);
+                s1 += rem_product(p, k + 1, ee, colS, valS, x_policy);
+                s2 += rem_product(p, k + 2, ee, colS, valS, x_policy);
+                s3 += rem_product(p, k + 3, ee, colS, valS, x_policy);
             }
             acc = (s0 + s1) + (s2 + s3);
             uint32_t lm = __ballot_sync(FULL, lng);
@@ -267,10 +279,10 @@ __device__ __forceinline__ void group_item2(const Params &p, const WItem &it, ui
 #pragma unroll 1
                 for (int t = 0; t < t2; ++t) {
                     const int k = bb + lane + 128 * t;
-                    q0 += lds_f64_lt(k, e2, valS + 8 * k);
-                    q1 += lds_f64_lt(k + 32, e2, valS + 8 * k + 256);
-                    q2 += lds_f64_lt(k + 64, e2, valS + 8 * k + 512);
-                    q3 += lds_f64_lt(k + 96, e2, valS + 8 * k + 768);
+                    q0 += rem_product(p, k, e2, colS, valS, x_policy);
+                    q1 += rem_product(p, k + 32, e2, colS, valS, x_policy);
+                    q2 += rem_product(p, k + 64, e2, colS, valS, x_policy);
+                    q3 += rem_product(p, k + 96, e2, colS, valS, x_policy);
                 }
                 double sq = (q0 + q1) + (q2 + q3);
                 sq += __shfl_xor_sync(FULL, sq, 16);
