@@ -75,13 +75,23 @@ __device__ __forceinline__ WItem load_witem(const WItem *w, int k) {
 //    each, one round trip of gathers;
 //  * every row <= MED entries (kShortRow, or kMedRow for the TM kernels):
 //    two lanes per row, all rows at once;
-//  * a longer row (power-law hubs): the flat pass (flat_products, flat_rows),
-//    all gathers of the item in flight together.
+//  * a longer row (power-law hubs): the flat pass (flat_rows), each product
+//    formed where it is summed.
 // The path and the order of every sum depend only on the item's content: y
 // stays bitwise deterministic.
-__device__ __forceinline__ void flat_products(const Params &p, uint32_t colS, uint32_t valS, int E,
-                                              uint64_t x_policy, int lane);
-__device__ __forceinline__ double flat_rows(uint32_t rq, uint32_t valS, int rows, int lane);
+__device__ __forceinline__ double flat_rows(const Params &p, uint32_t rq, uint32_t colS, uint32_t valS, int rows,
+                                            uint64_t x_policy, int lane);
+
+// product of remainder entry k (rounded on its own, as the earlier
+// shared-memory product pass stored it) if k < e, else +0.0 -- the term the row sums would have read
+__device__ __forceinline__ double rem_product(const Params &p, int k, int e, uint32_t colS, uint32_t valS,
+                                              uint64_t x_policy) {
+    int c;
+    double v;
+    lds_entry_lt(k, e, colS + 4 * k, valS + 8 * k, c, v);
+    const double pr = __dmul_rn(v, ldg_hint(p.x + (uint32_t)c, x_policy));
+    return k < e ? pr : 0.0;
+}
 
 template <int MED>
 __device__ __forceinline__ void remainder(const Params &p, uint32_t rpS, uint32_t colS, uint32_t valS, int rows,
@@ -105,8 +115,7 @@ __device__ __forceinline__ void remainder(const Params &p, uint32_t rpS, uint32_
     }
     if (maxlen > MED) {
         dirty = true;  // the slot now holds products written by the generic proxy
-        flat_products(p, colS, valS, lds_s32(rpS + 4 * rows), x_policy, lane);
-        acc += flat_rows(rpS, valS, rows, lane);
+        acc += flat_rows(p, rpS, colS, valS, rows, x_policy, lane);
         return;
     }
     const int trips = (int)__reduce_max_sync(FULL, (unsigned)((e - b + 1 - h) >> 1));
@@ -123,37 +132,13 @@ __device__ __forceinline__ void remainder(const Params &p, uint32_t rpS, uint32_
     }
 }
 
-// Flat remainder pass, step 1: one lane per entry, the x gathers of 256
-// entries in flight at once; each value in the slot is overwritten by its
-// product (rounded, so every later order of summation sees the same terms).
-__device__ __forceinline__ void flat_products(const Params &p, uint32_t colS, uint32_t valS, int E,
-                                              uint64_t x_policy, int lane) {
-#pragma unroll 1
-    for (int k0 = 0; k0 < E; k0 += 256) {
-        double pv[8];
-#pragma unroll
-        for (int j = 0; j < 8; ++j) {
-            const int k = k0 + 32 * j + lane;
-            int c;
-            double v;
-            lds_entry_lt(k, E, colS + 4 * k, valS + 8 * k, c, v);
-            pv[j] = __dmul_rn(v, ldg_hint(p.x + (uint32_t)c, x_policy));
-        }
-#pragma unroll
-        for (int j = 0; j < 8; ++j) {
-            const int k = k0 + 32 * j + lane;
-            if (k < E) sts_f64(valS + 8 * k, pv[j]);
-        }
-    }
-    __syncwarp();
-}
-
-// Flat remainder pass, step 2, for one tile row (rows <= 16, row pointers at
+// Flat remainder pass for one tile row (rows <= 16, row pointers at
 // rq): rows of <= kShortRow products two lanes per row, longer rows a
 // half-warp per row (two rows at a time, the whole warp for the last one)
 // with an xor tree.  Returns lane r's (or r + 16's) share of row r.  The order
 // of every sum depends only on this tile row.
-__device__ __forceinline__ double flat_rows(uint32_t rq, uint32_t valS, int rows, int lane) {
+__device__ __forceinline__ double flat_rows(const Params &p, uint32_t rq, uint32_t colS, uint32_t valS, int rows,
+                                            uint64_t x_policy, int lane) {
     const int r = lane & 15, h = lane >> 4;
     const int b = lds_s32(rq + 4 * min(r, rows)), e = lds_s32(rq + 4 * min(r + 1, rows));
     const bool lng = e - b > kShortRow;
@@ -163,8 +148,8 @@ __device__ __forceinline__ double flat_rows(uint32_t rq, uint32_t valS, int rows
 #pragma unroll 1
     for (int i = 0; i < trips; i += 2) {
         const int k0 = b + h + 2 * i;
-        s0 += lds_f64_lt(k0, ee, valS + 8 * k0);
-        s1 += lds_f64_lt(k0 + 2, ee, valS + 8 * k0 + 16);
+        s0 += rem_product(p, k0, ee, colS, valS, x_policy);
+        s1 += rem_product(p, k0 + 2, ee, colS, valS, x_policy);
     }
     double acc = s0 + s1;
     uint32_t lm = __ballot_sync(FULL, lng && h == 0 && r < rows);
@@ -183,10 +168,10 @@ __device__ __forceinline__ double flat_rows(uint32_t rq, uint32_t valS, int rows
 #pragma unroll 1
         for (int t = 0; t < t2; ++t) {
             const int k = bb + off + 4 * stride * t;
-            q0 += lds_f64_lt(k, e2, valS + 8 * k);
-            q1 += lds_f64_lt(k + stride, e2, valS + 8 * (k + stride));
-            q2 += lds_f64_lt(k + 2 * stride, e2, valS + 8 * (k + 2 * stride));
-            q3 += lds_f64_lt(k + 3 * stride, e2, valS + 8 * (k + 3 * stride));
+            q0 += rem_product(p, k, e2, colS, valS, x_policy);
+            q1 += rem_product(p, k + stride, e2, colS, valS, x_policy);
+            q2 += rem_product(p, k + 2 * stride, e2, colS, valS, x_policy);
+            q3 += rem_product(p, k + 3 * stride, e2, colS, valS, x_policy);
         }
         double sq = (q0 + q1) + (q2 + q3);
         if (!pair) sq += __shfl_xor_sync(FULL, sq, 16);
@@ -211,25 +196,14 @@ __device__ __forceinline__ void group_item(const Params &p, const WItem &it, uin
     const uint32_t total = it.val_tot >> 16, rp = it.rp_col & 0xFFFFu;
     const bool has_rem = total > rp;
     const uint32_t rpS = slot + rp, colS = slot + (it.rp_col >> 16), valS = slot + (it.val_tot & 0xFFFFu);
-    if (has_rem) flat_products(p, colS, valS, lds_s32(rpS + 4 * (16 * (ntr - 1) + rows_last)), x_policy, lane);
 #pragma unroll 1
     for (int g = 0; g < ntr; ++g) {
-        double acc = has_rem ? flat_rows(rpS + 64u * (uint32_t)g, valS, g + 1 < ntr ? 16 : rows_last, lane) : 0.0;
+        double acc = has_rem ? flat_rows(p, rpS + 64u * (uint32_t)g, colS, valS, g + 1 < ntr ? 16 : rows_last, x_policy,
+                                         lane) : 0.0;
         acc += __shfl_xor_sync(FULL, acc, 16);
         const int64_t row = 16 * ((int64_t)it.I + g) + lane;
         if (lane < 16 && row < p.m) p.y[row] = acc;
     }
-}
-
-// product of remainder entry k (rounded on its own, exactly as flat_products
-// stores it) if k < e, else +0.0 -- the term the row sums would have read
-__device__ __forceinline__ double rem_product(const Params &p, int k, int e, uint32_t colS, uint32_t valS,
-                                              uint64_t x_policy) {
-    int c;
-    double v;
-    lds_entry_lt(k, e, colS + 4 * k, valS + 8 * k, c, v);
-    const double pr = __dmul_rn(v, ldg_hint(p.x + (uint32_t)c, x_policy));
-    return k < e ? pr : 0.0;
 }
 
 // Row-group item, TM kernels: two tile rows at a time, half-warp h on tile
