@@ -43,6 +43,15 @@ extern "C" {
 #define TILESPMV_MODE_AUTO 2      /* DEFERRED iff nnz >= 1.8e6 (reading R18), else ADPT */
 #define TILESPMV_MODE_FORCE_CSR 3 /* TileSpMV_CSR: every tile CSR */
 
+/* SpMV kernel of a handle (tilespmv_opts_t.kernel).  Both compute the same
+ * y within the north-star bound; the work-item byte budget (and so the
+ * order of the sums) is the kernel's, so handles that must agree bitwise
+ * (row slices of one matrix, tilespmv sharding) must use the same kernel. */
+#define TILESPMV_KERNEL_AUTO 0       /* DENSE_ROWS if the mean stored payload per tile row exceeds
+                                        6 KiB (dense, FEM-like tile rows), else SM_QUEUE          */
+#define TILESPMV_KERNEL_SM_QUEUE 1   /* one 32-warp CTA per SM, 4.5 KiB items, shared-memory queue */
+#define TILESPMV_KERNEL_DENSE_ROWS 2 /* 16 warps per SM, 10.5 KiB items, static per-warp chunks    */
+
 /* tile format codes, in the order of P:20 / P:96 */
 #define TILESPMV_FMT_CSR 0
 #define TILESPMV_FMT_COO 1
@@ -67,8 +76,13 @@ extern "C" {
 typedef struct tilespmv_matrix *tilespmv_handle_t; /* opaque; owns all its device storage */
 
 typedef struct {
-    int32_t mode;     /* TILESPMV_MODE_*; default DEFERRED                               */
-    int32_t validate; /* 1 (default): check the CSR is canonical; 0: trust the caller   */
+    int32_t mode;        /* TILESPMV_MODE_*; default DEFERRED                               */
+    int32_t validate;    /* 1 (default): check the CSR is canonical; 0: trust the caller   */
+    int32_t kernel;      /* TILESPMV_KERNEL_*; default AUTO                                 */
+    int32_t keep_layout; /* 0 (default): after create the handle keeps only what the SpMV
+                            kernel reads (the execution schedule, about the matrix's
+                            algorithmic bytes); 1: also keep the canonical tiled arrays for
+                            tilespmv_export (bit-exact parity tests)                       */
 } tilespmv_opts_t;
 
 typedef struct {
@@ -88,6 +102,8 @@ typedef struct {
     int64_t num_split_rows;             /* tile rows split over several items */
     int64_t device_bytes;               /* device memory owned by the handle */
     double create_ms;                   /* wall time of tilespmv_create_from_csr */
+    int32_t kernel;                     /* resolved TILESPMV_KERNEL_* (never AUTO) */
+    int32_t reserved;
 } tilespmv_info_t;
 
 /* Build a tiled matrix from a canonical device CSR ("converting a basic
@@ -97,9 +113,11 @@ typedef struct {
  *   d_rowptr    int32[m+1], d_colidx int32[nnz], d_val double[nnz]: device,
  *               caller-owned, read only during this call.  Explicit zeros
  *               are entries.  d_colidx/d_val may be NULL when nnz == 0.
- *   opts        NULL = defaults {DEFERRED, validate=1}
- *   stream      work is queued on it; the call synchronises it before return,
- *               so the inputs may be freed immediately afterwards.
+ *   opts        NULL = defaults {DEFERRED, validate=1, kernel=AUTO, keep_layout=0}
+ *   stream      every kernel, copy and temporary allocation of the call is
+ *               queued on it (stream-ordered; no device-wide synchronisation,
+ *               other streams keep running); the call synchronises `stream`
+ *               before return, so the inputs may be freed immediately.
  * On success *out receives a handle bound to the current device.
  * Errors: INVALID_ARG, NOT_CANONICAL (only detected with validate=1),
  * OVERFLOW, OOM, CUDA.  On error *out is set to NULL and nothing leaks.     */
@@ -148,8 +166,17 @@ int64_t tilespmv_export_size(tilespmv_handle_t h, int32_t which);
 
 /* Copy one array of the canonical tiled layout to host memory (synchronous);
  * `bytes` must equal tilespmv_export_size(h, which).  Used for bit-exact
- * parity against the reference tiler.                                        */
+ * parity against the reference tiler.  Needs a handle created with
+ * opts.keep_layout = 1 (else INVALID_ARG; tilespmv_export_size returns the
+ * size either way).                                                          */
 int tilespmv_export(tilespmv_handle_t h, int32_t which, void *host_dst, size_t bytes);
+
+/* The kernel TILESPMV_KERNEL_AUTO resolves to for a matrix whose stored
+ * tile payload is payload_bytes over tilem tile rows (tilespmv_info_t).
+ * Sharded callers apply it to the whole matrix's totals so that every shard
+ * runs the kernel (and the item byte budget) of the unsharded matrix, and so
+ * the unsharded summation order.                                            */
+int32_t tilespmv_auto_kernel(int64_t payload_bytes, int64_t tilem);
 
 /* Static description of a status code. */
 const char *tilespmv_status_string(int status);

@@ -11,6 +11,10 @@
  * DESIGN.md §"Readings of the paper" (SURVEY.md §8c C3 #k).
  *
  * Contents
+ *   oracle_spmv_f64    Alg. 1 word for word in double: the plain
+ *                      fp64 row loop, the CPU baseline bench.py times
+ *                      (BASELINE.md D5 item 1); correctness uses
+ *                      oracle_spmv_rows
  *   oracle_spmv_rows   Alg. 1: y_i = sum_j a_ij * x_j, every row
  *                      independent, accumulated in x87 long double and rounded
  *                      once; also sum_j |a_ij * x_j| for the tolerance test.
@@ -68,6 +72,19 @@ int oracle_spmv_rows(int64_t m, const int32_t *rowptr, const int32_t *colidx,
         if (absy) absy[q] = (double)ai;
     }
     return 0;
+}
+
+/* Alg. 1 as printed, in double: y_i <- 0, then y_i <- y_i +
+ * a_ij * x_j in entry order, each product and sum rounded to double (gcc
+ * -O2 without -ffast-math and without FMA contraction keeps that order). */
+void oracle_spmv_f64(int64_t m, const int32_t *rowptr, const int32_t *colidx,
+                     const double *val, const double *x, double *y)
+{
+    for (int64_t i = 0; i < m; ++i) {
+        double yi = 0.0;
+        for (int64_t k = rowptr[i]; k < rowptr[i + 1]; ++k) yi = yi + val[k] * x[colidx[k]];
+        y[i] = yi;
+    }
 }
 
 /* ------------------------------------------------------------------------ */

@@ -30,7 +30,7 @@ def build(force: bool = False) -> str:
     """gcc the oracle (plain C, -O2, no fast-math) and the multi-threaded CPU
     CSR baseline beside it (not the oracle; bench context only)."""
     if force or not os.path.exists(LIB) or os.path.getmtime(LIB) < os.path.getmtime(SRC):
-        subprocess.check_call(["gcc", "-O2", "-std=c11", "-Wall", "-fPIC", "-shared",
+        subprocess.check_call(["gcc", "-O2", "-ffp-contract=off", "-std=c11", "-Wall", "-fPIC", "-shared",
                                "-o", LIB, SRC])
     if force or not os.path.exists(OMP_LIB) or os.path.getmtime(OMP_LIB) < os.path.getmtime(OMP_SRC):
         subprocess.check_call(["gcc", "-O3", "-std=c11", "-Wall", "-fopenmp", "-fPIC", "-shared",
@@ -64,6 +64,8 @@ def lib():
         p = ctypes.c_void_p
         L.oracle_spmv_rows.argtypes = [ctypes.c_int64, p, p, p, p, p, ctypes.c_int64, p, p]
         L.oracle_spmv_rows.restype = ctypes.c_int
+        L.oracle_spmv_f64.argtypes = [ctypes.c_int64, p, p, p, p, p]
+        L.oracle_spmv_f64.restype = None
         L.oracle_select.argtypes = [p, ctypes.c_int32, p]
         L.oracle_select.restype = ctypes.c_int
         L.oracle_hyb_width.argtypes = [p]
@@ -113,6 +115,18 @@ def spmv(A, x: np.ndarray, rows: np.ndarray | None = None):
                                 None if rws is None else _ptr(rws), nr, _ptr(y), _ptr(ay))
     assert rc == 0
     return y[:nr], ay[:nr]
+
+
+def spmv_f64(A, x: np.ndarray) -> np.ndarray:
+    """Alg. 1 as printed, in double (oracle_spmv_f64): the plain
+    fp64 row loop timed as the CPU baseline.  Correctness checks use spmv()."""
+    rp, ci, va = _csr_arrays(A)
+    x = np.ascontiguousarray(x, dtype=np.float64)
+    if x.size == 0:
+        x = np.zeros(1)
+    y = np.zeros(max(A.m, 1))
+    lib().oracle_spmv_f64(A.m, _ptr(rp), _ptr(ci), _ptr(va), _ptr(x), _ptr(y))
+    return y[:A.m]
 
 
 def select(masks, force_csr: bool = False):

@@ -8,7 +8,7 @@ PKG = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(PKG)
 LIB = os.path.join(PKG, "libtilespmv.so")
 SOURCES = [os.path.join(PKG, "csrc", f)
-           for f in ("abi.cu", "tiler.cu", "schedule.cu", "spmv_v1.cu", "spmv_warp.cu", "cg.cu")]
+           for f in ("abi.cu", "tiler.cu", "schedule.cu", "spmv_warp.cu", "cg.cu")]
 HEADERS = [os.path.join(PKG, "csrc", f) for f in ("internal.cuh", "spmv_common.cuh", "spmv_tiles.cuh")] + \
           [os.path.join(ROOT, "include", "tilespmv.h")]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")

@@ -1,6 +1,6 @@
 // abi.cu -- the extern "C" boundary declared in include/tilespmv.h.
 // Argument checking, handle lifetime, info/export, error strings.  All
-// compute is in tiler.cu (create) and spmv.cu (run).
+// compute is in tiler.cu, schedule.cu (create) and spmv_warp.cu (run).
 #include <chrono>
 #include <cstring>
 #include <string>
@@ -36,7 +36,8 @@ static void free_matrix(tilespmv_matrix *M) {
     if (cur != M->device) cudaSetDevice(M->device);
     void *ptrs[] = {M->tilePtr, M->tileColIdx, M->tileNnz, M->tileFmt, M->tileAux, M->tileOff,
                     M->payload, M->remRowPtr, M->remCol, M->remVal, M->items, M->split_info,
-                    M->partials, M->counters, M->xstage, M->ystage, M->tdesc, M->cta_begin, M->blob, M->witems, M->jcols, M->wfirst, M->units};
+                    M->partials, M->counters, M->xstage, M->ystage, M->tdesc, M->cta_begin, M->blob,
+                    M->witems, M->jcols, M->wfirst, M->units};
     for (void *p : ptrs)
         if (p) cudaFree(p);
     if (cur >= 0 && cur != M->device) cudaSetDevice(cur);
@@ -84,9 +85,12 @@ int tilespmv_create_from_csr(tilespmv_handle_t *out, int64_t m, int64_t n, int64
     if (!d_rowptr) return set_error(TILESPMV_INVALID_ARG, "rowptr is NULL");
     if (m == 0 && nnz != 0) return set_error(TILESPMV_NOT_CANONICAL, "m == 0 requires nnz == 0");
     if (nnz > 0 && (!d_colidx || !d_val)) return set_error(TILESPMV_INVALID_ARG, "colidx/val is NULL");
-    tilespmv_opts_t o{TILESPMV_MODE_DEFERRED, 1};
+    tilespmv_opts_t o{TILESPMV_MODE_DEFERRED, 1, TILESPMV_KERNEL_AUTO, 0};
     if (opts) o = *opts;
     if (o.mode < 0 || o.mode > 3) return set_error(TILESPMV_INVALID_ARG, "unknown mode");
+    if (o.kernel < TILESPMV_KERNEL_AUTO || o.kernel > TILESPMV_KERNEL_DENSE_ROWS)
+        return set_error(TILESPMV_INVALID_ARG, "unknown kernel");
+    if (o.keep_layout != 0 && o.keep_layout != 1) return set_error(TILESPMV_INVALID_ARG, "keep_layout must be 0 or 1");
     auto t0 = std::chrono::steady_clock::now();
     cudaStream_t st = static_cast<cudaStream_t>(stream);
     tilespmv_matrix *M = new (std::nothrow) tilespmv_matrix();
@@ -96,12 +100,18 @@ int tilespmv_create_from_csr(tilespmv_handle_t *out, int64_t m, int64_t n, int64
         return cuda_status(cudaGetLastError(), "cudaGetDevice");
     }
     {  // the CSR arrays must live on the current device
-        cudaPointerAttributes a;
-        if (cudaPointerGetAttributes(&a, d_rowptr) != cudaSuccess || a.type != cudaMemoryTypeDevice ||
-            a.device != M->device) {
-            cudaGetLastError();
-            delete M;
-            return set_error(TILESPMV_INVALID_ARG, "rowptr is not device memory of the current device");
+        const void *ptrs[3] = {d_rowptr, nnz > 0 ? d_colidx : nullptr, nnz > 0 ? d_val : nullptr};
+        const char *names[3] = {"rowptr", "colidx", "val"};
+        for (int i = 0; i < 3; ++i) {
+            if (!ptrs[i]) continue;
+            cudaPointerAttributes a;
+            if (cudaPointerGetAttributes(&a, ptrs[i]) != cudaSuccess || a.type != cudaMemoryTypeDevice ||
+                a.device != M->device) {
+                cudaGetLastError();
+                delete M;
+                return set_error(TILESPMV_INVALID_ARG,
+                                 std::string(names[i]) + " is not device memory of the current device");
+            }
         }
     }
     M->m = m;
@@ -109,11 +119,13 @@ int tilespmv_create_from_csr(tilespmv_handle_t *out, int64_t m, int64_t n, int64
     M->nnz = nnz;
     M->mode = o.mode == TILESPMV_MODE_AUTO ? (nnz >= 1800000 ? TILESPMV_MODE_DEFERRED : TILESPMV_MODE_ADPT)
                                            : o.mode;
+    M->keep_layout = o.keep_layout != 0;
     int rc = build_tiled(*M, d_rowptr, d_colidx, d_val, o.validate, st);
-    if (!rc) rc = choose_kernel(*M);
+    if (!rc) rc = choose_kernel(*M, o.kernel);
     if (!rc) rc = build_schedule(*M, st);
     if (!rc) rc = build_tdesc(*M, st);
-    if (!rc) rc = configure_launch(*M);
+    if (!rc) rc = configure_launch(*M, st);
+    if (!rc) release_create_time(*M, st);
     if (!rc) {
         cudaError_t e = cudaStreamSynchronize(st);
         if (e != cudaSuccess) rc = cuda_status(e, "cudaStreamSynchronize(create)");
@@ -151,11 +163,16 @@ int tilespmv_run_host(tilespmv_handle_t h, const double *h_x, double *h_y, void 
     if (int rc = check_handle(h)) return rc;
     if ((h->m > 0 && !h_y) || (h->n > 0 && !h_x)) return set_error(TILESPMV_INVALID_ARG, "NULL host buffer");
     cudaStream_t st = static_cast<cudaStream_t>(stream);
-    if (!h->xstage) {
-        if (cudaMalloc(&h->xstage, std::max<int64_t>(h->n, 1) * 8) != cudaSuccess)
-            return cuda_status(cudaGetLastError(), "cudaMalloc(xstage)");
-        if (cudaMalloc(&h->ystage, std::max<int64_t>(h->m, 1) * 8) != cudaSuccess)
-            return cuda_status(cudaGetLastError(), "cudaMalloc(ystage)");
+    if (!h->xstage || !h->ystage) {  // both staging buffers or neither
+        double *xs = nullptr, *ys = nullptr;
+        if (cudaMalloc(&xs, std::max<int64_t>(h->n, 1) * 8) != cudaSuccess ||
+            cudaMalloc(&ys, std::max<int64_t>(h->m, 1) * 8) != cudaSuccess) {
+            const int rc = cuda_status(cudaGetLastError(), "cudaMalloc(host-staging buffers)");
+            if (xs) cudaFree(xs);
+            return rc;
+        }
+        h->xstage = xs;
+        h->ystage = ys;
         h->device_bytes += 8 * (h->m + h->n);
     }
     cudaError_t e;
@@ -217,6 +234,7 @@ int tilespmv_get_info(tilespmv_handle_t h, tilespmv_info_t *info) {
     info->num_split_rows = h->num_split;
     info->device_bytes = h->device_bytes;
     info->create_ms = h->create_ms;
+    info->kernel = h->kernel;
     return TILESPMV_OK;
 }
 
@@ -231,7 +249,7 @@ static int64_t export_size(const Matrix &M, int32_t which, const void **src) {
     case TILESPMV_ARR_TILEAUX: p = M.tileAux; b = M.numtile; break;
     case TILESPMV_ARR_TILEOFF: p = M.tileOff; b = 4 * (M.numtile + 1); break;
     case TILESPMV_ARR_PAYLOAD: p = M.payload; b = M.payload_bytes; break;
-    case TILESPMV_ARR_REMROWPTR: p = M.remRowPtr; b = M.remRowPtr ? 4 * (M.m + 1) : 0; break;
+    case TILESPMV_ARR_REMROWPTR: p = M.remRowPtr; b = M.rem_nnz > 0 ? 4 * (M.m + 1) : 0; break;
     case TILESPMV_ARR_REMCOL: p = M.remCol; b = 4 * M.rem_nnz; break;
     case TILESPMV_ARR_REMVAL: p = M.remVal; b = 8 * M.rem_nnz; break;
     default: return TILESPMV_INVALID_ARG;
@@ -254,6 +272,8 @@ int tilespmv_export(tilespmv_handle_t h, int32_t which, void *host_dst, size_t b
     if (b < 0) return set_error(TILESPMV_INVALID_ARG, "unknown array id");
     if ((int64_t)bytes != b) return set_error(TILESPMV_INVALID_ARG, "byte count mismatch");
     if (b == 0) return TILESPMV_OK;
+    if (!h->keep_layout)
+        return set_error(TILESPMV_INVALID_ARG, "the canonical layout was not kept (create with opts.keep_layout = 1)");
     if (!host_dst) return set_error(TILESPMV_INVALID_ARG, "host_dst is NULL");
     cudaError_t e = cudaMemcpy(host_dst, src, b, cudaMemcpyDeviceToHost);
     if (e != cudaSuccess) return cuda_status(e, "cudaMemcpy(export)");
@@ -269,5 +289,7 @@ int tilespmv_launch_shape(tilespmv_handle_t h, int32_t *grid, int32_t *block, in
 }
 
 const char *tilespmv_kernel_name(tilespmv_handle_t h) { return h ? h->kernel_name : ""; }
+
+int32_t tilespmv_auto_kernel(int64_t payload_bytes, int64_t tilem) { return auto_kernel(payload_bytes, tilem); }
 
 }  // extern "C"

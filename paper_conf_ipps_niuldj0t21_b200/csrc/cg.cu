@@ -18,7 +18,6 @@
 // kCheckEvery iterations.
 #include <algorithm>
 #include <cmath>
-#include <cstdlib>
 
 #include "spmv_common.cuh"
 
@@ -223,7 +222,6 @@ int cg_solve(const Matrix &M, const double *d_b, double *d_x, double tol, int ma
     do {
         if ((rc = launch_spmv(M, d_x, q, st))) break;  // q = A x0
         int G = kBlocks;
-        if (const char *ev = getenv("TILESPMV_CG_BLOCKS")) G = std::min(kBlocks, std::max(1, atoi(ev)));
         k_cg_init<<<G, kThreads, 0, st>>>(d_b, q, r, p, n, S);
         k_cg_init_scalars<<<1, kThreads, 0, st>>>(S, G);
         const double tol2 = tol * tol;

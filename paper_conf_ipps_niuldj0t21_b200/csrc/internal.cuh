@@ -29,9 +29,6 @@ enum : uint8_t { F_CSR = 0, F_COO = 1, F_ELL = 2, F_HYB = 3, F_DNS = 4, F_DNSROW
 // ---------------------------------------------------------------------------
 constexpr int kItemTiles = 16;
 constexpr int kItemBytesMax = 12288;  // largest shared-memory slot of any kernel
-constexpr int kShortRow = 16;     // remainder rows up to this length: 2 lanes per row
-constexpr int kMedRow = 32;       // TM kernels: item remainder rows up to this length stay 2 lanes per row
-                                  // (the 27-point stencil's wrap rows hold up to 21; hubs take the flat pass)
 
 struct __align__(16) Item {
     int32_t I;        // tile row
@@ -73,14 +70,13 @@ struct __align__(16) WItem {
                            // bit 30: the last tile column's x segment passes x[n-1] (ragged tail)
 };
 
-// Per-warp start record of the warp kernel: the warp's item chunk and a copy
-// of its first item (and the second item's record, for the double-buffered
-// kernel), so the prologue needs one round trip before the blob copies.
+// Per-warp start record of the dense-row kernel: the warp's item chunk and a
+// copy of its first item, so the prologue needs one round trip before the
+// blob copy.
 struct __align__(16) WFirst {
     int32_t kbeg, kend, pad0, pad1;
     WItem w;
     int32_t J[16];
-    WItem w2;
 };
 
 // The parts of a split tile row form groups of kLocalParts consecutive parts.
@@ -92,8 +88,8 @@ struct __align__(16) WFirst {
 constexpr int kLocalParts = 4;
 // per-item fixed cost (bytes-equivalent of an item's latency chain: record,
 // blob, x gathers) used to balance the warps' item chunks; measured on R-MAT
-// (power-law, many small items): 2048 gives 174 us against 188 us for 512,
-// neutral on the stencil and mixed matrices
+// (power-law, many small items): 2048 gave 174 us against 188 us for 512,
+// neutral on the stencil and mixed matrices (round 1)
 constexpr int64_t kItemFixedCost = 2048;
 __host__ __device__ __forceinline__ int item_nt(const Item &it) { return (it.part_nt >> 24) & 31; }
 __host__ __device__ __forceinline__ int item_part(const Item &it) { return it.part_nt & 0xFFFFFF; }
@@ -104,7 +100,9 @@ struct Matrix {
     int device = 0;
     int64_t m = 0, n = 0, nnz = 0, tilem = 0, tilen = 0, numtile = 0;
     int32_t mode = TILESPMV_MODE_DEFERRED;
-    // level 1 + format bytes + payload offsets
+    bool keep_layout = false;  // keep the canonical arrays after create (tilespmv_export)
+    // level 1 + format bytes + payload offsets; create-time only
+    // unless keep_layout
     int32_t *tilePtr = nullptr, *tileColIdx = nullptr, *tileNnz = nullptr;
     uint8_t *tileFmt = nullptr, *tileAux = nullptr;
     uint32_t *tileOff = nullptr;
@@ -115,34 +113,33 @@ struct Matrix {
     int32_t *remRowPtr = nullptr, *remCol = nullptr;
     double *remVal = nullptr;
     int64_t rem_nnz = 0;
-    // SpMV schedule
+    // SpMV schedule (create-time: items, tdesc)
     Item *items = nullptr;
     int64_t num_items = 0;
+    uint2 *tdesc = nullptr;        // per-item tile-descriptor lists (dlist)
+    int64_t num_dsc = 0;
     int2 *split_info = nullptr;  // {first partial slot, number of parts}
     int64_t num_split = 0;
     double *partials = nullptr;
     int32_t *counters = nullptr;
+    // what the kernels read
+    uint8_t *blob = nullptr;       // per-item execution blobs (blob_parts)
+    WItem *witems = nullptr;       // compact per-item records
+    int32_t *jcols = nullptr;      // 16 tile columns per item
+    WFirst *wfirst = nullptr;      // dense-row kernel: per-warp chunk + first item
+    int64_t blob_bytes = 0;
+    int64_t *cta_begin = nullptr;  // dense-row kernel: item chunk per warp (row-aligned, cost-balanced);
+                                   // SM-queue kernel: unit range per CTA
+    int32_t *units = nullptr;      // SM-queue kernel: first item of each unit, num_units + 1
+    int64_t num_units = 0;
     // host-staging buffers for tilespmv_run_host
     double *xstage = nullptr, *ystage = nullptr;
     // statistics
     int64_t sel_tiles[7] = {0}, sel_nnz[7] = {0}, kept_tiles[7] = {0}, kept_nnz[7] = {0};
     int64_t device_bytes = 0;
     double create_ms = 0;
-    // v2 kernel inputs derived from the canonical arrays
-    uint2 *tdesc = nullptr;        // per-item tile-descriptor lists (dlist), create-time only
-    int64_t num_dsc = 0;
-    uint8_t *blob = nullptr;       // per-item execution blobs (blob_parts), read by the kernels
-    WItem *witems = nullptr;       // compact per-item records for the warp kernel
-    int32_t *jcols = nullptr;      // 16 tile columns per item (warp kernel)
-    WFirst *wfirst = nullptr;      // per-warp chunk + first item (warp kernel)
-    int64_t blob_bytes = 0;
-    int64_t *cta_begin = nullptr;  // contiguous item chunk per warp (row-aligned, cost-balanced),
-                                   // or unit range per CTA (SM-queue kernel)
-    int32_t *units = nullptr;      // SM-queue kernel: first item of each unit, num_units + 1
-    int64_t num_units = 0;
-    int local_parts = kLocalParts;  // parts per group of a split tile row (TILESPMV_LOCAL_PARTS)
     // launch shape
-    int kernel_version = 20;
+    int kernel = TILESPMV_KERNEL_SM_QUEUE;  // resolved kernel (never AUTO)
     const char *kernel_name = "";
     int item_bytes = kItemBytesMax;  // slot size the schedule was built for
     int grid = 0, block = 0, smem = 0;
@@ -155,11 +152,13 @@ int cuda_status(cudaError_t e, const char *what);
 // tiler.cu
 int build_tiled(Matrix &M, const int32_t *d_rowptr, const int32_t *d_colidx, const double *d_val,
                 int validate, cudaStream_t stream);
-// spmv.cu
-int choose_kernel(Matrix &M);
+// schedule.cu
+int auto_kernel(int64_t payload_bytes, int64_t tilem);
+int choose_kernel(Matrix &M, int requested);
 int build_schedule(Matrix &M, cudaStream_t stream);
 int build_tdesc(Matrix &M, cudaStream_t stream);
-int configure_launch(Matrix &M);
+int configure_launch(Matrix &M, cudaStream_t stream);
+void release_create_time(Matrix &M, cudaStream_t stream);
 int launch_spmv(const Matrix &M, const double *d_x, double *d_y, cudaStream_t stream);
 // cg.cu
 int cg_solve(const Matrix &M, const double *d_b, double *d_x, double tol, int maxit, int *iters, double *relres,

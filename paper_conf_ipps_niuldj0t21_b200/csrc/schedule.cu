@@ -1,13 +1,16 @@
 // schedule.cu -- create-time SpMV schedule and launch dispatch.
 //   * work items: byte-bounded pieces of one tile row (internal.cuh), built
 //     by one thread per tile row in two passes (count, scan, write);
-//   * 8-byte tile descriptors derived from the canonical level-1 arrays;
-//   * kernel choice (TILESPMV_KERNEL env: 1 = v1 baseline, 20-29 = warp kernel
-//     variants, default 20).
+//   * 8-byte tile descriptors derived from the canonical level-1 arrays, and
+//     the per-item execution blobs the kernels stage with one TMA copy;
+//   * kernel choice (tilespmv_opts_t.kernel) and the per-CTA / per-warp
+//     work ranges.
+// Everything runs on the caller's stream: temporaries are stream-ordered
+// (cudaMallocAsync / cudaFreeAsync), and the only host waits are
+// cudaStreamSynchronize(stream) for the sizes the next allocation needs.
 #include <cub/cub.cuh>
 
 #include <algorithm>
-#include <cstdlib>
 
 #include "spmv_common.cuh"
 
@@ -331,7 +334,7 @@ __global__ void k_item_cost(const Item *items, int64_t n, int64_t m, int64_t fix
     int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     if (k >= n) return;
     const Item it = items[k];
-    cost[k] = (int64_t)item_parts(it, m).total + 40 * (item_nt(it)) + fixed;
+    cost[k] = (int64_t)blob_parts(it, m).total + 40 * (item_nt(it)) + fixed;
 }
 
 __global__ void k_warp_first(const int64_t *begin, const WItem *witems, const int32_t *jcols, int W, WFirst *wf) {
@@ -348,7 +351,6 @@ __global__ void k_warp_first(const int64_t *begin, const WItem *witems, const in
         f.w = WItem{};
         for (int i = 0; i < 16; ++i) f.J[i] = 0;
     }
-    f.w2 = f.kbeg + 1 < f.kend ? witems[f.kbeg + 1] : WItem{};
     wf[b] = f;
 }
 
@@ -414,21 +416,32 @@ __global__ void k_cta_units(const int64_t *incl, const int32_t *units, int64_t n
     cta_begin[b] = lo;
 }
 
+// stream-ordered temporary device buffer
+struct Tmp {
+    void *p = nullptr;
+    cudaStream_t st;
+    explicit Tmp(cudaStream_t s) : st(s) {}
+    Tmp(const Tmp &) = delete;
+    ~Tmp() { if (p) cudaFreeAsync(p, st); }
+    int alloc(size_t bytes) {
+        if (cudaMallocAsync(&p, bytes ? bytes : 1, st) != cudaSuccess) {
+            p = nullptr;
+            return cuda_status(cudaGetLastError(), "cudaMallocAsync(schedule temporary)");
+        }
+        return 0;
+    }
+    template <class T> T *as() const { return static_cast<T *>(p); }
+};
+
+// a CUB device-wide call with a stream-ordered temporary
 template <class F>
-int scan(F &&f) {
+int scan(F &&f, cudaStream_t st) {
     size_t bytes = 0;
     TSP_CK(f(nullptr, bytes));
-    void *tmp = nullptr;
-    TSP_CK(cudaMalloc(&tmp, std::max<size_t>(bytes, 1)));
-    cudaError_t e = f(tmp, bytes);
-    cudaFree(tmp);
-    TSP_CK(e);
+    Tmp tmp(st);
+    if (int rc = tmp.alloc(bytes)) return rc;
+    TSP_CK(f(tmp.p, bytes));
     return 0;
-}
-
-KernelChoice choose(int version) {
-    if (version == 1) return kernel_v1();
-    return kernel_warp(version);
 }
 
 }  // namespace
@@ -439,183 +452,151 @@ int build_schedule(Matrix &M, cudaStream_t st) {
     if (T == 0) return 0;
     auto blocks = [&](int64_t n) { return (unsigned)std::max<int64_t>(1, (n + TB - 1) / TB); };
     const int64_t NW = (T + kGroupWindow - 1) / kGroupWindow;
-    // row-group items only for the kernels that run them (compute_item)
-    const int group = M.kernel_version != 1 && !getenv("TILESPMV_NO_GROUPS");
-    int32_t *buf = nullptr;
-    TSP_CK(cudaMalloc(&buf, (5 * (T + 1) + 2 * (NW + 1)) * sizeof(int32_t)));
-    int32_t *nitems = buf, *nsplit = buf + (T + 1), *parts = buf + 2 * (T + 1), *splitId = buf + 3 * (T + 1),
-            *partBase = buf + 4 * (T + 1), *wcount = buf + 5 * (T + 1), *wbase = wcount + (NW + 1);
-    int rc = 0;
-    do {
-        if (cudaMemsetAsync(buf, 0, 3 * (T + 1) * sizeof(int32_t), st) != cudaSuccess ||
-            cudaMemsetAsync(wcount, 0, (NW + 1) * sizeof(int32_t), st) != cudaSuccess) { rc = cuda_status(cudaGetLastError(), "memset"); break; }
-        k_items_count<<<blocks(T), TB, 0, st>>>(M.tilePtr, M.tileOff, M.remRowPtr, M.m, M.item_bytes, T, nitems, nsplit, parts);
-        k_window_count<<<blocks(NW), TB, 0, st>>>(M.tilePtr, M.tileOff, M.remRowPtr, M.m, M.item_bytes, T, group, nitems,
-                                                   NW, wcount);
-        if ((rc = scan([&](void *t, size_t &b) { return cub::DeviceScan::ExclusiveSum(t, b, wcount, wbase, (int)(NW + 1), st); }))) break;
-        if ((rc = scan([&](void *t, size_t &b) { return cub::DeviceScan::ExclusiveSum(t, b, nsplit, splitId, (int)(T + 1), st); }))) break;
-        if ((rc = scan([&](void *t, size_t &b) { return cub::DeviceScan::ExclusiveSum(t, b, parts, partBase, (int)(T + 1), st); }))) break;
-        int32_t h[3];
-        cudaMemcpyAsync(&h[0], wbase + NW, 4, cudaMemcpyDeviceToHost, st);
-        cudaMemcpyAsync(&h[1], splitId + T, 4, cudaMemcpyDeviceToHost, st);
-        cudaMemcpyAsync(&h[2], partBase + T, 4, cudaMemcpyDeviceToHost, st);
-        if (cudaStreamSynchronize(st) != cudaSuccess) { rc = cuda_status(cudaGetLastError(), "schedule sizes"); break; }
-        M.num_items = h[0];
-        M.num_split = h[1];
-        const int64_t nparts = h[2];
-        if (cudaMalloc(&M.items, std::max<int64_t>(M.num_items, 1) * sizeof(Item)) != cudaSuccess ||
-            cudaMalloc(&M.split_info, std::max<int64_t>(M.num_split, 1) * sizeof(int2)) != cudaSuccess ||
-            cudaMalloc(&M.counters, std::max<int64_t>(M.num_split, 1) * sizeof(int32_t)) != cudaSuccess ||
-            cudaMalloc(&M.partials, std::max<int64_t>(nparts, 1) * 16 * sizeof(double)) != cudaSuccess) {
-            rc = cuda_status(cudaGetLastError(), "cudaMalloc(schedule)");
-            break;
-        }
-        M.device_bytes += M.num_items * (int64_t)sizeof(Item) + M.num_split * 12 + nparts * 128;
-        // whole records (padding included) are copied later: start from zeros
-        cudaMemsetAsync(M.items, 0, std::max<int64_t>(M.num_items, 1) * sizeof(Item), st);
-        cudaMemsetAsync(M.counters, 0, std::max<int64_t>(M.num_split, 1) * sizeof(int32_t), st);
-        k_window_write<<<blocks(NW), TB, 0, st>>>(M.tilePtr, M.tileOff, M.remRowPtr, M.m, M.item_bytes, T, group, nitems,
-                                                   NW, wbase, splitId, partBase, M.items, M.split_info, M.local_parts);
-        if (cudaStreamSynchronize(st) != cudaSuccess) rc = cuda_status(cudaGetLastError(), "k_window_write");
-    } while (0);
-    cudaFree(buf);
-    return rc;
+    const int group = 1;  // both kernels run row-group items (compute_item)
+    Tmp buf(st);
+    if (int rc = buf.alloc((5 * (T + 1) + 2 * (NW + 1)) * sizeof(int32_t))) return rc;
+    int32_t *nitems = buf.as<int32_t>(), *nsplit = nitems + (T + 1), *parts = nitems + 2 * (T + 1),
+            *splitId = nitems + 3 * (T + 1), *partBase = nitems + 4 * (T + 1), *wcount = nitems + 5 * (T + 1),
+            *wbase = wcount + (NW + 1);
+    TSP_CK(cudaMemsetAsync(nitems, 0, 3 * (T + 1) * sizeof(int32_t), st));
+    TSP_CK(cudaMemsetAsync(wcount, 0, (NW + 1) * sizeof(int32_t), st));
+    k_items_count<<<blocks(T), TB, 0, st>>>(M.tilePtr, M.tileOff, M.remRowPtr, M.m, M.item_bytes, T, nitems, nsplit, parts);
+    k_window_count<<<blocks(NW), TB, 0, st>>>(M.tilePtr, M.tileOff, M.remRowPtr, M.m, M.item_bytes, T, group, nitems,
+                                               NW, wcount);
+    TSP_CK(cudaGetLastError());
+    if (int rc = scan([&](void *t, size_t &b) { return cub::DeviceScan::ExclusiveSum(t, b, wcount, wbase, (int)(NW + 1), st); }, st)) return rc;
+    if (int rc = scan([&](void *t, size_t &b) { return cub::DeviceScan::ExclusiveSum(t, b, nsplit, splitId, (int)(T + 1), st); }, st)) return rc;
+    if (int rc = scan([&](void *t, size_t &b) { return cub::DeviceScan::ExclusiveSum(t, b, parts, partBase, (int)(T + 1), st); }, st)) return rc;
+    int32_t h[3];
+    TSP_CK(cudaMemcpyAsync(&h[0], wbase + NW, 4, cudaMemcpyDeviceToHost, st));
+    TSP_CK(cudaMemcpyAsync(&h[1], splitId + T, 4, cudaMemcpyDeviceToHost, st));
+    TSP_CK(cudaMemcpyAsync(&h[2], partBase + T, 4, cudaMemcpyDeviceToHost, st));
+    TSP_CK(cudaStreamSynchronize(st));
+    M.num_items = h[0];
+    M.num_split = h[1];
+    const int64_t nparts = h[2];
+    TSP_CK(cudaMalloc(&M.items, std::max<int64_t>(M.num_items, 1) * sizeof(Item)));
+    TSP_CK(cudaMalloc(&M.split_info, std::max<int64_t>(M.num_split, 1) * sizeof(int2)));
+    TSP_CK(cudaMalloc(&M.counters, std::max<int64_t>(M.num_split, 1) * sizeof(int32_t)));
+    TSP_CK(cudaMalloc(&M.partials, std::max<int64_t>(nparts, 1) * 16 * sizeof(double)));
+    M.device_bytes += M.num_split * 12 + nparts * 128;
+    // whole records (padding included) are copied later: start from zeros
+    TSP_CK(cudaMemsetAsync(M.items, 0, std::max<int64_t>(M.num_items, 1) * sizeof(Item), st));
+    TSP_CK(cudaMemsetAsync(M.counters, 0, std::max<int64_t>(M.num_split, 1) * sizeof(int32_t), st));
+    k_window_write<<<blocks(NW), TB, 0, st>>>(M.tilePtr, M.tileOff, M.remRowPtr, M.m, M.item_bytes, T, group, nitems,
+                                               NW, wbase, splitId, partBase, M.items, M.split_info, kLocalParts);
+    TSP_CK(cudaGetLastError());
+    return 0;
 }
 
 int build_tdesc(Matrix &M, cudaStream_t st) {
     const int64_t n = M.num_items;
     if (n == 0) {
-        TSP_CK(cudaMalloc(&M.tdesc, 4 * sizeof(uint2)));
         TSP_CK(cudaMalloc(&M.blob, 256));
         TSP_CK(cudaMalloc(&M.witems, sizeof(WItem)));
         TSP_CK(cudaMalloc(&M.jcols, 16 * sizeof(int32_t)));
+        M.device_bytes += 256 + sizeof(WItem) + 64;
         return 0;
     }
-    int32_t *cnt = nullptr;
-    TSP_CK(cudaMalloc(&cnt, 2 * (n + 1) * sizeof(int32_t)));
-    int32_t *beg = cnt + (n + 1);
+    Tmp cntb(st);
+    if (int rc = cntb.alloc(2 * (n + 1) * sizeof(int32_t))) return rc;
+    int32_t *cnt = cntb.as<int32_t>(), *beg = cnt + (n + 1);
     const unsigned nb = (unsigned)((n + 255) / 256);
-    int rc = 0;
-    do {
-        if (cudaMemsetAsync(cnt + n, 0, sizeof(int32_t), st) != cudaSuccess) { rc = cuda_status(cudaGetLastError(), "memset"); break; }
-        k_dsc_count<<<nb, 256, 0, st>>>(M.items, n, M.tileFmt, cnt);
-        if ((rc = scan([&](void *t, size_t &b) { return cub::DeviceScan::ExclusiveSum(t, b, cnt, beg, (int)(n + 1), st); }))) break;
-        int32_t total = 0;
-        cudaMemcpyAsync(&total, beg + n, 4, cudaMemcpyDeviceToHost, st);
-        if (cudaStreamSynchronize(st) != cudaSuccess) { rc = cuda_status(cudaGetLastError(), "dsc sizes"); break; }
-        M.num_dsc = total;
-        if (cudaMalloc(&M.tdesc, (total + 4) * sizeof(uint2)) != cudaSuccess) { rc = cuda_status(cudaGetLastError(), "cudaMalloc(dlist)"); break; }
-        M.device_bytes += (total + 4) * 8;
-        k_dsc_write<<<nb, 256, 0, st>>>(M.items, n, beg, cnt, M.tileColIdx, M.tileFmt, M.tileAux, M.tileNnz, M.tileOff,
-                                         M.tdesc);
-        if (cudaStreamSynchronize(st) != cudaSuccess) { rc = cuda_status(cudaGetLastError(), "k_dsc_write"); break; }
-        // execution blobs
-        int64_t *len16 = nullptr;
-        if (cudaMalloc(&len16, 2 * (n + 1) * sizeof(int64_t)) != cudaSuccess) { rc = cuda_status(cudaGetLastError(), "cudaMalloc(blob sizes)"); break; }
-        int64_t *start16 = len16 + (n + 1);
-        cudaMemsetAsync(len16 + n, 0, sizeof(int64_t), st);
-        cudaMemsetAsync(cnt + n, 0, sizeof(int32_t), st);  // cnt[n]: slot overflow flag
-        k_blob_len<<<nb, 256, 0, st>>>(M.items, n, M.m, (uint32_t)choose(M.kernel_version).slot_bytes, len16, cnt + n);
-        if ((rc = scan([&](void *t, size_t &b) { return cub::DeviceScan::ExclusiveSum(t, b, len16, start16, (int)(n + 1), st); }))) { cudaFree(len16); break; }
-        int64_t total16 = 0;
-        int32_t over = 0;
-        cudaMemcpyAsync(&total16, start16 + n, 8, cudaMemcpyDeviceToHost, st);
-        cudaMemcpyAsync(&over, cnt + n, 4, cudaMemcpyDeviceToHost, st);
-        if (cudaStreamSynchronize(st) != cudaSuccess) { rc = cuda_status(cudaGetLastError(), "blob size"); cudaFree(len16); break; }
-        if (over) { rc = set_error(TILESPMV_CUDA, "schedule: an item's blob exceeds the kernel's slot"); cudaFree(len16); break; }
-        if (total16 >= (int64_t(1) << 32)) { rc = set_error(TILESPMV_OVERFLOW, "execution blob >= 64 GiB"); cudaFree(len16); break; }
-        M.blob_bytes = total16 * 16;
-        if (cudaMalloc(&M.blob, M.blob_bytes + 256) != cudaSuccess) { rc = cuda_status(cudaGetLastError(), "cudaMalloc(blob)"); cudaFree(len16); break; }
-        M.device_bytes += M.blob_bytes + 256;
-        if (cudaMalloc(&M.witems, n * sizeof(WItem)) != cudaSuccess ||
-            cudaMalloc(&M.jcols, n * 16 * sizeof(int32_t)) != cudaSuccess) {
-            rc = cuda_status(cudaGetLastError(), "cudaMalloc(witems)");
-            cudaFree(len16);
-            break;
-        }
-        M.device_bytes += n * (int64_t)(sizeof(WItem) + 64);
-        k_blob_fill<<<(unsigned)((n * 32 + 255) / 256), 256, 0, st>>>(M.items, n, M.m, M.n, start16, M.tdesc, M.tileColIdx,
-                                                                     M.tileFmt, M.payload, M.remRowPtr, M.remCol,
-                                                                     M.remVal, M.blob, M.witems, M.jcols);
-        if (cudaStreamSynchronize(st) != cudaSuccess) rc = cuda_status(cudaGetLastError(), "k_blob_fill");
-        cudaFree(len16);
-    } while (0);
-    cudaFree(cnt);
-    return rc;
+    TSP_CK(cudaMemsetAsync(cnt + n, 0, sizeof(int32_t), st));
+    k_dsc_count<<<nb, 256, 0, st>>>(M.items, n, M.tileFmt, cnt);
+    if (int rc = scan([&](void *t, size_t &b) { return cub::DeviceScan::ExclusiveSum(t, b, cnt, beg, (int)(n + 1), st); }, st)) return rc;
+    int32_t total = 0;
+    TSP_CK(cudaMemcpyAsync(&total, beg + n, 4, cudaMemcpyDeviceToHost, st));
+    TSP_CK(cudaStreamSynchronize(st));
+    M.num_dsc = total;
+    TSP_CK(cudaMallocAsync(&M.tdesc, (total + 4) * sizeof(uint2), st));  // create-time only
+    k_dsc_write<<<nb, 256, 0, st>>>(M.items, n, beg, cnt, M.tileColIdx, M.tileFmt, M.tileAux, M.tileNnz, M.tileOff,
+                                     M.tdesc);
+    TSP_CK(cudaGetLastError());
+    // execution blobs
+    Tmp lenb(st);
+    if (int rc = lenb.alloc(2 * (n + 1) * sizeof(int64_t))) return rc;
+    int64_t *len16 = lenb.as<int64_t>(), *start16 = len16 + (n + 1);
+    TSP_CK(cudaMemsetAsync(len16 + n, 0, sizeof(int64_t), st));
+    TSP_CK(cudaMemsetAsync(cnt + n, 0, sizeof(int32_t), st));  // cnt[n]: slot overflow flag
+    k_blob_len<<<nb, 256, 0, st>>>(M.items, n, M.m, (uint32_t)M.item_bytes, len16, cnt + n);
+    if (int rc = scan([&](void *t, size_t &b) { return cub::DeviceScan::ExclusiveSum(t, b, len16, start16, (int)(n + 1), st); }, st)) return rc;
+    int64_t total16 = 0;
+    int32_t over = 0;
+    TSP_CK(cudaMemcpyAsync(&total16, start16 + n, 8, cudaMemcpyDeviceToHost, st));
+    TSP_CK(cudaMemcpyAsync(&over, cnt + n, 4, cudaMemcpyDeviceToHost, st));
+    TSP_CK(cudaStreamSynchronize(st));
+    if (over) return set_error(TILESPMV_CUDA, "schedule: an item's blob exceeds the kernel's slot");
+    if (total16 >= (int64_t(1) << 32)) return set_error(TILESPMV_OVERFLOW, "execution blob >= 64 GiB");
+    M.blob_bytes = total16 * 16;
+    TSP_CK(cudaMalloc(&M.blob, M.blob_bytes + 256));
+    M.device_bytes += M.blob_bytes + 256;
+    TSP_CK(cudaMalloc(&M.witems, n * sizeof(WItem)));
+    TSP_CK(cudaMalloc(&M.jcols, n * 16 * sizeof(int32_t)));
+    M.device_bytes += n * (int64_t)(sizeof(WItem) + 64);
+    k_blob_fill<<<(unsigned)((n * 32 + 255) / 256), 256, 0, st>>>(M.items, n, M.m, M.n, start16, M.tdesc, M.tileColIdx,
+                                                                 M.tileFmt, M.payload, M.remRowPtr, M.remCol,
+                                                                 M.remVal, M.blob, M.witems, M.jcols);
+    TSP_CK(cudaGetLastError());
+    return 0;
 }
 
-int choose_kernel(Matrix &M) {
-    // default: the SM-queue kernel (one CTA of 32 warps per SM, 4.5 KB slots,
+int auto_kernel(int64_t payload_bytes, int64_t tilem) {
+    // integer form of "mean payload per tile row > 6 KiB"
+    return tilem > 0 && payload_bytes > 6144 * tilem ? TILESPMV_KERNEL_DENSE_ROWS : TILESPMV_KERNEL_SM_QUEUE;
+}
+
+int choose_kernel(Matrix &M, int requested) {
+    // AUTO: the SM-queue kernel (one CTA of 32 warps per SM, 4.5 KB slots,
     // warps claim units from a shared-memory counter); matrices whose tile
-    // rows average more than 6 KB of payload (dense, FEM-like) use the warp
-    // kernel with 10.5 KB slots (16 warps/SM) so a tile row stays one item.
-    // The SM-queue kernel runs CSR and ELL tiles with the pair extent known
-    // (variant 43, descriptor bits 20-24): C5 -9%, mixed -8% against 40.
-    // Measured (graph-replayed launches, profiles/): C5 498 us (sm<32,4608>)
-    // vs 512 us (warp<8,4608>); R-MAT 145 vs 163 us; mixed 113 vs 116 us;
-    // C2 6.9 us for warp<4,10752> vs 7.5 us for sm<16,10752>.
-    const double row_bytes = M.tilem ? (double)M.payload_bytes / (double)M.tilem : 0.0;
-    int version = row_bytes > 6144.0 ? 25 : 43;
-    if (const char *e = getenv("TILESPMV_KERNEL")) version = atoi(e);
-    if (const char *e = getenv("TILESPMV_LOCAL_PARTS")) M.local_parts = std::max(1, atoi(e));
-    M.kernel_version = version;
-    M.item_bytes = choose(version).slot_bytes;
+    // rows average more than 6 KB of payload (dense, FEM-like) use the
+    // dense-row kernel with 10.5 KB slots (16 warps/SM) so a tile row stays
+    // one item.  Measured in round 1 (graph-replayed launches, profiles/):
+    // C5 498 us (SM queue) vs 512 us (static chunks); R-MAT 145 vs 163 us;
+    // mixed 113 vs 116 us; C2 6.9 us (dense-row) vs 7.5 us (SM queue, 10.5 KB).
+    const int k = requested == TILESPMV_KERNEL_AUTO ? auto_kernel(M.payload_bytes, M.tilem) : requested;
+    M.kernel = k;
+    M.item_bytes = kernel_choice(k).slot_bytes;
     return 0;
 }
 
 // SM-queue kernel: units (items, or whole groups of parts) and a
 // contiguous, cost-balanced unit range per CTA
-static int configure_sm_queue(Matrix &M, int G) {
+static int configure_sm_queue(Matrix &M, int G, cudaStream_t st) {
     M.grid = G;
     const int64_t n = M.num_items;
-    if (M.cta_begin) cudaFree(M.cta_begin);
-    if (M.units) cudaFree(M.units);
-    M.cta_begin = nullptr;
-    M.units = nullptr;
     TSP_CK(cudaMalloc(&M.cta_begin, (G + 1) * sizeof(int64_t)));
     TSP_CK(cudaMalloc(&M.units, (n + 1) * sizeof(int32_t)));
     M.device_bytes += (G + 1) * 8 + (n + 1) * 4;
     if (n == 0) {
-        TSP_CK(cudaMemset(M.cta_begin, 0, (G + 1) * sizeof(int64_t)));
-        TSP_CK(cudaMemset(M.units, 0, sizeof(int32_t)));
+        TSP_CK(cudaMemsetAsync(M.cta_begin, 0, (G + 1) * sizeof(int64_t), st));
+        TSP_CK(cudaMemsetAsync(M.units, 0, sizeof(int32_t), st));
         M.num_units = 0;
         return 0;
     }
-    int64_t *cost = nullptr;
-    int32_t *flag = nullptr;
-    TSP_CK(cudaMalloc(&cost, 2 * n * sizeof(int64_t)));
-    if (cudaMalloc(&flag, 2 * (n + 1) * sizeof(int32_t)) != cudaSuccess) {
-        cudaFree(cost);
-        return cuda_status(cudaGetLastError(), "cudaMalloc(unit flags)");
-    }
-    int32_t *pos = flag + (n + 1);
-    int64_t *incl = cost + n;
-    int rc = 0;
-    do {
-        int64_t fixed = kItemFixedCost;
-        if (const char *e = getenv("TILESPMV_ITEM_COST")) fixed = atoll(e);
-        const unsigned nb = (unsigned)((n + 1 + 255) / 256);
-        k_item_cost<<<nb, 256>>>(M.items, n, M.m, fixed, cost);
-        if ((rc = scan([&](void *t, size_t &b) { return cub::DeviceScan::InclusiveSum(t, b, cost, incl, (int)n); }))) break;
-        cudaMemset(flag + n, 0, sizeof(int32_t));
-        k_unit_flags<<<nb, 256>>>(M.items, n, M.local_parts, flag);
-        if ((rc = scan([&](void *t, size_t &b) { return cub::DeviceScan::ExclusiveSum(t, b, flag, pos, (int)(n + 1)); }))) break;
-        int32_t nu = 0;
-        cudaMemcpy(&nu, pos + n, 4, cudaMemcpyDeviceToHost);
-        M.num_units = nu;
-        k_unit_write<<<nb, 256>>>(flag, pos, n, M.units);
-        k_cta_units<<<(G + 1 + 255) / 256, 256>>>(incl, M.units, nu, n, G, M.cta_begin);
-        cudaError_t e = cudaDeviceSynchronize();
-        if (e != cudaSuccess) rc = cuda_status(e, "k_cta_units");
-    } while (0);
-    cudaFree(cost);
-    cudaFree(flag);
-    return rc;
+    Tmp costb(st), flagb(st);
+    if (int rc = costb.alloc(2 * n * sizeof(int64_t))) return rc;
+    if (int rc = flagb.alloc(2 * (n + 1) * sizeof(int32_t))) return rc;
+    int64_t *cost = costb.as<int64_t>(), *incl = cost + n;
+    int32_t *flag = flagb.as<int32_t>(), *pos = flag + (n + 1);
+    const unsigned nb = (unsigned)((n + 1 + 255) / 256);
+    k_item_cost<<<nb, 256, 0, st>>>(M.items, n, M.m, kItemFixedCost, cost);
+    if (int rc = scan([&](void *t, size_t &b) { return cub::DeviceScan::InclusiveSum(t, b, cost, incl, (int)n, st); }, st)) return rc;
+    TSP_CK(cudaMemsetAsync(flag + n, 0, sizeof(int32_t), st));
+    k_unit_flags<<<nb, 256, 0, st>>>(M.items, n, kLocalParts, flag);
+    if (int rc = scan([&](void *t, size_t &b) { return cub::DeviceScan::ExclusiveSum(t, b, flag, pos, (int)(n + 1), st); }, st)) return rc;
+    int32_t nu = 0;
+    TSP_CK(cudaMemcpyAsync(&nu, pos + n, 4, cudaMemcpyDeviceToHost, st));
+    TSP_CK(cudaStreamSynchronize(st));
+    M.num_units = nu;
+    k_unit_write<<<nb, 256, 0, st>>>(flag, pos, n, M.units);
+    k_cta_units<<<(G + 1 + 255) / 256, 256, 0, st>>>(incl, M.units, nu, n, G, M.cta_begin);
+    TSP_CK(cudaGetLastError());
+    return 0;
 }
 
-int configure_launch(Matrix &M) {
-    const int version = M.kernel_version;
-    const KernelChoice kc = choose(version);
+int configure_launch(Matrix &M, cudaStream_t st) {
+    const KernelChoice kc = kernel_choice(M.kernel);
     TSP_CK(cudaFuncSetAttribute(kc.fn, cudaFuncAttributeMaxDynamicSharedMemorySize, kc.smem));
     int sms = 0, per_sm = 0;
     TSP_CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, M.device));
@@ -624,65 +605,72 @@ int configure_launch(Matrix &M) {
     M.kernel_name = kc.name;
     M.block = kc.threads;
     M.smem = kc.smem;
-    if (kc.ring) return set_error(TILESPMV_CUDA, "no ring kernel in this build");
+    if (kc.sm_queue) return configure_sm_queue(M, sms * per_sm, st);
+    // dense-row kernel: persistent grid, one contiguous, cost-balanced,
+    // row-aligned item chunk per warp
     const int64_t warps = kc.threads / 32;
-    if (version == 1) {  // v1: grid-stride over items
-        const int64_t need = (M.num_items + warps - 1) / warps;
-        M.grid = (int)std::max<int64_t>(1, std::min<int64_t>(need, (int64_t)sms * per_sm));
-        return 0;
-    }
-    if (kc.sm_queue) return configure_sm_queue(M, sms * per_sm);
-    // warp kernel: persistent grid, one contiguous, cost-balanced, row-aligned
-    // item chunk per warp
     const int64_t need = (M.num_items + warps - 1) / warps;
     M.grid = (int)std::max<int64_t>(1, std::min<int64_t>(need, (int64_t)sms * per_sm));
     const int W = (int)(M.grid * warps);
-    if (M.cta_begin) cudaFree(M.cta_begin);
-    M.cta_begin = nullptr;
     TSP_CK(cudaMalloc(&M.cta_begin, (W + 1) * sizeof(int64_t)));
     M.device_bytes += (W + 1) * 8;
     if (M.num_items > 0) {
-        int64_t *cost = nullptr;
-        TSP_CK(cudaMalloc(&cost, 2 * M.num_items * sizeof(int64_t)));
-        int64_t *incl = cost + M.num_items;
-        // TILESPMV_ITEM_COST overrides the per-item fixed cost for sweeps
-        int64_t fixed = kItemFixedCost;
-        if (const char *e = getenv("TILESPMV_ITEM_COST")) fixed = atoll(e);
-        k_item_cost<<<(unsigned)((M.num_items + 255) / 256), 256>>>(M.items, M.num_items, M.m, fixed, cost);
-        int rc = scan([&](void *t, size_t &b) { return cub::DeviceScan::InclusiveSum(t, b, cost, incl, (int)M.num_items); });
-        if (!rc) {
-            k_cta_begin<<<(W + 1 + 255) / 256, 256>>>(incl, M.items, M.num_items, W, M.local_parts, M.cta_begin);
-            cudaError_t e = cudaDeviceSynchronize();
-            if (e != cudaSuccess) rc = cuda_status(e, "k_cta_begin");
-        }
-        cudaFree(cost);
-        if (rc) return rc;
+        Tmp costb(st);
+        if (int rc = costb.alloc(2 * M.num_items * sizeof(int64_t))) return rc;
+        int64_t *cost = costb.as<int64_t>(), *incl = cost + M.num_items;
+        k_item_cost<<<(unsigned)((M.num_items + 255) / 256), 256, 0, st>>>(M.items, M.num_items, M.m, kItemFixedCost,
+                                                                         cost);
+        if (int rc = scan([&](void *t, size_t &b) { return cub::DeviceScan::InclusiveSum(t, b, cost, incl, (int)M.num_items, st); }, st))
+            return rc;
+        k_cta_begin<<<(W + 1 + 255) / 256, 256, 0, st>>>(incl, M.items, M.num_items, W, kLocalParts, M.cta_begin);
+        TSP_CK(cudaGetLastError());
     } else {
-        TSP_CK(cudaMemset(M.cta_begin, 0, (W + 1) * sizeof(int64_t)));
+        TSP_CK(cudaMemsetAsync(M.cta_begin, 0, (W + 1) * sizeof(int64_t), st));
     }
-    if (M.wfirst) cudaFree(M.wfirst);
-    M.wfirst = nullptr;
     TSP_CK(cudaMalloc(&M.wfirst, W * sizeof(WFirst)));
     M.device_bytes += W * (int64_t)sizeof(WFirst);
-    k_warp_first<<<(W + 255) / 256, 256>>>(M.cta_begin, M.witems, M.jcols, W, M.wfirst);
-    TSP_CK(cudaDeviceSynchronize());
+    k_warp_first<<<(W + 255) / 256, 256, 0, st>>>(M.cta_begin, M.witems, M.jcols, W, M.wfirst);
+    TSP_CK(cudaGetLastError());
     return 0;
+}
+
+// After the schedule is built: free what only create needed (items, the
+// descriptor lists) and, unless the caller asked to keep the canonical
+// layout (tilespmv_export), the canonical level-1/level-2 arrays and the
+// remainder CSR, which the kernels never read (they read the blobs).
+void release_create_time(Matrix &M, cudaStream_t st) {
+    auto drop = [&](auto *&p) {
+        if (p) cudaFreeAsync(p, st);
+        p = nullptr;
+    };
+    drop(M.items);
+    drop(M.tdesc);
+    if (M.keep_layout) {
+        M.device_bytes += (M.tilem + 1) * 4 + M.numtile * 14 + 8 + M.payload_bytes + 64;
+        if (M.rem_nnz > 0) M.device_bytes += (M.m + 1 + 8) * 4 + (M.rem_nnz + 4) * 4 + (M.rem_nnz + 2) * 8;
+        return;
+    }
+    drop(M.tilePtr);
+    drop(M.tileColIdx);
+    drop(M.tileNnz);
+    drop(M.tileFmt);
+    drop(M.tileAux);
+    drop(M.tileOff);
+    drop(M.payload);
+    drop(M.remRowPtr);
+    drop(M.remCol);
+    drop(M.remVal);
 }
 
 int launch_spmv(const Matrix &M, const double *d_x, double *d_y, cudaStream_t st) {
     if (M.m == 0) return 0;
     Params p;
-    p.items = M.items;
-    p.num_items = M.num_items;
-    p.tileColIdx = M.tileColIdx;
-    p.tileFmt = M.tileFmt;
-    p.tileAux = M.tileAux;
-    p.tileNnz = M.tileNnz;
-    p.tileOff = M.tileOff;
-    p.payload = M.payload;
-    p.remRowPtr = M.remRowPtr;
-    p.remCol = M.remCol;
-    p.remVal = M.remVal;
+    p.blob = M.blob;
+    p.witems = M.witems;
+    p.jcols = M.jcols;
+    p.wfirst = M.wfirst;
+    p.cta_begin = M.cta_begin;
+    p.units = M.units;
     p.split_info = M.split_info;
     p.partials = M.partials;
     p.counters = M.counters;
@@ -690,26 +678,20 @@ int launch_spmv(const Matrix &M, const double *d_x, double *d_y, cudaStream_t st
     p.y = d_y;
     p.m = M.m;
     p.n = M.n;
-    p.tdesc = M.tdesc;
-    p.blob = M.blob;
-    p.witems = M.witems;
-    p.jcols = M.jcols;
-    p.wfirst = M.wfirst;
-    p.cta_begin = M.cta_begin;
     p.x_vec = (reinterpret_cast<uintptr_t>(d_x) & 15u) == 0;
-    p.units = M.units;
-    p.local_parts = M.local_parts;
-    const KernelChoice kc = choose(M.kernel_version);
+    const KernelChoice kc = kernel_choice(M.kernel);
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3(M.grid);
     cfg.blockDim = dim3(M.block);
     cfg.dynamicSmemBytes = M.smem;
     cfg.stream = st;
+    // programmatic dependent launch: the kernel waits (griddepcontrol.wait)
+    // before its first read of x or write of y
     cudaLaunchAttribute attr[1];
     attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
     attr[0].val.programmaticStreamSerializationAllowed = 1;
     cfg.attrs = attr;
-    cfg.numAttrs = kc.pdl ? 1 : 0;
+    cfg.numAttrs = 1;
     TSP_CK(cudaLaunchKernelEx(&cfg, kc.fn, p));
     return 0;
 }

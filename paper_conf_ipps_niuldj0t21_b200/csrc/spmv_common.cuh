@@ -1,5 +1,5 @@
-// spmv_common.cuh -- pieces shared by the SpMV kernels (spmv_v1.cu,
-// spmv_warp.cu) and the schedule builder (schedule.cu).
+// spmv_common.cuh -- pieces shared by the SpMV kernels (spmv_warp.cu) and
+// the schedule builder (schedule.cu).
 #pragma once
 
 #include "internal.cuh"
@@ -8,34 +8,23 @@ namespace tsp {
 
 constexpr unsigned FULL = 0xffffffffu;
 
-// Everything a launch reads; passed by value in constant memory.
+// Everything a launch reads; passed by value in constant memory.  The
+// kernels read only the schedule's execution records (schedule.cu), never the
+// canonical level-1/level-2 arrays, which the handle may free after create.
 struct Params {
-    const Item *items;
-    int64_t num_items;
-    const int32_t *tileColIdx;
-    const uint8_t *tileFmt;
-    const uint8_t *tileAux;
-    const int32_t *tileNnz;
-    const uint32_t *tileOff;
-    const uint8_t *payload;
-    const int32_t *remRowPtr;
-    const int32_t *remCol;
-    const double *remVal;
-    const int2 *split_info;
+    const uint8_t *blob;       // per-item execution blobs (blob_parts)
+    const WItem *witems;       // compact per-item records
+    const int32_t *jcols;      // tile column J of each item's tiles, 16 per item
+    const WFirst *wfirst;      // warp kernel: per-warp chunk and first item
+    const int64_t *cta_begin;  // SM-queue kernel: unit range of each CTA
+    const int32_t *units;      // SM-queue kernel: first item of each unit (+ end)
+    const int2 *split_info;    // split tile rows: {first partial slot, parts}
     double *partials;
     int32_t *counters;
     const double *x;
     double *y;
     int64_t m, n;
-    const uint2 *tdesc;        // per-item tile-descriptor lists (schedule.cu)
-    const uint8_t *blob;       // per-item execution blobs (schedule.cu)
-    const WItem *witems;       // compact per-item records (schedule.cu)
-    const int32_t *jcols;      // tile column J of each item's tiles, 16 per item
-    const WFirst *wfirst;      // per-warp chunk and first item (warp kernel)
-    const int64_t *cta_begin;  // warp kernel: item chunk of each warp
     int x_vec;                 // x is 16-byte aligned: x segments load as double2
-    const int32_t *units;      // SM-queue kernel: first item of each unit (+ end), see schedule.cu
-    int local_parts;           // parts per group of a split tile row (Matrix::local_parts)
 };
 
 // ------------------------------------------------------------------ PTX ----
@@ -54,16 +43,6 @@ __device__ __forceinline__ void fence_proxy_async() {
 __device__ __forceinline__ void mbar_expect_tx(uint32_t bar, uint32_t bytes) {
     asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes)
                  : "memory");
-}
-__device__ __forceinline__ void mbar_arrive(uint32_t bar) {
-    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(bar) : "memory");
-}
-// 1-D TMA: global -> shared, completion counted on an mbarrier (bytes % 16 == 0)
-__device__ __forceinline__ void bulk_g2s(uint32_t dst, const void *src, uint32_t bytes, uint32_t bar) {
-    asm volatile(
-        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(dst),
-        "l"(src), "r"(bytes), "r"(bar)
-        : "memory");
 }
 __device__ __forceinline__ bool mbar_try_wait(uint32_t bar, uint32_t parity) {
     uint32_t ok;
@@ -84,42 +63,9 @@ __device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
 __host__ __device__ __forceinline__ int64_t imin64(int64_t a, int64_t b) { return a < b ? a : b; }
 __host__ __device__ __forceinline__ uint32_t up16(uint32_t v) { return (v + 15u) & ~15u; }
 
-__device__ __forceinline__ int nib(const uint8_t *base, int idx) {
-    return (base[idx >> 1] >> ((idx & 1) * 4)) & 15;
-}
-
-// ------------------------------------------------- one item's staged bytes --
-// payload | tile descriptors | remRowPtr[16I..16I+rows] | remCol[kb..ke) | remVal[kb..ke)
-// Each part is 16-byte aligned in shared memory; the unaligned arrays are
-// copied as their enclosing 16-byte-aligned superset ("skew" = offset of the
-// first wanted byte inside it).
-struct ItemParts {
-    uint32_t pay, dsc, rp, col, val, total;
-    uint32_t dsc_skew, col_skew, val_skew;
-};
-
 // rows the item's remainder row pointers cover
 __host__ __device__ __forceinline__ int64_t item_rows(const Item &it, int64_t m) {
     return imin64(it.ntr > 0 ? 16 * (int64_t)it.ntr : 16, m - 16 * (int64_t)it.I);
-}
-
-__host__ __device__ __forceinline__ ItemParts item_parts(const Item &it, int64_t m) {
-    ItemParts r;
-    r.pay = (it.offe - it.offb) * 16u;
-    r.dsc_skew = (uint32_t)(it.dbeg & 1) * 8u;
-    r.dsc = it.ndsc ? up16(r.dsc_skew + 8u * (uint32_t)it.ndsc) : 0u;
-    if (it.ke > it.kb) {
-        const int64_t rows = item_rows(it, m);
-        r.rp = up16((uint32_t)(rows + 1) * 4u);
-        r.col_skew = ((uint32_t)it.kb * 4u) & 15u;
-        r.col = up16(r.col_skew + 4u * (uint32_t)(it.ke - it.kb));
-        r.val_skew = ((uint32_t)it.kb * 8u) & 15u;
-        r.val = up16(r.val_skew + 8u * (uint32_t)(it.ke - it.kb));
-    } else {
-        r.rp = r.col = r.val = r.col_skew = r.val_skew = 0u;
-    }
-    r.total = r.pay + r.dsc + r.rp + r.col + r.val;
-    return r;
 }
 
 // ---------------------------------------------- one item's execution blob --
@@ -174,11 +120,6 @@ __device__ __forceinline__ double ldg_hint(const double *p, uint64_t policy) {
     asm volatile("ld.global.nc.L2::cache_hint.f64 %0, [%1], %2;" : "=d"(v) : "l"(p), "l"(policy));
     return v;
 }
-__device__ __forceinline__ double2 ldg2_hint(const double *p, uint64_t policy) {
-    double2 v;
-    asm volatile("ld.global.nc.L2::cache_hint.v2.f64 {%0, %1}, [%2], %3;" : "=d"(v.x), "=d"(v.y) : "l"(p), "l"(policy));
-    return v;
-}
 __device__ __forceinline__ void sts_v2f64(uint32_t a, double2 v) {
     asm volatile("st.shared.v2.f64 [%0], {%1, %2};" ::"r"(a), "d"(v.x), "d"(v.y) : "memory");
 }
@@ -205,46 +146,15 @@ __device__ __forceinline__ void fma_if(bool pred, double a, double b, double &ac
         : "d"(a), "d"(b), "r"((unsigned)pred));
 }
 
-// ----------------------------------------------------------- y output ------
-// Lanes 0..15 hold the 16 row sums of the item.  A whole tile row writes y
-// directly (one 128-byte store); a split tile row writes its partial and the
-// last finishing part sums all parts in part order (deterministic).
-__device__ __forceinline__ void write_rows(const Params &p, const Item &item, int lane, double acc) {
-    const int64_t row = 16 * (int64_t)item.I + lane;
-    if (item.split < 0) {
-        if (lane < 16 && row < p.m) p.y[row] = acc;
-        return;
-    }
-    const int2 si = p.split_info[item.split];
-    const int part = item_part(item);
-    if (lane < 16) __stcg(p.partials + (int64_t)(si.x + part) * 16 + lane, acc);
-    __threadfence();
-    __syncwarp();
-    int old = 0;
-    if (lane == 0) old = atomicAdd(p.counters + item.split, 1);
-    old = __shfl_sync(FULL, old, 0);
-    if (old == si.y - 1) {
-        __threadfence();
-        const int r = lane & 15, hh = lane >> 4;
-        double s = 0.0;
-        for (int q = hh; q < si.y; q += 2) s += __ldcg(p.partials + (int64_t)(si.x + q) * 16 + r);
-        s += __shfl_xor_sync(FULL, s, 16);
-        if (lane < 16 && row < p.m) p.y[row] = s;
-        if (lane == 0) p.counters[item.split] = 0;  // ready for the next run
-    }
-}
-
-// kernels (spmv_v1.cu, spmv_warp.cu)
+// the two SpMV kernels (spmv_warp.cu)
 struct KernelChoice {
     const char *name;
     void (*fn)(Params);
-    int threads, smem, ctas_per_sm;
-    bool ring;       // one CTA per SM with cta_begin chunks (no current kernel)
+    int threads, smem;
     int slot_bytes;  // item budget the schedule must respect
-    bool pdl;        // launched with programmatic dependent launch (kernel waits on griddepcontrol)
     bool sm_queue;   // one CTA per SM; its warps claim units from a shared-memory counter
 };
-KernelChoice kernel_v1();
-KernelChoice kernel_warp(int variant);
+// TILESPMV_KERNEL_SM_QUEUE or TILESPMV_KERNEL_DENSE_ROWS
+KernelChoice kernel_choice(int kernel);
 
 }  // namespace tsp

@@ -107,71 +107,6 @@ __device__ __forceinline__ void csr_rot16(uint32_t RP, int beg, uint32_t V, uint
     }
 }
 
-// CSR: csrVal row-major | csrRowPtr[16] u8 | 4-bit columns (Alg. 2).
-// RP: shared address of csrRowPtr.  The 8 column nibbles from entry beg on
-// come from two 32-bit words and one funnel shift.
-__device__ __forceinline__ void half_csr(uint32_t RP, int nz, uint32_t X, int r, bool ok, double &acc) {
-    const int beg = (int)lds_u8(RP + r);
-    const int end = r < 15 ? (int)lds_u8(RP + r + 1) : nz;
-    const int len = ok ? end - beg : 0;
-    const int trips = (int)__reduce_max_sync(FULL, (unsigned)len);
-    const uint32_t V = RP + 8 * (beg - nz);
-    if ((trips >= 6 && trips <= 8) || trips >= 13) {  // long equal rows: lane-rotated
-        const uint32_t wa = RP + 16 + 4 * (beg >> 3);
-        const uint32_t u = funnel_r(lds_u32(wa), lds_u32(wa + 4), 4u * beg);
-        if (trips <= 8) csr_rot8(V, u, X, r, len, acc);
-        else csr_rot16(RP, beg, V, u, X, r, len, acc);
-        return;
-    }
-    {
-        const uint32_t wa = RP + 16 + 4 * (beg >> 3);
-        const uint32_t u = funnel_r(lds_u32(wa), lds_u32(wa + 4), 4u * beg);
-        const double x0 = lds_f64(xaddr(u << 3, X)), x1 = lds_f64(xaddr(u >> 1, X));
-        const double x2 = lds_f64(xaddr(u >> 5, X)), x3 = lds_f64(xaddr(u >> 9, X));
-        const double v0 = lds_f64_lt(0, len, V), v1 = lds_f64_lt(1, len, V + 8);
-        const double v2 = lds_f64_lt(2, len, V + 16), v3 = lds_f64_lt(3, len, V + 24);
-        acc = fma(v0, x0, acc);
-        acc = fma(v1, x1, acc);
-        acc = fma(v2, x2, acc);
-        acc = fma(v3, x3, acc);
-    }
-#pragma unroll 1
-    for (int i = 4; i < trips; i += 4) {
-        const uint32_t wa = RP + 16 + 4 * ((beg + i) >> 3);
-        const uint32_t u = funnel_r(lds_u32(wa), lds_u32(wa + 4), 4u * (beg + i));
-        const double x0 = lds_f64(xaddr(u << 3, X)), x1 = lds_f64(xaddr(u >> 1, X));
-        const double x2 = lds_f64(xaddr(u >> 5, X)), x3 = lds_f64(xaddr(u >> 9, X));
-        const double v0 = lds_f64_lt(i, len, V + 8 * i), v1 = lds_f64_lt(i + 1, len, V + 8 * i + 8);
-        const double v2 = lds_f64_lt(i + 2, len, V + 8 * i + 16), v3 = lds_f64_lt(i + 3, len, V + 8 * i + 24);
-        acc = fma(v0, x0, acc);
-        acc = fma(v1, x1, acc);
-        acc = fma(v2, x2, acc);
-        acc = fma(v3, x3, acc);
-    }
-}
-
-// ELL: slots k*16 + r column-major | 4-bit columns (Alg. 4).
-// Pads hold +0.0 at column 0 (reading R10) and are multiplied like entries:
-// +0.0 * x adds nothing (x finite, R19).
-__device__ __forceinline__ void half_ell(uint32_t P, int w, uint32_t X, int r, bool ok, double &acc) {
-    const int wq = ok ? w : 0;
-    const int trips = (int)__reduce_max_sync(FULL, (unsigned)wq);
-    const uint32_t ci = P + 128 * w + (r >> 1);
-    const uint32_t sh = 4 * (r & 1);
-    const uint32_t V = P + 8 * r;
-#pragma unroll 1
-    for (int k = 0; k < trips; k += 4) {
-        double xv[4], v[4];
-#pragma unroll
-        for (int j = 0; j < 4; ++j) {
-            xv[j] = lds_f64(X + 8 * ((lds_u8(ci + 8 * (k + j)) >> sh) & 15u));
-            v[j] = lds_f64_lt(k + j, wq, V + 128 * (k + j));
-        }
-#pragma unroll
-        for (int j = 0; j < 4; ++j) acc = fma(v[j], xv[j], acc);
-    }
-}
-
 // Dns: 256 values column-major; x[c], x[c+1] arrive as one
 // 16-byte broadcast load
 __device__ __forceinline__ void half_dns(uint32_t P, uint32_t X, int r, bool ok, double &acc) {
@@ -217,27 +152,6 @@ __device__ __forceinline__ void half_dnsrow_tree(uint32_t P, int nr, uint32_t X,
     }
 }
 
-// DnsRow: full row q (id rowid[q]) holds values q*16 + c; the
-// lane of row rowid[q] sums the 16 products of its row.
-__device__ __forceinline__ void half_dnsrow(uint32_t P, int nr, uint32_t X, int r, bool ok, double &acc) {
-    const uint32_t rid = P + 128 * nr;
-    int q_r = -1;
-    const int nq = ok ? nr : 0;
-    for (int q = 0; q < 7; ++q)
-        if (q < nq && (int)lds_u8(rid + q) == r) q_r = q;
-    const bool mine = q_r >= 0;
-    if (__any_sync(FULL, mine)) {
-        const uint32_t Vr = P + 128 * (mine ? q_r : 0);
-        double a0 = 0.0, a1 = 0.0;
-#pragma unroll
-        for (int c = 0; c < 16; c += 2) {
-            a0 = fma(lds_f64(Vr + 8 * c), lds_f64(X + 8 * c), a0);
-            a1 = fma(lds_f64(Vr + 8 * c + 8), lds_f64(X + 8 * c + 8), a1);
-        }
-        if (mine) acc += a0 + a1;
-    }
-}
-
 // COO with at most N entries per tile of the pair (tm <= N): every lane of
 // the half walks the entries, the lane of the entry's row adds it
 template <int N>
@@ -248,20 +162,6 @@ __device__ __forceinline__ void half_coo_n(uint32_t V, uint32_t rc, int n, uint3
         const uint32_t b = lds_u8(rc + j);
         const double v = lds_f64_lt(j, (int)(b >> 4) == r ? nq : 0, V + 8 * j);
         acc = fma(v, lds_f64(X + 8 * (b & 15u)), acc);
-    }
-}
-
-// COO entries: value j, packed (row << 4 | col) byte (Alg. 3); the lane
-// of the entry's row adds it (no atomics, fixed order)
-__device__ __forceinline__ void half_coo(uint32_t V, uint32_t rc, int n, uint32_t X, int r, bool ok, double &acc) {
-    const int nq = ok ? n : 0;
-    const int trips = (int)__reduce_max_sync(FULL, (unsigned)nq);
-#pragma unroll 2
-    for (int j = 0; j < trips; ++j) {
-        const uint32_t b = lds_u8(rc + j);
-        const double v = lds_f64(V + 8 * j);
-        const double xv = lds_f64(X + 8 * (b & 15u));
-        fma_if(j < nq && (int)(b >> 4) == r, v, xv, acc);
     }
 }
 
@@ -428,21 +328,6 @@ __device__ __forceinline__ void half_hyb_scan(uint32_t P, int w, int nz, uint32_
     const int passes = (int)__reduce_max_sync(FULL, (unsigned)(ok ? (kc + 15) >> 4 : 0));
 #pragma unroll 1
     for (int c = 0; c < passes; ++c) half_coo_scan(P + 128 * w, ei + 8 * w, kc, X, r, h, S, ok, acc, 16 * c);
-}
-
-// HYB: ELL(w) values | COO values | ELL 4-bit columns | COO (row<<4|col)
-__device__ __forceinline__ void half_hyb(uint32_t P, int w, int nz, uint32_t X, int r, bool ok, double &acc) {
-    const int kc = nz - 16 * w;
-    const uint32_t ei = P + 128 * w + 8 * kc;
-    const int wq = ok ? w : 0;
-    const int trips = (int)__reduce_max_sync(FULL, (unsigned)wq);
-    const uint32_t sh = 4 * (r & 1);
-    for (int k = 0; k < trips; ++k) {
-        const double v = lds_f64_lt(k, wq, P + 8 * (16 * k + r));
-        const double xv = lds_f64(X + 8 * ((lds_u8(ei + 8 * k + (r >> 1)) >> sh) & 15u));
-        acc = fma(v, xv, acc);
-    }
-    half_coo(P + 128 * w, ei + 8 * w, kc, X, r, ok, acc);
 }
 
 }  // namespace tsp

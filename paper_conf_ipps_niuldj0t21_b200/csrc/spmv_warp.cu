@@ -1,12 +1,12 @@
-// spmv_warp.cu -- the default SpMV kernel (TILESPMV_KERNEL 20-29): y =
-// A_tiles*x + A_rem*x in fp64 on sm_100a (§III.C P:118-173 warp-level
-// tile SpMV, P:199 load balancing, P:201 DeferredCOO remainder).
+// spmv_warp.cu -- the SpMV kernels: y = A_tiles*x + A_rem*x in fp64 on
+// sm_100a (§III.C P:118-173 warp-level tile SpMV, P:199 load
+// balancing, P:201 DeferredCOO remainder).
 //
-// High occupancy (32 warps/SM): every warp is its own producer and consumer.
-// Per work item, lane 0 stages the item's execution blob (descriptor list,
-// tile columns, tile payloads, remainder rowptr/col/val; blob_parts) into the
-// warp's shared-memory slot with ONE TMA bulk copy (cp.async.bulk, L2
-// evict-first) completing on the warp's mbarrier.  The warp then
+// Every warp is its own producer and consumer.  Per work item, lane 0 stages
+// the item's execution blob (descriptor list, tile payloads, remainder
+// rowptr/col/val; blob_parts) into the warp's shared-memory slot with ONE TMA
+// bulk copy (cp.async.bulk, L2 evict-first) completing on the warp's
+// mbarrier.  The warp then
 //   1. starts the x segment of every tile (one 128-byte line) with cp.async
 //      (L2 evict-last; the tail of x past n reads as 0),
 //   2. runs the fused CSR remainder rows of the tile row,
@@ -16,6 +16,13 @@
 //      of parts, one partial per group for hub rows).
 // Latency is hidden by warp count; the next item's record is prefetched into
 // registers.  No floating-point atomics: y is bitwise deterministic.
+//
+// Two kernels share this item code (schedule.cu picks one per handle):
+//   tilespmv_fp64_sm<32,4608>    one CTA of 32 warps per SM, 4.5 KB slots,
+//                                 warps claim units from a shared-memory queue
+//   tilespmv_fp64_warp<4,10752>  16 warps per SM, 10.5 KB slots, a static
+//                                 cost-balanced item chunk per warp (dense
+//                                 tile rows: one tile row stays one item)
 #include "spmv_tiles.cuh"
 
 namespace tsp {
@@ -48,14 +55,14 @@ __device__ __forceinline__ unsigned long long gtimer() {
 
 namespace {
 
-template <int WARPS, int SLOT, int NBUF = 1, int RACC = 128>
+template <int WARPS, int SLOT>
 struct WarpCfg {
     static_assert(SLOT % 16 == 0 && SLOT <= kItemBytesMax, "slot size");
-    // [x stage of every warp, 2 KB each, 128-byte aligned] [per warp: NBUF
-    // slots | row-sum scratch (RACC bytes) | mbarriers]
+    // [x stage of every warp, 2 KB each, 128-byte aligned] [per warp: slot |
+    // row-sum scratch of the COO scan (256 B) | mbarrier]
     static constexpr uint32_t kX = kItemTiles * 16 * 8;
-    static constexpr uint32_t kRacc = RACC;
-    static constexpr uint32_t kPer = NBUF * SLOT + RACC + 16;
+    static constexpr uint32_t kRacc = 256;
+    static constexpr uint32_t kPer = SLOT + kRacc + 16;
     static constexpr uint32_t kSmem = WARPS * (kX + kPer) + 256;  // +256: loads may overrun a slot
     static constexpr int kThreads = 32 * WARPS;
 };
@@ -69,126 +76,92 @@ __device__ __forceinline__ WItem load_witem(const WItem *w, int k) {
     return it;
 }
 
-// fused CSR remainder of the item's rows; adds row sums into acc of
-// lane r (and r + 16).  rpS: rebased row pointers (rows + 1), colS/valS: entries.
-//  * every row <= 4 entries (stencil-like): two lanes per row, two entries
-//    each, one round trip of gathers;
-//  * every row <= MED entries (kShortRow, or kMedRow for the TM kernels):
-//    two lanes per row, all rows at once;
-//  * a longer row (power-law hubs): the flat pass (flat_rows), each product
-//    formed where it is summed.
-// The path and the order of every sum depend only on the item's content: y
-// stays bitwise deterministic.
-__device__ __forceinline__ double flat_rows(const Params &p, uint32_t rq, uint32_t colS, uint32_t valS, int rows,
-                                            uint64_t x_policy, int lane);
-
-// product of remainder entry k (rounded on its own, as the earlier
-// shared-memory product pass stored it) if k < e, else +0.0 -- the term the row sums would have read
-__device__ __forceinline__ double rem_product(const Params &p, int k, int e, uint32_t colS, uint32_t valS,
-                                              uint64_t x_policy) {
-    int c;
-    double v;
-    lds_entry_lt(k, e, colS + 4 * k, valS + 8 * k, c, v);
-    const double pr = __dmul_rn(v, ldg_hint(p.x + (uint32_t)c, x_policy));
-    return k < e ? pr : 0.0;
+// ------------------------------------------------ fused CSR remainder -------
+// One 32-entry chunk of remainder products, p = lane's product (0.0 past the
+// end), chunk entries [base, base + 32).  Lane r < 16 owns row r with entries
+// [b, e) (live: r is a row of the item and is not empty).  An inclusive
+// segmented scan (Hillis-Steele, segments = rows, lane 0 always starts one)
+// leaves each row's sum of this chunk on its last lane, which the row's lane
+// fetches.  For a row wholly inside the chunk the tree depends only on the
+// row's length, and the chunk grid is anchored at the first entry of the
+// tile row (or of the item's part of it), so every sum order is a function
+// of the tile row's own content (shard and grouping invariant).
+__device__ __forceinline__ double chunk_piece(double p, int base, int b, int e, bool live, int lane) {
+    const int s = b - base;
+    const bool hd = live && s >= 0 && s < 32;
+    const uint32_t heads = __reduce_or_sync(FULL, hd ? 1u << s : 0u) | 1u;
+    const int seg = 31 - __clz(heads & (0xFFFFFFFFu >> (31 - lane)));  // the lane's segment head
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+        const double t = __shfl_up_sync(FULL, p, d);
+        if (lane - d >= seg) p += t;
+    }
+    const bool in = live && s < 32 && e > base;
+    const double piece = __shfl_sync(FULL, p, in ? min(e - base, 32) - 1 : lane);
+    return in ? piece : 0.0;
 }
 
-template <int MED>
-__device__ __forceinline__ void remainder(const Params &p, uint32_t rpS, uint32_t colS, uint32_t valS, int rows,
-                                          uint64_t x_policy, int lane, double &acc, bool &dirty) {
-    const int r = lane & 15, h = lane >> 4;
-    const int b = lds_s32(rpS + 4 * min(r, rows)), e = lds_s32(rpS + 4 * min(r + 1, rows));
-    const double *x = p.x;
-    const int maxlen = (int)__reduce_max_sync(FULL, (unsigned)(e - b));
-    if (maxlen <= 4) {
-        // entries b + h and b + h + 2 of row r; a masked entry reads column 0
-        // and value 0.0 (x[0] exists whenever the item has remainder entries)
-        const int k0 = b + h, k1 = k0 + 2;
-        int c0, c1;
-        double v0, v1;
-        lds_entry_lt(k0, e, colS + 4 * k0, valS + 8 * k0, c0, v0);
-        lds_entry_lt(k1, e, colS + 4 * k1, valS + 8 * k1, c1, v1);
-        const double x0 = ldg_hint(x + (uint32_t)c0, x_policy), x1 = ldg_hint(x + (uint32_t)c1, x_policy);
-        acc = fma(v0, x0, acc);
-        acc = fma(v1, x1, acc);
-        return;
-    }
-    if (maxlen > MED) {
-        dirty = true;  // the slot now holds products written by the generic proxy
-        acc += flat_rows(p, rpS, colS, valS, rows, x_policy, lane);
-        return;
-    }
-    const int trips = (int)__reduce_max_sync(FULL, (unsigned)((e - b + 1 - h) >> 1));
-#pragma unroll 1
-    for (int i = 0; i < trips; i += 2) {
-        const int k0 = b + h + 2 * i, k1 = k0 + 2;
-        int c0, c1;
-        double v0, v1;
-        lds_entry_lt(k0, e, colS + 4 * k0, valS + 8 * k0, c0, v0);
-        lds_entry_lt(k1, e, colS + 4 * k1, valS + 8 * k1, c1, v1);
-        const double x0 = ldg_hint(x + (uint32_t)c0, x_policy), x1 = ldg_hint(x + (uint32_t)c1, x_policy);
-        acc = fma(v0, x0, acc);
-        acc = fma(v1, x1, acc);
-    }
-}
-
-// Flat remainder pass for one tile row (rows <= 16, row pointers at
-// rq): rows of <= kShortRow products two lanes per row, longer rows a
-// half-warp per row (two rows at a time, the whole warp for the last one)
-// with an xor tree.  Returns lane r's (or r + 16's) share of row r.  The order
-// of every sum depends only on this tile row.
-__device__ __forceinline__ double flat_rows(const Params &p, uint32_t rq, uint32_t colS, uint32_t valS, int rows,
-                                            uint64_t x_policy, int lane) {
-    const int r = lane & 15, h = lane >> 4;
+// The remainder rows 0..rows-1 of one tile row (rq: its rebased row pointers
+// rq[0..rows] in shared memory; colS/valS: the entries), lane per entry in
+// chunks of 32 anchored at rq[0], two chunks (two x gathers) in flight.
+// Returns row r's sum in lane r < 16 (lanes >= 16: 0).  Each product is
+// rounded on its own (v * x, not fused): masked lanes contribute an exact
+// 0.0 however x[0] reads (a halo rank need not hold x[0]).
+__device__ __forceinline__ double rem_chunks(const Params &p, uint32_t rq, int rows, uint32_t colS, uint32_t valS,
+                                             uint64_t x_policy, int lane) {
+    const int r = lane & 15;
     const int b = lds_s32(rq + 4 * min(r, rows)), e = lds_s32(rq + 4 * min(r + 1, rows));
-    const bool lng = e - b > kShortRow;
-    const int ee = lng ? b : e;
-    const int trips = (int)__reduce_max_sync(FULL, (unsigned)((ee - b + 1 - h) >> 1));
-    double s0 = 0.0, s1 = 0.0;
+    const bool live = lane < 16 && e > b;  // r >= rows: b = e = rq[rows]
+    const int kb = lds_s32(rq), ke = lds_s32(rq + 4 * rows);
+    double acc = 0.0;
 #pragma unroll 1
-    for (int i = 0; i < trips; i += 2) {
-        const int k0 = b + h + 2 * i;
-        s0 += rem_product(p, k0, ee, colS, valS, x_policy);
-        s1 += rem_product(p, k0 + 2, ee, colS, valS, x_policy);
-    }
-    double acc = s0 + s1;
-    uint32_t lm = __ballot_sync(FULL, lng && h == 0 && r < rows);
-#pragma unroll 1
-    while (lm) {
-        const int r0 = __ffs(lm) - 1;
-        lm &= lm - 1;
-        const int r1 = lm ? __ffs(lm) - 1 : -1;
-        if (lm) lm &= lm - 1;
-        const bool pair = r1 >= 0;  // warp-uniform
-        const int myrow = (pair && h) ? r1 : r0;
-        const int off = pair ? r : lane, stride = pair ? 16 : 32;
-        const int bb = lds_s32(rq + 4 * myrow), e2 = lds_s32(rq + 4 * myrow + 4);
-        const int t2 = (int)__reduce_max_sync(FULL, (unsigned)((e2 - bb + 4 * stride - 1) >> (pair ? 6 : 7)));
-        double q0 = 0.0, q1 = 0.0, q2 = 0.0, q3 = 0.0;
-#pragma unroll 1
-        for (int t = 0; t < t2; ++t) {
-            const int k = bb + off + 4 * stride * t;
-            q0 += rem_product(p, k, e2, colS, valS, x_policy);
-            q1 += rem_product(p, k + stride, e2, colS, valS, x_policy);
-            q2 += rem_product(p, k + 2 * stride, e2, colS, valS, x_policy);
-            q3 += rem_product(p, k + 3 * stride, e2, colS, valS, x_policy);
+    for (int base = kb; base < ke; base += 64) {
+        const int k0 = base + lane, k1 = k0 + 32;
+        const bool two = base + 32 < ke;  // warp-uniform
+        int c0, c1 = 0;
+        double v0, v1 = 0.0, x1 = 0.0;
+        lds_entry_lt(k0, ke, colS + 4 * k0, valS + 8 * k0, c0, v0);
+        const double x0 = ldg_hint(p.x + (uint32_t)c0, x_policy);
+        if (two) {
+            lds_entry_lt(k1, ke, colS + 4 * k1, valS + 8 * k1, c1, v1);
+            x1 = ldg_hint(p.x + (uint32_t)c1, x_policy);
         }
-        double sq = (q0 + q1) + (q2 + q3);
-        if (!pair) sq += __shfl_xor_sync(FULL, sq, 16);
-        sq += __shfl_xor_sync(FULL, sq, 8);
-        sq += __shfl_xor_sync(FULL, sq, 4);
-        sq += __shfl_xor_sync(FULL, sq, 2);
-        sq += __shfl_xor_sync(FULL, sq, 1);
-        if (pair ? r == myrow : lane == r0) acc += sq;
+        acc += chunk_piece(k0 < ke ? v0 * x0 : 0.0, base, b, e, live, lane);
+        if (two) acc += chunk_piece(k1 < ke ? v1 * x1 : 0.0, base + 32, b, e, live, lane);
     }
     return acc;
 }
 
+// fused CSR remainder of an item's rows; adds row r's sum into acc
+// of lane r (or r + 16).  rpS: rebased row pointers (rows + 1), colS/valS:
+// entries.  Rows of <= 4 entries (stencil-like) run two lanes per row, two
+// entries each, one round trip of gathers; anything longer runs rem_chunks.
+// The path depends only on the item's content.
+__device__ __forceinline__ void remainder(const Params &p, uint32_t rpS, uint32_t colS, uint32_t valS, int rows,
+                                          uint64_t x_policy, int lane, double &acc) {
+    const int r = lane & 15, h = lane >> 4;
+    const int b = lds_s32(rpS + 4 * min(r, rows)), e = lds_s32(rpS + 4 * min(r + 1, rows));
+    const int maxlen = (int)__reduce_max_sync(FULL, (unsigned)(e - b));
+    if (maxlen > 4) {
+        acc += rem_chunks(p, rpS, rows, colS, valS, x_policy, lane);
+        return;
+    }
+    // entries b + h and b + h + 2 of row r; a masked entry adds nothing
+    // (predicated FMA: the x it read is never used)
+    const int k0 = b + h, k1 = k0 + 2;
+    int c0, c1;
+    double v0, v1;
+    lds_entry_lt(k0, e, colS + 4 * k0, valS + 8 * k0, c0, v0);
+    lds_entry_lt(k1, e, colS + 4 * k1, valS + 8 * k1, c1, v1);
+    const double x0 = ldg_hint(p.x + (uint32_t)c0, x_policy), x1 = ldg_hint(p.x + (uint32_t)c1, x_policy);
+    fma_if(k0 < e, v0, x0, acc);
+    fma_if(k1 < e, v1, x1, acc);
+}
+
 // Row-group item (internal.cuh): ntr consecutive tile rows without stored
-// tiles, only remainder rows: the flat pass over all their entries,
-// then per tile row the row sums from shared memory and y written once per
-// row.  Every tile row is summed exactly as it would be alone, so grouping
-// never changes a bit of y.
+// tiles, only remainder rows.  Each tile row runs rem_chunks with its
+// chunk grid anchored at its own first entry and writes y once per row, so a
+// tile row's sums never depend on which tile rows share its item.
 __device__ __forceinline__ void group_item(const Params &p, const WItem &it, uint32_t slot, uint64_t x_policy,
                                            int lane) {
     const int ntr = (int)(it.jt_rows_pay & 0xFFu);
@@ -198,86 +171,19 @@ __device__ __forceinline__ void group_item(const Params &p, const WItem &it, uin
     const uint32_t rpS = slot + rp, colS = slot + (it.rp_col >> 16), valS = slot + (it.val_tot & 0xFFFFu);
 #pragma unroll 1
     for (int g = 0; g < ntr; ++g) {
-        double acc = has_rem ? flat_rows(p, rpS + 64u * (uint32_t)g, colS, valS, g + 1 < ntr ? 16 : rows_last, x_policy,
-                                         lane) : 0.0;
-        acc += __shfl_xor_sync(FULL, acc, 16);
+        const int rows = g + 1 < ntr ? 16 : rows_last;
+        const double acc = has_rem ? rem_chunks(p, rpS + 64u * (uint32_t)g, rows, colS, valS, x_policy, lane) : 0.0;
         const int64_t row = 16 * ((int64_t)it.I + g) + lane;
         if (lane < 16 && row < p.m) p.y[row] = acc;
-    }
-}
-
-// Row-group item, TM kernels: two tile rows at a time, half-warp h on tile
-// row g + h and lane r on its row r alone (4 running sums over the row's
-// products, in entry order mod 4); rows longer than kShortRow are summed by
-// the whole warp with an xor tree.  Each product is formed where it is summed
-// (no shared-memory round trip), rounded on its own, so the terms and their
-// order are those of the flat pass.  A tile row's sums depend only on its own
-// entries (grouping never changes a bit of y).
-__device__ __forceinline__ void group_item2(const Params &p, const WItem &it, uint32_t slot, uint64_t x_policy,
-                                            int lane) {
-    const int ntr = (int)(it.jt_rows_pay & 0xFFu);
-    const int rows_last = (int)((it.jt_rows_pay >> 8) & 31u);
-    const uint32_t total = it.val_tot >> 16, rp = it.rp_col & 0xFFFFu;
-    const bool has_rem = total > rp;
-    const uint32_t rpS = slot + rp, colS = slot + (it.rp_col >> 16), valS = slot + (it.val_tot & 0xFFFFu);
-    const int h = lane >> 4, r = lane & 15;
-#pragma unroll 1
-    for (int g = 0; g < ntr; g += 2) {
-        const int gg = g + h;
-        const int rows = gg < ntr ? (gg + 1 < ntr ? 16 : rows_last) : 0;
-        double acc = 0.0;
-        if (has_rem) {
-            const uint32_t rq = rpS + 64u * (uint32_t)gg;
-            const int b = lds_s32(rq + 4 * min(r, rows)), e = lds_s32(rq + 4 * min(r + 1, rows));
-            const bool lng = e - b > kShortRow;
-            const int ee = lng ? b : e;
-            const int trips = (int)__reduce_max_sync(FULL, (unsigned)((ee - b + 3) >> 2));
-            double s0 = 0.0, s1 = 0.0, s2 = 0.0, s3 = 0.0;
-#pragma unroll 1
-            for (int t = 0; t < trips; ++t) {
-                const int k = b + 4 * t;
-                s0 += rem_product(p, k, ee, colS, valS, x_policy);
-                s1 += rem_product(p, k + 1, ee, colS, valS, x_policy);
-                s2 += rem_product(p, k + 2, ee, colS, valS, x_policy);
-                s3 += rem_product(p, k + 3, ee, colS, valS, x_policy);
-            }
-            acc = (s0 + s1) + (s2 + s3);
-            uint32_t lm = __ballot_sync(FULL, lng);
-#pragma unroll 1
-            while (lm) {  // one long row at a time, the whole warp
-                const int src = __ffs(lm) - 1;
-                lm &= lm - 1;
-                const int bb = __shfl_sync(FULL, b, src), e2 = __shfl_sync(FULL, e, src);
-                const int t2 = (e2 - bb + 127) >> 7;
-                double q0 = 0.0, q1 = 0.0, q2 = 0.0, q3 = 0.0;
-#pragma unroll 1
-                for (int t = 0; t < t2; ++t) {
-                    const int k = bb + lane + 128 * t;
-                    q0 += rem_product(p, k, e2, colS, valS, x_policy);
-                    q1 += rem_product(p, k + 32, e2, colS, valS, x_policy);
-                    q2 += rem_product(p, k + 64, e2, colS, valS, x_policy);
-                    q3 += rem_product(p, k + 96, e2, colS, valS, x_policy);
-                }
-                double sq = (q0 + q1) + (q2 + q3);
-                sq += __shfl_xor_sync(FULL, sq, 16);
-                sq += __shfl_xor_sync(FULL, sq, 8);
-                sq += __shfl_xor_sync(FULL, sq, 4);
-                sq += __shfl_xor_sync(FULL, sq, 2);
-                sq += __shfl_xor_sync(FULL, sq, 1);
-                if (lane == src) acc += sq;
-            }
-        }
-        const int64_t row = 16 * ((int64_t)it.I + gg) + r;
-        if (gg < ntr && row < p.m) p.y[row] = acc;
     }
 }
 
 // the tiles of one format group, two per step.  d: shared address of this
 // half's descriptor (see k_blob_fill): x = distance from the descriptor to the
 // tile's payload (CSR: to its csrRowPtr), y = aux | t*128 | nz << 11 | tm << 20 |
-// invalid << 31 (tm: the pair's longest CSR row / larger ELL width).  TM:
-// run CSR and ELL with the tm routines.
-template <int F, bool TM, int N = 0>
+// invalid << 31 (tm: the pair's longest CSR row / larger ELL width / larger
+// COO entry count).  N = 3: every CSR row / ELL width of the item is <= 3.
+template <int F, int N = 0>
 __device__ __forceinline__ void run_group(int np, uint32_t &d, uint32_t xs, int r, double &acc, uint32_t racc = 0) {
     const int lane_h = (int)(threadIdx.x >> 4) & 1;
 #pragma unroll 1
@@ -289,48 +195,38 @@ __device__ __forceinline__ void run_group(int np, uint32_t &d, uint32_t xs, int 
         const int aux = (int)(e.y & 31u), nz = (int)(e.y >> 11) & 511;
         const int tm = (int)(e.y >> 20) & 31;
         if (F == F_CSR && N == 3) half_csr_n<3>(P, nz, X, r, ok, acc);
-        if (F == F_CSR && TM && N == 0) half_csr_tm(P, nz, tm, X, r, ok, acc);
-        if (F == F_CSR && !TM) half_csr(P, nz, X, r, ok, acc);
+        if (F == F_CSR && N == 0) half_csr_tm(P, nz, tm, X, r, ok, acc);
         if (F == F_ELL && N == 3) half_ell_n<3>(P, aux, X, r, ok, acc);
-        if (F == F_ELL && TM && N == 0) half_ell_tm(P, aux, tm, X, r, ok, acc);
-        if (F == F_ELL && !TM) half_ell(P, aux, X, r, ok, acc);
+        if (F == F_ELL && N == 0) half_ell_tm(P, aux, tm, X, r, ok, acc);
         if (F == F_DNS) half_dns(P, X, r, ok, acc);
         if (F == F_DNSCOL) half_dnscol(P, aux, X, r, ok, acc);
-        if (F == F_DNSROW && TM) half_dnsrow_tree(P, aux, X, r, ok, acc);
-        if (F == F_DNSROW && !TM) half_dnsrow(P, aux, X, r, ok, acc);
-        if (F == F_COO && TM) {  // tiny tiles (power-law, stencil corners): walk; else scan
+        if (F == F_DNSROW) half_dnsrow_tree(P, aux, X, r, ok, acc);
+        if (F == F_COO) {  // tiny tiles (power-law, stencil corners): walk; else scan
             if (tm <= 2) half_coo_n<2>(P, P + 8 * nz, nz, X, r, ok, acc);
             else half_coo_scan(P, P + 8 * nz, nz, X, r, lane_h, racc, ok, acc);
         }
-        if (F == F_COO && !TM) half_coo(P, P + 8 * nz, nz, X, r, ok, acc);
-        if (F == F_HYB && TM) half_hyb_scan(P, aux, nz, X, r, lane_h, racc, ok, acc);
-        if (F == F_HYB && !TM) half_hyb(P, aux, nz, X, r, ok, acc);
+        if (F == F_HYB) half_hyb_scan(P, aux, nz, X, r, lane_h, racc, ok, acc);
     }
 }
 
-// lane 0: the whole item (descriptors, payload, remainder) in ONE TMA bulk copy.
-// fence: the previous item wrote the slot with generic-proxy stores (flat
-// pass), which must be ordered before the async-proxy write
+// lane 0: the whole item (descriptors, payload, remainder) in ONE TMA bulk
+// copy.  The slot is only ever read through the generic proxy (the kernels
+// never store to it), so no proxy fence precedes the async-proxy write.
 __device__ __forceinline__ void issue_blob(const Params &p, const WItem &it, uint32_t slot, uint32_t bar,
-                                           uint64_t policy, int lane, bool fence = true) {
+                                           uint64_t policy, int lane) {
     const uint32_t total = it.val_tot >> 16;
     if (lane == 0 && total) {
-        if (fence) fence_proxy_async();
         mbar_expect_tx(bar, total);
         bulk_g2s_hint(slot, p.blob + (size_t)it.blob16 * 16, total, bar, policy);
     }
 }
 
 // the x segment of every tile of the item (J: tile column of tile `lane`),
-// issued before the blob lands
-// tail: -1 = find out here, else the item's WItem bit 30 (its last tile
-// column reaches the ragged end of x)
+// issued before the blob lands.  tail: the item's WItem bit 30 (its last
+// tile column reaches the ragged end of x)
 __device__ __forceinline__ void issue_x(const Params &p, int J, int nt, uint32_t xs, uint64_t x_policy, int lane,
-                                        int tail = -1) {
+                                        bool tail) {
     const uint32_t n32 = (uint32_t)p.n;
-    // tile columns ascend within an item: only the last one can reach the
-    // ragged end of x
-    if (tail < 0) tail = 16u * (uint32_t)__shfl_sync(FULL, J, max(nt - 1, 0)) + 16u > n32;
     if (p.x_vec && !tail) {  // lane l: tile 4k + (l >> 3), 16 bytes at elements 2(l & 7)
         const double *xq = p.x + 2 * (lane & 7);
         const uint32_t xs_l = xs + 16 * (lane & 7);
@@ -357,7 +253,7 @@ __device__ __forceinline__ void issue_x(const Params &p, int J, int nt, uint32_t
             }
         }
         cp_async_commit();
-    } else {  // lane l: tile 2k + h, element r
+    } else {  // x not 16-byte aligned: lane l: tile 2k + h, element r
         const int h = lane >> 4, r = lane & 15;
 #pragma unroll
         for (int kk = 0; kk < kItemTiles / 2; ++kk) {
@@ -370,15 +266,10 @@ __device__ __forceinline__ void issue_x(const Params &p, int J, int nt, uint32_t
 
 // steps 2-4 of an item whose blob is in `slot` and whose x segments are in
 // flight into `xs`: remainder, tiles, y (or the split-row carry)
-template <bool TM>
 __device__ __forceinline__ void compute_item(const Params &p, const WItem &it, uint32_t slot, uint32_t xs,
-                                             uint32_t racc, uint64_t x_policy, int lane, double &carry,
-                                             bool &dirty) {
-    if (it.jt_rows_pay & 0xFFu) {  // row-group item
-        dirty = true;
-        if (p.x_vec) cp_async_wait_all();
-        if (TM) group_item2(p, it, slot, x_policy, lane);
-        else group_item(p, it, slot, x_policy, lane);
+                                             uint32_t racc, uint64_t x_policy, int lane, double &carry) {
+    if (it.jt_rows_pay & 0xFFu) {  // row-group item (no tiles, no x segments)
+        group_item(p, it, slot, x_policy, lane);
         return;
     }
     const int h = lane >> 4, r = lane & 15;
@@ -387,26 +278,26 @@ __device__ __forceinline__ void compute_item(const Params &p, const WItem &it, u
     double acc = 0.0;
     const uint32_t rp = it.rp_col & 0xFFFFu;
     if (total > rp)
-        remainder<TM ? kMedRow : kShortRow>(p, slot + rp, slot + (it.rp_col >> 16), slot + (it.val_tot & 0xFFFFu),
-                  (int)((it.jt_rows_pay >> 8) & 31u), x_policy, lane, acc, dirty);
+        remainder(p, slot + rp, slot + (it.rp_col >> 16), slot + (it.val_tot & 0xFFFFu),
+                  (int)((it.jt_rows_pay >> 8) & 31u), x_policy, lane, acc);
     if (p.x_vec) cp_async_wait_all();
     __syncwarp();
     // 3. tiles: format group by format group, two tiles per step
     {
         const uint32_t g = it.groups;
         uint32_t d = slot + 8 * h;
-        // TM: items whose CSR rows / ELL widths are all <= 3 (bits 28, 29)
-        // run those groups without per-pair dispatch
-        if (TM && ((g >> 28) & 1u)) run_group<F_CSR, TM, 3>((int)(g & 15u), d, xs, r, acc);
-        else run_group<F_CSR, TM>((int)(g & 15u), d, xs, r, acc);
-        if (!TM || (g & 0xF0u)) run_group<F_COO, TM>((int)((g >> 4) & 15u), d, xs, r, acc, racc);
-        if (TM && ((g >> 29) & 1u)) run_group<F_ELL, TM, 3>((int)((g >> 8) & 15u), d, xs, r, acc);
-        else run_group<F_ELL, TM>((int)((g >> 8) & 15u), d, xs, r, acc);
-        if (!TM || (g & 0x0FFFF000u)) {  // TM: one test skips the four rarer formats
-            run_group<F_HYB, TM>((int)((g >> 12) & 15u), d, xs, r, acc, racc);
-            run_group<F_DNS, TM>((int)((g >> 16) & 15u), d, xs, r, acc);
-            run_group<F_DNSROW, TM>((int)((g >> 20) & 15u), d, xs, r, acc);
-            run_group<F_DNSCOL, TM>((int)((g >> 24) & 15u), d, xs, r, acc);
+        // items whose CSR rows / ELL widths are all <= 3 (bits 28, 29) run
+        // those groups without per-pair dispatch
+        if ((g >> 28) & 1u) run_group<F_CSR, 3>((int)(g & 15u), d, xs, r, acc);
+        else run_group<F_CSR>((int)(g & 15u), d, xs, r, acc);
+        if (g & 0xF0u) run_group<F_COO>((int)((g >> 4) & 15u), d, xs, r, acc, racc);
+        if ((g >> 29) & 1u) run_group<F_ELL, 3>((int)((g >> 8) & 15u), d, xs, r, acc);
+        else run_group<F_ELL>((int)((g >> 8) & 15u), d, xs, r, acc);
+        if (g & 0x0FFFF000u) {  // one test skips the four rarer formats
+            run_group<F_HYB>((int)((g >> 12) & 15u), d, xs, r, acc, racc);
+            run_group<F_DNS>((int)((g >> 16) & 15u), d, xs, r, acc);
+            run_group<F_DNSROW>((int)((g >> 20) & 15u), d, xs, r, acc);
+            run_group<F_DNSCOL>((int)((g >> 24) & 15u), d, xs, r, acc);
         }
     }
     acc += __shfl_xor_sync(FULL, acc, 16);
@@ -423,8 +314,8 @@ __device__ __forceinline__ void compute_item(const Params &p, const WItem &it, u
             if (lane < 16 && row < p.m) p.y[row] = sum;
         } else {  // hub row: one partial per group, the last group sums them in order
             const int2 si = p.split_info[it.split];
-            const int ngroups = (si.y + p.local_parts - 1) / p.local_parts;
-            const int gidx = (it.part_nt & 0xFFFFFF) / p.local_parts;
+            const int ngroups = (si.y + kLocalParts - 1) / kLocalParts;
+            const int gidx = (it.part_nt & 0xFFFFFF) / kLocalParts;
             if (lane < 16) __stcg(p.partials + (int64_t)(si.x + gidx) * 16 + lane, sum);
             __threadfence();
             __syncwarp();
@@ -452,7 +343,9 @@ __device__ __forceinline__ void compute_item(const Params &p, const WItem &it, u
     }
 }
 
-// one blob in flight per warp: latency hidden by warp count (32 warps/SM)
+// Dense-row kernel: WARPS warps per CTA, several CTAs per SM, one blob in
+// flight per warp; each warp owns a contiguous, cost-balanced, row-aligned
+// item chunk (schedule.cu) and its start record (chunk + first item).
 template <int WARPS, int SLOT, int MINB>
 __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, MINB) tilespmv_fp64_warp(const Params p) {
     using Cfg = WarpCfg<WARPS, SLOT>;
@@ -469,16 +362,12 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, MINB) tilespmv
     // PDL: the next SpMV in the stream may start its prologue now; it waits
     // (griddep_wait) before touching x or y, and so do we
     griddep_launch_dependents();
-    // contiguous, cost-balanced, row-aligned item chunk per warp (schedule.cu);
-    // neighbouring tile rows share x segments.  The warp's start record holds
-    // the chunk and a copy of the first item (one round trip).
     const int64_t gw = (int64_t)blockIdx.x * WARPS + warp;
     TSP_SMID(gw, (int64_t)gridDim.x * WARPS);
     const WFirst *wf = p.wfirst + gw;
     const int4 wb = __ldg(reinterpret_cast<const int4 *>(wf));
     const int kbeg = wb.x, kend = wb.y;
     double carry = 0.0;  // partial row sums inside a group of parts of a split tile row
-    bool dirty = true;   // the slot may hold generic-proxy writes (TM kernels track it)
     uint32_t phase = 0;
     const uint64_t stream_policy = policy_evict_first(), x_policy = policy_evict_last();
     WItem nxt = load_witem(&wf->w, 0);
@@ -491,7 +380,7 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, MINB) tilespmv
         // the matrix is immutable; x and y may belong to the previous kernel
         if (k == kbeg) griddep_wait();
         // 1. x segments, issued before the blob lands (J came with the record)
-        issue_x(p, J, (it.part_nt >> 24) & 31, xs, x_policy, lane);
+        issue_x(p, J, (it.part_nt >> 24) & 31, xs, x_policy, lane, (it.groups >> 30) & 1u);
         if (k + 1 < kend) {  // the next record and its columns, in flight during this item
             nxt = load_witem(p.witems, k + 1);
             Jn = lane < 16 ? __ldg(p.jcols + (int64_t)(k + 1) * 16 + lane) : 0;
@@ -502,24 +391,24 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, MINB) tilespmv
         }
         TSP_STAMP(gw, k - kbeg, 1);
         TSP_INFO(gw, k - kbeg, k, it);
-        compute_item<false>(p, it, slot, xs, racc, x_policy, lane, carry, dirty);
+        compute_item(p, it, slot, xs, racc, x_policy, lane, carry);
         __syncwarp();  // slot and x scratch free for the next item
         TSP_STAMP(gw, k - kbeg, 3);
     }
 }
 
-// One CTA per SM (WARPS warps, one blob in flight each).  The CTA owns a
-// contiguous, cost-balanced range of units (schedule.cu: a unit is one item,
-// or the items of a group of parts of a split tile row, which must run in
-// order in one warp); its warps claim units from a shared-memory counter, so
-// warps that draw slow units take fewer and all warps of the SM finish
-// together (with several CTAs per SM the hardware's oldest-first issue
-// priority leaves the youngest CTAs as a serial tail).  Each warp claims its
-// next unit when it starts one, so the claim and the unit's bounds are in
-// flight while the current unit runs.
-template <int WARPS, int SLOT, bool TM>
+// SM-queue kernel: one CTA per SM (WARPS warps, one blob in flight each).
+// The CTA owns a contiguous, cost-balanced range of units (schedule.cu: a
+// unit is one item, or the items of a group of parts of a split tile row,
+// which must run in order in one warp); its warps claim units from a
+// shared-memory counter, so warps that draw slow units take fewer and all
+// warps of the SM finish together (with several CTAs per SM the hardware's
+// oldest-first issue priority leaves the youngest CTAs as a serial tail).
+// Each warp claims its next unit when it starts one, so the claim and the
+// unit's bounds are in flight while the current unit runs.
+template <int WARPS, int SLOT>
 __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, 1) tilespmv_fp64_sm(const Params p) {
-    using Cfg = WarpCfg<WARPS, SLOT, 1, TM ? 256 : 128>;
+    using Cfg = WarpCfg<WARPS, SLOT>;
     extern __shared__ __align__(128) uint8_t smem[];
     __shared__ int s_next;
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -538,7 +427,6 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, 1) tilespmv_fp
     TSP_SMID(gw, (int64_t)gridDim.x * WARPS);
     (void)gw;
     double carry = 0.0;  // partial row sums inside a group of parts of a split tile row
-    bool dirty = true;   // the slot may hold generic-proxy writes (TM kernels track it)
     uint32_t phase = 0;
     const uint64_t stream_policy = policy_evict_first(), x_policy = policy_evict_last();
     int k = -1, ke = 0, nb = -1, ne = 0;
@@ -559,8 +447,7 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, 1) tilespmv_fp
         const WItem it = nxt;
         const int J = Jn;
         TSP_STAMP(gw, j, 0);
-        issue_blob(p, it, slot, bar, stream_policy, lane, !TM || dirty);
-        dirty = false;
+        issue_blob(p, it, slot, bar, stream_policy, lane);
         // the matrix is immutable; x and y may belong to the previous kernel
         if (!waited) {
             griddep_wait();
@@ -577,7 +464,7 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, 1) tilespmv_fp
             }
         }
         // 1. x segments, issued before the blob lands (J came with the record)
-        issue_x(p, J, (it.part_nt >> 24) & 31, xs, x_policy, lane, TM ? (int)((it.groups >> 30) & 1u) : -1);
+        issue_x(p, J, (it.part_nt >> 24) & 31, xs, x_policy, lane, (it.groups >> 30) & 1u);
         const int kn = k + 1 < ke ? k + 1 : nb;
         if (kn >= 0) {  // the next record and its columns, in flight during this item
             nxt = load_witem(p.witems, kn);
@@ -589,7 +476,7 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, 1) tilespmv_fp
         }
         TSP_STAMP(gw, j, 1);
         TSP_INFO(gw, j, k, it);
-        compute_item<TM>(p, it, slot, xs, racc, x_policy, lane, carry, dirty);
+        compute_item(p, it, slot, xs, racc, x_policy, lane, carry);
         __syncwarp();  // slot and x scratch free for the next item
         TSP_STAMP(gw, j, 3);
         ++j;
@@ -601,106 +488,16 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, 1) tilespmv_fp
     }
 }
 
-// two blobs in flight per warp: item k+1 streams in while item k computes
-// (dense tile rows, where few large slots fit per SM)
-template <int WARPS, int SLOT, int MINB>
-__global__ void __launch_bounds__(WarpCfg<WARPS, SLOT, 2>::kThreads, MINB) tilespmv_fp64_warp2(const Params p) {
-    using Cfg = WarpCfg<WARPS, SLOT, 2>;
-    extern __shared__ __align__(128) uint8_t smem[];
-    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    const uint32_t xs = smem_u32(smem) + (uint32_t)warp * Cfg::kX;
-    const uint32_t base = smem_u32(smem) + WARPS * Cfg::kX + (uint32_t)warp * Cfg::kPer;
-    const uint32_t racc = base + 2 * SLOT, bar0 = racc + Cfg::kRacc;
-    if (lane == 0) {
-        mbar_init(bar0, 1);
-        mbar_init(bar0 + 8, 1);
-        fence_mbar_init();
-    }
-    __syncwarp();
-    griddep_launch_dependents();
-    const int64_t gw = (int64_t)blockIdx.x * WARPS + warp;
-    const WFirst *wf = p.wfirst + gw;
-    const int4 wb = __ldg(reinterpret_cast<const int4 *>(wf));
-    const int kbeg = wb.x, kend = wb.y;
-    double carry = 0.0;
-    bool dirty = true;
-    uint32_t phases = 0;  // bit s: parity of slot s's barrier
-    const uint64_t stream_policy = policy_evict_first(), x_policy = policy_evict_last();
-    WItem cur = load_witem(&wf->w, 0), nx{};
-    int Jc = lane < 16 ? __ldg(wf->J + lane) : 0, Jx = 0;
-    // both slots start streaming before the dependency wait (matrix data only)
-    if (kbeg < kend) issue_blob(p, cur, base, bar0, stream_policy, lane);
-    if (kbeg + 1 < kend) {
-        nx = load_witem(&wf->w2, 0);
-        issue_blob(p, nx, base + SLOT, bar0 + 8, stream_policy, lane);
-        Jx = lane < 16 ? __ldg(p.jcols + (int64_t)(kbeg + 1) * 16 + lane) : 0;
-    }
-    for (int k = kbeg; k < kend; ++k) {
-        const uint32_t s = (uint32_t)(k - kbeg) & 1u;
-        const uint32_t slot = base + s * SLOT, bar = bar0 + 8 * s;
-        if (k == kbeg) griddep_wait();
-        issue_x(p, Jc, (cur.part_nt >> 24) & 31, xs, x_policy, lane);
-        WItem n2{};
-        int J2 = 0;
-        if (k + 2 < kend) {  // the record of the item that refills this slot
-            n2 = load_witem(p.witems, k + 2);
-            J2 = lane < 16 ? __ldg(p.jcols + (int64_t)(k + 2) * 16 + lane) : 0;
-        }
-        if (cur.val_tot >> 16) {
-            mbar_wait(bar, (phases >> s) & 1u);
-            phases ^= 1u << s;
-        }
-        compute_item<false>(p, cur, slot, xs, racc, x_policy, lane, carry, dirty);
-        __syncwarp();  // slot s and the x stage are free
-        if (k + 2 < kend) issue_blob(p, n2, slot, bar, stream_policy, lane);
-        cur = nx;
-        Jc = Jx;
-        nx = n2;
-        Jx = J2;
-    }
-}
-
-template <int WARPS, int SLOT, int MINB>
-KernelChoice warp_choice(const char *name) {
-    using Cfg = WarpCfg<WARPS, SLOT>;
-    return {name, tilespmv_fp64_warp<WARPS, SLOT, MINB>, Cfg::kThreads, (int)Cfg::kSmem, 0, false, SLOT, true, false};
-}
-
-template <int WARPS, int SLOT, bool TM = false>
-KernelChoice sm_choice(const char *name) {
-    using Cfg = WarpCfg<WARPS, SLOT, 1, TM ? 256 : 128>;
-    return {name, tilespmv_fp64_sm<WARPS, SLOT, TM>, Cfg::kThreads, (int)Cfg::kSmem, 1, false, SLOT, true, true};
-}
-
-template <int WARPS, int SLOT, int MINB>
-KernelChoice warp2_choice(const char *name) {
-    using Cfg = WarpCfg<WARPS, SLOT, 2>;
-    return {name, tilespmv_fp64_warp2<WARPS, SLOT, MINB>, Cfg::kThreads, (int)Cfg::kSmem, 0, false, SLOT, true, false};
-}
-
 }  // namespace
 
-KernelChoice kernel_warp(int variant) {
-    switch (variant) {
-    case 21: return warp_choice<8, 4608, 4>("tilespmv_fp64_warp<8,4608>");
-    case 22: return warp_choice<8, 5120, 3>("tilespmv_fp64_warp<8,5120>");
-    case 23: return warp_choice<4, 4608, 8>("tilespmv_fp64_warp<4,4608>");
-    case 24: return warp_choice<8, 4096, 4>("tilespmv_fp64_warp<8,4096>");
-    case 25: return warp_choice<4, 10752, 4>("tilespmv_fp64_warp<4,10752>");  // dense tile rows
-    case 26: return warp_choice<4, 8704, 5>("tilespmv_fp64_warp<4,8704>");
-    // double-buffered
-    case 30: return warp2_choice<4, 6016, 4>("tilespmv_fp64_warp2<4,6016>");
-    case 31: return warp2_choice<6, 4608, 3>("tilespmv_fp64_warp2<6,4608>");
-    case 32: return warp2_choice<4, 8448, 3>("tilespmv_fp64_warp2<4,8448>");
-    case 33: return warp2_choice<4, 10752, 2>("tilespmv_fp64_warp2<4,10752>");
-    case 34: return warp2_choice<3, 6192, 5>("tilespmv_fp64_warp2<3,6192>");
-    // one CTA per SM, shared-memory unit queue
-    case 40: return sm_choice<32, 4608>("tilespmv_fp64_sm<32,4608>");
-    case 41: return sm_choice<16, 10752>("tilespmv_fp64_sm<16,10752>");
-    case 42: return sm_choice<24, 6144>("tilespmv_fp64_sm<24,6144>");
-    case 43: return sm_choice<32, 4608, true>("tilespmv_fp64_sm<32,4608,tm>");
-    default: return warp_choice<8, 4608, 4>("tilespmv_fp64_warp<8,4608>");
+KernelChoice kernel_choice(int kernel) {
+    if (kernel == TILESPMV_KERNEL_DENSE_ROWS) {
+        using Cfg = WarpCfg<4, 10752>;
+        return {"tilespmv_fp64_warp<4,10752>", tilespmv_fp64_warp<4, 10752, 4>, Cfg::kThreads, (int)Cfg::kSmem,
+                10752, false};
     }
+    using Cfg = WarpCfg<32, 4608>;
+    return {"tilespmv_fp64_sm<32,4608>", tilespmv_fp64_sm<32, 4608>, Cfg::kThreads, (int)Cfg::kSmem, 4608, true};
 }
 
 }  // namespace tsp

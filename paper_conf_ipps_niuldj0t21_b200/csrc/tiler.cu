@@ -32,23 +32,29 @@ namespace tsp {
 
 namespace {
 
+// stream-ordered temporary (cudaMallocAsync / cudaFreeAsync on the create
+// stream: no device-wide synchronisation, other streams keep running)
 template <class T>
 struct DevBuf {
     T *p = nullptr;
-    DevBuf() = default;
+    cudaStream_t st = nullptr;
+    explicit DevBuf(cudaStream_t s) : st(s) {}
     DevBuf(const DevBuf &) = delete;
-    ~DevBuf() { if (p) cudaFree(p); }
+    ~DevBuf() { free(); }
+    void free() {
+        if (p) cudaFreeAsync(p, st);
+        p = nullptr;
+    }
     int alloc(size_t n) {
-        if (p) { cudaFree(p); p = nullptr; }
-        cudaError_t e = cudaMalloc(&p, std::max<size_t>(n, 1) * sizeof(T));
+        free();
+        cudaError_t e = cudaMallocAsync(&p, std::max<size_t>(n, 1) * sizeof(T), st);
         if (e != cudaSuccess) {
             cudaGetLastError();
             p = nullptr;
-            return set_error(TILESPMV_OOM, "cudaMalloc of a tiler temporary failed");
+            return set_error(TILESPMV_OOM, "cudaMallocAsync of a tiler temporary failed");
         }
         return 0;
     }
-    T *release() { T *q = p; p = nullptr; return q; }
 };
 
 inline unsigned blocks_for(int64_t n, int threads) {
@@ -381,10 +387,9 @@ template <class F>
 int cub_call(F &&f, cudaStream_t stream) {
     size_t bytes = 0;
     TSP_CK(f((void *)nullptr, bytes));
-    DevBuf<uint8_t> tmp;
+    DevBuf<uint8_t> tmp(stream);
     if (int rc = tmp.alloc(bytes)) return rc;
     TSP_CK(f((void *)tmp.p, bytes));
-    (void)stream;
     return 0;
 }
 
@@ -402,8 +407,8 @@ int build_tiled_k(Matrix &M, const int32_t *d_rowptr, const int32_t *d_colidx, c
     const int64_t nnz = M.nnz;
     const int ibits = bits_for(M.tilem);
     // ---- a2: keys, stable radix sort (tiles by (I,J); entries stay row-major)
-    DevBuf<K> keyA, keyB;
-    DevBuf<int32_t> idxA, idxB;
+    DevBuf<K> keyA(st), keyB(st);
+    DevBuf<int32_t> idxA(st), idxB(st);
     if (int rc = keyA.alloc(nnz)) return rc;
     if (int rc = keyB.alloc(nnz)) return rc;
     if (int rc = idxA.alloc(nnz)) return rc;
@@ -420,12 +425,12 @@ int build_tiled_k(Matrix &M, const int32_t *d_rowptr, const int32_t *d_colidx, c
         if (kb.Current() != keyA.p) std::swap(keyA.p, keyB.p);
         if (vb.Current() != idxA.p) std::swap(idxA.p, idxB.p);
     }
-    cudaFree(keyB.p); keyB.p = nullptr;
-    cudaFree(idxB.p); idxB.p = nullptr;
+    keyB.free();
+    idxB.free();
     const K *key = keyA.p;
     const int32_t *idx = idxA.p;
     // ---- tile heads and ids
-    DevBuf<int32_t> head, tid;
+    DevBuf<int32_t> head(st), tid(st);
     if (int rc = head.alloc(nnz)) return rc;
     if (int rc = tid.alloc(nnz)) return rc;
     k_heads<K><<<blocks_for(nnz, TB), TB, 0, st>>>(key, nnz, head.p);
@@ -435,22 +440,22 @@ int build_tiled_k(Matrix &M, const int32_t *d_rowptr, const int32_t *d_colidx, c
     int32_t numtile32 = 0;
     if (int rc = read_scalar(tid.p + nnz - 1, &numtile32, st)) return rc;
     const int64_t numtile = numtile32;
-    DevBuf<int32_t> tileStart;
+    DevBuf<int32_t> tileStart(st);
     if (int rc = tileStart.alloc(numtile + 1)) return rc;
     k_tile_ids<<<blocks_for(nnz, TB), TB, 0, st>>>(head.p, tid.p, nnz, tileStart.p);
     TSP_CK(cudaGetLastError());
-    cudaFree(head.p); head.p = nullptr;
+    head.free();
     // ---- a3: census masks
-    DevBuf<uint32_t> mask32;
+    DevBuf<uint32_t> mask32(st);
     if (int rc = mask32.alloc(numtile * 8)) return rc;
     TSP_CK(cudaMemsetAsync(mask32.p, 0, numtile * 8 * sizeof(uint32_t), st));
     k_masks<<<blocks_for(nnz, TB), TB, 0, st>>>(idx, tid.p, rowOf, d_colidx, nnz, mask32.p);
     TSP_CK(cudaGetLastError());
     // ---- a4: selection
-    DevBuf<uint8_t> fmt0, aux0, sfmt;
-    DevBuf<int32_t> held, keep;
-    DevBuf<int64_t> size16;
-    DevBuf<unsigned long long> stats;
+    DevBuf<uint8_t> fmt0(st), aux0(st), sfmt(st);
+    DevBuf<int32_t> held(st), keep(st);
+    DevBuf<int64_t> size16(st);
+    DevBuf<unsigned long long> stats(st);
     if (int rc = fmt0.alloc(numtile)) return rc;
     if (int rc = aux0.alloc(numtile)) return rc;
     if (int rc = sfmt.alloc(numtile)) return rc;
@@ -467,7 +472,7 @@ int build_tiled_k(Matrix &M, const int32_t *d_rowptr, const int32_t *d_colidx, c
     TSP_CK(cudaGetLastError());
     // ---- remainder (DEFERRED)
     if (M.mode == TILESPMV_MODE_DEFERRED) {
-        DevBuf<int32_t> ext, pos;
+        DevBuf<int32_t> ext(st), pos(st);
         if (int rc = ext.alloc(nnz + 1)) return rc;
         if (int rc = pos.alloc(nnz + 1)) return rc;
         TSP_CK(cudaMemsetAsync(ext.p + nnz, 0, sizeof(int32_t), st));
@@ -481,10 +486,9 @@ int build_tiled_k(Matrix &M, const int32_t *d_rowptr, const int32_t *d_colidx, c
         if (int rc = read_scalar(pos.p + nnz, &nrem, st)) return rc;
         M.rem_nnz = nrem;
         if (nrem > 0) {
-            TSP_CK(cudaMalloc(&M.remRowPtr, (M.m + 1 + 8) * sizeof(int32_t)));  // + bulk-copy slack
-            TSP_CK(cudaMalloc(&M.remCol, (nrem + 4) * sizeof(int32_t)));
-            TSP_CK(cudaMalloc(&M.remVal, (nrem + 2) * sizeof(double)));
-            M.device_bytes += (M.m + 1) * 4 + (nrem + 4) * 4 + (nrem + 2) * 8;
+            TSP_CK(cudaMallocAsync(&M.remRowPtr, (M.m + 1 + 8) * sizeof(int32_t), st));  // + bulk-copy slack
+            TSP_CK(cudaMallocAsync(&M.remCol, (nrem + 4) * sizeof(int32_t), st));
+            TSP_CK(cudaMallocAsync(&M.remVal, (nrem + 2) * sizeof(double), st));
             k_rem_rowptr<<<blocks_for(M.m + 1, TB), TB, 0, st>>>(d_rowptr, pos.p, M.m, M.remRowPtr);
             k_rem_scatter<<<blocks_for(nnz, TB), TB, 0, st>>>(ext.p, pos.p, d_colidx, d_val, nnz,
                                                               M.remCol, M.remVal);
@@ -492,8 +496,8 @@ int build_tiled_k(Matrix &M, const int32_t *d_rowptr, const int32_t *d_colidx, c
         }
     }
     // ---- a5: kept tiles, prefix sums, tilePtr
-    DevBuf<int32_t> newId, nnzOff;
-    DevBuf<int64_t> off16;
+    DevBuf<int32_t> newId(st), nnzOff(st);
+    DevBuf<int64_t> off16(st);
     if (int rc = newId.alloc(numtile + 1)) return rc;
     if (int rc = nnzOff.alloc(numtile + 1)) return rc;
     if (int rc = off16.alloc(numtile + 1)) return rc;
@@ -513,16 +517,15 @@ int build_tiled_k(Matrix &M, const int32_t *d_rowptr, const int32_t *d_colidx, c
     if (total16 >= (int64_t(1) << 32)) return set_error(TILESPMV_OVERFLOW, "payload >= 64 GiB");
     M.numtile = nkept;
     M.payload_bytes = total16 * 16;
-    TSP_CK(cudaMalloc(&M.tilePtr, (M.tilem + 1) * sizeof(int32_t)));
-    TSP_CK(cudaMalloc(&M.tileColIdx, std::max<int64_t>(nkept, 1) * sizeof(int32_t)));
-    TSP_CK(cudaMalloc(&M.tileNnz, (nkept + 1) * sizeof(int32_t)));
-    TSP_CK(cudaMalloc(&M.tileFmt, std::max<int64_t>(nkept, 1)));
-    TSP_CK(cudaMalloc(&M.tileAux, std::max<int64_t>(nkept, 1)));
-    TSP_CK(cudaMalloc(&M.tileOff, (nkept + 1) * sizeof(uint32_t)));
+    TSP_CK(cudaMallocAsync(&M.tilePtr, (M.tilem + 1) * sizeof(int32_t), st));
+    TSP_CK(cudaMallocAsync(&M.tileColIdx, std::max<int64_t>(nkept, 1) * sizeof(int32_t), st));
+    TSP_CK(cudaMallocAsync(&M.tileNnz, (nkept + 1) * sizeof(int32_t), st));
+    TSP_CK(cudaMallocAsync(&M.tileFmt, std::max<int64_t>(nkept, 1), st));
+    TSP_CK(cudaMallocAsync(&M.tileAux, std::max<int64_t>(nkept, 1), st));
+    TSP_CK(cudaMallocAsync(&M.tileOff, (nkept + 1) * sizeof(uint32_t), st));
     // +64 bytes: the SpMV kernel never reads past the end, but keep a pad
-    TSP_CK(cudaMalloc(&M.payload, M.payload_bytes + 64));
-    M.device_bytes += (M.tilem + 1) * 4 + int64_t(nkept) * 14 + 8 + M.payload_bytes + 64;
-    DevBuf<int32_t> rowCount;
+    TSP_CK(cudaMallocAsync(&M.payload, M.payload_bytes + 64, st));
+    DevBuf<int32_t> rowCount(st);
     if (int rc = rowCount.alloc(M.tilem + 1)) return rc;
     TSP_CK(cudaMemsetAsync(rowCount.p, 0, (M.tilem + 1) * sizeof(int32_t), st));
     k_compact<K><<<blocks_for(numtile, TB), TB, 0, st>>>(
@@ -569,7 +572,7 @@ int build_tiled(Matrix &M, const int32_t *d_rowptr, const int32_t *d_colidx, con
     M.tilen = (M.n + kTile - 1) / kTile;
     // a1: validation
     if (validate && M.m > 0) {
-        DevBuf<int> bad;
+        DevBuf<int> bad(st);
         if (int rc = bad.alloc(1)) return rc;
         TSP_CK(cudaMemsetAsync(bad.p, 0, sizeof(int), st));
         k_check_rowptr<<<blocks_for(M.m + 1, TB), TB, 0, st>>>(d_rowptr, M.m, M.nnz, bad.p);
@@ -579,23 +582,22 @@ int build_tiled(Matrix &M, const int32_t *d_rowptr, const int32_t *d_colidx, con
         if (hbad) return set_error(TILESPMV_NOT_CANONICAL, "rowptr is not a monotone 0..nnz sequence");
     }
     if (M.nnz == 0) {  // no tiles, empty remainder
-        TSP_CK(cudaMalloc(&M.tilePtr, (M.tilem + 1) * sizeof(int32_t)));
+        TSP_CK(cudaMallocAsync(&M.tilePtr, (M.tilem + 1) * sizeof(int32_t), st));
         TSP_CK(cudaMemsetAsync(M.tilePtr, 0, (M.tilem + 1) * sizeof(int32_t), st));
-        TSP_CK(cudaMalloc(&M.tileNnz, sizeof(int32_t)));
+        TSP_CK(cudaMallocAsync(&M.tileNnz, sizeof(int32_t), st));
         TSP_CK(cudaMemsetAsync(M.tileNnz, 0, sizeof(int32_t), st));
-        TSP_CK(cudaMalloc(&M.tileOff, sizeof(uint32_t)));
+        TSP_CK(cudaMallocAsync(&M.tileOff, sizeof(uint32_t), st));
         TSP_CK(cudaMemsetAsync(M.tileOff, 0, sizeof(uint32_t), st));
-        TSP_CK(cudaMalloc(&M.payload, 64));
+        TSP_CK(cudaMallocAsync(&M.payload, 64, st));
         TSP_CK(cudaStreamSynchronize(st));
-        M.device_bytes += (M.tilem + 1) * 4 + 72;
         return 0;
     }
-    DevBuf<int32_t> rowOf;
+    DevBuf<int32_t> rowOf(st);
     if (int rc = rowOf.alloc(M.nnz)) return rc;
     k_expand_rows<<<blocks_for(M.m * 32, TB), TB, 0, st>>>(d_rowptr, M.m, rowOf.p);
     TSP_CK(cudaGetLastError());
     if (validate) {
-        DevBuf<int> bad;
+        DevBuf<int> bad(st);
         if (int rc = bad.alloc(1)) return rc;
         TSP_CK(cudaMemsetAsync(bad.p, 0, sizeof(int), st));
         k_check_cols<<<blocks_for(M.nnz, TB), TB, 0, st>>>(d_rowptr, d_colidx, rowOf.p, M.nnz, M.n, bad.p);

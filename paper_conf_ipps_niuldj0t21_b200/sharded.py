@@ -10,7 +10,10 @@ order as on one GPU and the gathered vector equals the 1-GPU y bitwise.
 
 The collective is torch.distributed (backend "nccl" on B200s, "gloo" in the
 CPU tests); `spmv` is any callable (x_full, y_out) -> None, normally
-TiledMatrix.run.
+TiledMatrix.run.  The bitwise claim needs every shard to run the kernel and
+mode of the unsharded matrix (the kernel fixes the work-item byte budget and
+so the order of the sums): build_shard_handles resolves AUTO from the global
+totals.
 """
 from __future__ import annotations
 
@@ -37,12 +40,54 @@ def partition_tile_rows(nrows: int, P: int, weights=None) -> list[int]:
     return [min(16 * t, nrows) for t in cuts[:-1]] + [nrows]
 
 
+def build_shard_handles(create, slices, nnz_local: int, mode="DEFERRED", kernel="AUTO", group=None,
+                        device=None):
+    """One handle per row slice of this rank, all with the mode and kernel the
+    unsharded matrix resolves to.
+
+    create(slice, mode_id, kernel_id) -> a handle with .info() and .close()
+    (normally TiledMatrix.from_csr of that slice).  AUTO mode follows reading
+    R18 on the global nnz (DEFERRED iff nnz >= 1.8e6); AUTO kernel is
+    tilespmv_auto_kernel of the global payload bytes and tile rows.  Both are
+    all-reduced over `group` (a collective: every rank calls this).
+    Returns (handles, mode_id, kernel_id)."""
+    import torch
+    import torch.distributed as dist
+    from .tilespmv import KERNELS, MODES, auto_kernel
+
+    def allsum(vals):
+        t = torch.tensor(vals, dtype=torch.int64, device=device)
+        if dist.is_available() and dist.is_initialized():
+            dist.all_reduce(t, group=group)
+        return [int(v) for v in t.cpu().tolist()]
+
+    md = MODES[mode] if isinstance(mode, str) else int(mode)
+    if md == MODES["AUTO"]:
+        (nnz,) = allsum([nnz_local])
+        md = MODES["DEFERRED"] if nnz >= 1_800_000 else MODES["ADPT"]
+    kn = KERNELS[kernel] if isinstance(kernel, str) else int(kernel)
+    k0 = KERNELS["SM_QUEUE"] if kn == KERNELS["AUTO"] else kn
+    hs = [create(s, md, k0) for s in slices]
+    if kn == KERNELS["AUTO"]:
+        infos = [h.info() for h in hs]
+        pay, tm = allsum([sum(i["payload_bytes"] for i in infos), sum(i["tilem"] for i in infos)])
+        kn = auto_kernel(pay, tm)
+        if kn != k0:
+            for h in hs:
+                h.close()
+            hs = [create(s, md, kn) for s in slices]
+    return hs, md, kn
+
+
 class ShardedSpMV:
     """One rank's side of the sharded iterated SpMV x_{k+1} = A x_k."""
 
     def __init__(self, spmv, bounds: list[int], rank: int, world: int, group=None, device=None,
-                 dtype=None):
+                 dtype=None, host_staging: bool = False):
+        """host_staging: gather through host buffers (a backend such as gloo
+        that cannot gather device tensors; development runs only)."""
         import torch
+        self.host_staging = host_staging
         self.spmv = spmv
         self.bounds = bounds
         self.rank, self.world, self.group = rank, world, group
@@ -60,12 +105,27 @@ class ShardedSpMV:
 
     def step(self, x_full, x_next=None):
         """y_local = A_local x_full, then all-gather into x_next (length m)."""
-        import torch
-        import torch.distributed as dist
         self.spmv(x_full, self.local_out())
+        self.exchange()
+        return self.assemble(x_next)
+
+    def exchange(self):
+        """All-gather of the ranks' y chunks into `gathered` (NCCL over
+        NVLink on B200s); a no-op without a process group."""
+        import torch.distributed as dist
         chunk = self.gathered[self.rank * self.maxrows:(self.rank + 1) * self.maxrows]
-        if self.world > 1:
+        if not (dist.is_available() and dist.is_initialized()):
+            return
+        if self.host_staging:
+            hg = self.gathered.new_empty(self.gathered.shape, device="cpu")
+            dist.all_gather_into_tensor(hg, chunk.cpu(), group=self.group)
+            self.gathered.copy_(hg)
+        else:
             dist.all_gather_into_tensor(self.gathered, chunk, group=self.group)
+
+    def assemble(self, x_next=None):
+        """The gathered vector as x_{k+1} (a view when shards are equal)."""
+        import torch
         if self.equal and x_next is None:
             return self.gathered[:self.m]
         if x_next is None:
@@ -118,7 +178,14 @@ class HaloPlan:
 
 def halo_needs(rowptr, colidx, bounds, rank):
     """(recv ranges, row parts) of rank's slice (rowptr rebased, global
-    columns).  Pure host logic: depends only on the slice's column pattern."""
+    columns).  Pure host logic: depends only on the slice's column pattern.
+
+    A received range covers whole 16-column tile segments: the tile kernels
+    stage x one 16-entry segment per tile (the x segment of a tile
+    column) and multiply stored zeros (Dns fill, ELL pads) by its entries, so
+    every entry of a touched segment must be a valid x value, not just the
+    columns that hold non-zeros.  Rank boundaries are multiples of 16, so a
+    widened range stays inside the peer's rows."""
     world = len(bounds) - 1
     a, b = int(bounds[rank]), int(bounds[rank + 1])
     cols = np.asarray(colidx)
@@ -129,7 +196,7 @@ def halo_needs(rowptr, colidx, bounds, rank):
         lo, hi = int(bounds[q]), int(bounds[q + 1])
         c = cols[(cols >= lo) & (cols < hi)]
         if c.size:
-            recv.append((q, int(c.min()), int(c.max()) + 1))
+            recv.append((q, max(lo, int(c.min()) // 16 * 16), min(hi, (int(c.max()) // 16 + 1) * 16)))
     # interior tile rows: every entry's column inside [a, b)
     mloc = b - a
     T = (mloc + 15) // 16

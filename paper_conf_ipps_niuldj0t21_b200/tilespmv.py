@@ -16,6 +16,7 @@ from . import _build
 
 FORMATS = ["CSR", "COO", "ELL", "HYB", "DNS", "DNSROW", "DNSCOL"]
 MODES = {"ADPT": 0, "DEFERRED": 1, "AUTO": 2, "FORCE_CSR": 3}
+KERNELS = {"AUTO": 0, "SM_QUEUE": 1, "DENSE_ROWS": 2}
 ARRAYS = {"tilePtr": (0, np.int32), "tileColIdx": (1, np.int32), "tileNnz": (2, np.int32),
           "tileFmt": (3, np.uint8), "tileAux": (4, np.uint8), "tileOff": (5, np.uint32),
           "payload": (6, np.uint8), "remRowPtr": (7, np.int32), "remCol": (8, np.int32),
@@ -23,7 +24,8 @@ ARRAYS = {"tilePtr": (0, np.int32), "tileColIdx": (1, np.int32), "tileNnz": (2, 
 EXPORTED_SYMBOLS = ["tilespmv_create_from_csr", "tilespmv_run", "tilespmv_run_host",
                     "tilespmv_destroy", "tilespmv_get_info", "tilespmv_export_size",
                     "tilespmv_export", "tilespmv_status_string", "tilespmv_last_error",
-                    "tilespmv_launch_shape", "tilespmv_kernel_name", "tilespmv_cg"]
+                    "tilespmv_launch_shape", "tilespmv_kernel_name", "tilespmv_cg",
+                    "tilespmv_auto_kernel"]
 
 
 class TileSpMVError(RuntimeError):
@@ -31,7 +33,8 @@ class TileSpMVError(RuntimeError):
 
 
 class Opts(ctypes.Structure):
-    _fields_ = [("mode", ctypes.c_int32), ("validate", ctypes.c_int32)]
+    _fields_ = [("mode", ctypes.c_int32), ("validate", ctypes.c_int32), ("kernel", ctypes.c_int32),
+                ("keep_layout", ctypes.c_int32)]
 
 
 class Info(ctypes.Structure):
@@ -44,7 +47,7 @@ class Info(ctypes.Structure):
                 ("meta_bytes", ctypes.c_int64), ("alg_bytes", ctypes.c_int64),
                 ("flops", ctypes.c_int64), ("num_items", ctypes.c_int64),
                 ("num_split_rows", ctypes.c_int64), ("device_bytes", ctypes.c_int64),
-                ("create_ms", ctypes.c_double)]
+                ("create_ms", ctypes.c_double), ("kernel", ctypes.c_int32), ("reserved", ctypes.c_int32)]
 
     def as_dict(self) -> dict:
         d = {}
@@ -87,6 +90,9 @@ def load(build_if_missing: bool = True):
     L.tilespmv_launch_shape.argtypes = [p, ctypes.POINTER(i32), ctypes.POINTER(i32),
                                         ctypes.POINTER(i32)]
     L.tilespmv_cg.argtypes = [p, p, p, ctypes.c_double, i32, ctypes.POINTER(i32), ctypes.POINTER(ctypes.c_double), p]
+    if hasattr(L, "tilespmv_auto_kernel"):  # (absent from round-1 builds used in A/B runs)
+        L.tilespmv_auto_kernel.argtypes = [i64, i64]
+        L.tilespmv_auto_kernel.restype = i32
     L.tilespmv_kernel_name.argtypes = [p]
     L.tilespmv_kernel_name.restype = ctypes.c_char_p
     for name in ("tilespmv_create_from_csr", "tilespmv_run", "tilespmv_run_host",
@@ -95,6 +101,11 @@ def load(build_if_missing: bool = True):
         getattr(L, name).restype = ctypes.c_int
     _lib = L
     return L
+
+
+def auto_kernel(payload_bytes: int, tilem: int) -> int:
+    """TILESPMV_KERNEL_AUTO's choice for these totals (tilespmv_auto_kernel)."""
+    return int(load().tilespmv_auto_kernel(int(payload_bytes), int(tilem)))
 
 
 def _check(rc: int, what: str):
@@ -127,8 +138,11 @@ class TiledMatrix:
     # ---------------------------------------------------------------- create
     @classmethod
     def from_csr(cls, rowptr, colidx, val, m: int, n: int, mode: str | int = "DEFERRED",
-                 validate: bool = True, stream=None) -> "TiledMatrix":
-        """rowptr/colidx (int32) and val (float64) are CUDA tensors."""
+                 validate: bool = True, stream=None, kernel: str | int = "AUTO",
+                 keep_layout: bool = False) -> "TiledMatrix":
+        """rowptr/colidx (int32) and val (float64) are CUDA tensors.  kernel:
+        TILESPMV_KERNEL_* by name or number; keep_layout: keep the canonical
+        tiled arrays for export() (tests)."""
         import torch
         _require_cuda()
         for t, dt in ((rowptr, torch.int32), (colidx, torch.int32), (val, torch.float64)):
@@ -136,7 +150,8 @@ class TiledMatrix:
                 raise TileSpMVError("rowptr/colidx must be contiguous CUDA int32, val CUDA float64")
         L = load()
         md = MODES[mode] if isinstance(mode, str) else int(mode)
-        opts = Opts(md, int(validate))
+        kn = KERNELS[kernel] if isinstance(kernel, str) else int(kernel)
+        opts = Opts(md, int(validate), kn, int(keep_layout))
         h = ctypes.c_void_p()
         nnz = int(colidx.numel())
         rc = L.tilespmv_create_from_csr(ctypes.byref(h), m, n, nnz, rowptr.data_ptr(),
@@ -147,7 +162,8 @@ class TiledMatrix:
         return cls(h.value, m, n)
 
     @classmethod
-    def from_host_csr(cls, A, mode="DEFERRED", validate=True, device=None, stream=None):
+    def from_host_csr(cls, A, mode="DEFERRED", validate=True, device=None, stream=None, kernel="AUTO",
+                      keep_layout=False):
         """Copies a host CSR (synthetic.gen.CSR-like: m, n, rowptr, colidx, val)."""
         import torch
         _require_cuda()
@@ -155,7 +171,7 @@ class TiledMatrix:
         rp = torch.from_numpy(np.ascontiguousarray(A.rowptr, np.int32)).to(dev)
         ci = torch.from_numpy(np.ascontiguousarray(A.colidx, np.int32)).to(dev)
         va = torch.from_numpy(np.ascontiguousarray(A.val, np.float64)).to(dev)
-        return cls.from_csr(rp, ci, va, A.m, A.n, mode, validate, stream)
+        return cls.from_csr(rp, ci, va, A.m, A.n, mode, validate, stream, kernel, keep_layout)
 
     # -------------------------------------------------------------------- run
     def run(self, x, y=None, stream=None):

@@ -20,12 +20,13 @@ for A in mats:
     x = gen.dense_x(A.n, 101)
     yref, absy = O.spmv(A, x)
     for mode in ("ADPT", "DEFERRED"):
-        M = TiledMatrix.from_host_csr(A, mode=mode)
-        y = M.run(torch.from_numpy(x).cuda()).cpu().numpy()
-        ok = np.all(np.abs(y - yref) <= 1e-12 * absy + 1e-300)
-        bad += not ok
-        print(A.name, mode, "ok" if ok else "MISMATCH", flush=True)
-        M.close()
+        for kernel in ("SM_QUEUE", "DENSE_ROWS"):
+            M = TiledMatrix.from_host_csr(A, mode=mode, kernel=kernel)
+            y = M.run(torch.from_numpy(x).cuda()).cpu().numpy()
+            ok = np.all(np.abs(y - yref) <= 1e-12 * absy + 1e-300)
+            bad += not ok
+            print(A.name, mode, kernel, "ok" if ok else "MISMATCH", flush=True)
+            M.close()
 torch.cuda.synchronize()
 print("sanitize_small done, mismatches:", bad)
 sys.exit(1 if bad else 0)

@@ -5,7 +5,7 @@ pair extents 6..8 and 13..16 -- and ragged rows of 0..16 entries), mixed with
 sparse COO-sized tiles, dense tiles and remainder-heavy rows, on ragged
 m, n.  Each run is checked against the oracle SpMV within the north_star
 tolerance (fp64) and for run-to-run bitwise determinism, in every mode
- and on the default and two other kernel variants."""
+ on both SpMV kernels."""
 import numpy as np
 import pytest
 
@@ -52,21 +52,20 @@ CASES = [(128, 128, 0, "equal"), (125, 131, 1, "equal"), (200, 96, 2, "ragged"),
 
 
 @pytest.mark.gpu
-@pytest.mark.parametrize("variant", ["43", "40", "25"])
-def test_tile_profile_fuzz(cuda_device, variant, monkeypatch):
+@pytest.mark.parametrize("kernel", ["SM_QUEUE", "DENSE_ROWS"])
+def test_tile_profile_fuzz(cuda_device, kernel):
     import torch
     from paper_conf_ipps_niuldj0t21_b200 import TiledMatrix
-    monkeypatch.setenv("TILESPMV_KERNEL", variant)
     for (m, n, seed, profile) in CASES:
         A = tile_profile_matrix(m, n, seed, profile)
         x = gen.dense_x(n, 7 + seed)
         yref, absy = O.spmv(A, x)
         xd = torch.from_numpy(x).to(cuda_device)
         for mode in ("ADPT", "DEFERRED", "FORCE_CSR"):
-            M = TiledMatrix.from_host_csr(A, mode=mode, device=cuda_device)
+            M = TiledMatrix.from_host_csr(A, mode=mode, device=cuda_device, kernel=kernel)
             y1 = M.run(xd).cpu().numpy()
             y2 = M.run(xd).cpu().numpy()
-            assert_spmv_close(y1, yref, absy, f"{profile}{seed}/{mode}/v{variant}")
+            assert_spmv_close(y1, yref, absy, f"{profile}{seed}/{mode}/{kernel}")
             assert np.array_equal(y1.view(np.uint64), y2.view(np.uint64))
             M.close()
 

@@ -154,3 +154,45 @@ def test_cpu_csr_omp_baseline_matches_oracle():
         yr, absy = O.spmv(A, x)
         assert threads >= 1
         assert np.all(np.abs(y - yr) <= 1e-12 * absy + 1e-300), name
+
+
+# ---------------------------------------------------------------------------
+# oracle_spmv_f64: Alg. 1 as printed, in double (the CPU baseline of bench.py)
+# ---------------------------------------------------------------------------
+
+def test_f64_row_loop_identity_diagonal_permutation_exact():
+    A = gen.identity(300)
+    x = gen.dense_x(300, 5)
+    assert np.array_equal(O.spmv_f64(A, x), x)
+    D = gen.diagonal(257)
+    assert np.array_equal(O.spmv_f64(D, gen.dense_x(257, 6)), D.val * gen.dense_x(257, 6))
+    P, pi = gen.permutation(129)
+    xp = gen.dense_x(129, 7)
+    assert np.array_equal(O.spmv_f64(P, xp), O.spmv(P, xp)[0])
+
+
+def test_f64_row_loop_sums_left_to_right_in_double():
+    """y_i <- y_i + a_ij x_j in entry order, each step rounded to double
+    (ulp(1e16) = 2, so 1e16 + 1 rounds back to 1e16): the three orders of
+    {1e16, 1, -1e16} give 0, 0 and 1, where the extended-precision oracle
+    gives 1 for all three."""
+    rows = [0, 0, 0, 1, 1, 1, 2, 2, 2]
+    cols = [0, 1, 2, 0, 1, 2, 0, 1, 2]
+    vals = [1e16, 1.0, -1e16, 1.0, 1e16, -1e16, 1e16, -1e16, 1.0]
+    A = gen.csr_from_coo(3, 3, rows, cols, vals=vals, name="order")
+    y = O.spmv_f64(A, np.ones(3))
+    assert y.tolist() == [0.0, 0.0, 1.0]
+    assert O.spmv(A, np.ones(3))[0].tolist() == [1.0, 1.0, 1.0]
+
+
+def test_f64_row_loop_integer_exact_and_within_bound():
+    A = gen.stencil27(11, values="int", seed=3)
+    x = gen.dense_x(A.n, 5, kind="int")
+    assert np.array_equal(O.spmv_f64(A, x), O.spmv(A, x)[0])
+    for name in ("rmat12", "mixed_small", "lap2d_37x29"):
+        A, x = gen.make(name)
+        y = O.spmv_f64(A, x)
+        yref, absy = O.spmv(A, x)
+        k = np.diff(A.rowptr.astype(np.int64))
+        # sequential fp64 sum of k products: |err| <= (k + 1) u sum|a x| (u = 2^-53)
+        assert np.all(np.abs(y - yref) <= (k + 1) * 2.0 ** -53 * absy * (1 + 1e-9))
