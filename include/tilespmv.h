@@ -47,10 +47,15 @@ extern "C" {
  * y within the north-star bound; the work-item byte budget (and so the
  * order of the sums) is the kernel's, so handles that must agree bitwise
  * (row slices of one matrix, tilespmv sharding) must use the same kernel. */
-#define TILESPMV_KERNEL_AUTO 0       /* DENSE_ROWS if the mean stored payload per tile row exceeds
+#define TILESPMV_KERNEL_AUTO 0       /* GATHER if the CSR remainder holds more than half of the
+                                        algorithmic bytes (power-law graphs in DEFERRED mode), else
+                                        DENSE_ROWS if the mean stored payload per tile row exceeds
                                         6 KiB (dense, FEM-like tile rows), else SM_QUEUE          */
 #define TILESPMV_KERNEL_SM_QUEUE 1   /* one 32-warp CTA per SM, 4.5 KiB items, shared-memory queue */
 #define TILESPMV_KERNEL_DENSE_ROWS 2 /* 16 warps per SM, 10.5 KiB items, static per-warp chunks    */
+#define TILESPMV_KERNEL_GATHER 3     /* SM_QUEUE with 2.25 KiB items of at most 8 tiles: 115 KiB of
+                                        shared memory per SM instead of 222 KiB leaves ~140 KiB of
+                                        L1 to the remainder's x gathers                            */
 
 /* tile format codes, in the order of P:20 / P:96 */
 #define TILESPMV_FMT_CSR 0
@@ -172,11 +177,12 @@ int64_t tilespmv_export_size(tilespmv_handle_t h, int32_t which);
 int tilespmv_export(tilespmv_handle_t h, int32_t which, void *host_dst, size_t bytes);
 
 /* The kernel TILESPMV_KERNEL_AUTO resolves to for a matrix whose stored
- * tile payload is payload_bytes over tilem tile rows (tilespmv_info_t).
+ * tile payload is payload_bytes over tilem tile rows, with rem_nnz
+ * remainder entries and alg_bytes algorithmic bytes (tilespmv_info_t).
  * Sharded callers apply it to the whole matrix's totals so that every shard
  * runs the kernel (and the item byte budget) of the unsharded matrix, and so
  * the unsharded summation order.                                            */
-int32_t tilespmv_auto_kernel(int64_t payload_bytes, int64_t tilem);
+int32_t tilespmv_auto_kernel(int64_t payload_bytes, int64_t tilem, int64_t rem_nnz, int64_t alg_bytes);
 
 /* Static description of a status code. */
 const char *tilespmv_status_string(int status);

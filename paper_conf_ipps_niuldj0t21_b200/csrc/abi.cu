@@ -44,7 +44,7 @@ static void free_matrix(tilespmv_matrix *M) {
     delete M;
 }
 
-static int64_t alg_bytes(const Matrix &M) {
+int64_t alg_bytes(const Matrix &M) {
     // DESIGN.md §"Bytes model": payload + 14 B of level-1 meta
     // per stored tile + tilePtr + remainder CSR (if any) + x read once + y
     // written once.
@@ -88,7 +88,7 @@ int tilespmv_create_from_csr(tilespmv_handle_t *out, int64_t m, int64_t n, int64
     tilespmv_opts_t o{TILESPMV_MODE_DEFERRED, 1, TILESPMV_KERNEL_AUTO, 0};
     if (opts) o = *opts;
     if (o.mode < 0 || o.mode > 3) return set_error(TILESPMV_INVALID_ARG, "unknown mode");
-    if (o.kernel < TILESPMV_KERNEL_AUTO || o.kernel > TILESPMV_KERNEL_DENSE_ROWS)
+    if (o.kernel < TILESPMV_KERNEL_AUTO || o.kernel > TILESPMV_KERNEL_GATHER)
         return set_error(TILESPMV_INVALID_ARG, "unknown kernel");
     if (o.keep_layout != 0 && o.keep_layout != 1) return set_error(TILESPMV_INVALID_ARG, "keep_layout must be 0 or 1");
     auto t0 = std::chrono::steady_clock::now();
@@ -290,6 +290,8 @@ int tilespmv_launch_shape(tilespmv_handle_t h, int32_t *grid, int32_t *block, in
 
 const char *tilespmv_kernel_name(tilespmv_handle_t h) { return h ? h->kernel_name : ""; }
 
-int32_t tilespmv_auto_kernel(int64_t payload_bytes, int64_t tilem) { return auto_kernel(payload_bytes, tilem); }
+int32_t tilespmv_auto_kernel(int64_t payload_bytes, int64_t tilem, int64_t rem_nnz, int64_t alg) {
+    return auto_kernel(payload_bytes, tilem, rem_nnz, alg);
+}
 
 }  // extern "C"

@@ -18,10 +18,11 @@ enum : uint8_t { F_CSR = 0, F_COO = 1, F_ELL = 2, F_HYB = 3, F_DNS = 4, F_DNSROW
 
 // ---------------------------------------------------------------------------
 // SpMV schedule.  A work item is a byte-bounded piece of one tile row: a run
-// of at most kItemTiles consecutive tiles and/or a range of remainder entries
-// of the tile row's 16 rows, such that everything the kernel stages for it
-// (payloads, 8-byte tile descriptors, remainder rowptr/col/val) fits one
-// shared-memory slot (the kernel's slot size, <= kItemBytesMax).  A tile row split over several items writes
+// of at most kItemTiles (the kernel's item_tiles) consecutive tiles and/or a
+// range of remainder entries of the tile row's 16 rows, such that everything
+// the kernel stages for it (payloads, 8-byte tile descriptors, remainder
+// rowptr/col/val) fits one shared-memory slot (the kernel's slot size,
+// <= kItemBytesMax).  A tile row split over several items writes
 // per-item partials that the last finishing item sums in item order
 // (deterministic; replaces the atomic merge of tbalance).  Item
 // boundaries depend only on the tile row's own content, so a tile-row-sharded
@@ -142,6 +143,7 @@ struct Matrix {
     int kernel = TILESPMV_KERNEL_SM_QUEUE;  // resolved kernel (never AUTO)
     const char *kernel_name = "";
     int item_bytes = kItemBytesMax;  // slot size the schedule was built for
+    int item_tiles = kItemTiles;     // tiles per item (the kernel's x stage)
     int grid = 0, block = 0, smem = 0;
 };
 
@@ -153,7 +155,8 @@ int cuda_status(cudaError_t e, const char *what);
 int build_tiled(Matrix &M, const int32_t *d_rowptr, const int32_t *d_colidx, const double *d_val,
                 int validate, cudaStream_t stream);
 // schedule.cu
-int auto_kernel(int64_t payload_bytes, int64_t tilem);
+int auto_kernel(int64_t payload_bytes, int64_t tilem, int64_t rem_nnz, int64_t alg_bytes);
+int64_t alg_bytes(const Matrix &M);  // abi.cu
 int choose_kernel(Matrix &M, int requested);
 int build_schedule(Matrix &M, cudaStream_t stream);
 int build_tdesc(Matrix &M, cudaStream_t stream);

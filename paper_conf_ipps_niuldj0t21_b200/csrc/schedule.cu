@@ -29,7 +29,8 @@ namespace {
 // row's remainder entries.  Depends only on the tile row's own content.
 template <bool WRITE>
 __device__ int items_for_row(int64_t I, const int32_t *tilePtr, const uint32_t *tileOff, const int32_t *remRowPtr,
-                             int64_t m, int budget, Item *out, int split, int nparts = 0, int lp = kLocalParts) {
+                             int64_t m, int budget, int max_tiles, Item *out, int split, int nparts = 0,
+                             int lp = kLocalParts) {
     const int tp0 = tilePtr[I], tp1 = tilePtr[I + 1];
     int k0 = 0, k1 = 0;
     if (remRowPtr) {
@@ -42,7 +43,7 @@ __device__ int items_for_row(int64_t I, const int32_t *tilePtr, const uint32_t *
     do {
         const int tb = t;
         uint32_t used = 0;
-        while (t < tp1 && t - tb < kItemTiles) {
+        while (t < tp1 && t - tb < max_tiles) {
             const uint32_t pay = (tileOff[t + 1] - tileOff[tb]) * 16u;
             // blob: descriptor list (<= ntiles + 7 pads) + J array (blob_parts)
             const uint32_t dsc = up16(8u * (uint32_t)(t - tb + 1 + 7)) + up16(4u * (uint32_t)(t - tb + 1));
@@ -88,10 +89,11 @@ __device__ int items_for_row(int64_t I, const int32_t *tilePtr, const uint32_t *
 }
 
 __global__ void k_items_count(const int32_t *tilePtr, const uint32_t *tileOff, const int32_t *remRowPtr, int64_t m,
-                              int budget, int64_t tilem, int32_t *nitems, int32_t *nsplit, int32_t *parts) {
+                              int budget, int max_tiles, int64_t tilem, int32_t *nitems, int32_t *nsplit,
+                              int32_t *parts) {
     int64_t I = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     if (I >= tilem) return;
-    const int c = items_for_row<false>(I, tilePtr, tileOff, remRowPtr, m, budget, nullptr, -1);
+    const int c = items_for_row<false>(I, tilePtr, tileOff, remRowPtr, m, budget, max_tiles, nullptr, -1);
     nitems[I] = c;
     nsplit[I] = c > 1 ? 1 : 0;
     parts[I] = c > 1 ? c : 0;
@@ -108,14 +110,14 @@ __device__ __forceinline__ bool groupable(int64_t I, const int32_t *tilePtr, con
 // within budget).  group = false: no row-group items (kernels without them).
 template <bool WRITE>
 __device__ int window_items(int64_t w, const int32_t *tilePtr, const uint32_t *tileOff, const int32_t *remRowPtr,
-                            int64_t m, int budget, int64_t tilem, bool group, const int32_t *nitems,
-                            const int32_t *splitId, Item *out, int lp) {
+                            int64_t m, int budget, int max_tiles, int64_t tilem, bool group,
+                            const int32_t *nitems, const int32_t *splitId, Item *out, int lp) {
     const int64_t I0 = w * kGroupWindow, I1 = imin64(I0 + kGroupWindow, tilem);
     int cnt = 0;
     int64_t I = I0;
     while (I < I1) {
         if (!group || !groupable(I, tilePtr, nitems)) {
-            if (WRITE) items_for_row<true>(I, tilePtr, tileOff, remRowPtr, m, budget, out + cnt,
+            if (WRITE) items_for_row<true>(I, tilePtr, tileOff, remRowPtr, m, budget, max_tiles, out + cnt,
                                            nitems[I] > 1 ? splitId[I] : -1, nitems[I], lp);
             cnt += nitems[I];
             ++I;
@@ -152,21 +154,21 @@ __device__ int window_items(int64_t w, const int32_t *tilePtr, const uint32_t *t
 }
 
 __global__ void k_window_count(const int32_t *tilePtr, const uint32_t *tileOff, const int32_t *remRowPtr, int64_t m,
-                               int budget, int64_t tilem, int group, const int32_t *nitems, int64_t nwin,
-                               int32_t *wcount) {
+                               int budget, int max_tiles, int64_t tilem, int group, const int32_t *nitems,
+                               int64_t nwin, int32_t *wcount) {
     const int64_t w = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     if (w >= nwin) return;
-    wcount[w] = window_items<false>(w, tilePtr, tileOff, remRowPtr, m, budget, tilem, group != 0, nitems, nullptr,
-                                    nullptr, kLocalParts);
+    wcount[w] = window_items<false>(w, tilePtr, tileOff, remRowPtr, m, budget, max_tiles, tilem, group != 0, nitems,
+                                    nullptr, nullptr, kLocalParts);
 }
 
 __global__ void k_window_write(const int32_t *tilePtr, const uint32_t *tileOff, const int32_t *remRowPtr, int64_t m,
-                               int budget, int64_t tilem, int group, const int32_t *nitems, int64_t nwin,
-                               const int32_t *wbase, const int32_t *splitId, const int32_t *partBase, Item *items,
-                               int2 *split_info, int lp) {
+                               int budget, int max_tiles, int64_t tilem, int group,
+                               const int32_t *nitems, int64_t nwin, const int32_t *wbase, const int32_t *splitId,
+                               const int32_t *partBase, Item *items, int2 *split_info, int lp) {
     const int64_t w = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     if (w >= nwin) return;
-    window_items<true>(w, tilePtr, tileOff, remRowPtr, m, budget, tilem, group != 0, nitems, splitId,
+    window_items<true>(w, tilePtr, tileOff, remRowPtr, m, budget, max_tiles, tilem, group != 0, nitems, splitId,
                        items + wbase[w], lp);
     const int64_t I1 = imin64((w + 1) * kGroupWindow, tilem);
     for (int64_t I = w * kGroupWindow; I < I1; ++I)
@@ -460,9 +462,10 @@ int build_schedule(Matrix &M, cudaStream_t st) {
             *wbase = wcount + (NW + 1);
     TSP_CK(cudaMemsetAsync(nitems, 0, 3 * (T + 1) * sizeof(int32_t), st));
     TSP_CK(cudaMemsetAsync(wcount, 0, (NW + 1) * sizeof(int32_t), st));
-    k_items_count<<<blocks(T), TB, 0, st>>>(M.tilePtr, M.tileOff, M.remRowPtr, M.m, M.item_bytes, T, nitems, nsplit, parts);
-    k_window_count<<<blocks(NW), TB, 0, st>>>(M.tilePtr, M.tileOff, M.remRowPtr, M.m, M.item_bytes, T, group, nitems,
-                                               NW, wcount);
+    k_items_count<<<blocks(T), TB, 0, st>>>(M.tilePtr, M.tileOff, M.remRowPtr, M.m, M.item_bytes, M.item_tiles, T,
+                                            nitems, nsplit, parts);
+    k_window_count<<<blocks(NW), TB, 0, st>>>(M.tilePtr, M.tileOff, M.remRowPtr, M.m, M.item_bytes, M.item_tiles, T,
+                                               group, nitems, NW, wcount);
     TSP_CK(cudaGetLastError());
     if (int rc = scan([&](void *t, size_t &b) { return cub::DeviceScan::ExclusiveSum(t, b, wcount, wbase, (int)(NW + 1), st); }, st)) return rc;
     if (int rc = scan([&](void *t, size_t &b) { return cub::DeviceScan::ExclusiveSum(t, b, nsplit, splitId, (int)(T + 1), st); }, st)) return rc;
@@ -483,8 +486,9 @@ int build_schedule(Matrix &M, cudaStream_t st) {
     // whole records (padding included) are copied later: start from zeros
     TSP_CK(cudaMemsetAsync(M.items, 0, std::max<int64_t>(M.num_items, 1) * sizeof(Item), st));
     TSP_CK(cudaMemsetAsync(M.counters, 0, std::max<int64_t>(M.num_split, 1) * sizeof(int32_t), st));
-    k_window_write<<<blocks(NW), TB, 0, st>>>(M.tilePtr, M.tileOff, M.remRowPtr, M.m, M.item_bytes, T, group, nitems,
-                                               NW, wbase, splitId, partBase, M.items, M.split_info, kLocalParts);
+    k_window_write<<<blocks(NW), TB, 0, st>>>(M.tilePtr, M.tileOff, M.remRowPtr, M.m, M.item_bytes, M.item_tiles, T,
+                                               group, nitems, NW, wbase, splitId, partBase, M.items, M.split_info,
+                                               kLocalParts);
     TSP_CK(cudaGetLastError());
     return 0;
 }
@@ -541,7 +545,10 @@ int build_tdesc(Matrix &M, cudaStream_t st) {
     return 0;
 }
 
-int auto_kernel(int64_t payload_bytes, int64_t tilem) {
+int auto_kernel(int64_t payload_bytes, int64_t tilem, int64_t rem_nnz, int64_t alg) {
+    // the remainder's bytes (12 per entry) are most of what the SpMV moves:
+    // its x gathers need the L1 that the big-slot kernels give to shared memory
+    if (2 * 12 * rem_nnz > alg) return TILESPMV_KERNEL_GATHER;
     // integer form of "mean payload per tile row > 6 KiB"
     return tilem > 0 && payload_bytes > 6144 * tilem ? TILESPMV_KERNEL_DENSE_ROWS : TILESPMV_KERNEL_SM_QUEUE;
 }
@@ -554,9 +561,12 @@ int choose_kernel(Matrix &M, int requested) {
     // one item.  Measured in round 1 (graph-replayed launches, profiles/):
     // C5 498 us (SM queue) vs 512 us (static chunks); R-MAT 145 vs 163 us;
     // mixed 113 vs 116 us; C2 6.9 us (dense-row) vs 7.5 us (SM queue, 10.5 KB).
-    const int k = requested == TILESPMV_KERNEL_AUTO ? auto_kernel(M.payload_bytes, M.tilem) : requested;
+    const int k = requested == TILESPMV_KERNEL_AUTO ? auto_kernel(M.payload_bytes, M.tilem, M.rem_nnz, alg_bytes(M))
+                                                    : requested;
+    const KernelChoice kc = kernel_choice(k);
     M.kernel = k;
-    M.item_bytes = kernel_choice(k).slot_bytes;
+    M.item_bytes = kc.slot_bytes;
+    M.item_tiles = kc.item_tiles;
     return 0;
 }
 

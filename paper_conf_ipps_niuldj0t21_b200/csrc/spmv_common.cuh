@@ -129,6 +129,11 @@ __device__ __forceinline__ void cp_async16(uint32_t dst, const void *src, uint32
                  "r"(src_bytes), "l"(policy)
                  : "memory");
 }
+// 8-byte async copy global -> shared (an x gather; .ca: the L1 may hold hot x lines)
+__device__ __forceinline__ void cp_async8(uint32_t dst, const void *src, uint64_t policy) {
+    asm volatile("cp.async.ca.shared.global.L2::cache_hint [%0], [%1], 8, %2;" ::"r"(dst), "l"(src), "l"(policy)
+                 : "memory");
+}
 __device__ __forceinline__ void cp_async_wait_all() {
     asm volatile("cp.async.commit_group;\n\tcp.async.wait_group 0;" ::: "memory");
 }
@@ -146,15 +151,16 @@ __device__ __forceinline__ void fma_if(bool pred, double a, double b, double &ac
         : "d"(a), "d"(b), "r"((unsigned)pred));
 }
 
-// the two SpMV kernels (spmv_warp.cu)
+// the SpMV kernels (spmv_warp.cu)
 struct KernelChoice {
     const char *name;
     void (*fn)(Params);
     int threads, smem;
-    int slot_bytes;  // item budget the schedule must respect
-    bool sm_queue;   // one CTA per SM; its warps claim units from a shared-memory counter
+    int slot_bytes;   // item budget the schedule must respect
+    int item_tiles;   // tiles per item (x stage segments)
+    bool sm_queue;    // one CTA per SM; its warps claim units from a shared-memory counter
 };
-// TILESPMV_KERNEL_SM_QUEUE or TILESPMV_KERNEL_DENSE_ROWS
+// TILESPMV_KERNEL_SM_QUEUE, _DENSE_ROWS or _GATHER
 KernelChoice kernel_choice(int kernel);
 
 }  // namespace tsp

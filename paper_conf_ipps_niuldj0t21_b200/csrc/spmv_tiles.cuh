@@ -48,6 +48,15 @@ __device__ __forceinline__ double lds_f64_lt(int i, int len, uint32_t a) {
         : "r"(i), "r"(len), "r"(a));
     return v;
 }
+// a remainder entry k (column, value) if k < e, else (cdef, 0.0): cdef is a
+// column the item itself references (so x[cdef] is a valid, finite x entry
+// on any rank that runs the item) and 0.0 * x[cdef] adds an exact zero
+__device__ __forceinline__ void lds_entry_or(int k, int e, uint32_t ca, uint32_t va, int cdef, int &c, double &v) {
+    asm("{\n\t.reg .pred q;\n\tsetp.lt.s32 q, %2, %3;\n\tmov.b32 %0, %6;\n\tmov.b64 %1, 0;\n\t"
+        "@q ld.shared.s32 %0, [%4];\n\t@q ld.shared.f64 %1, [%5];\n\t}"
+        : "=r"(c), "=d"(v)
+        : "r"(k), "r"(e), "r"(ca), "r"(va), "r"(cdef));
+}
 // a remainder entry k (column, value) if k < e, else (0, 0.0)
 __device__ __forceinline__ void lds_entry_lt(int k, int e, uint32_t ca, uint32_t va, int &c, double &v) {
     asm("{\n\t.reg .pred q;\n\tsetp.lt.s32 q, %2, %3;\n\tmov.b32 %0, 0;\n\tmov.b64 %1, 0;\n\t"

@@ -17,12 +17,18 @@
 // Latency is hidden by warp count; the next item's record is prefetched into
 // registers.  No floating-point atomics: y is bitwise deterministic.
 //
-// Two kernels share this item code (schedule.cu picks one per handle):
-//   tilespmv_fp64_sm<32,4608>    one CTA of 32 warps per SM, 4.5 KB slots,
-//                                 warps claim units from a shared-memory queue
-//   tilespmv_fp64_warp<4,10752>  16 warps per SM, 10.5 KB slots, a static
-//                                 cost-balanced item chunk per warp (dense
-//                                 tile rows: one tile row stays one item)
+// Three kernels share this item code (schedule.cu picks one per handle):
+//   tilespmv_fp64_sm<32,4608,16> SM_QUEUE: one CTA of 32 warps per SM, 4.5 KB
+//                                 slots, warps claim units from a
+//                                 shared-memory queue (222 KB of shared memory)
+//   tilespmv_fp64_sm<32,2304,8>  GATHER: the same with 2.25 KB slots and at
+//                                 most 8 tiles per item (115 KB): the L1 left
+//                                 to the remainder's x gathers grows from ~30
+//                                 to ~140 KB (power-law matrices in DEFERRED
+//                                 mode: R-MAT 127.6 -> 114.2 us)
+//   tilespmv_fp64_warp<4,10752>  DENSE_ROWS: 16 warps per SM, 10.5 KB slots,
+//                                 a static cost-balanced item chunk per warp
+//                                 (dense tile rows: one tile row stays one item)
 #include "spmv_tiles.cuh"
 
 namespace tsp {
@@ -55,12 +61,13 @@ __device__ __forceinline__ unsigned long long gtimer() {
 
 namespace {
 
-template <int WARPS, int SLOT>
+
+template <int WARPS, int SLOT, int XT = kItemTiles>
 struct WarpCfg {
-    static_assert(SLOT % 16 == 0 && SLOT <= kItemBytesMax, "slot size");
-    // [x stage of every warp, 2 KB each, 128-byte aligned] [per warp: slot |
+    static_assert(SLOT % 16 == 0 && SLOT <= kItemBytesMax && XT % 4 == 0 && XT <= kItemTiles, "slot size");
+    // [x stage of every warp, XT x 128 B, 128-byte aligned] [per warp: slot |
     // row-sum scratch of the COO scan (256 B) | mbarrier]
-    static constexpr uint32_t kX = kItemTiles * 16 * 8;
+    static constexpr uint32_t kX = XT * 16 * 8;
     static constexpr uint32_t kRacc = 256;
     static constexpr uint32_t kPer = SLOT + kRacc + 16;
     static constexpr uint32_t kSmem = WARPS * (kX + kPer) + 256;  // +256: loads may overrun a slot
@@ -77,91 +84,114 @@ __device__ __forceinline__ WItem load_witem(const WItem *w, int k) {
 }
 
 // ------------------------------------------------ fused CSR remainder -------
-// One 32-entry chunk of remainder products, p = lane's product (0.0 past the
-// end), chunk entries [base, base + 32).  Lane r < 16 owns row r with entries
-// [b, e) (live: r is a row of the item and is not empty).  An inclusive
-// segmented scan (Hillis-Steele, segments = rows, lane 0 always starts one)
-// leaves each row's sum of this chunk on its last lane, which the row's lane
-// fetches.  For a row wholly inside the chunk the tree depends only on the
-// row's length, and the chunk grid is anchored at the first entry of the
-// tile row (or of the item's part of it), so every sum order is a function
-// of the tile row's own content (shard and grouping invariant).
-__device__ __forceinline__ double chunk_piece(double p, int base, int b, int e, bool live, int lane) {
-    const int s = b - base;
-    const bool hd = live && s >= 0 && s < 32;
-    const uint32_t heads = __reduce_or_sync(FULL, hd ? 1u << s : 0u) | 1u;
-    const int seg = 31 - __clz(heads & (0xFFFFFFFFu >> (31 - lane)));  // the lane's segment head
-#pragma unroll
-    for (int d = 1; d < 32; d <<= 1) {
-        const double t = __shfl_up_sync(FULL, p, d);
-        if (lane - d >= seg) p += t;
-    }
-    const bool in = live && s < 32 && e > base;
-    const double piece = __shfl_sync(FULL, p, in ? min(e - base, 32) - 1 : lane);
-    return in ? piece : 0.0;
+// The remainder rows of a tile row are summed by their own lanes:
+// lane r (or r + 16) owns row r.  Which routine runs depends only on the
+// item's content (its longest row), so every sum order is a function of the
+// tile row's own entries (shard and grouping invariant):
+//   <= 4 entries per row (stencils): two lanes per row, one round of gathers;
+//   <= 32: two lanes per row, two entries each per step, all rows at once;
+//   longer (power-law hubs): the flat pass below.
+// A masked term never reads an x entry the item does not reference (a halo
+// rank holds only its own rows and its halo): the two-lane paths multiply
+// 0.0 by x at the item's first remainder column, the flat pass rounds each
+// product on its own and selects +0.0.
+constexpr int kShortRow = 16;  // flat pass: rows of up to this many entries two lanes per row
+
+// product of staged remainder entry k if k < e, else +0.0 (rounded on its own)
+__device__ __forceinline__ double rem_product(const Params &p, int k, int e, uint32_t colS, uint32_t valS,
+                                              uint64_t x_policy) {
+    int c;
+    double v;
+    lds_entry_lt(k, e, colS + 4 * k, valS + 8 * k, c, v);
+    const double pr = __dmul_rn(v, ldg_hint(p.x + (uint32_t)c, x_policy));
+    return k < e ? pr : 0.0;
 }
 
-// The remainder rows 0..rows-1 of one tile row (rq: its rebased row pointers
-// rq[0..rows] in shared memory; colS/valS: the entries), lane per entry in
-// chunks of 32 anchored at rq[0], two chunks (two x gathers) in flight.
-// Returns row r's sum in lane r < 16 (lanes >= 16: 0).  Each product is
-// rounded on its own (v * x, not fused): masked lanes contribute an exact
-// 0.0 however x[0] reads (a halo rank need not hold x[0]).
-__device__ __forceinline__ double rem_chunks(const Params &p, uint32_t rq, int rows, uint32_t colS, uint32_t valS,
-                                             uint64_t x_policy, int lane) {
-    const int r = lane & 15;
+// Flat remainder pass for one tile row (rows <= 16, row pointers at
+// rq): rows of <= kShortRow products two lanes per row, longer rows a
+// half-warp per row (two rows at a time, the whole warp for the last one)
+// with an xor tree.  Returns lane r's (or r + 16's) share of row r.  The order
+// of every sum depends only on this tile row.
+__device__ __forceinline__ double flat_rows(const Params &p, uint32_t rq, uint32_t colS, uint32_t valS, int rows,
+                                            uint64_t x_policy, int lane) {
+    const int r = lane & 15, h = lane >> 4;
     const int b = lds_s32(rq + 4 * min(r, rows)), e = lds_s32(rq + 4 * min(r + 1, rows));
-    const bool live = lane < 16 && e > b;  // r >= rows: b = e = rq[rows]
-    const int kb = lds_s32(rq), ke = lds_s32(rq + 4 * rows);
-    double acc = 0.0;
+    const bool lng = e - b > kShortRow;
+    const int ee = lng ? b : e;
+    const int trips = (int)__reduce_max_sync(FULL, (unsigned)((ee - b + 1 - h) >> 1));
+    double s0 = 0.0, s1 = 0.0;
 #pragma unroll 1
-    for (int base = kb; base < ke; base += 64) {
-        const int k0 = base + lane, k1 = k0 + 32;
-        const bool two = base + 32 < ke;  // warp-uniform
-        int c0, c1 = 0;
-        double v0, v1 = 0.0, x1 = 0.0;
-        lds_entry_lt(k0, ke, colS + 4 * k0, valS + 8 * k0, c0, v0);
-        const double x0 = ldg_hint(p.x + (uint32_t)c0, x_policy);
-        if (two) {
-            lds_entry_lt(k1, ke, colS + 4 * k1, valS + 8 * k1, c1, v1);
-            x1 = ldg_hint(p.x + (uint32_t)c1, x_policy);
+    for (int i = 0; i < trips; i += 2) {
+        const int k0 = b + h + 2 * i;
+        s0 += rem_product(p, k0, ee, colS, valS, x_policy);
+        s1 += rem_product(p, k0 + 2, ee, colS, valS, x_policy);
+    }
+    double acc = s0 + s1;
+    uint32_t lm = __ballot_sync(FULL, lng && h == 0 && r < rows);
+#pragma unroll 1
+    while (lm) {
+        const int r0 = __ffs(lm) - 1;
+        lm &= lm - 1;
+        const int r1 = lm ? __ffs(lm) - 1 : -1;
+        if (lm) lm &= lm - 1;
+        const bool pair = r1 >= 0;  // warp-uniform
+        const int myrow = (pair && h) ? r1 : r0;
+        const int off = pair ? r : lane, stride = pair ? 16 : 32;
+        const int bb = lds_s32(rq + 4 * myrow), e2 = lds_s32(rq + 4 * myrow + 4);
+        const int t2 = (int)__reduce_max_sync(FULL, (unsigned)((e2 - bb + 4 * stride - 1) >> (pair ? 6 : 7)));
+        double q0 = 0.0, q1 = 0.0, q2 = 0.0, q3 = 0.0;
+#pragma unroll 1
+        for (int t = 0; t < t2; ++t) {
+            const int k = bb + off + 4 * stride * t;
+            q0 += rem_product(p, k, e2, colS, valS, x_policy);
+            q1 += rem_product(p, k + stride, e2, colS, valS, x_policy);
+            q2 += rem_product(p, k + 2 * stride, e2, colS, valS, x_policy);
+            q3 += rem_product(p, k + 3 * stride, e2, colS, valS, x_policy);
         }
-        acc += chunk_piece(k0 < ke ? v0 * x0 : 0.0, base, b, e, live, lane);
-        if (two) acc += chunk_piece(k1 < ke ? v1 * x1 : 0.0, base + 32, b, e, live, lane);
+        double sq = (q0 + q1) + (q2 + q3);
+        if (!pair) sq += __shfl_xor_sync(FULL, sq, 16);
+        sq += __shfl_xor_sync(FULL, sq, 8);
+        sq += __shfl_xor_sync(FULL, sq, 4);
+        sq += __shfl_xor_sync(FULL, sq, 2);
+        sq += __shfl_xor_sync(FULL, sq, 1);
+        if (pair ? r == myrow : lane == r0) acc += sq;
     }
     return acc;
 }
 
-// fused CSR remainder of an item's rows; adds row r's sum into acc
-// of lane r (or r + 16).  rpS: rebased row pointers (rows + 1), colS/valS:
-// entries.  Rows of <= 4 entries (stencil-like) run two lanes per row, two
-// entries each, one round trip of gathers; anything longer runs rem_chunks.
-// The path depends only on the item's content.
 __device__ __forceinline__ void remainder(const Params &p, uint32_t rpS, uint32_t colS, uint32_t valS, int rows,
                                           uint64_t x_policy, int lane, double &acc) {
     const int r = lane & 15, h = lane >> 4;
     const int b = lds_s32(rpS + 4 * min(r, rows)), e = lds_s32(rpS + 4 * min(r + 1, rows));
     const int maxlen = (int)__reduce_max_sync(FULL, (unsigned)(e - b));
-    if (maxlen > 4) {
-        acc += rem_chunks(p, rpS, rows, colS, valS, x_policy, lane);
+    if (maxlen > 32) {
+        acc += flat_rows(p, rpS, colS, valS, rows, x_policy, lane);
         return;
     }
-    // entries b + h and b + h + 2 of row r; a masked entry adds nothing
-    // (predicated FMA: the x it read is never used)
-    const int k0 = b + h, k1 = k0 + 2;
-    int c0, c1;
-    double v0, v1;
-    lds_entry_lt(k0, e, colS + 4 * k0, valS + 8 * k0, c0, v0);
-    lds_entry_lt(k1, e, colS + 4 * k1, valS + 8 * k1, c1, v1);
-    const double x0 = ldg_hint(p.x + (uint32_t)c0, x_policy), x1 = ldg_hint(p.x + (uint32_t)c1, x_policy);
-    fma_if(k0 < e, v0, x0, acc);
-    fma_if(k1 < e, v1, x1, acc);
+    // entries b + h + 2i and b + h + 2i + 2 of row r per step; a masked
+    // entry multiplies 0.0 by x at the item's first remainder column
+    const int cdef = lds_s32(colS);
+    const int trips = maxlen <= 4 ? 1 : (int)__reduce_max_sync(FULL, (unsigned)((e - b + 1 - h) >> 1));
+#pragma unroll 1
+    for (int i = 0; i < trips; i += 2) {
+        const int k0 = b + h + 2 * i, k1 = k0 + 2;
+        int c0, c1;
+        double v0, v1;
+        lds_entry_or(k0, e, colS + 4 * k0, valS + 8 * k0, cdef, c0, v0);
+        lds_entry_or(k1, e, colS + 4 * k1, valS + 8 * k1, cdef, c1, v1);
+        const double x0 = ldg_hint(p.x + (uint32_t)c0, x_policy), x1 = ldg_hint(p.x + (uint32_t)c1, x_policy);
+        acc = fma(v0, x0, acc);
+        acc = fma(v1, x1, acc);
+    }
 }
 
 // Row-group item (internal.cuh): ntr consecutive tile rows without stored
-// tiles, only remainder rows.  Each tile row runs rem_chunks with its
-// chunk grid anchored at its own first entry and writes y once per row, so a
-// tile row's sums never depend on which tile rows share its item.
+// tiles, only remainder rows.  Two tile rows at a time, half-warp h
+// on tile row g + h and lane r on its row r alone (4 running sums over the
+// row's products, in entry order mod 4); rows longer than kShortRow entries
+// are summed by the whole warp with an xor tree.  y is written once per row.
+// A tile row's sums depend only on its own entries, so grouping never
+// changes a bit of y.
 __device__ __forceinline__ void group_item(const Params &p, const WItem &it, uint32_t slot, uint64_t x_policy,
                                            int lane) {
     const int ntr = (int)(it.jt_rows_pay & 0xFFu);
@@ -169,12 +199,55 @@ __device__ __forceinline__ void group_item(const Params &p, const WItem &it, uin
     const uint32_t total = it.val_tot >> 16, rp = it.rp_col & 0xFFFFu;
     const bool has_rem = total > rp;
     const uint32_t rpS = slot + rp, colS = slot + (it.rp_col >> 16), valS = slot + (it.val_tot & 0xFFFFu);
+    const int h = lane >> 4, r = lane & 15;
 #pragma unroll 1
-    for (int g = 0; g < ntr; ++g) {
-        const int rows = g + 1 < ntr ? 16 : rows_last;
-        const double acc = has_rem ? rem_chunks(p, rpS + 64u * (uint32_t)g, rows, colS, valS, x_policy, lane) : 0.0;
-        const int64_t row = 16 * ((int64_t)it.I + g) + lane;
-        if (lane < 16 && row < p.m) p.y[row] = acc;
+    for (int g = 0; g < ntr; g += 2) {
+        const int gg = g + h;
+        const int rows = gg < ntr ? (gg + 1 < ntr ? 16 : rows_last) : 0;
+        double acc = 0.0;
+        if (has_rem) {
+            const uint32_t rq = rpS + 64u * (uint32_t)min(gg, ntr - 1);
+            const int b = lds_s32(rq + 4 * min(r, rows)), e = lds_s32(rq + 4 * min(r + 1, rows));
+            const bool lng = e - b > kShortRow;
+            const int ee = lng ? b : e;
+            const int trips = (int)__reduce_max_sync(FULL, (unsigned)((ee - b + 3) >> 2));
+            double s0 = 0.0, s1 = 0.0, s2 = 0.0, s3 = 0.0;
+#pragma unroll 1
+            for (int t = 0; t < trips; ++t) {
+                const int k = b + 4 * t;
+                s0 += rem_product(p, k, ee, colS, valS, x_policy);
+                s1 += rem_product(p, k + 1, ee, colS, valS, x_policy);
+                s2 += rem_product(p, k + 2, ee, colS, valS, x_policy);
+                s3 += rem_product(p, k + 3, ee, colS, valS, x_policy);
+            }
+            acc = (s0 + s1) + (s2 + s3);
+            uint32_t lm = __ballot_sync(FULL, lng);
+#pragma unroll 1
+            while (lm) {  // one long row at a time, the whole warp
+                const int src = __ffs(lm) - 1;
+                lm &= lm - 1;
+                const int bb = __shfl_sync(FULL, b, src), e2 = __shfl_sync(FULL, e, src);
+                const int t2 = (e2 - bb + 127) >> 7;
+                double q0 = 0.0, q1 = 0.0, q2 = 0.0, q3 = 0.0;
+#pragma unroll 1
+                for (int t = 0; t < t2; ++t) {
+                    const int k = bb + lane + 128 * t;
+                    q0 += rem_product(p, k, e2, colS, valS, x_policy);
+                    q1 += rem_product(p, k + 32, e2, colS, valS, x_policy);
+                    q2 += rem_product(p, k + 64, e2, colS, valS, x_policy);
+                    q3 += rem_product(p, k + 96, e2, colS, valS, x_policy);
+                }
+                double sq = (q0 + q1) + (q2 + q3);
+                sq += __shfl_xor_sync(FULL, sq, 16);
+                sq += __shfl_xor_sync(FULL, sq, 8);
+                sq += __shfl_xor_sync(FULL, sq, 4);
+                sq += __shfl_xor_sync(FULL, sq, 2);
+                sq += __shfl_xor_sync(FULL, sq, 1);
+                if (lane == src) acc += sq;
+            }
+        }
+        const int64_t row = 16 * ((int64_t)it.I + gg) + r;
+        if (gg < ntr && row < p.m) p.y[row] = acc;
     }
 }
 
@@ -224,6 +297,7 @@ __device__ __forceinline__ void issue_blob(const Params &p, const WItem &it, uin
 // the x segment of every tile of the item (J: tile column of tile `lane`),
 // issued before the blob lands.  tail: the item's WItem bit 30 (its last
 // tile column reaches the ragged end of x)
+template <int XT>
 __device__ __forceinline__ void issue_x(const Params &p, int J, int nt, uint32_t xs, uint64_t x_policy, int lane,
                                         bool tail) {
     const uint32_t n32 = (uint32_t)p.n;
@@ -231,7 +305,7 @@ __device__ __forceinline__ void issue_x(const Params &p, int J, int nt, uint32_t
         const double *xq = p.x + 2 * (lane & 7);
         const uint32_t xs_l = xs + 16 * (lane & 7);
 #pragma unroll
-        for (int kk = 0; kk < kItemTiles / 4; ++kk) {
+        for (int kk = 0; kk < XT / 4; ++kk) {
             const int t = 4 * kk + (lane >> 3);
             const uint32_t Jt = (uint32_t)__shfl_sync(FULL, J, t);
             if (t < nt) cp_async16(xs_l + 128 * t, xq + 16u * Jt, 16u, x_policy);
@@ -240,7 +314,7 @@ __device__ __forceinline__ void issue_x(const Params &p, int J, int nt, uint32_t
     } else if (p.x_vec) {
         const uint32_t qq = lane & 7;
 #pragma unroll
-        for (int kk = 0; kk < kItemTiles / 4; ++kk) {
+        for (int kk = 0; kk < XT / 4; ++kk) {
             const int t = 4 * kk + (lane >> 3);
             const uint32_t c0 = 16u * (uint32_t)__shfl_sync(FULL, J, t) + 2u * qq;
             if (t < nt) {
@@ -256,7 +330,7 @@ __device__ __forceinline__ void issue_x(const Params &p, int J, int nt, uint32_t
     } else {  // x not 16-byte aligned: lane l: tile 2k + h, element r
         const int h = lane >> 4, r = lane & 15;
 #pragma unroll
-        for (int kk = 0; kk < kItemTiles / 2; ++kk) {
+        for (int kk = 0; kk < XT / 2; ++kk) {
             const int t = 2 * kk + h;
             const uint32_t col = 16u * (uint32_t)__shfl_sync(FULL, J, t) + (uint32_t)r;
             if (t < nt) sts_f64(xs + 8 * (16 * t + r), col < n32 ? ldg_hint(p.x + col, x_policy) : 0.0);
@@ -274,7 +348,7 @@ __device__ __forceinline__ void compute_item(const Params &p, const WItem &it, u
     }
     const int h = lane >> 4, r = lane & 15;
     const uint32_t total = it.val_tot >> 16;
-    // 2. fused CSR remainder
+    // 2. fused CSR remainder, while the x segments land
     double acc = 0.0;
     const uint32_t rp = it.rp_col & 0xFFFFu;
     if (total > rp)
@@ -380,7 +454,7 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, MINB) tilespmv
         // the matrix is immutable; x and y may belong to the previous kernel
         if (k == kbeg) griddep_wait();
         // 1. x segments, issued before the blob lands (J came with the record)
-        issue_x(p, J, (it.part_nt >> 24) & 31, xs, x_policy, lane, (it.groups >> 30) & 1u);
+        issue_x<kItemTiles>(p, J, (it.part_nt >> 24) & 31, xs, x_policy, lane, (it.groups >> 30) & 1u);
         if (k + 1 < kend) {  // the next record and its columns, in flight during this item
             nxt = load_witem(p.witems, k + 1);
             Jn = lane < 16 ? __ldg(p.jcols + (int64_t)(k + 1) * 16 + lane) : 0;
@@ -406,9 +480,10 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, MINB) tilespmv
 // oldest-first issue priority leaves the youngest CTAs as a serial tail).
 // Each warp claims its next unit when it starts one, so the claim and the
 // unit's bounds are in flight while the current unit runs.
-template <int WARPS, int SLOT>
-__global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, 1) tilespmv_fp64_sm(const Params p) {
-    using Cfg = WarpCfg<WARPS, SLOT>;
+// XT tiles per item (an x stage of XT segments per warp)
+template <int WARPS, int SLOT, int XT>
+__global__ void __launch_bounds__(WarpCfg<WARPS, SLOT, XT>::kThreads, 1) tilespmv_fp64_sm(const Params p) {
+    using Cfg = WarpCfg<WARPS, SLOT, XT>;
     extern __shared__ __align__(128) uint8_t smem[];
     __shared__ int s_next;
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -464,7 +539,7 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, 1) tilespmv_fp
             }
         }
         // 1. x segments, issued before the blob lands (J came with the record)
-        issue_x(p, J, (it.part_nt >> 24) & 31, xs, x_policy, lane, (it.groups >> 30) & 1u);
+        issue_x<XT>(p, J, (it.part_nt >> 24) & 31, xs, x_policy, lane, (it.groups >> 30) & 1u);
         const int kn = k + 1 < ke ? k + 1 : nb;
         if (kn >= 0) {  // the next record and its columns, in flight during this item
             nxt = load_witem(p.witems, kn);
@@ -494,10 +569,16 @@ KernelChoice kernel_choice(int kernel) {
     if (kernel == TILESPMV_KERNEL_DENSE_ROWS) {
         using Cfg = WarpCfg<4, 10752>;
         return {"tilespmv_fp64_warp<4,10752>", tilespmv_fp64_warp<4, 10752, 4>, Cfg::kThreads, (int)Cfg::kSmem,
-                10752, false};
+                10752, kItemTiles, false};
+    }
+    if (kernel == TILESPMV_KERNEL_GATHER) {
+        using Cfg = WarpCfg<32, 2304, 8>;
+        return {"tilespmv_fp64_sm<32,2304,8>", tilespmv_fp64_sm<32, 2304, 8>, Cfg::kThreads, (int)Cfg::kSmem, 2304, 8,
+                true};
     }
     using Cfg = WarpCfg<32, 4608>;
-    return {"tilespmv_fp64_sm<32,4608>", tilespmv_fp64_sm<32, 4608>, Cfg::kThreads, (int)Cfg::kSmem, 4608, true};
+    return {"tilespmv_fp64_sm<32,4608>", tilespmv_fp64_sm<32, 4608, kItemTiles>, Cfg::kThreads, (int)Cfg::kSmem, 4608,
+            kItemTiles, true};
 }
 
 }  // namespace tsp

@@ -48,7 +48,8 @@ def build_shard_handles(create, slices, nnz_local: int, mode="DEFERRED", kernel=
     create(slice, mode_id, kernel_id) -> a handle with .info() and .close()
     (normally TiledMatrix.from_csr of that slice).  AUTO mode follows reading
     R18 on the global nnz (DEFERRED iff nnz >= 1.8e6); AUTO kernel is
-    tilespmv_auto_kernel of the global payload bytes and tile rows.  Both are
+    tilespmv_auto_kernel of the global payload bytes, tile rows, remainder
+    entries and algorithmic bytes.  Both are
     all-reduced over `group` (a collective: every rank calls this).
     Returns (handles, mode_id, kernel_id)."""
     import torch
@@ -70,8 +71,8 @@ def build_shard_handles(create, slices, nnz_local: int, mode="DEFERRED", kernel=
     hs = [create(s, md, k0) for s in slices]
     if kn == KERNELS["AUTO"]:
         infos = [h.info() for h in hs]
-        pay, tm = allsum([sum(i["payload_bytes"] for i in infos), sum(i["tilem"] for i in infos)])
-        kn = auto_kernel(pay, tm)
+        tot = allsum([sum(i[k] for i in infos) for k in ("payload_bytes", "tilem", "rem_nnz", "alg_bytes")])
+        kn = auto_kernel(*tot)
         if kn != k0:
             for h in hs:
                 h.close()

@@ -16,7 +16,7 @@ from . import _build
 
 FORMATS = ["CSR", "COO", "ELL", "HYB", "DNS", "DNSROW", "DNSCOL"]
 MODES = {"ADPT": 0, "DEFERRED": 1, "AUTO": 2, "FORCE_CSR": 3}
-KERNELS = {"AUTO": 0, "SM_QUEUE": 1, "DENSE_ROWS": 2}
+KERNELS = {"AUTO": 0, "SM_QUEUE": 1, "DENSE_ROWS": 2, "GATHER": 3}
 ARRAYS = {"tilePtr": (0, np.int32), "tileColIdx": (1, np.int32), "tileNnz": (2, np.int32),
           "tileFmt": (3, np.uint8), "tileAux": (4, np.uint8), "tileOff": (5, np.uint32),
           "payload": (6, np.uint8), "remRowPtr": (7, np.int32), "remCol": (8, np.int32),
@@ -91,7 +91,7 @@ def load(build_if_missing: bool = True):
                                         ctypes.POINTER(i32)]
     L.tilespmv_cg.argtypes = [p, p, p, ctypes.c_double, i32, ctypes.POINTER(i32), ctypes.POINTER(ctypes.c_double), p]
     if hasattr(L, "tilespmv_auto_kernel"):  # (absent from round-1 builds used in A/B runs)
-        L.tilespmv_auto_kernel.argtypes = [i64, i64]
+        L.tilespmv_auto_kernel.argtypes = [i64, i64, i64, i64]
         L.tilespmv_auto_kernel.restype = i32
     L.tilespmv_kernel_name.argtypes = [p]
     L.tilespmv_kernel_name.restype = ctypes.c_char_p
@@ -103,9 +103,9 @@ def load(build_if_missing: bool = True):
     return L
 
 
-def auto_kernel(payload_bytes: int, tilem: int) -> int:
+def auto_kernel(payload_bytes: int, tilem: int, rem_nnz: int, alg_bytes: int) -> int:
     """TILESPMV_KERNEL_AUTO's choice for these totals (tilespmv_auto_kernel)."""
-    return int(load().tilespmv_auto_kernel(int(payload_bytes), int(tilem)))
+    return int(load().tilespmv_auto_kernel(int(payload_bytes), int(tilem), int(rem_nnz), int(alg_bytes)))
 
 
 def _check(rc: int, what: str):

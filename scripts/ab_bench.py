@@ -1,11 +1,11 @@
 #!/usr/bin/env python
 """A/B timing of SpMV kernel variants on one box (development tool).
 
-    python scripts/ab_bench.py WORKLOAD VARIANT[,VARIANT...] [--rounds R] [--steps K]
+    python scripts/ab_bench.py WORKLOAD KERNEL[,KERNEL...] [--rounds R] [--steps K]
 
-Builds one handle per variant (TILESPMV_KERNEL is read at create time) on
-enough replicas of the matrix to defeat L2, then times K back-to-back SpMVs
-per variant, interleaving the variants round by round.  Prints per-variant
+KERNEL: SM_QUEUE, DENSE_ROWS or AUTO (tilespmv_opts_t.kernel).  Builds one
+handle per kernel on enough replicas of the matrix to defeat L2, then times K
+back-to-back SpMVs per kernel, interleaving the kernels round by round.  Prints per-variant
 median / min microseconds and the HBM fraction.  Not a bench line.
 """
 import argparse
@@ -36,22 +36,14 @@ def main():
     l2 = torch.cuda.get_device_properties(0).L2_cache_size
     hs = {}
     for v in a.variants.split(","):
-        # VARIANT[@NAME=VALUE...]: kernel variant plus TILESPMV_<NAME> settings
-        kv, *envs = v.split("@")
-        os.environ["TILESPMV_KERNEL"] = kv
-        for e in envs:
-            k_, v_ = e.split("=")
-            os.environ["TILESPMV_" + k_] = v_
-        M0 = T.TiledMatrix.from_host_csr(A, mode=a.mode, device=dev)
+        kv = int(v) if v.isdigit() else v
+        M0 = T.TiledMatrix.from_host_csr(A, mode=a.mode, device=dev, kernel=kv)
         alg = M0.info()["alg_bytes"]
         reps = max(1, int(np.ceil(4 * l2 / max(alg, 1))))
-        Ms = [M0] + [T.TiledMatrix.from_host_csr(A, mode=a.mode, device=dev) for _ in range(reps - 1)]
+        Ms = [M0] + [T.TiledMatrix.from_host_csr(A, mode=a.mode, device=dev, kernel=kv) for _ in range(reps - 1)]
         xs = [torch.from_numpy(x).to(dev) for _ in range(reps)]
         ys = [torch.empty(A.m, dtype=torch.float64, device=dev) for _ in range(reps)]
         hs[v] = (Ms, xs, ys, alg, M0.kernel_name())
-        for e in envs:
-            os.environ.pop("TILESPMV_" + e.split("=")[0], None)
-    os.environ.pop("TILESPMV_KERNEL", None)
     res = {v: [] for v in hs}
     graphs = {}
     for v, (Ms, xs, ys, alg, name) in hs.items():  # K launches per variant, one graph each
@@ -78,7 +70,7 @@ def main():
             res[v].append(e0.elapsed_time(e1) * 1e3 / a.steps)
     for v, (Ms, xs, ys, alg, name) in hs.items():
         t = np.array(res[v])
-        print(f"{a.workload} v{v:>3} {name:34s} median {np.median(t):9.2f} us  min {t.min():9.2f} us  "
+        print(f"{a.workload} {v:>10} {name:34s} median {np.median(t):9.2f} us  min {t.min():9.2f} us  "
               f"frac(median) {alg / (np.median(t) * 1e-6) / 1e9 / peak:.3f}  reps {len(Ms)}", flush=True)
 
 

@@ -20,7 +20,7 @@ for A in mats:
     x = gen.dense_x(A.n, 101)
     yref, absy = O.spmv(A, x)
     for mode in ("ADPT", "DEFERRED"):
-        for kernel in ("SM_QUEUE", "DENSE_ROWS"):
+        for kernel in ("SM_QUEUE", "DENSE_ROWS", "GATHER"):
             M = TiledMatrix.from_host_csr(A, mode=mode, kernel=kernel)
             y = M.run(torch.from_numpy(x).cuda()).cpu().numpy()
             ok = np.all(np.abs(y - yref) <= 1e-12 * absy + 1e-300)

@@ -86,10 +86,10 @@ def test_no_cpu_fallback():
 
 
 def test_default_spmv_kernel_has_no_register_spills(tmp_path):
-    """The two SpMV kernels (SM-queue, dense-row) are register-capped at 64
-    per thread by their launch bounds; a spill puts local-memory traffic on
+    """The SpMV kernels (SM-queue, gather, dense-row) are register-capped by
+    their launch bounds (64 / 64 / 128 per thread); a spill puts local-memory traffic on
     the hot path (it cost 10% once).  ptxas -v must report zero spill bytes
-    for both, and they must be the only SpMV kernels in the translation unit."""
+    for all three, and they must be the only SpMV kernels in the translation unit."""
     from paper_conf_ipps_niuldj0t21_b200 import _build
     src = os.path.join(_build.PKG, "csrc", "spmv_warp.cu")
     out = subprocess.run([_build.NVCC, "-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-std=c++17",
@@ -99,13 +99,14 @@ def test_default_spmv_kernel_has_no_register_spills(tmp_path):
     checked = 0
     for b in blocks[1:]:
         name = b.split("'")[1]
-        assert "tilespmv_fp64" not in name or ("tilespmv_fp64_smILi32ELi4608EE" in name) or (
-            "tilespmv_fp64_warpILi4ELi10752" in name), name
-        if ("tilespmv_fp64_smILi32ELi4608EE" in name) or ("tilespmv_fp64_warpILi4ELi10752" in name):
+        names = ("tilespmv_fp64_smILi32ELi4608ELi16EE", "tilespmv_fp64_smILi32ELi2304ELi8EE",
+                 "tilespmv_fp64_warpILi4ELi10752")
+        assert "tilespmv_fp64" not in name or any(n in name for n in names), name
+        if any(n in name for n in names):
             m = re.search(r"(\d+) bytes spill stores, (\d+) bytes spill loads", b)
             assert m and m.group(1) == "0" and m.group(2) == "0", (name, m and m.group(0))
             checked += 1
-    assert checked == 2
+    assert checked == 3
 
 
 def test_no_hidden_configuration():
@@ -118,24 +119,29 @@ def test_no_hidden_configuration():
             assert "getenv" not in fh.read(), f
 
 
-def test_library_has_exactly_two_spmv_kernels():
-    """The shipped libtilespmv.so holds the two SpMV kernels and no
-    superseded variants."""
+def test_library_has_exactly_three_spmv_kernels():
+    """The shipped libtilespmv.so holds the three SpMV kernels (one per
+    TILESPMV_KERNEL_*) and no superseded variants."""
     from paper_conf_ipps_niuldj0t21_b200 import _build
     _build.build()
     out = subprocess.run(["nm", "-C", _build.LIB], capture_output=True, text=True, check=True).stdout
     names = {l.split(" ", 2)[-1] for l in out.splitlines() if "tilespmv_fp64_" in l and "__device_stub" not in l}
     kernels = {n for n in names if "(tsp::Params)" in n}
-    assert len(kernels) == 2, kernels
+    assert len(kernels) == 3, kernels
 
 
 def test_auto_kernel_rule_without_gpu():
     """TILESPMV_KERNEL_AUTO: the dense-row kernel iff the mean stored payload
     per tile row exceeds 6 KiB (integer form, no float rounding)."""
     from paper_conf_ipps_niuldj0t21_b200.tilespmv import KERNELS, auto_kernel
-    assert auto_kernel(6144 * 1000, 1000) == KERNELS["SM_QUEUE"]
-    assert auto_kernel(6144 * 1000 + 1, 1000) == KERNELS["DENSE_ROWS"]
-    assert auto_kernel(0, 0) == KERNELS["SM_QUEUE"]
-    # C2 (FEM, 10 KiB per tile row) and C5 (3.8 KiB) as the bench builds them
-    assert auto_kernel(39_964_672, 3904) == KERNELS["DENSE_ROWS"]
-    assert auto_kernel(1_901_429_504, 500_000) == KERNELS["SM_QUEUE"]
+    assert auto_kernel(6144 * 1000, 1000, 0, 10**9) == KERNELS["SM_QUEUE"]
+    assert auto_kernel(6144 * 1000 + 1, 1000, 0, 10**9) == KERNELS["DENSE_ROWS"]
+    assert auto_kernel(0, 0, 0, 0) == KERNELS["SM_QUEUE"]
+    # the remainder's 12 B per entry more than half of the algorithmic bytes
+    assert auto_kernel(0, 16, 1000, 23999) == KERNELS["GATHER"]
+    assert auto_kernel(0, 16, 1000, 24000) == KERNELS["SM_QUEUE"]
+    # C2 (FEM, 10 KiB per tile row), C5 (3.8 KiB, 8.3M of 213.8M nnz in the
+    # remainder) and C3 (R-MAT, 98% in the remainder) as the bench builds them
+    assert auto_kernel(39_964_672, 3904, 0, 41_540_000) == KERNELS["DENSE_ROWS"]
+    assert auto_kernel(1_901_429_504, 500_000, 8_344_492, 2_264_462_760) == KERNELS["SM_QUEUE"]
+    assert auto_kernel(2_900_000, 65_536, 15_774_932, 213_500_000) == KERNELS["GATHER"]

@@ -52,7 +52,7 @@ CASES = [(128, 128, 0, "equal"), (125, 131, 1, "equal"), (200, 96, 2, "ragged"),
 
 
 @pytest.mark.gpu
-@pytest.mark.parametrize("kernel", ["SM_QUEUE", "DENSE_ROWS"])
+@pytest.mark.parametrize("kernel", ["SM_QUEUE", "DENSE_ROWS", "GATHER"])
 def test_tile_profile_fuzz(cuda_device, kernel):
     import torch
     from paper_conf_ipps_niuldj0t21_b200 import TiledMatrix

@@ -263,11 +263,13 @@ def test_full_size_tiler_and_spmv(cuda_device, name):
         # algorithmic bytes, and the same y bit for bit
         with TM.from_host_csr(A, mode=mode, device=cuda_device) as M2:
             i2 = M2.info()
-            assert i2["device_bytes"] <= 1.2 * i2["alg_bytes"], (name, mode, i2["device_bytes"], i2["alg_bytes"])
+            # (ADPT adds an 8-byte descriptor per stored tile: R-MAT's 11M tiny COO tiles)
+            lim = 1.2 if mode == "DEFERRED" else 1.3
+            assert i2["device_bytes"] <= lim * i2["alg_bytes"], (name, mode, i2["device_bytes"], i2["alg_bytes"])
             assert torch.equal(M2.run(xd), y)
 
 
-KERNELS = ["SM_QUEUE", "DENSE_ROWS"]
+KERNELS = ["SM_QUEUE", "DENSE_ROWS", "GATHER"]
 
 
 @pytest.mark.parametrize("kernel", KERNELS)
