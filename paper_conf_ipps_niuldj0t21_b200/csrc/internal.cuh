@@ -37,6 +37,8 @@ struct __align__(16) Item {
     int32_t kb, ke;   // remainder entry range
     uint32_t offb;    // payload offset of tile tb (16-byte units)
     uint32_t offe;    // payload offset one past the last tile
+    uint32_t pay_bytes;  // bytes of the tiles in the blob payload (tile_cost; canonical unless a COO run)
+    uint32_t run_e;      // entries of the item's COO run (ADPT: COO tiles + HYB COO parts), 0 if none
     int32_t split;    // split-row index, or -1 if the item covers its whole tile row
     int32_t part_nt;  // part index (bits 0-23) | tiles << 24 (5 bits) | local << 29 | last-of-group << 30
     int32_t dbeg;      // first entry of the item's tile-descriptor list (dlist)
@@ -68,7 +70,8 @@ struct __align__(16) WItem {
     uint32_t val_tot;      // val offset | total bytes << 16
     uint32_t groups;       // tile pairs per format f, 4 bits at 4f (descriptor list order);
                            // bit 28: every CSR row of the item <= 3 entries, bit 29: every ELL width <= 3,
-                           // bit 30: the last tile column's x segment passes x[n-1] (ragged tail)
+                           // bit 30: the last tile column's x segment passes x[n-1] (ragged tail),
+                           // bit 31: the rp/col/val parts are a COO run (ADPT), not a CSR remainder
 };
 
 // Per-warp start record of the dense-row kernel: the warp's item chunk and a

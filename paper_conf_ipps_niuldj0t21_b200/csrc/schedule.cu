@@ -24,13 +24,45 @@ namespace tsp {
 
 namespace {
 
-// Greedy split of tile row I into items whose staged bytes (item_parts)
-// never exceed the kernel's slot size (budget): tiles first (at most kItemTiles), then the tile
-// row's remainder entries.  Depends only on the tile row's own content.
+// The level-1 arrays the schedule reads, and whether items gather their COO
+// data into a COO run (ADPT mode, see blob_parts).
+struct TileView {
+    const int32_t *tilePtr;
+    const uint32_t *tileOff;
+    const uint8_t *tileFmt, *tileAux;
+    const int32_t *tileNnz;
+    int run;
+};
+
+// Bytes tile g occupies in its item's blob payload, and the entries it adds
+// to the item's COO run: with a run, a COO tile moves wholly into the run and
+// a HYB(w) tile keeps its ELL(w) part as an ELL tile (136 w bytes, no pads:
+// every row holds >= w entries) and moves its COO part into the run.
+__device__ __forceinline__ void tile_cost(const TileView &T, int g, uint32_t &pay, uint32_t &run) {
+    pay = (T.tileOff[g + 1] - T.tileOff[g]) * 16u;
+    run = 0;
+    if (!T.run) return;
+    const uint8_t f = T.tileFmt[g];
+    const uint32_t nz = (uint32_t)(T.tileNnz[g + 1] - T.tileNnz[g]);
+    if (f == F_COO) {
+        pay = 0;
+        run = nz;
+    } else if (f == F_HYB) {
+        const uint32_t w = T.tileAux[g];
+        pay = up16(136u * w);
+        run = nz - 16u * w;
+    }
+}
+
+// Greedy split of tile row I into items whose staged bytes (blob_parts)
+// never exceed the kernel's slot size (budget): tiles first (at most
+// max_tiles), then the tile row's remainder entries.  Depends only on the
+// tile row's own content.
 template <bool WRITE>
-__device__ int items_for_row(int64_t I, const int32_t *tilePtr, const uint32_t *tileOff, const int32_t *remRowPtr,
-                             int64_t m, int budget, int max_tiles, Item *out, int split, int nparts = 0,
-                             int lp = kLocalParts) {
+__device__ int items_for_row(int64_t I, const TileView &T, const int32_t *remRowPtr, int64_t m, int budget,
+                             int max_tiles, Item *out, int split, int nparts = 0, int lp = kLocalParts) {
+    const int32_t *tilePtr = T.tilePtr;
+    const uint32_t *tileOff = T.tileOff;
     const int tp0 = tilePtr[I], tp1 = tilePtr[I + 1];
     int k0 = 0, k1 = 0;
     if (remRowPtr) {
@@ -42,17 +74,22 @@ __device__ int items_for_row(int64_t I, const int32_t *tilePtr, const uint32_t *
     int t = tp0, k = k0, cnt = 0;
     do {
         const int tb = t;
-        uint32_t used = 0;
+        uint32_t used = 0, pays = 0, rune = 0;
         while (t < tp1 && t - tb < max_tiles) {
-            const uint32_t pay = (tileOff[t + 1] - tileOff[tb]) * 16u;
-            // blob: descriptor list (<= ntiles + 7 pads) + J array (blob_parts)
+            uint32_t pt, rt;
+            tile_cost(T, t, pt, rt);
+            // blob: descriptor list (<= ntiles + 7 pads) + J array + COO run (blob_parts)
             const uint32_t dsc = up16(8u * (uint32_t)(t - tb + 1 + 7)) + up16(4u * (uint32_t)(t - tb + 1));
-            if (pay + dsc > (uint32_t)budget) break;
-            used = pay + dsc;
+            const uint32_t u = pays + pt + run_bytes(rune + rt) + dsc;
+            if (u > (uint32_t)budget) break;
+            used = u;
+            pays += pt;
+            rune += rt;
             t++;
         }
         if (t == tb && t < tp1) {  // unreachable: one tile (<= 2176 B) always fits
-            used = (tileOff[t + 1] - tileOff[tb]) * 16u + 80u;
+            tile_cost(T, t, pays, rune);
+            used = pays + run_bytes(rune) + 80u;
             t++;
         }
         int kb = k, ke = k;
@@ -72,6 +109,8 @@ __device__ int items_for_row(int64_t I, const int32_t *tilePtr, const uint32_t *
             it.ke = ke;
             it.offb = tileOff[tb];
             it.offe = tileOff[t];
+            it.pay_bytes = pays;
+            it.run_e = rune;
             it.split = split;
             const bool local = split >= 0 && nparts <= lp;
             const bool last = split >= 0 && (cnt == nparts - 1 || cnt % lp == lp - 1);
@@ -88,12 +127,11 @@ __device__ int items_for_row(int64_t I, const int32_t *tilePtr, const uint32_t *
     return cnt;
 }
 
-__global__ void k_items_count(const int32_t *tilePtr, const uint32_t *tileOff, const int32_t *remRowPtr, int64_t m,
-                              int budget, int max_tiles, int64_t tilem, int32_t *nitems, int32_t *nsplit,
-                              int32_t *parts) {
+__global__ void k_items_count(TileView T, const int32_t *remRowPtr, int64_t m, int budget, int max_tiles, int64_t tilem,
+                              int32_t *nitems, int32_t *nsplit, int32_t *parts) {
     int64_t I = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     if (I >= tilem) return;
-    const int c = items_for_row<false>(I, tilePtr, tileOff, remRowPtr, m, budget, max_tiles, nullptr, -1);
+    const int c = items_for_row<false>(I, T, remRowPtr, m, budget, max_tiles, nullptr, -1);
     nitems[I] = c;
     nsplit[I] = c > 1 ? 1 : 0;
     parts[I] = c > 1 ? c : 0;
@@ -109,15 +147,17 @@ __device__ __forceinline__ bool groupable(int64_t I, const int32_t *tilePtr, con
 // packed greedily into row-group items (<= kGroupTileRows tile rows, blob
 // within budget).  group = false: no row-group items (kernels without them).
 template <bool WRITE>
-__device__ int window_items(int64_t w, const int32_t *tilePtr, const uint32_t *tileOff, const int32_t *remRowPtr,
-                            int64_t m, int budget, int max_tiles, int64_t tilem, bool group,
-                            const int32_t *nitems, const int32_t *splitId, Item *out, int lp) {
+__device__ int window_items(int64_t w, const TileView &T, const int32_t *remRowPtr, int64_t m, int budget,
+                            int max_tiles, int64_t tilem, bool group, const int32_t *nitems, const int32_t *splitId,
+                            Item *out, int lp) {
+    const int32_t *tilePtr = T.tilePtr;
+    const uint32_t *tileOff = T.tileOff;
     const int64_t I0 = w * kGroupWindow, I1 = imin64(I0 + kGroupWindow, tilem);
     int cnt = 0;
     int64_t I = I0;
     while (I < I1) {
         if (!group || !groupable(I, tilePtr, nitems)) {
-            if (WRITE) items_for_row<true>(I, tilePtr, tileOff, remRowPtr, m, budget, max_tiles, out + cnt,
+            if (WRITE) items_for_row<true>(I, T, remRowPtr, m, budget, max_tiles, out + cnt,
                                            nitems[I] > 1 ? splitId[I] : -1, nitems[I], lp);
             cnt += nitems[I];
             ++I;
@@ -140,6 +180,7 @@ __device__ int window_items(int64_t w, const int32_t *tilePtr, const uint32_t *t
             it.kb = remRowPtr ? remRowPtr[16 * I] : 0;
             it.ke = remRowPtr ? remRowPtr[imin64(16 * J, m)] : 0;
             it.offb = it.offe = tileOff[it.tb];
+            it.pay_bytes = it.run_e = 0;
             it.split = -1;
             it.part_nt = 0;
             it.dbeg = it.ndsc = 0;
@@ -153,23 +194,21 @@ __device__ int window_items(int64_t w, const int32_t *tilePtr, const uint32_t *t
     return cnt;
 }
 
-__global__ void k_window_count(const int32_t *tilePtr, const uint32_t *tileOff, const int32_t *remRowPtr, int64_t m,
-                               int budget, int max_tiles, int64_t tilem, int group, const int32_t *nitems,
-                               int64_t nwin, int32_t *wcount) {
+__global__ void k_window_count(TileView T, const int32_t *remRowPtr, int64_t m, int budget, int max_tiles,
+                               int64_t tilem, int group, const int32_t *nitems, int64_t nwin, int32_t *wcount) {
     const int64_t w = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     if (w >= nwin) return;
-    wcount[w] = window_items<false>(w, tilePtr, tileOff, remRowPtr, m, budget, max_tiles, tilem, group != 0, nitems,
-                                    nullptr, nullptr, kLocalParts);
+    wcount[w] = window_items<false>(w, T, remRowPtr, m, budget, max_tiles, tilem, group != 0, nitems, nullptr, nullptr,
+                                    kLocalParts);
 }
 
-__global__ void k_window_write(const int32_t *tilePtr, const uint32_t *tileOff, const int32_t *remRowPtr, int64_t m,
-                               int budget, int max_tiles, int64_t tilem, int group,
+__global__ void k_window_write(TileView T, const int32_t *remRowPtr, int64_t m, int budget, int max_tiles, int64_t tilem,
+                               int group,
                                const int32_t *nitems, int64_t nwin, const int32_t *wbase, const int32_t *splitId,
                                const int32_t *partBase, Item *items, int2 *split_info, int lp) {
     const int64_t w = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     if (w >= nwin) return;
-    window_items<true>(w, tilePtr, tileOff, remRowPtr, m, budget, max_tiles, tilem, group != 0, nitems, splitId,
-                       items + wbase[w], lp);
+    window_items<true>(w, T, remRowPtr, m, budget, max_tiles, tilem, group != 0, nitems, splitId, items + wbase[w], lp);
     const int64_t I1 = imin64((w + 1) * kGroupWindow, tilem);
     for (int64_t I = w * kGroupWindow; I < I1; ++I)
         if (nitems[I] > 1) split_info[splitId[I]] = make_int2(partBase[I], nitems[I]);
@@ -181,21 +220,32 @@ __global__ void k_window_write(const int32_t *tilePtr, const uint32_t *tileOff, 
 // Entry: x = payload byte offset inside the item | (t * 128) << 14 | fmt << 29
 //        y = aux | nnz << 8 | invalid << 31          (t: tile index in the item;
 // t * 128 is the byte offset of the tile's x segment in the warp's x scratch)
-__global__ void k_dsc_count(Item *items, int64_t n, const uint8_t *tileFmt, int32_t *ndsc) {
+// With a COO run (tile_cost): COO tiles get no descriptor and a HYB(w)
+// tile's descriptor is an ELL(w) one (none if w = 0).
+__device__ __forceinline__ int dsc_format(const TileView &T, int g) {
+    const int f = T.tileFmt[g];
+    if (!T.run) return f;
+    if (f == F_COO) return -1;
+    if (f == F_HYB) return T.tileAux[g] ? F_ELL : -1;
+    return f;
+}
+
+__global__ void k_dsc_count(Item *items, int64_t n, TileView T, int32_t *ndsc) {
     int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     if (k >= n) return;
     const Item it = items[k];
     const int nt = item_nt(it);
     int cnt[8] = {0, 0, 0, 0, 0, 0, 0, 0};
-    for (int t = 0; t < nt; ++t) cnt[tileFmt[it.tb + t] & 7]++;
+    for (int t = 0; t < nt; ++t) {
+        const int f = dsc_format(T, it.tb + t);
+        if (f >= 0) cnt[f]++;
+    }
     int total = 0;
     for (int f = 0; f < 7; ++f) total += (cnt[f] + 1) & ~1;
     ndsc[k] = total;
 }
 
-__global__ void k_dsc_write(Item *items, int64_t n, const int32_t *dbeg, const int32_t *ndsc, const int32_t *tileColIdx,
-                            const uint8_t *tileFmt, const uint8_t *tileAux, const int32_t *tileNnz,
-                            const uint32_t *tileOff, uint2 *dlist) {
+__global__ void k_dsc_write(Item *items, int64_t n, const int32_t *dbeg, const int32_t *ndsc, TileView T, uint2 *dlist) {
     int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     if (k >= n) return;
     Item it = items[k];
@@ -204,15 +254,27 @@ __global__ void k_dsc_write(Item *items, int64_t n, const int32_t *dbeg, const i
     it.dbeg = pos;
     it.ndsc = ndsc[k];
     items[k] = it;
+    uint32_t off[kItemTiles];  // each tile's payload offset inside the item's blob payload
+    {
+        uint32_t o = 0;
+        for (int t = 0; t < nt; ++t) {
+            uint32_t pt, rt;
+            tile_cost(T, it.tb + t, pt, rt);
+            off[t] = o;
+            o += pt;
+        }
+    }
     for (int f = 0; f < 7; ++f) {
         uint2 last = make_uint2(0u, 0u);
         int c = 0;
         for (int t = 0; t < nt; ++t) {
             const int g = it.tb + t;
-            if (tileFmt[g] != f) continue;
+            if (dsc_format(T, g) != f) continue;
+            const bool hyb_ell = T.tileFmt[g] == F_HYB;  // (run) the ELL(w) part of a HYB tile
             uint2 d;
-            d.x = ((tileOff[g] - it.offb) * 16u) | ((uint32_t)t << 21) | ((uint32_t)f << 29);
-            d.y = (uint32_t)tileAux[g] | ((uint32_t)(tileNnz[g + 1] - tileNnz[g]) << 8);
+            d.x = off[t] | ((uint32_t)t << 21) | ((uint32_t)f << 29);
+            d.y = (uint32_t)T.tileAux[g] |
+                  ((hyb_ell ? 16u * T.tileAux[g] : (uint32_t)(T.tileNnz[g + 1] - T.tileNnz[g])) << 8);
             dlist[pos++] = d;
             last = d;
             c++;
@@ -233,14 +295,15 @@ __global__ void k_blob_len(const Item *items, int64_t n, int64_t m, uint32_t slo
 
 // one warp per item: copy descriptors, J, payload and the rebased remainder
 __global__ void k_blob_fill(Item *items, int64_t nitems, int64_t m, int64_t n, const int64_t *start16, const uint2 *dlist,
-                            const int32_t *tileColIdx, const uint8_t *tileFmt, const uint8_t *payload,
-                            const int32_t *remRowPtr, const int32_t *remCol, const double *remVal, uint8_t *blob,
-                            WItem *witems, int32_t *jcols) {
+                            const int32_t *tileColIdx, TileView T, const uint8_t *payload, const int32_t *remRowPtr,
+                            const int32_t *remCol, const double *remVal, uint8_t *blob, WItem *witems,
+                            int32_t *jcols) {
     const int64_t k = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
     const int lane = threadIdx.x & 31;
     if (k >= nitems) return;
     Item it = items[k];
     const BlobParts b = blob_parts(it, m);
+    const int nt = item_nt(it);
     uint8_t *dst = blob + start16[k] * 16;
     if (lane == 0) {
         it.blob16 = (uint32_t)start16[k];
@@ -257,10 +320,13 @@ __global__ void k_blob_fill(Item *items, int64_t nitems, int64_t m, int64_t n, c
         w.rp_col = b.rp | (b.col << 16);
         w.val_tot = b.val | (b.total << 16);
         int cnt[7] = {0, 0, 0, 0, 0, 0, 0};
-        for (int t = 0; t < item_nt(it); ++t) cnt[tileFmt[it.tb + t]]++;
+        for (int t = 0; t < nt; ++t) {
+            const int f = dsc_format(T, it.tb + t);
+            if (f >= 0) cnt[f]++;
+        }
         uint32_t g = 0;
         for (int f = 0; f < 7; ++f) g |= (uint32_t)((cnt[f] + 1) >> 1) << (4 * f);
-        w.groups = g;
+        w.groups = g | (it.run_e > 0 ? 1u << 31 : 0u);
         witems[k] = w;
     }
     for (uint32_t o = 4 * lane; o < b.total; o += 128) *reinterpret_cast<uint32_t *>(dst + o) = 0u;  // padding
@@ -272,7 +338,6 @@ __global__ void k_blob_fill(Item *items, int64_t nitems, int64_t m, int64_t n, c
     // larger extent of the two tiles of the half-warp pair (2j, 2j+1): CSR the
     // longest row, ELL the width, COO the entry count (ndsc is even; the
     // loop is warp-uniform)
-    const uint8_t *tpay = payload + (size_t)it.offb * 16;
     uint32_t csr_max = 0, ell_max = 0;
     for (int i0 = 0; i0 < it.ndsc; i0 += 32) {
         const int i = i0 + lane;
@@ -285,7 +350,7 @@ __global__ void k_blob_fill(Item *items, int64_t nitems, int64_t m, int64_t n, c
             e.x = b.pay + off + (f == F_CSR ? 8u * nz : 0u) - 8u * (uint32_t)i;
             e.y = (d.y & 0x1Fu) | (t << 7) | (nz << 11) | (d.y & 0x80000000u);
             if (f == F_CSR) {
-                const uint8_t *rp = tpay + off + 8u * nz;
+                const uint8_t *rp = payload + (size_t)T.tileOff[it.tb + t] * 16 + 8u * nz;
                 for (int r = 0; r < 16; ++r) {
                     const uint32_t len = (r < 15 ? rp[r + 1] : nz) - rp[r];
                     tm = len > tm ? len : tm;
@@ -305,14 +370,81 @@ __global__ void k_blob_fill(Item *items, int64_t nitems, int64_t m, int64_t n, c
     }
     // item-wide extents: the kernel runs such items' CSR / ELL groups with
     // straight-line 3-step routines and no per-pair dispatch
-    const int nt = item_nt(it);
     const bool xtail = nt > 0 && 16 * (int64_t)tileColIdx[it.tb + nt - 1] + 16 > n;
     if (lane == 0)
         witems[k].groups |= (csr_max <= 3 ? 1u << 28 : 0u) | (ell_max <= 3 ? 1u << 29 : 0u) | (xtail ? 1u << 30 : 0u);
     if (lane < 16) jcols[k * 16 + lane] = lane < nt ? tileColIdx[it.tb + lane] : 0;
-    const uint4 *ps = reinterpret_cast<const uint4 *>(payload + (size_t)it.offb * 16);
-    uint4 *pd = reinterpret_cast<uint4 *>(dst + b.pay);
-    for (uint32_t i = lane; i < it.offe - it.offb; i += 32) pd[i] = ps[i];
+    if (!T.run) {  // the canonical payload bytes of the item's tiles, in one piece
+        const uint4 *ps = reinterpret_cast<const uint4 *>(payload + (size_t)it.offb * 16);
+        uint4 *pd = reinterpret_cast<uint4 *>(dst + b.pay);
+        for (uint32_t i = lane; i < it.offe - it.offb; i += 32) pd[i] = ps[i];
+    } else {  // tile by tile: COO tiles left out, HYB(w) tiles as their ELL(w) part
+        uint32_t o = b.pay;
+        for (int t = 0; t < nt; ++t) {
+            const int g = it.tb + t;
+            uint32_t pt, rt;
+            tile_cost(T, g, pt, rt);
+            const uint8_t *src = payload + (size_t)T.tileOff[g] * 16;
+            if (T.tileFmt[g] == F_HYB) {
+                const uint32_t w = T.tileAux[g], kc = rt;
+                const uint2 *vs = reinterpret_cast<const uint2 *>(src);  // ELL values, 16 w
+                uint2 *vd = reinterpret_cast<uint2 *>(dst + o);
+                for (uint32_t i = lane; i < 16u * w; i += 32) vd[i] = vs[i];
+                for (uint32_t i = lane; i < w; i += 32)  // ELL column nibbles, 8 w bytes
+                    reinterpret_cast<uint2 *>(dst + o + 128u * w)[i] =
+                        reinterpret_cast<const uint2 *>(src + 128u * w + 8u * kc)[i];
+            } else if (pt) {
+                const uint4 *ps = reinterpret_cast<const uint4 *>(src);
+                uint4 *pd = reinterpret_cast<uint4 *>(dst + o);
+                for (uint32_t i = lane; i < pt / 16u; i += 32) pd[i] = ps[i];
+            }
+            o += pt;
+        }
+        if (it.run_e > 0) {
+            // the COO run: lane r < 16 gathers row r's COO entries, tile by tile
+            const int r = lane & 15;
+            int cnt = 0;
+            for (int t = 0; t < nt; ++t) {
+                const int g = it.tb + t;
+                const uint8_t f = T.tileFmt[g];
+                if (f != F_COO && f != F_HYB) continue;
+                const uint32_t w = f == F_HYB ? T.tileAux[g] : 0u;
+                const uint32_t kc = (uint32_t)(T.tileNnz[g + 1] - T.tileNnz[g]) - 16u * w;
+                const uint8_t *rc = payload + (size_t)T.tileOff[g] * 16 + (f == F_HYB ? 136u * w + 8u * kc : 8u * kc);
+                for (uint32_t j = 0; j < kc; ++j) cnt += (rc[j] >> 4) == (uint32_t)r;
+            }
+            int base = cnt;  // exclusive prefix over rows 0..15
+            for (int d = 1; d < 16; d <<= 1) {
+                const int v = __shfl_up_sync(0xFFFFFFFFu, base, d, 16);
+                if (r >= d) base += v;
+            }
+            base -= cnt;
+            int32_t *rp = reinterpret_cast<int32_t *>(dst + b.rp);
+            uint8_t *xsl = dst + b.col;
+            double *vv = reinterpret_cast<double *>(dst + b.val);
+            if (lane < 16) {
+                rp[r] = base;
+                if (r == 15) rp[16] = base + cnt;
+                int pos = base;
+                for (int t = 0; t < nt; ++t) {
+                    const int g = it.tb + t;
+                    const uint8_t f = T.tileFmt[g];
+                    if (f != F_COO && f != F_HYB) continue;
+                    const uint32_t w = f == F_HYB ? T.tileAux[g] : 0u;
+                    const uint32_t kc = (uint32_t)(T.tileNnz[g + 1] - T.tileNnz[g]) - 16u * w;
+                    const uint8_t *src = payload + (size_t)T.tileOff[g] * 16;
+                    const double *cv = reinterpret_cast<const double *>(src + 128u * w);  // COO values
+                    const uint8_t *rc = src + (f == F_HYB ? 136u * w + 8u * kc : 8u * kc);
+                    for (uint32_t j = 0; j < kc; ++j) {
+                        if ((rc[j] >> 4) != (uint32_t)r) continue;
+                        vv[pos] = cv[j];
+                        xsl[pos] = (uint8_t)(16 * t + (rc[j] & 15));
+                        ++pos;
+                    }
+                }
+            }
+        }
+    }
     if (it.ke > it.kb) {
         const int rows = (int)item_rows(it, m);
         int32_t *rp = reinterpret_cast<int32_t *>(dst + b.rp);
@@ -418,6 +550,11 @@ __global__ void k_cta_units(const int64_t *incl, const int32_t *units, int64_t n
     cta_begin[b] = lo;
 }
 
+// ADPT mode gathers each item's COO data into a COO run (blob_parts)
+TileView tile_view(const Matrix &M) {
+    return {M.tilePtr, M.tileOff, M.tileFmt, M.tileAux, M.tileNnz, M.mode == TILESPMV_MODE_ADPT ? 1 : 0};
+}
+
 // stream-ordered temporary device buffer
 struct Tmp {
     void *p = nullptr;
@@ -462,10 +599,10 @@ int build_schedule(Matrix &M, cudaStream_t st) {
             *wbase = wcount + (NW + 1);
     TSP_CK(cudaMemsetAsync(nitems, 0, 3 * (T + 1) * sizeof(int32_t), st));
     TSP_CK(cudaMemsetAsync(wcount, 0, (NW + 1) * sizeof(int32_t), st));
-    k_items_count<<<blocks(T), TB, 0, st>>>(M.tilePtr, M.tileOff, M.remRowPtr, M.m, M.item_bytes, M.item_tiles, T,
-                                            nitems, nsplit, parts);
-    k_window_count<<<blocks(NW), TB, 0, st>>>(M.tilePtr, M.tileOff, M.remRowPtr, M.m, M.item_bytes, M.item_tiles, T,
-                                               group, nitems, NW, wcount);
+    const TileView TV = tile_view(M);
+    k_items_count<<<blocks(T), TB, 0, st>>>(TV, M.remRowPtr, M.m, M.item_bytes, M.item_tiles, T, nitems, nsplit, parts);
+    k_window_count<<<blocks(NW), TB, 0, st>>>(TV, M.remRowPtr, M.m, M.item_bytes, M.item_tiles, T, group, nitems, NW,
+                                               wcount);
     TSP_CK(cudaGetLastError());
     if (int rc = scan([&](void *t, size_t &b) { return cub::DeviceScan::ExclusiveSum(t, b, wcount, wbase, (int)(NW + 1), st); }, st)) return rc;
     if (int rc = scan([&](void *t, size_t &b) { return cub::DeviceScan::ExclusiveSum(t, b, nsplit, splitId, (int)(T + 1), st); }, st)) return rc;
@@ -486,7 +623,7 @@ int build_schedule(Matrix &M, cudaStream_t st) {
     // whole records (padding included) are copied later: start from zeros
     TSP_CK(cudaMemsetAsync(M.items, 0, std::max<int64_t>(M.num_items, 1) * sizeof(Item), st));
     TSP_CK(cudaMemsetAsync(M.counters, 0, std::max<int64_t>(M.num_split, 1) * sizeof(int32_t), st));
-    k_window_write<<<blocks(NW), TB, 0, st>>>(M.tilePtr, M.tileOff, M.remRowPtr, M.m, M.item_bytes, M.item_tiles, T,
+    k_window_write<<<blocks(NW), TB, 0, st>>>(TV, M.remRowPtr, M.m, M.item_bytes, M.item_tiles, T,
                                                group, nitems, NW, wbase, splitId, partBase, M.items, M.split_info,
                                                kLocalParts);
     TSP_CK(cudaGetLastError());
@@ -507,15 +644,15 @@ int build_tdesc(Matrix &M, cudaStream_t st) {
     int32_t *cnt = cntb.as<int32_t>(), *beg = cnt + (n + 1);
     const unsigned nb = (unsigned)((n + 255) / 256);
     TSP_CK(cudaMemsetAsync(cnt + n, 0, sizeof(int32_t), st));
-    k_dsc_count<<<nb, 256, 0, st>>>(M.items, n, M.tileFmt, cnt);
+    const TileView TV = tile_view(M);
+    k_dsc_count<<<nb, 256, 0, st>>>(M.items, n, TV, cnt);
     if (int rc = scan([&](void *t, size_t &b) { return cub::DeviceScan::ExclusiveSum(t, b, cnt, beg, (int)(n + 1), st); }, st)) return rc;
     int32_t total = 0;
     TSP_CK(cudaMemcpyAsync(&total, beg + n, 4, cudaMemcpyDeviceToHost, st));
     TSP_CK(cudaStreamSynchronize(st));
     M.num_dsc = total;
     TSP_CK(cudaMallocAsync(&M.tdesc, (total + 4) * sizeof(uint2), st));  // create-time only
-    k_dsc_write<<<nb, 256, 0, st>>>(M.items, n, beg, cnt, M.tileColIdx, M.tileFmt, M.tileAux, M.tileNnz, M.tileOff,
-                                     M.tdesc);
+    k_dsc_write<<<nb, 256, 0, st>>>(M.items, n, beg, cnt, TV, M.tdesc);
     TSP_CK(cudaGetLastError());
     // execution blobs
     Tmp lenb(st);
@@ -539,8 +676,8 @@ int build_tdesc(Matrix &M, cudaStream_t st) {
     TSP_CK(cudaMalloc(&M.jcols, n * 16 * sizeof(int32_t)));
     M.device_bytes += n * (int64_t)(sizeof(WItem) + 64);
     k_blob_fill<<<(unsigned)((n * 32 + 255) / 256), 256, 0, st>>>(M.items, n, M.m, M.n, start16, M.tdesc, M.tileColIdx,
-                                                                 M.tileFmt, M.payload, M.remRowPtr, M.remCol,
-                                                                 M.remVal, M.blob, M.witems, M.jcols);
+                                                                 TV, M.payload, M.remRowPtr, M.remCol, M.remVal,
+                                                                 M.blob, M.witems, M.jcols);
     TSP_CK(cudaGetLastError());
     return 0;
 }

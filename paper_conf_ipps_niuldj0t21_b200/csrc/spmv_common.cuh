@@ -72,10 +72,23 @@ __host__ __device__ __forceinline__ int64_t item_rows(const Item &it, int64_t m)
 // A create-time copy of everything one work item reads, contiguous and
 // 16-byte aligned part by part, so a single TMA bulk copy stages it:
 //   dsc : the descriptor list (k_dsc_write), ndsc x 8 B
-//   pay : the tiles' canonical payload bytes
+//   pay : the tiles' payload bytes: canonical, except that with a
+//         COO run a COO tile is absent and a HYB(w) tile is its ELL(w) part
 //   rp  : remainder row pointers of the item's rows, rebased to the item's
 //         entry range and clamped to it (rows + 1 ints)
 //   col, val : the item's remainder entries
+// ADPT mode instead gathers the item's COO data -- its COO tiles and the
+// COO parts of its HYB tiles, at most 11 and 15 entries per tile (P:181,
+// P:105) -- into one COO run in the same three parts: rp = the 16 row
+// pointers (+ end) of the run, col = one byte per entry holding its x slot
+// (tile index * 16 + column in the tile), val = the values, entries in row
+// order and, within a row, in tile then column order.  The kernel sums the
+// run two lanes per row from the staged x segments (coo_run) instead of
+// running each 1..11-entry tile on its own half-warp.
+__host__ __device__ __forceinline__ uint32_t run_bytes(uint32_t e) {
+    return e ? 80u + up16(e) + up16(8u * e) : 0u;
+}
+
 struct BlobParts {
     uint32_t pay, rp, col, val, total;
 };
@@ -83,8 +96,12 @@ struct BlobParts {
 __host__ __device__ __forceinline__ BlobParts blob_parts(const Item &it, int64_t m) {
     BlobParts b;
     b.pay = up16(8u * (uint32_t)it.ndsc);
-    b.rp = b.pay + (it.offe - it.offb) * 16u;
-    if (it.ke > it.kb) {
+    b.rp = b.pay + it.pay_bytes;
+    if (it.run_e > 0) {
+        b.col = b.rp + 80u;
+        b.val = b.col + up16(it.run_e);
+        b.total = b.val + up16(8u * it.run_e);
+    } else if (it.ke > it.kb) {
         const uint32_t rows = (uint32_t)item_rows(it, m);
         const uint32_t e = (uint32_t)(it.ke - it.kb);
         b.col = b.rp + up16(4u * (rows + 1));

@@ -48,6 +48,14 @@ __device__ __forceinline__ double lds_f64_lt(int i, int len, uint32_t a) {
         : "r"(i), "r"(len), "r"(a));
     return v;
 }
+// u8 at a if i < len, else 0
+__device__ __forceinline__ uint32_t lds_u8_lt(int i, int len, uint32_t a) {
+    uint32_t v;
+    asm("{\n\t.reg .pred q;\n\tsetp.lt.s32 q, %1, %2;\n\tmov.b32 %0, 0;\n\t@q ld.shared.u8 %0, [%3];\n\t}"
+        : "=r"(v)
+        : "r"(i), "r"(len), "r"(a));
+    return v;
+}
 // a remainder entry k (column, value) if k < e, else (cdef, 0.0): cdef is a
 // column the item itself references (so x[cdef] is a valid, finite x entry
 // on any rank that runs the item) and 0.0 * x[cdef] adds an exact zero

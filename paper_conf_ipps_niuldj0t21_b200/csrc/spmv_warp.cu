@@ -251,6 +251,28 @@ __device__ __forceinline__ void group_item(const Params &p, const WItem &it, uin
     }
 }
 
+// ADPT's COO run (blob_parts): the item's COO tiles and HYB COO parts as one
+// row-sorted list, summed two lanes per row like the remainder's short rows
+// (lane (r, h) takes entries b + h, b + h + 2, ...; the halves meet in the
+// final acc(r) + acc(r + 16)), each value times x from the staged segment of
+// its tile (x slot = tile index * 16 + column).  Replaces the per-tile COO
+// routines: 1..11-entry tiles left most of a half-warp idle.
+// A masked step multiplies 0.0 by x slot 0 (a staged x entry: finite).
+__device__ __forceinline__ void coo_run(uint32_t rpS, uint32_t xslS, uint32_t valS, int rows, uint32_t xs, int lane,
+                                        double &acc) {
+    const int r = lane & 15, h = lane >> 4;
+    const int b = lds_s32(rpS + 4 * min(r, rows)), e = lds_s32(rpS + 4 * min(r + 1, rows));
+    const int trips = (int)__reduce_max_sync(FULL, (unsigned)((e - b + 1 - h) >> 1));
+#pragma unroll 1
+    for (int i = 0; i < trips; i += 2) {
+        const int k0 = b + h + 2 * i, k1 = k0 + 2;
+        const double v0 = lds_f64_lt(k0, e, valS + 8 * k0), v1 = lds_f64_lt(k1, e, valS + 8 * k1);
+        const double x0 = lds_f64(xs + 8 * lds_u8_lt(k0, e, xslS + k0)), x1 = lds_f64(xs + 8 * lds_u8_lt(k1, e, xslS + k1));
+        acc = fma(v0, x0, acc);
+        acc = fma(v1, x1, acc);
+    }
+}
+
 // the tiles of one format group, two per step.  d: shared address of this
 // half's descriptor (see k_blob_fill): x = distance from the descriptor to the
 // tile's payload (CSR: to its csrRowPtr), y = aux | t*128 | nz << 11 | tm << 20 |
@@ -351,11 +373,15 @@ __device__ __forceinline__ void compute_item(const Params &p, const WItem &it, u
     // 2. fused CSR remainder, while the x segments land
     double acc = 0.0;
     const uint32_t rp = it.rp_col & 0xFFFFu;
-    if (total > rp)
+    const bool run = it.groups >> 31;  // the rp/col/val parts hold a COO run (ADPT), not a remainder
+    if (total > rp && !run)
         remainder(p, slot + rp, slot + (it.rp_col >> 16), slot + (it.val_tot & 0xFFFFu),
                   (int)((it.jt_rows_pay >> 8) & 31u), x_policy, lane, acc);
     if (p.x_vec) cp_async_wait_all();
     __syncwarp();
+    if (run)
+        coo_run(slot + rp, slot + (it.rp_col >> 16), slot + (it.val_tot & 0xFFFFu), (int)((it.jt_rows_pay >> 8) & 31u),
+                xs, lane, acc);
     // 3. tiles: format group by format group, two tiles per step
     {
         const uint32_t g = it.groups;
