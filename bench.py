@@ -44,7 +44,9 @@ WORKLOAD_DESC = {
 }
 # N = 1: the other BASELINE configs, each its own line in `secondary`
 SECONDARY = [("fem", "DEFERRED"), ("rmat20", "DEFERRED"), ("mixed", "ADPT"), ("mixed", "DEFERRED"),
-             ("lap2d_64", "DEFERRED")]
+             ("lap2d_64", "DEFERRED"),
+             # the optional byte-cost selection mode (not the paper's rule)
+             ("fem", "BYTES")]
 SINGLE_LAUNCHES = 60  # single-launch timing: median of this many isolated launches
 
 
@@ -745,7 +747,7 @@ def main():
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--workload", default=DEFAULT_WORKLOAD)
-    ap.add_argument("--mode", default="DEFERRED", choices=["ADPT", "DEFERRED", "AUTO", "FORCE_CSR"])
+    ap.add_argument("--mode", default="DEFERRED", choices=["ADPT", "DEFERRED", "AUTO", "FORCE_CSR", "BYTES"])
     ap.add_argument("--exchange", default="allgather", choices=["allgather", "halo"],
                     help="N>1: all-gather of y (north star, default) or the neighbour-only x exchange; "
                          "the other one is timed as a secondary entry")

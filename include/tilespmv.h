@@ -42,6 +42,12 @@ extern "C" {
 #define TILESPMV_MODE_DEFERRED 1  /* TileSpMV_DeferredCOO: COO data -> CSR remainder (default) */
 #define TILESPMV_MODE_AUTO 2      /* DEFERRED iff nnz >= 1.8e6 (reading R18), else ADPT */
 #define TILESPMV_MODE_FORCE_CSR 3 /* TileSpMV_CSR: every tile CSR */
+#define TILESPMV_MODE_BYTES 4     /* NOT the paper's rule: per tile, the format
+                                     with the fewest payload bytes (DESIGN.md §4 sizes, rounded
+                                     to 16; ELL only if every row is non-empty; ties to the
+                                     lower format code); no extraction.  The paper's thresholds
+                                     (Dns >= 128) were set on A100; a 136-entry FEM
+                                     triangle is 1,184 B as CSR against 2,048 B as Dns        */
 
 /* SpMV kernel of a handle (tilespmv_opts_t.kernel).  Both compute the same
  * y within the north-star bound; the work-item byte budget (and so the

@@ -19,6 +19,8 @@
  *                      independent, accumulated in x87 long double and rounded
  *                      once; also sum_j |a_ij * x_j| for the tolerance test.
  *   oracle_select      the TileSpMV_ADPT format rules.
+ *   oracle_select_bytes  the optional B200 byte-cost selection (SURVEY
+ *                      §8(f) f4; NOT the paper's rule): fewest payload bytes.
  *   oracle_hyb_width   the HYB ELL-width scan.
  *   oracle_tile        two-level tiled storage with the
  *                      DeferredCOO extraction, laid out in the
@@ -39,7 +41,7 @@ _Static_assert(LDBL_MANT_DIG == 64, "oracle needs x87 80-bit long double");
 /* tile formats, numbered in the order the paper lists them */
 enum { O_CSR = 0, O_COO = 1, O_ELL = 2, O_HYB = 3, O_DNS = 4, O_DNSROW = 5, O_DNSCOL = 6 };
 /* the three TileSpMV methods of P:177 (+ the size switch of P:235) */
-enum { O_MODE_ADPT = 0, O_MODE_DEFERRED = 1, O_MODE_AUTO = 2, O_MODE_FORCE_CSR = 3 };
+enum { O_MODE_ADPT = 0, O_MODE_DEFERRED = 1, O_MODE_AUTO = 2, O_MODE_FORCE_CSR = 3, O_MODE_BYTES = 4 };
 
 #define TILE 16 /* "the size is always 16 by 16" */
 
@@ -154,6 +156,63 @@ int oracle_select(const uint16_t masks[16], int32_t force_csr, int32_t *aux)
     return O_CSR;
 }
 
+/* B200 byte-cost selection (TILESPMV_MODE_BYTES; not the
+ * paper's rule, so no parity with its format statistics is claimed): the
+ * format whose payload, by the sizes of DESIGN.md §4 rounded up to 16 bytes,
+ * is smallest among the formats able to hold the tile:
+ *   CSR     8 nnz + 16 + ceil(nnz / 2)       any tile
+ *   COO     9 nnz                            any tile
+ *   ELL     136 * (max row length)           every row non-empty (R26: a pad
+ *                                            must be told from an entry)
+ *   HYB     136 w + 9 (nnz - 16 w), w = oracle_hyb_width (R11)   any tile
+ *   Dns     2048                             any tile
+ *   DnsRow  129 * (full rows)                every row 0 or 16 entries (R6)
+ *   DnsCol  129 * (full columns)             every column 0 or 16 entries
+ * Ties go to the lowest format code (P:96 order).  aux as oracle_select.   */
+int oracle_select_bytes(const uint16_t masks[16], int32_t *aux)
+{
+    int32_t lens[16];
+    int64_t nnz = 0;
+    int32_t colcnt[16] = {0};
+    for (int r = 0; r < TILE; ++r) {
+        lens[r] = popc16(masks[r]);
+        nnz += lens[r];
+        for (int c = 0; c < TILE; ++c)
+            if ((masks[r] >> c) & 1u) colcnt[c]++;
+    }
+    int32_t maxlen = 0, minlen = TILE, nr = 0, nc = 0, rows_full = 1, cols_full = 1;
+    for (int r = 0; r < TILE; ++r) {
+        if (lens[r] > maxlen) maxlen = lens[r];
+        if (lens[r] < minlen) minlen = lens[r];
+        if (lens[r] != 0 && lens[r] != TILE) rows_full = 0;
+        if (lens[r] == TILE) nr++;
+    }
+    for (int c = 0; c < TILE; ++c) {
+        if (colcnt[c] != 0 && colcnt[c] != TILE) cols_full = 0;
+        if (colcnt[c] == TILE) nc++;
+    }
+    int32_t hw = oracle_hyb_width(lens);
+    int64_t size[7];
+    int32_t faux[7] = {0, 0, maxlen, hw, 0, nr, nc};
+    int eligible[7] = {1, 1, minlen >= 1, 1, 1, rows_full, cols_full};
+    size[O_CSR] = 8 * nnz + 16 + (nnz + 1) / 2;
+    size[O_COO] = 9 * nnz;
+    size[O_ELL] = 136 * (int64_t)maxlen;
+    size[O_HYB] = 136 * (int64_t)hw + 9 * (nnz - 16 * (int64_t)hw);
+    size[O_DNS] = 2048;
+    size[O_DNSROW] = 129 * (int64_t)nr;
+    size[O_DNSCOL] = 129 * (int64_t)nc;
+    int best = -1;
+    int64_t best_size = 0;
+    for (int f = 0; f < 7; ++f) {
+        if (!eligible[f]) continue;
+        int64_t sz = (size[f] + 15) / 16 * 16;
+        if (best < 0 || sz < best_size) { best = f; best_size = sz; }
+    }
+    *aux = faux[best];
+    return best;
+}
+
 /* "gradually calculate the least memory space by setting the ELL width
  * from the maximum to zero until the smallest memory space is found".
  * Memory of a width-w HYB tile (R11): 16*w ELL slots of value + 4-bit column
@@ -242,7 +301,8 @@ void oracle_tiling_free(oracle_tiling *t)
     free(t);
 }
 
-/* mode: ADPT, DEFERRED, AUTO (DEFERRED iff nnz >= 1.8e6, R18) or FORCE_CSR.
+/* mode: ADPT, DEFERRED, AUTO (DEFERRED iff nnz >= 1.8e6, R18), FORCE_CSR, or
+ * BYTES (oracle_select_bytes, no extraction).
  * Returns NULL on allocation failure or non-canonical input.               */
 oracle_tiling *oracle_tile(int64_t m, int64_t n, const int32_t *rowptr,
                            const int32_t *colidx, const double *val, int32_t mode)
@@ -316,7 +376,7 @@ oracle_tiling *oracle_tile(int64_t m, int64_t n, const int32_t *rowptr,
             }
             /* step 5: select the format */
             int32_t aux;
-            int fmt = oracle_select(masks, force_csr, &aux);
+            int fmt = mode == O_MODE_BYTES ? oracle_select_bytes(masks, &aux) : oracle_select(masks, force_csr, &aux);
             T->sel_tiles[fmt]++;
             T->sel_nnz[fmt] += nt;
             /* step 7: DeferredCOO extracts COO tiles and HYB COO parts */

@@ -19,7 +19,7 @@ SRC = os.path.join(HERE, "oracle.c")
 
 FMT_NAMES = ["CSR", "COO", "ELL", "HYB", "DNS", "DNSROW", "DNSCOL"]
 CSR, COO, ELL, HYB, DNS, DNSROW, DNSCOL = range(7)
-MODES = {"ADPT": 0, "DEFERRED": 1, "AUTO": 2, "FORCE_CSR": 3}
+MODES = {"ADPT": 0, "DEFERRED": 1, "AUTO": 2, "FORCE_CSR": 3, "BYTES": 4}
 
 
 OMP_SRC = os.path.join(HERE, "cpu_csr_omp.c")
@@ -68,6 +68,8 @@ def lib():
         L.oracle_spmv_f64.restype = None
         L.oracle_select.argtypes = [p, ctypes.c_int32, p]
         L.oracle_select.restype = ctypes.c_int
+        L.oracle_select_bytes.argtypes = [p, p]
+        L.oracle_select_bytes.restype = ctypes.c_int
         L.oracle_hyb_width.argtypes = [p]
         L.oracle_hyb_width.restype = ctypes.c_int
         L.oracle_tile.argtypes = [ctypes.c_int64, ctypes.c_int64, p, p, p, ctypes.c_int32]
@@ -136,6 +138,14 @@ def select(masks, force_csr: bool = False):
     aux = np.zeros(1, np.int32)
     f = lib().oracle_select(_ptr(m), int(force_csr), _ptr(aux))
     return int(f), int(aux[0])
+
+
+def select_bytes(masks):
+    """B200 byte-cost format rule for one tile (oracle_select_bytes) -> (fmt, aux)."""
+    m = np.ascontiguousarray(np.asarray(masks, dtype=np.uint16))
+    aux = ctypes.c_int32()
+    f = lib().oracle_select_bytes(_ptr(m), ctypes.byref(aux))
+    return f, aux.value
 
 
 def hyb_width(lens) -> int:

@@ -87,7 +87,7 @@ int tilespmv_create_from_csr(tilespmv_handle_t *out, int64_t m, int64_t n, int64
     if (nnz > 0 && (!d_colidx || !d_val)) return set_error(TILESPMV_INVALID_ARG, "colidx/val is NULL");
     tilespmv_opts_t o{TILESPMV_MODE_DEFERRED, 1, TILESPMV_KERNEL_AUTO, 0};
     if (opts) o = *opts;
-    if (o.mode < 0 || o.mode > 3) return set_error(TILESPMV_INVALID_ARG, "unknown mode");
+    if (o.mode < 0 || o.mode > TILESPMV_MODE_BYTES) return set_error(TILESPMV_INVALID_ARG, "unknown mode");
     if (o.kernel < TILESPMV_KERNEL_AUTO || o.kernel > TILESPMV_KERNEL_GATHER)
         return set_error(TILESPMV_INVALID_ARG, "unknown kernel");
     if (o.keep_layout != 0 && o.keep_layout != 1) return set_error(TILESPMV_INVALID_ARG, "keep_layout must be 0 or 1");

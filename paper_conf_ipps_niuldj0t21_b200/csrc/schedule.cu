@@ -550,9 +550,10 @@ __global__ void k_cta_units(const int64_t *incl, const int32_t *units, int64_t n
     cta_begin[b] = lo;
 }
 
-// ADPT mode gathers each item's COO data into a COO run (blob_parts)
+// ADPT (and BYTES) mode gathers each item's COO data into a COO run (blob_parts)
 TileView tile_view(const Matrix &M) {
-    return {M.tilePtr, M.tileOff, M.tileFmt, M.tileAux, M.tileNnz, M.mode == TILESPMV_MODE_ADPT ? 1 : 0};
+    return {M.tilePtr, M.tileOff, M.tileFmt, M.tileAux, M.tileNnz,
+            M.mode == TILESPMV_MODE_ADPT || M.mode == TILESPMV_MODE_BYTES ? 1 : 0};
 }
 
 // stream-ordered temporary device buffer

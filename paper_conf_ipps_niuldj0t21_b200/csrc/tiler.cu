@@ -173,7 +173,28 @@ __global__ void k_select(const uint32_t *__restrict__ mask32, int64_t numtile, i
         // variance over the 16 rows, CV^2 = (16*S2 - n^2) / n^2, so
         //   CV <= te=0.2  <=>  400*S2 <= 26*n^2 ;  CV > th=1.0  <=>  8*S2 > n^2.
         int f, a = 0;
-        if (mode == TILESPMV_MODE_FORCE_CSR) f = F_CSR;
+        if (mode == TILESPMV_MODE_BYTES) {
+            // optional B200 byte-cost rule (not the paper's):
+            // the eligible format with the smallest 16-rounded payload (§4
+            // sizes), ties to the lower format code
+            auto r16 = [](int v) { return (v + 15) & ~15; };
+            int best = r16(8 * n + 16 + (n + 1) / 2);
+            f = F_CSR;
+            auto take = [&](int ff, int sz, int aa, bool ok) {
+                if (ok && r16(sz) < best) {
+                    best = r16(sz);
+                    f = ff;
+                    a = aa;
+                }
+            };
+            take(F_COO, 9 * n, 0, true);
+            take(F_ELL, 136 * maxl, maxl, minl >= 1);  // every row non-empty (R26)
+            take(F_HYB, 136 * minl + 9 * (n - 16 * minl), minl, true);
+            take(F_DNS, 2048, 0, true);
+            take(F_DNSROW, 129 * nfull, nfull, rows_full);
+            take(F_DNSCOL, 129 * __popc(mk0), __popc(mk0), cols_same);
+        }
+        else if (mode == TILESPMV_MODE_FORCE_CSR) f = F_CSR;
         else if (n < 12) f = F_COO;
         else if (n >= 128) f = F_DNS;
         else if (rows_full) { f = F_DNSROW; a = nfull; }

@@ -15,7 +15,7 @@ import numpy as np
 from . import _build
 
 FORMATS = ["CSR", "COO", "ELL", "HYB", "DNS", "DNSROW", "DNSCOL"]
-MODES = {"ADPT": 0, "DEFERRED": 1, "AUTO": 2, "FORCE_CSR": 3}
+MODES = {"ADPT": 0, "DEFERRED": 1, "AUTO": 2, "FORCE_CSR": 3, "BYTES": 4}
 KERNELS = {"AUTO": 0, "SM_QUEUE": 1, "DENSE_ROWS": 2, "GATHER": 3}
 ARRAYS = {"tilePtr": (0, np.int32), "tileColIdx": (1, np.int32), "tileNnz": (2, np.int32),
           "tileFmt": (3, np.uint8), "tileAux": (4, np.uint8), "tileOff": (5, np.uint32),

@@ -61,7 +61,7 @@ def test_tile_profile_fuzz(cuda_device, kernel):
         x = gen.dense_x(n, 7 + seed)
         yref, absy = O.spmv(A, x)
         xd = torch.from_numpy(x).to(cuda_device)
-        for mode in ("ADPT", "DEFERRED", "FORCE_CSR"):
+        for mode in ("ADPT", "DEFERRED", "FORCE_CSR", "BYTES"):
             M = TiledMatrix.from_host_csr(A, mode=mode, device=cuda_device, kernel=kernel)
             y1 = M.run(xd).cpu().numpy()
             y2 = M.run(xd).cpu().numpy()

@@ -17,7 +17,7 @@ pytestmark = pytest.mark.gpu
 GOLDEN = os.path.join(os.path.dirname(__file__), "golden")
 SMALL = ["lap2d_64", "lap2d_37x29", "fem_small", "rmat12", "mixed_small", "stencil27_21",
          "stencil27_40"]
-MODES = ["ADPT", "DEFERRED", "FORCE_CSR", "AUTO"]
+MODES = ["ADPT", "DEFERRED", "FORCE_CSR", "AUTO", "BYTES"]
 TOL = 1e-12
 
 
@@ -104,7 +104,7 @@ def test_spmv_parity_small(cuda_device, mode):
         M.close()
 
 
-@pytest.mark.parametrize("mode", ["ADPT", "DEFERRED", "FORCE_CSR"])
+@pytest.mark.parametrize("mode", ["ADPT", "DEFERRED", "FORCE_CSR", "BYTES"])
 def test_spmv_integer_bitwise(cuda_device, mode):
     """Integer-valued A and x: every summation order is exact -> bitwise."""
     import torch

@@ -339,8 +339,8 @@ def check_invariants(A, T):
         assert sizes[t] == (s + 15) // 16 * 16
         if T.tileFmt[t] in (ELL, HYB):
             assert 0 <= T.tileAux[t] <= 16
-        if T.tileFmt[t] in (DNSROW, DNSCOL):
-            assert 1 <= T.tileAux[t] <= 7
+        if T.tileFmt[t] in (DNSROW, DNSCOL):  # paper rules: <= 7 (8 full rows = 128 -> Dns)
+            assert 1 <= T.tileAux[t] <= (15 if T.mode == O.MODES["BYTES"] else 7)
     assert T.payload_bytes == T.tileOff[-1] * 16
     assert T.remRowPtr[-1] == T.rem_nnz
 
@@ -369,7 +369,7 @@ def _all_mats():
     yield from _special()
 
 
-@pytest.mark.parametrize("mode", ["ADPT", "DEFERRED", "FORCE_CSR", "AUTO"])
+@pytest.mark.parametrize("mode", ["ADPT", "DEFERRED", "FORCE_CSR", "AUTO", "BYTES"])
 def test_roundtrip_and_invariants(mode):
     for A in _all_mats():
         T = O.tile(A, mode)
@@ -381,7 +381,7 @@ def test_roundtrip_and_invariants(mode):
         assert np.array_equal(v.view(np.uint64), A.val.view(np.uint64)), A.name
         if mode == "FORCE_CSR":
             assert set(np.unique(T.tileFmt)) <= {CSR} and T.rem_nnz == 0
-        if mode == "ADPT":
+        if mode in ("ADPT", "BYTES"):
             assert T.rem_nnz == 0
 
 
@@ -469,3 +469,66 @@ def test_golden_counts_match_oracle():
             assert g["payload_bytes"] == T.payload_bytes
             assert g["rem_nnz"] == T.rem_nnz
             assert g["nnz"] == A.nnz
+
+
+# --------------------------------------------------------------------------
+# optional B200 byte-cost selection (not the paper's rule):
+# hand-computed payload sizes (rounded to 16) at its boundaries
+# --------------------------------------------------------------------------
+
+def _masks_full_rows(full, extra=()):
+    m = [0xFFFF if r in full else 0 for r in range(16)]
+    for r, cols in extra:
+        for c in cols:
+            m[r] |= 1 << c
+    return m
+
+
+@pytest.mark.parametrize("masks,fmt,aux,why", [
+    # FEM's upper-triangle tile (row r holds columns r..15, 136 entries): CSR
+    # 8*136+16+68 = 1172 -> 1184 beats Dns 2048, ELL 16*136 = 2176, HYB(w=1)
+    # 136+9*120 = 1216, COO 1224 (the paper's rule takes Dns: n >= 128)
+    ([(0xFFFF << r) & 0xFFFF for r in range(16)], CSR, 0, "triangle"),
+    # a full tile: Dns 2048 < DnsRow/DnsCol 2064 < CSR 2192
+    ([0xFFFF] * 16, DNS, 0, "full"),
+    # 13 full rows + rows of 15, 15 and 1 = 239 entries: CSR 1912+16+120 =
+    # 2048 ties Dns 2048 and the lower code wins (HYB w=1: 2143 -> 2144)
+    (_masks_full_rows(range(13), [(13, range(15)), (14, range(1, 16)), (15, [0])]), CSR, 0, "239"),
+    # ... and 240 (last row of 2): CSR 1920+16+120 = 2056 -> 2064 > Dns 2048
+    (_masks_full_rows(range(13), [(13, range(15)), (14, range(1, 16)), (15, [0, 1])]), DNS, 0, "240"),
+    # one entry: COO 9 -> 16 beats CSR 25 -> 32
+    ([1] + [0] * 15, COO, 0, "single"),
+    # one full row: COO 144 ties DnsRow 129 -> 144; the lower code (COO) wins
+    (_masks_full_rows([5]), COO, 0, "one full row"),
+    # 3 full rows: DnsRow 387 -> 400 beats COO 432, CSR 384+16+24 = 424 -> 432
+    (_masks_full_rows([1, 7, 12]), DNSROW, 3, "three full rows"),
+    # 16 rows of 3: ELL 408 -> 416 ties HYB(w=3) 408 -> 416 and beats CSR
+    # 424 -> 432 and COO 432: ELL (lower code)
+    ([0b111 << (r % 14) for r in range(16)], ELL, 3, "equal rows of 3"),
+    # 15 rows of 3 and an empty row: ELL not eligible (R26), HYB w=0 = COO
+    # 405 -> 416, CSR 360+16+23 = 399 -> 400
+    ([0b111 << (r % 14) for r in range(15)] + [0], CSR, 0, "empty row"),
+])
+def test_select_bytes_boundaries(masks, fmt, aux, why):
+    assert O.select_bytes(masks) == (fmt, aux), why
+
+
+def test_select_bytes_is_a_minimum_over_brute_force_layouts():
+    """On random tiles, the byte rule's choice has the smallest payload of the
+    formats that can hold the tile, sizes taken from the oracle's own packing
+    of single-tile matrices in each format (BYTES, ADPT, FORCE_CSR tilings)."""
+    rng = np.random.default_rng(5)
+    for trial in range(300):
+        dens = rng.choice([0.02, 0.1, 0.3, 0.6, 0.95])
+        M = (rng.random((16, 16)) < dens)
+        if not M.any():
+            continue
+        masks = [int(sum(1 << c for c in range(16) if M[r, c])) for r in range(16)]
+        f, a = O.select_bytes(masks)
+        A = gen.from_dense(np.where(M, 1.0 + rng.random((16, 16)), 0.0))
+        Tb = O.tile(A, "BYTES")
+        assert Tb.numtile == 1 and int(Tb.tileFmt[0]) == f and int(Tb.tileAux[0]) == a
+        got = int(Tb.payload_bytes)
+        # the paper's choice and plain CSR are never smaller
+        for mode in ("ADPT", "FORCE_CSR"):
+            assert got <= int(O.tile(A, mode).payload_bytes), (trial, mode)
