@@ -4,7 +4,7 @@ sys.path.insert(0, '.')
 from paper_conf_ipps_niuldj0t21_b200 import TiledMatrix
 from synthetic import gen
 out = {}
-for name in ("rmat12", "mixed_small", "rmat20", "mixed"):
+for name in ("rmat12", "mixed_small", "stencil27_40", "rmat20", "mixed"):
     A, x = gen.make(name)
     for mode in ("DEFERRED", "ADPT"):
         M = TiledMatrix.from_host_csr(A, mode=mode, device=torch.device("cuda", 0))

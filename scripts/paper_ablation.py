@@ -4,7 +4,8 @@
 
   * Fig. 6: TileSpMV_CSR (FORCE_CSR) vs TileSpMV_ADPT vs
     TileSpMV_DeferredCOO (and AUTO, the 1.8M switch of P:235, reading R18)
-    GFLOP/s of the same matrix;
+    GFLOP/s of the same matrix, plus the optional byte-cost selection
+    (BYTES, SURVEY §8(f) f4; not the paper's rule);
   * Fig. 7 (P:229): tiles and nonzeros per format (ADPT selection);
   * Fig. 10: space of the tiled form against plain CSR
     (12 B per nonzero + 4 B per row pointer);
@@ -32,7 +33,7 @@ FMTS = ["CSR", "COO", "ELL", "HYB", "DNS", "DNSROW", "DNSCOL"]
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--workloads", default="lap2d_64,fem,rmat20,mixed,stencil27_200")
-    ap.add_argument("--modes", default="FORCE_CSR,ADPT,DEFERRED,AUTO")
+    ap.add_argument("--modes", default="FORCE_CSR,ADPT,DEFERRED,AUTO,BYTES")
     ap.add_argument("--steps", type=int, default=100)
     a = ap.parse_args()
     import numpy as np
