@@ -38,7 +38,10 @@ struct __align__(16) Item {
     uint32_t offb;    // payload offset of tile tb (16-byte units)
     uint32_t offe;    // payload offset one past the last tile
     uint32_t pay_bytes;  // bytes of the tiles in the blob payload (tile_cost; canonical unless a COO run)
-    uint32_t run_e;      // entries of the item's COO run (ADPT: COO tiles + HYB COO parts), 0 if none
+    uint32_t run_e;      // entries of the item's COO run (ADPT: COO tiles + HYB COO parts; DEFERRED:
+                         // a remainder whose x lies in the item's staged segments), 0 if none
+    uint32_t xseg;       // x segments the kernel stages: the tiles' J, then (local remainder) the
+                         // remainder's other tile columns
     int32_t split;    // split-row index, or -1 if the item covers its whole tile row
     int32_t part_nt;  // part index (bits 0-23) | tiles << 24 (5 bits) | local << 29 | last-of-group << 30
     int32_t dbeg;      // first entry of the item's tile-descriptor list (dlist)

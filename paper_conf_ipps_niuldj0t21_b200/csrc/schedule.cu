@@ -31,7 +31,9 @@ struct TileView {
     const uint32_t *tileOff;
     const uint8_t *tileFmt, *tileAux;
     const int32_t *tileNnz;
-    int run;
+    const int32_t *tileColIdx;
+    int run;        // ADPT / BYTES: COO data as a COO run
+    int local_rem;  // DEFERRED: remainders that fit the x stage as a local run (rem_local)
 };
 
 // Bytes tile g occupies in its item's blob payload, and the entries it adds
@@ -111,6 +113,7 @@ __device__ int items_for_row(int64_t I, const TileView &T, const int32_t *remRow
             it.offe = tileOff[t];
             it.pay_bytes = pays;
             it.run_e = rune;
+            it.xseg = (uint32_t)(t - tb);
             it.split = split;
             const bool local = split >= 0 && nparts <= lp;
             const bool last = split >= 0 && (cnt == nparts - 1 || cnt % lp == lp - 1);
@@ -180,7 +183,7 @@ __device__ int window_items(int64_t w, const TileView &T, const int32_t *remRowP
             it.kb = remRowPtr ? remRowPtr[16 * I] : 0;
             it.ke = remRowPtr ? remRowPtr[imin64(16 * J, m)] : 0;
             it.offb = it.offe = tileOff[it.tb];
-            it.pay_bytes = it.run_e = 0;
+            it.pay_bytes = it.run_e = it.xseg = 0;
             it.split = -1;
             it.part_nt = 0;
             it.dbeg = it.ndsc = 0;
@@ -285,10 +288,58 @@ __global__ void k_dsc_write(Item *items, int64_t n, const int32_t *dbeg, const i
 
 // blob length per item; *over is set if one exceeds the kernel's slot (a
 // schedule bug: the kernel would stage past its shared-memory slot)
-__global__ void k_blob_len(const Item *items, int64_t n, int64_t m, uint32_t slot, int64_t *len16, int32_t *over) {
+// DEFERRED, an ordinary item with remainder rows of <= 32 entries: the tile
+// columns of its remainder entries that are not among its tiles' (ascending),
+// if they fit the x stage beside the tiles' segments (returns their count,
+// the list in extra[]), else -1.  Such an item runs its remainder as a local
+// run (blob_parts): x from the staged segments through a one-byte x slot per
+// entry instead of a global gather, the two-lanes-per-row sum of the
+// remainder's short rows unchanged (coo_run), so y keeps every bit.
+__device__ int rem_local(const Item &it, int64_t m, const TileView &T, const int32_t *remRowPtr, const int32_t *remCol,
+                         int max_tiles, int32_t *extra) {
+    if (!T.local_rem || it.ntr > 0 || it.ke <= it.kb) return -1;
+    const int nt = item_nt(it);
+    const int rows = (int)item_rows(it, m);
+    for (int r = 0; r < rows; ++r) {  // the MED path's domain: every row <= 32 entries
+        int b = remRowPtr[16 * (int64_t)it.I + r], e = remRowPtr[16 * (int64_t)it.I + r + 1];
+        b = b < it.kb ? it.kb : (b > it.ke ? it.ke : b);
+        e = e < it.kb ? it.kb : (e > it.ke ? it.ke : e);
+        if (e - b > 32) return -1;
+    }
+    int nx = 0;
+    for (int k = it.kb; k < it.ke; ++k) {
+        const int J = remCol[k] >> 4;
+        bool seen = false;
+        for (int t = 0; t < nt && !seen; ++t) seen = T.tileColIdx[it.tb + t] == J;
+        for (int q = 0; q < nx && !seen; ++q) seen = extra[q] == J;
+        if (seen) continue;
+        if (nt + nx >= max_tiles) return -1;
+        int q = nx++;  // insertion keeps extra[] ascending
+        while (q > 0 && extra[q - 1] > J) {
+            extra[q] = extra[q - 1];
+            --q;
+        }
+        extra[q] = J;
+    }
+    return nx;
+}
+
+// blob length per item (deciding the DEFERRED local runs first); *over is
+// set if one exceeds the kernel's slot (a schedule bug: the kernel would
+// stage past its shared-memory slot)
+__global__ void k_blob_len(Item *items, int64_t n, int64_t m, uint32_t slot, TileView T, const int32_t *remRowPtr,
+                           const int32_t *remCol, int max_tiles, int64_t *len16, int32_t *over) {
     int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     if (k >= n) return;
-    const uint32_t total = blob_parts(items[k], m).total;
+    Item it = items[k];
+    int32_t extra[kItemTiles];
+    const int nx = rem_local(it, m, T, remRowPtr, remCol, max_tiles, extra);
+    if (nx >= 0) {
+        it.run_e = (uint32_t)(it.ke - it.kb);
+        it.xseg = (uint32_t)(item_nt(it) + nx);
+        items[k] = it;
+    }
+    const uint32_t total = blob_parts(it, m).total;
     len16[k] = total / 16;
     if (total > slot) atomicOr(over, 1);
 }
@@ -313,7 +364,7 @@ __global__ void k_blob_fill(Item *items, int64_t nitems, int64_t m, int64_t n, c
         w.blob16 = it.blob16;
         w.I = (uint32_t)it.I;
         w.split = it.split;
-        w.part_nt = it.part_nt;
+        w.part_nt = (it.part_nt & ~(31 << 24)) | (int32_t)(it.xseg << 24);  // x segments to stage
         const uint32_t rows = (uint32_t)item_rows(it, m);
         const uint32_t last = it.ntr > 0 ? rows - 16u * (uint32_t)(it.ntr - 1) : rows;
         w.jt_rows_pay = (uint32_t)it.ntr | (last << 8) | (b.pay << 16);
@@ -326,7 +377,7 @@ __global__ void k_blob_fill(Item *items, int64_t nitems, int64_t m, int64_t n, c
         }
         uint32_t g = 0;
         for (int f = 0; f < 7; ++f) g |= (uint32_t)((cnt[f] + 1) >> 1) << (4 * f);
-        w.groups = g | (it.run_e > 0 ? 1u << 31 : 0u);
+        w.groups = g | (it.run_e > 0 ? 1u << 31 : 0u);  // a COO run or a local remainder run
         witems[k] = w;
     }
     for (uint32_t o = 4 * lane; o < b.total; o += 128) *reinterpret_cast<uint32_t *>(dst + o) = 0u;  // padding
@@ -368,12 +419,21 @@ __global__ void k_blob_fill(Item *items, int64_t nitems, int64_t m, int64_t n, c
         csr_max = max(csr_max, __reduce_max_sync(0xFFFFFFFFu, fi == F_CSR ? tm : 0u));
         ell_max = max(ell_max, __reduce_max_sync(0xFFFFFFFFu, fi == F_ELL ? tm : 0u));
     }
+    // the x segments: the tiles' columns, then a DEFERRED local run's others
+    const bool local = !T.run && it.run_e > 0;
+    int32_t extra[kItemTiles];
+    const int nx = local ? rem_local(it, m, T, remRowPtr, remCol, kItemTiles, extra) : 0;
+    int jseg = 0;
+    if (lane < 16) {
+        jseg = lane < nt ? tileColIdx[it.tb + lane] : (lane < nt + nx ? extra[lane - nt] : 0);
+        jcols[k * 16 + lane] = jseg;
+    }
     // item-wide extents: the kernel runs such items' CSR / ELL groups with
-    // straight-line 3-step routines and no per-pair dispatch
-    const bool xtail = nt > 0 && 16 * (int64_t)tileColIdx[it.tb + nt - 1] + 16 > n;
+    // straight-line 3-step routines and no per-pair dispatch; bit 30: some
+    // staged segment reaches past x[n-1]
+    const bool xtail = __any_sync(0xFFFFFFFFu, lane < nt + nx && 16 * (int64_t)jseg + 16 > n);
     if (lane == 0)
         witems[k].groups |= (csr_max <= 3 ? 1u << 28 : 0u) | (ell_max <= 3 ? 1u << 29 : 0u) | (xtail ? 1u << 30 : 0u);
-    if (lane < 16) jcols[k * 16 + lane] = lane < nt ? tileColIdx[it.tb + lane] : 0;
     if (!T.run) {  // the canonical payload bytes of the item's tiles, in one piece
         const uint4 *ps = reinterpret_cast<const uint4 *>(payload + (size_t)it.offb * 16);
         uint4 *pd = reinterpret_cast<uint4 *>(dst + b.pay);
@@ -445,7 +505,26 @@ __global__ void k_blob_fill(Item *items, int64_t nitems, int64_t m, int64_t n, c
             }
         }
     }
-    if (it.ke > it.kb) {
+    if (local) {  // the remainder as a local run: rows' pointers, x slots, values
+        const int rows = (int)item_rows(it, m);
+        int32_t *rp = reinterpret_cast<int32_t *>(dst + b.rp);
+        for (int i = lane; i <= 16; i += 32) {
+            int v = remRowPtr[16 * (int64_t)it.I + min(i, rows)];
+            v = v < it.kb ? it.kb : (v > it.ke ? it.ke : v);
+            rp[i] = v - it.kb;
+        }
+        uint8_t *xsl = dst + b.col;
+        unsigned long long *vd = reinterpret_cast<unsigned long long *>(dst + b.val);
+        const unsigned long long *vs = reinterpret_cast<const unsigned long long *>(remVal);
+        for (int i = lane; i < it.ke - it.kb; i += 32) {
+            const int c = remCol[it.kb + i], J = c >> 4;
+            int s = 0;
+            for (int t = 0; t < nt + nx; ++t)
+                if ((t < nt ? tileColIdx[it.tb + t] : extra[t - nt]) == J) s = t;
+            xsl[i] = (uint8_t)(16 * s + (c & 15));
+            vd[i] = vs[it.kb + i];
+        }
+    } else if (it.ke > it.kb) {
         const int rows = (int)item_rows(it, m);
         int32_t *rp = reinterpret_cast<int32_t *>(dst + b.rp);
         for (int i = lane; i <= rows; i += 32) {
@@ -552,8 +631,9 @@ __global__ void k_cta_units(const int64_t *incl, const int32_t *units, int64_t n
 
 // ADPT (and BYTES) mode gathers each item's COO data into a COO run (blob_parts)
 TileView tile_view(const Matrix &M) {
-    return {M.tilePtr, M.tileOff, M.tileFmt, M.tileAux, M.tileNnz,
-            M.mode == TILESPMV_MODE_ADPT || M.mode == TILESPMV_MODE_BYTES ? 1 : 0};
+    return {M.tilePtr, M.tileOff, M.tileFmt, M.tileAux, M.tileNnz, M.tileColIdx,
+            M.mode == TILESPMV_MODE_ADPT || M.mode == TILESPMV_MODE_BYTES ? 1 : 0,
+            M.mode == TILESPMV_MODE_DEFERRED ? 1 : 0};
 }
 
 // stream-ordered temporary device buffer
@@ -661,7 +741,8 @@ int build_tdesc(Matrix &M, cudaStream_t st) {
     int64_t *len16 = lenb.as<int64_t>(), *start16 = len16 + (n + 1);
     TSP_CK(cudaMemsetAsync(len16 + n, 0, sizeof(int64_t), st));
     TSP_CK(cudaMemsetAsync(cnt + n, 0, sizeof(int32_t), st));  // cnt[n]: slot overflow flag
-    k_blob_len<<<nb, 256, 0, st>>>(M.items, n, M.m, (uint32_t)M.item_bytes, len16, cnt + n);
+    k_blob_len<<<nb, 256, 0, st>>>(M.items, n, M.m, (uint32_t)M.item_bytes, TV, M.remRowPtr, M.remCol, M.item_tiles,
+                                   len16, cnt + n);
     if (int rc = scan([&](void *t, size_t &b) { return cub::DeviceScan::ExclusiveSum(t, b, len16, start16, (int)(n + 1), st); }, st)) return rc;
     int64_t total16 = 0;
     int32_t over = 0;
