@@ -155,6 +155,12 @@ __device__ __forceinline__ void cp_async_wait_all() {
     asm volatile("cp.async.commit_group;\n\tcp.async.wait_group 0;" ::: "memory");
 }
 __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+// counter += v with acquire-release semantics at gpu scope; returns the old value
+__device__ __forceinline__ int atom_add_acq_rel_gpu(int32_t *a, int v) {
+    int old;
+    asm volatile("atom.acq_rel.gpu.global.add.s32 %0, [%1], %2;" : "=r"(old) : "l"(a), "r"(v) : "memory");
+    return old;
+}
 // Programmatic dependent launch: let the next kernel in the stream start its
 // prologue early / wait until the previous kernel's writes are visible
 __device__ __forceinline__ void griddep_launch_dependents() {

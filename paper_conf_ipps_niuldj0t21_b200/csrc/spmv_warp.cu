@@ -417,13 +417,15 @@ __device__ __forceinline__ void compute_item(const Params &p, const WItem &it, u
             const int ngroups = (si.y + kLocalParts - 1) / kLocalParts;
             const int gidx = (it.part_nt & 0xFFFFFF) / kLocalParts;
             if (lane < 16) __stcg(p.partials + (int64_t)(si.x + gidx) * 16 + lane, sum);
-            __threadfence();
+            // the warp's partial stores, then lane 0's counter increment with
+            // release (and acquire) semantics at gpu scope: the last group to
+            // arrive sees every group's partial (no full membar.gl fences)
             __syncwarp();
             int old = 0;
-            if (lane == 0) old = atomicAdd(p.counters + it.split, 1);
+            if (lane == 0) old = atom_add_acq_rel_gpu(p.counters + it.split, 1);
             old = __shfl_sync(FULL, old, 0);
             if (old == ngroups - 1) {  // half h sums groups h, h+2, ... in order, 4 loads in flight
-                __threadfence();
+                __syncwarp();
                 double s = 0.0;
                 for (int q0 = h; q0 < ngroups; q0 += 8) {
                     double v[4];
