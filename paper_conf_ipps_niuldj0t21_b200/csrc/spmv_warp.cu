@@ -21,11 +21,11 @@
 //   tilespmv_fp64_sm<32,4608,16> SM_QUEUE: one CTA of 32 warps per SM, 4.5 KB
 //                                 slots, warps claim units from a
 //                                 shared-memory queue (222 KB of shared memory)
-//   tilespmv_fp64_sm<32,2304,8>  GATHER: the same with 2.25 KB slots and at
-//                                 most 8 tiles per item (115 KB): the L1 left
+//   tilespmv_fp64_sm<32,3328,4>  GATHER: the same with 3.25 KB slots and at
+//                                 most 4 tiles per item (132 KB): the L1 left
 //                                 to the remainder's x gathers grows from ~30
-//                                 to ~140 KB (power-law matrices in DEFERRED
-//                                 mode: R-MAT 127.6 -> 114.2 us)
+//                                 to ~125 KB (power-law matrices in DEFERRED
+//                                 mode: R-MAT 127.6 -> 109.0 us)
 //   tilespmv_fp64_warp<4,10752>  DENSE_ROWS: 16 warps per SM, 10.5 KB slots,
 //                                 a static cost-balanced item chunk per warp
 //                                 (dense tile rows: one tile row stays one item)
@@ -600,8 +600,8 @@ KernelChoice kernel_choice(int kernel) {
                 10752, kItemTiles, false};
     }
     if (kernel == TILESPMV_KERNEL_GATHER) {
-        using Cfg = WarpCfg<32, 2304, 8>;
-        return {"tilespmv_fp64_sm<32,2304,8>", tilespmv_fp64_sm<32, 2304, 8>, Cfg::kThreads, (int)Cfg::kSmem, 2304, 8,
+        using Cfg = WarpCfg<32, 3328, 4>;
+        return {"tilespmv_fp64_sm<32,3328,4>", tilespmv_fp64_sm<32, 3328, 4>, Cfg::kThreads, (int)Cfg::kSmem, 3328, 4,
                 true};
     }
     using Cfg = WarpCfg<32, 4608>;
