@@ -23,4 +23,10 @@ for tool in memcheck racecheck synccheck initcheck; do
   timeout 900 /usr/local/cuda/bin/compute-sanitizer --tool $tool --num-cuda-barriers 64 --error-exitcode 9 python scripts/sanitize_small.py > $OUT/sanitizer_$tool.log 2>&1
   echo "rc=$?" >> $OUT/sanitizer_$tool.log
 done
+# the N > 1 code path on one GPU (two ranks on cuda:0 over gloo, host-staged exchange): a functional
+# check of bench.py's sharded step, not a bench number
+TILESPMV_BENCH_ONE_GPU=1 timeout 900 python -m torch.distributed.run --nnodes=1 --nproc-per-node 2 \
+   --master-addr 127.0.0.1 --master-port 29533 bench.py --gpus 2 --steps 5 --warmup 3 --workload stencil27_40 \
+   --e2e-steps 2 > $OUT/n2_devcheck.json 2> $OUT/n2_devcheck.err; echo "rc=$?" >> $OUT/n2_devcheck.err
+timeout 300 python bench.py --impl reference --steps 20 --warmup 5 > $OUT/reference.json 2> $OUT/reference.err
 echo done > $OUT/DONE

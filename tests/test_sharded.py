@@ -202,3 +202,72 @@ def test_halo_needs_stencil_closed_form():
     recv1, parts1 = halo_needs(S1.rowptr, S1.colidx, b, 1)
     assert recv1 == [(0, b[1] - pl, b[1])]
     assert parts1 == [(b[1], b[1] + pl, False), (b[1] + pl, b[2], True)]
+
+
+# ---------------------------------------------------------------------------
+# build_shard_handles: AUTO resolved on the global totals (host logic)
+# ---------------------------------------------------------------------------
+
+class _FakeHandle:
+    """Stands in for TiledMatrix: info() of a shard, records the mode/kernel."""
+
+    def __init__(self, sl, md, kn, stats):
+        self.sl, self.md, self.kn = sl, md, kn
+        self.stats = stats
+        self.closed = False
+
+    def info(self):
+        return dict(self.stats)
+
+    def close(self):
+        self.closed = True
+
+
+def _shard_worker(rank, world, port, q):
+    try:
+        from paper_conf_ipps_niuldj0t21_b200.sharded import build_shard_handles
+        os.environ["MASTER_ADDR"] = "127.0.0.1"
+        os.environ["MASTER_PORT"] = str(port)
+        dist.init_process_group("gloo", rank=rank, world_size=world)
+        # rank 0: 1.0M nnz, remainder-heavy; rank 1: 0.9M nnz, no remainder.
+        # Each alone would resolve AUTO to ADPT (< 1.8M) and its own kernel;
+        # together: 1.9M nnz -> DEFERRED, and the remainder's 12 B/entry are
+        # 12 * 1.2M = 14.4 MB of 27 MB -> GATHER
+        stats = [dict(payload_bytes=1_000_000, tilem=1000, rem_nnz=1_200_000, alg_bytes=16_000_000, nnz=1_000_000),
+                 dict(payload_bytes=9_000_000, tilem=1000, rem_nnz=0, alg_bytes=11_000_000, nnz=900_000)][rank]
+        made = []
+
+        def create(sl, md, kn):
+            h = _FakeHandle(sl, md, kn, stats)
+            made.append(h)
+            return h
+
+        hs, md, kn = build_shard_handles(create, [(0, 16), (16, 32)], stats["nnz"], mode="AUTO", kernel="AUTO")
+        q.put((rank, md, kn, [(h.md, h.kn) for h in hs], sum(h.closed for h in made)))
+        dist.destroy_process_group()
+    except Exception:  # pragma: no cover
+        import traceback
+        q.put((rank, None, traceback.format_exc(), None, None))
+
+
+def test_build_shard_handles_resolves_auto_globally():
+    """Every rank resolves AUTO mode (reading R18 on the global nnz) and the
+    AUTO kernel (tilespmv_auto_kernel on the global totals) identically, so
+    shards run the unsharded matrix's kernel and summation order; handles
+    built with a provisional kernel are closed and rebuilt."""
+    from paper_conf_ipps_niuldj0t21_b200.tilespmv import KERNELS, MODES
+    world = 2
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _port()
+    procs = [ctx.Process(target=_shard_worker, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = [q.get(timeout=300) for _ in range(world)]
+    for p in procs:
+        p.join(timeout=60)
+    for rank, md, kn, hs, closed in res:
+        assert md == MODES["DEFERRED"], (rank, md, kn)
+        assert kn == KERNELS["GATHER"], (rank, kn)
+        assert hs == [(MODES["DEFERRED"], KERNELS["GATHER"])] * 2
+        assert closed == 2  # the two provisional SM_QUEUE handles
