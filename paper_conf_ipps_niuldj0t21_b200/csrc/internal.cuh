@@ -98,6 +98,13 @@ constexpr int kLocalParts = 4;
 // (power-law, many small items): 2048 gave 174 us against 188 us for 512,
 // neutral on the stencil and mixed matrices (round 1)
 constexpr int64_t kItemFixedCost = 2048;
+// row-group items cost more per byte than their bytes say (two tile rows per
+// step, one chain of gather round trips each): per-item traces of R-MAT
+// (profiles/r02_ab/trace_items_rmat20.txt) put a row-group item at 5.99 us
+// for 2,392 B against 5.12 us for a 3,071 B remainder-only item; charging
+// 320 per tile row of a group moves R-MAT from 108.8 to 102.9 us
+// (profiles/r02_ab/group_row_cost_rmat20.txt; 160: 104.1, 640: 104.0)
+constexpr int64_t kGroupRowCost = 320;
 __host__ __device__ __forceinline__ int item_nt(const Item &it) { return (it.part_nt >> 24) & 31; }
 __host__ __device__ __forceinline__ int item_part(const Item &it) { return it.part_nt & 0xFFFFFF; }
 __host__ __device__ __forceinline__ bool item_local(const Item &it) { return (it.part_nt >> 29) & 1; }

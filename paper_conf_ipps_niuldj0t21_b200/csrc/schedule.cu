@@ -547,7 +547,7 @@ __global__ void k_item_cost(const Item *items, int64_t n, int64_t m, int64_t fix
     int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     if (k >= n) return;
     const Item it = items[k];
-    cost[k] = (int64_t)blob_parts(it, m).total + 40 * (item_nt(it)) + fixed;
+    cost[k] = (int64_t)blob_parts(it, m).total + 40 * (item_nt(it)) + fixed + kGroupRowCost * it.ntr;
 }
 
 __global__ void k_warp_first(const int64_t *begin, const WItem *witems, const int32_t *jcols, int W, WFirst *wf) {
