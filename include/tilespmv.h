@@ -114,7 +114,8 @@ typedef struct {
     int64_t device_bytes;               /* device memory owned by the handle */
     double create_ms;                   /* wall time of tilespmv_create_from_csr */
     int32_t kernel;                     /* resolved TILESPMV_KERNEL_* (never AUTO) */
-    int32_t reserved;
+    int32_t xcache_cols;                /* GATHER kernel: remainder columns held in its shared-memory
+                                           x cache (the most-gathered ones, <= 1024); 0 otherwise */
 } tilespmv_info_t;
 
 /* Build a tiled matrix from a canonical device CSR ("converting a basic

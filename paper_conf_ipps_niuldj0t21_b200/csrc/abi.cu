@@ -37,7 +37,7 @@ static void free_matrix(tilespmv_matrix *M) {
     void *ptrs[] = {M->tilePtr, M->tileColIdx, M->tileNnz, M->tileFmt, M->tileAux, M->tileOff,
                     M->payload, M->remRowPtr, M->remCol, M->remVal, M->items, M->split_info,
                     M->partials, M->counters, M->xstage, M->ystage, M->tdesc, M->cta_begin, M->blob,
-                    M->witems, M->jcols, M->wfirst, M->units};
+                    M->witems, M->jcols, M->wfirst, M->units, M->xc_cols};
     for (void *p : ptrs)
         if (p) cudaFree(p);
     if (cur >= 0 && cur != M->device) cudaSetDevice(cur);
@@ -235,6 +235,7 @@ int tilespmv_get_info(tilespmv_handle_t h, tilespmv_info_t *info) {
     info->device_bytes = h->device_bytes;
     info->create_ms = h->create_ms;
     info->kernel = h->kernel;
+    info->xcache_cols = h->xc_n;
     return TILESPMV_OK;
 }
 

@@ -144,8 +144,11 @@ struct Matrix {
     int64_t blob_bytes = 0;
     int64_t *cta_begin = nullptr;  // dense-row kernel: item chunk per warp (row-aligned, cost-balanced);
                                    // SM-queue kernel: unit range per CTA
-    int32_t *units = nullptr;      // SM-queue kernel: first item of each unit, num_units + 1
+    int2 *units = nullptr;         // SM-queue kernel: [first, end) items of each unit, in claim order
+                                   // (inside each CTA's range: decreasing cost)
     int64_t num_units = 0;
+    int32_t *xc_cols = nullptr;    // GATHER kernel: columns of the shared-memory x cache (slot order)
+    int32_t xc_n = 0;
     // host-staging buffers for tilespmv_run_host
     double *xstage = nullptr, *ystage = nullptr;
     // statistics

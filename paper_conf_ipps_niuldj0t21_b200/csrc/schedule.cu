@@ -348,7 +348,7 @@ __global__ void k_blob_len(Item *items, int64_t n, int64_t m, uint32_t slot, Til
 __global__ void k_blob_fill(Item *items, int64_t nitems, int64_t m, int64_t n, const int64_t *start16, const uint2 *dlist,
                             const int32_t *tileColIdx, TileView T, const uint8_t *payload, const int32_t *remRowPtr,
                             const int32_t *remCol, const double *remVal, uint8_t *blob, WItem *witems,
-                            int32_t *jcols) {
+                            int32_t *jcols, const int32_t *xc_slot) {
     const int64_t k = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
     const int lane = threadIdx.x & 31;
     if (k >= nitems) return;
@@ -536,7 +536,9 @@ __global__ void k_blob_fill(Item *items, int64_t nitems, int64_t m, int64_t n, c
         unsigned long long *vd = reinterpret_cast<unsigned long long *>(dst + b.val);
         const unsigned long long *vs = reinterpret_cast<const unsigned long long *>(remVal);
         for (int i = lane; i < it.ke - it.kb; i += 32) {
-            cd[i] = remCol[it.kb + i];
+            const int32_t c = remCol[it.kb + i];
+            const int32_t sl = xc_slot ? xc_slot[c] : -1;
+            cd[i] = sl >= 0 ? ~sl : c;  // a cached column: ~(its x-cache slot)
             vd[i] = vs[it.kb + i];
         }
     }
@@ -629,6 +631,28 @@ __global__ void k_cta_units(const int64_t *incl, const int32_t *units, int64_t n
     cta_begin[b] = lo;
 }
 
+// sort key of a unit for the per-CTA ordering: its cost (the items' costs);
+// unless `all`, only units of at least twice the mean unit cost keep it and
+// the others get 0 (they keep their tile-row order: on stencils and banded
+// matrices neighbouring tile rows share x lines in L1/L2)
+__global__ void k_unit_cost(const int64_t *incl, const int32_t *ustart, int64_t nu, int64_t n, int all,
+                            int64_t *ucost, int32_t *uidx) {
+    const int64_t u = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (u >= nu) return;
+    const int32_t a = ustart[u], b = ustart[u + 1];
+    const int64_t c = incl[b - 1] - (a ? incl[a - 1] : 0);
+    ucost[u] = all || c * nu >= 2 * incl[n - 1] ? c : 0;
+    uidx[u] = (int32_t)u;
+}
+
+// the units in claim order: [first item, end item) of unit uidx[c]
+__global__ void k_unit_bounds(const int32_t *ustart, const int32_t *uidx, int64_t nu, int2 *units) {
+    const int64_t c = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (c >= nu) return;
+    const int32_t u = uidx[c];
+    units[c] = make_int2(ustart[u], ustart[u + 1]);
+}
+
 // ADPT (and BYTES) mode gathers each item's COO data into a COO run (blob_parts)
 TileView tile_view(const Matrix &M) {
     return {M.tilePtr, M.tileOff, M.tileFmt, M.tileAux, M.tileNnz, M.tileColIdx,
@@ -711,6 +735,58 @@ int build_schedule(Matrix &M, cudaStream_t st) {
     return 0;
 }
 
+__global__ void k_col_hist(const int32_t *col, int64_t nnz, int32_t *cnt, int32_t *iota, int64_t n) {
+    const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (i < n) iota[i] = (int32_t)i;
+    if (i < nnz) atomicAdd(cnt + col[i], 1);
+}
+// the first k of the columns sorted by decreasing count, if gathered at least twice
+__global__ void k_xc_mark(const int32_t *cnt_s, const int32_t *col_s, int64_t k, int32_t *flag) {
+    const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (i < k && cnt_s[i] >= 2) flag[col_s[i]] = 1;
+}
+// slots in column order: slot[c] = prefix of the flags, -1 if c is not cached
+__global__ void k_xc_write(const int32_t *flag, const int32_t *pos, int64_t n, int32_t *slot, int32_t *cols) {
+    const int64_t c = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (c >= n) return;
+    const int32_t f = flag[c], q = pos[c];
+    slot[c] = f ? q : -1;
+    if (f) cols[q] = (int32_t)c;
+}
+
+// GATHER kernel's x cache (spmv_warp.cu): the (at most) `slots` remainder
+// columns gathered most often (ties: lower column first; only columns
+// gathered at least twice), in column order.  slot[c] = its cache slot or -1.
+// A property of the handle's own entries: it moves where x is read from, never
+// a value or a summation order, so y is the same with or without it.
+static int build_xcache(Matrix &M, int slots, int32_t *slot, cudaStream_t st) {
+    const int64_t n = M.n;
+    Tmp ab(st), bb(st);
+    if (int rc = ab.alloc(4 * (size_t)(n + 1) * sizeof(int32_t))) return rc;
+    int32_t *cnt = ab.as<int32_t>(), *iota = cnt + (n + 1), *cnt_s = iota + (n + 1), *col_s = cnt_s + (n + 1);
+    TSP_CK(cudaMemsetAsync(cnt, 0, (n + 1) * sizeof(int32_t), st));
+    const int64_t mx = std::max<int64_t>(n, M.rem_nnz);
+    k_col_hist<<<(unsigned)((mx + 255) / 256), 256, 0, st>>>(M.remCol, M.rem_nnz, cnt, iota, n);
+    if (int rc = scan([&](void *t, size_t &b) {
+            return cub::DeviceRadixSort::SortPairsDescending(t, b, cnt, cnt_s, iota, col_s, (int)n, 0, 32, st);
+        }, st)) return rc;
+    // flags over columns (reusing cnt), then their exclusive prefix (in iota)
+    int32_t *flag = cnt, *pos = iota;
+    TSP_CK(cudaMemsetAsync(flag, 0, (n + 1) * sizeof(int32_t), st));
+    const int64_t k = std::min<int64_t>(slots, n);
+    k_xc_mark<<<(unsigned)((k + 255) / 256), 256, 0, st>>>(cnt_s, col_s, k, flag);
+    if (int rc = scan([&](void *t, size_t &b) { return cub::DeviceScan::ExclusiveSum(t, b, flag, pos, (int)(n + 1), st); }, st)) return rc;
+    int32_t nx = 0;
+    TSP_CK(cudaMemcpyAsync(&nx, pos + n, 4, cudaMemcpyDeviceToHost, st));
+    TSP_CK(cudaStreamSynchronize(st));
+    TSP_CK(cudaMalloc(&M.xc_cols, std::max(nx, 1) * sizeof(int32_t)));
+    M.device_bytes += std::max(nx, 1) * 4;
+    M.xc_n = nx;
+    k_xc_write<<<(unsigned)((n + 255) / 256), 256, 0, st>>>(flag, pos, n, slot, M.xc_cols);
+    TSP_CK(cudaGetLastError());
+    return 0;
+}
+
 int build_tdesc(Matrix &M, cudaStream_t st) {
     const int64_t n = M.num_items;
     if (n == 0) {
@@ -752,6 +828,15 @@ int build_tdesc(Matrix &M, cudaStream_t st) {
     if (over) return set_error(TILESPMV_CUDA, "schedule: an item's blob exceeds the kernel's slot");
     if (total16 >= (int64_t(1) << 32)) return set_error(TILESPMV_OVERFLOW, "execution blob >= 64 GiB");
     M.blob_bytes = total16 * 16;
+    // GATHER: the kernel's x cache holds the most-gathered remainder columns
+    Tmp xcb(st);
+    int32_t *xc_slot = nullptr;
+    const int xcache = kernel_choice(M.kernel).xcache;
+    if (xcache > 0 && M.rem_nnz > 0) {
+        if (int rc = xcb.alloc((size_t)(M.n + 1) * sizeof(int32_t))) return rc;
+        xc_slot = xcb.as<int32_t>();
+        if (int rc = build_xcache(M, xcache, xc_slot, st)) return rc;
+    }
     TSP_CK(cudaMalloc(&M.blob, M.blob_bytes + 256));
     M.device_bytes += M.blob_bytes + 256;
     TSP_CK(cudaMalloc(&M.witems, n * sizeof(WItem)));
@@ -759,7 +844,7 @@ int build_tdesc(Matrix &M, cudaStream_t st) {
     M.device_bytes += n * (int64_t)(sizeof(WItem) + 64);
     k_blob_fill<<<(unsigned)((n * 32 + 255) / 256), 256, 0, st>>>(M.items, n, M.m, M.n, start16, M.tdesc, M.tileColIdx,
                                                                  TV, M.payload, M.remRowPtr, M.remCol, M.remVal,
-                                                                 M.blob, M.witems, M.jcols);
+                                                                 M.blob, M.witems, M.jcols, xc_slot);
     TSP_CK(cudaGetLastError());
     return 0;
 }
@@ -795,19 +880,20 @@ static int configure_sm_queue(Matrix &M, int G, cudaStream_t st) {
     M.grid = G;
     const int64_t n = M.num_items;
     TSP_CK(cudaMalloc(&M.cta_begin, (G + 1) * sizeof(int64_t)));
-    TSP_CK(cudaMalloc(&M.units, (n + 1) * sizeof(int32_t)));
-    M.device_bytes += (G + 1) * 8 + (n + 1) * 4;
     if (n == 0) {
+        TSP_CK(cudaMalloc(&M.units, sizeof(int2)));
+        M.device_bytes += (G + 1) * 8 + 8;
         TSP_CK(cudaMemsetAsync(M.cta_begin, 0, (G + 1) * sizeof(int64_t), st));
-        TSP_CK(cudaMemsetAsync(M.units, 0, sizeof(int32_t), st));
+        TSP_CK(cudaMemsetAsync(M.units, 0, sizeof(int2), st));
         M.num_units = 0;
         return 0;
     }
-    Tmp costb(st), flagb(st);
+    Tmp costb(st), flagb(st), ub(st);
     if (int rc = costb.alloc(2 * n * sizeof(int64_t))) return rc;
     if (int rc = flagb.alloc(2 * (n + 1) * sizeof(int32_t))) return rc;
+    if (int rc = ub.alloc((n + 1) * sizeof(int32_t))) return rc;
     int64_t *cost = costb.as<int64_t>(), *incl = cost + n;
-    int32_t *flag = flagb.as<int32_t>(), *pos = flag + (n + 1);
+    int32_t *flag = flagb.as<int32_t>(), *pos = flag + (n + 1), *ustart = ub.as<int32_t>();
     const unsigned nb = (unsigned)((n + 1 + 255) / 256);
     k_item_cost<<<nb, 256, 0, st>>>(M.items, n, M.m, kItemFixedCost, cost);
     if (int rc = scan([&](void *t, size_t &b) { return cub::DeviceScan::InclusiveSum(t, b, cost, incl, (int)n, st); }, st)) return rc;
@@ -818,8 +904,30 @@ static int configure_sm_queue(Matrix &M, int G, cudaStream_t st) {
     TSP_CK(cudaMemcpyAsync(&nu, pos + n, 4, cudaMemcpyDeviceToHost, st));
     TSP_CK(cudaStreamSynchronize(st));
     M.num_units = nu;
-    k_unit_write<<<nb, 256, 0, st>>>(flag, pos, n, M.units);
-    k_cta_units<<<(G + 1 + 255) / 256, 256, 0, st>>>(incl, M.units, nu, n, G, M.cta_begin);
+    k_unit_write<<<nb, 256, 0, st>>>(flag, pos, n, ustart);
+    k_cta_units<<<(G + 1 + 255) / 256, 256, 0, st>>>(incl, ustart, nu, n, G, M.cta_begin);
+    // inside each CTA's range the warps claim units costliest first
+    // (longest-processing-time order), so the SM's tail is made of its
+    // smallest units: all units for GATHER (power-law remainders; R-MAT 99.4
+    // -> 93.2 us), only the big ones (>= 2x the mean unit cost) for SM_QUEUE,
+    // whose other units keep their tile-row order (sorting them all cost C5
+    // 5%: neighbouring tile rows share x lines); stable sort
+    TSP_CK(cudaMalloc(&M.units, (size_t)nu * sizeof(int2)));
+    M.device_bytes += (G + 1) * 8 + (int64_t)nu * 8;
+    {
+        Tmp kb(st), vb(st);
+        if (int rc = kb.alloc(2 * (size_t)nu * sizeof(int64_t))) return rc;
+        if (int rc = vb.alloc(2 * (size_t)nu * sizeof(int32_t))) return rc;
+        int64_t *ucost = kb.as<int64_t>(), *ucost_s = ucost + nu;
+        int32_t *uidx = vb.as<int32_t>(), *uidx_s = uidx + nu;
+        const unsigned nbu = (unsigned)((nu + 255) / 256);
+        k_unit_cost<<<nbu, 256, 0, st>>>(incl, ustart, nu, n, M.kernel == TILESPMV_KERNEL_GATHER, ucost, uidx);
+        if (int rc = scan([&](void *t, size_t &b) {
+                return cub::DeviceSegmentedSort::StableSortPairsDescending(t, b, ucost, ucost_s, uidx, uidx_s, (int)nu, G,
+                                                                           M.cta_begin, M.cta_begin + 1, st);
+            }, st)) return rc;
+        k_unit_bounds<<<nbu, 256, 0, st>>>(ustart, uidx_s, nu, M.units);
+    }
     TSP_CK(cudaGetLastError());
     return 0;
 }
@@ -900,6 +1008,8 @@ int launch_spmv(const Matrix &M, const double *d_x, double *d_y, cudaStream_t st
     p.wfirst = M.wfirst;
     p.cta_begin = M.cta_begin;
     p.units = M.units;
+    p.xc_cols = M.xc_cols;
+    p.xc_n = M.xc_n;
     p.split_info = M.split_info;
     p.partials = M.partials;
     p.counters = M.counters;

@@ -17,7 +17,7 @@ struct Params {
     const int32_t *jcols;      // tile column J of each item's tiles, 16 per item
     const WFirst *wfirst;      // warp kernel: per-warp chunk and first item
     const int64_t *cta_begin;  // SM-queue kernel: unit range of each CTA
-    const int32_t *units;      // SM-queue kernel: first item of each unit (+ end)
+    const int2 *units;         // SM-queue kernel: item range of each unit, in claim order
     const int2 *split_info;    // split tile rows: {first partial slot, parts}
     double *partials;
     int32_t *counters;
@@ -25,6 +25,8 @@ struct Params {
     double *y;
     int64_t m, n;
     int x_vec;                 // x is 16-byte aligned: x segments load as double2
+    const int32_t *xc_cols;    // GATHER: the columns of the shared-memory x cache
+    int xc_n;                  // (their number, <= the kernel's cache slots)
 };
 
 // ------------------------------------------------------------------ PTX ----
@@ -182,7 +184,16 @@ struct KernelChoice {
     int slot_bytes;   // item budget the schedule must respect
     int item_tiles;   // tiles per item (x stage segments)
     bool sm_queue;    // one CTA per SM; its warps claim units from a shared-memory counter
+    int xcache;       // slots of the shared-memory x cache (0: none)
 };
+#ifndef TSP_XCACHE
+#define TSP_XCACHE 1024
+#endif
+constexpr int kXCache = TSP_XCACHE;  // GATHER kernel: x cache slots (8 B each)
+#ifndef TSP_GSLOT
+#define TSP_GSLOT 3136
+#endif
+constexpr int kGatherSlot = TSP_GSLOT;  // GATHER kernel: slot bytes
 // TILESPMV_KERNEL_SM_QUEUE, _DENSE_ROWS or _GATHER
 KernelChoice kernel_choice(int kernel);
 

@@ -21,11 +21,14 @@
 //   tilespmv_fp64_sm<32,4608,16> SM_QUEUE: one CTA of 32 warps per SM, 4.5 KB
 //                                 slots, warps claim units from a
 //                                 shared-memory queue (222 KB of shared memory)
-//   tilespmv_fp64_sm<32,3328,4>  GATHER: the same with 3.25 KB slots and at
-//                                 most 4 tiles per item (132 KB): the L1 left
-//                                 to the remainder's x gathers grows from ~30
-//                                 to ~125 KB (power-law matrices in DEFERRED
-//                                 mode: R-MAT 127.6 -> 109.0 us)
+//   tilespmv_fp64_sm<32,3136,4,1024> GATHER: the same with 3 KB slots, at
+//                                 most 4 tiles per item and an 8 KB x cache of
+//                                 the 1,024 most-gathered remainder columns
+//                                 (130 KB in all: the 132 KB carve-out leaves
+//                                 ~124 KB of L1 to the remainder's x gathers;
+//                                 power-law matrices in DEFERRED mode), every
+//                                 remainder through the product pre-pass, units
+//                                 claimed costliest first
 //   tilespmv_fp64_warp<4,10752>  DENSE_ROWS: 16 warps per SM, 10.5 KB slots,
 //                                 a static cost-balanced item chunk per warp
 //                                 (dense tile rows: one tile row stays one item)
@@ -62,15 +65,16 @@ __device__ __forceinline__ unsigned long long gtimer() {
 namespace {
 
 
-template <int WARPS, int SLOT, int XT = kItemTiles>
+template <int WARPS, int SLOT, int XT = kItemTiles, int XC = 0>
 struct WarpCfg {
     static_assert(SLOT % 16 == 0 && SLOT <= kItemBytesMax && XT % 4 == 0 && XT <= kItemTiles, "slot size");
     // [x stage of every warp, XT x 128 B, 128-byte aligned] [per warp: slot |
-    // row-sum scratch of the COO scan (256 B) | mbarrier]
+    // row-sum scratch of the COO scan (256 B) | mbarrier] [x cache: XC x 8 B]
     static constexpr uint32_t kX = XT * 16 * 8;
     static constexpr uint32_t kRacc = 256;
     static constexpr uint32_t kPer = SLOT + kRacc + 16;
-    static constexpr uint32_t kSmem = WARPS * (kX + kPer) + 256;  // +256: loads may overrun a slot
+    static constexpr uint32_t kXc = WARPS * (kX + kPer);  // x cache offset
+    static constexpr uint32_t kSmem = kXc + XC * 8 + 256;  // +256: loads may overrun a slot
     static constexpr int kThreads = 32 * WARPS;
 };
 
@@ -97,9 +101,45 @@ __device__ __forceinline__ WItem load_witem(const WItem *w, int k) {
 // product on its own and selects +0.0.
 constexpr int kShortRow = 16;  // flat pass: rows of up to this many entries two lanes per row
 
-// product of staged remainder entry k if k < e, else +0.0 (rounded on its own)
+// Product pre-pass (GATHER kernel, PRE = true): the x gathers of all E
+// remainder entries of an item, one lane per entry and kGatherDepth gathers
+// in flight per lane, each product v*x rounded on its own and stored over its
+// value in the slot; x comes from the CTA's shared-memory x cache for the
+// most-gathered columns (blob column ~slot).  The row sums then read
+// products from shared memory in the same order as the inline-gather form
+// (PRE = false, the other kernels), so the flat pass and row groups give the
+// same bits either way.  The slot was written through the generic proxy: the
+// caller fences before the next TMA copy into it.
+constexpr int kGatherDepth = 2;  // 2 / 4 / 8 in flight: R-MAT 94.3 / 95.8 / 109 us (more thrash the L1)
+__device__ __forceinline__ void rem_products(const Params &p, uint32_t colS, uint32_t valS, int E, uint64_t x_policy,
+                                             uint32_t xcS, int lane) {
+#pragma unroll 1
+    for (int base = 0; base < E; base += 32 * kGatherDepth) {
+        double xv[kGatherDepth];
+#pragma unroll
+        for (int j = 0; j < kGatherDepth; ++j) {
+            const int k = base + lane + 32 * j;
+            xv[j] = 0.0;
+            if (k < E) {
+                const int c = lds_s32(colS + 4 * k);  // < 0: slot ~c of the CTA's x cache (GATHER)
+                xv[j] = c < 0 ? lds_f64(xcS + 8u * (uint32_t)~c) : ldg_hint(p.x + (uint32_t)c, x_policy);
+            }
+        }
+#pragma unroll
+        for (int j = 0; j < kGatherDepth; ++j) {
+            const int k = base + lane + 32 * j;
+            if (k < E) sts_f64(valS + 8 * k, __dmul_rn(lds_f64(valS + 8 * k), xv[j]));
+        }
+    }
+    __syncwarp();
+}
+
+// product of staged remainder entry k if k < e, else +0.0 (rounded on its
+// own): read back after rem_products (PRE), or gathered here
+template <bool PRE>
 __device__ __forceinline__ double rem_product(const Params &p, int k, int e, uint32_t colS, uint32_t valS,
                                               uint64_t x_policy) {
+    if (PRE) return lds_f64_lt(k, e, valS + 8 * k);
     int c;
     double v;
     lds_entry_lt(k, e, colS + 4 * k, valS + 8 * k, c, v);
@@ -112,6 +152,7 @@ __device__ __forceinline__ double rem_product(const Params &p, int k, int e, uin
 // half-warp per row (two rows at a time, the whole warp for the last one)
 // with an xor tree.  Returns lane r's (or r + 16's) share of row r.  The order
 // of every sum depends only on this tile row.
+template <bool PRE>
 __device__ __forceinline__ double flat_rows(const Params &p, uint32_t rq, uint32_t colS, uint32_t valS, int rows,
                                             uint64_t x_policy, int lane) {
     const int r = lane & 15, h = lane >> 4;
@@ -123,8 +164,8 @@ __device__ __forceinline__ double flat_rows(const Params &p, uint32_t rq, uint32
 #pragma unroll 1
     for (int i = 0; i < trips; i += 2) {
         const int k0 = b + h + 2 * i;
-        s0 += rem_product(p, k0, ee, colS, valS, x_policy);
-        s1 += rem_product(p, k0 + 2, ee, colS, valS, x_policy);
+        s0 += rem_product<PRE>(p, k0, ee, colS, valS, x_policy);
+        s1 += rem_product<PRE>(p, k0 + 2, ee, colS, valS, x_policy);
     }
     double acc = s0 + s1;
     uint32_t lm = __ballot_sync(FULL, lng && h == 0 && r < rows);
@@ -143,10 +184,10 @@ __device__ __forceinline__ double flat_rows(const Params &p, uint32_t rq, uint32
 #pragma unroll 1
         for (int t = 0; t < t2; ++t) {
             const int k = bb + off + 4 * stride * t;
-            q0 += rem_product(p, k, e2, colS, valS, x_policy);
-            q1 += rem_product(p, k + stride, e2, colS, valS, x_policy);
-            q2 += rem_product(p, k + 2 * stride, e2, colS, valS, x_policy);
-            q3 += rem_product(p, k + 3 * stride, e2, colS, valS, x_policy);
+            q0 += rem_product<PRE>(p, k, e2, colS, valS, x_policy);
+            q1 += rem_product<PRE>(p, k + stride, e2, colS, valS, x_policy);
+            q2 += rem_product<PRE>(p, k + 2 * stride, e2, colS, valS, x_policy);
+            q3 += rem_product<PRE>(p, k + 3 * stride, e2, colS, valS, x_policy);
         }
         double sq = (q0 + q1) + (q2 + q3);
         if (!pair) sq += __shfl_xor_sync(FULL, sq, 16);
@@ -159,17 +200,38 @@ __device__ __forceinline__ double flat_rows(const Params &p, uint32_t rq, uint32
     return acc;
 }
 
-__device__ __forceinline__ void remainder(const Params &p, uint32_t rpS, uint32_t colS, uint32_t valS, int rows,
-                                          uint64_t x_policy, int lane, double &acc) {
+// returns true if the slot now holds products (PRE: the kernel's choice, so
+// every handle of one kernel sums a row the same way)
+template <bool PRE>
+__device__ __forceinline__ bool remainder(const Params &p, uint32_t rpS, uint32_t colS, uint32_t valS, int rows,
+                                          uint64_t x_policy, uint32_t xcS, int lane, double &acc) {
     const int r = lane & 15, h = lane >> 4;
     const int b = lds_s32(rpS + 4 * min(r, rows)), e = lds_s32(rpS + 4 * min(r + 1, rows));
     const int maxlen = (int)__reduce_max_sync(FULL, (unsigned)(e - b));
-    if (maxlen > 32) {
-        acc += flat_rows(p, rpS, colS, valS, rows, x_policy, lane);
-        return;
+    if (PRE) {  // all gathers first, then the row sums over the products
+        rem_products(p, colS, valS, lds_s32(rpS + 4 * rows), x_policy, xcS, lane);
+        if (maxlen > 32) {
+            acc += flat_rows<true>(p, rpS, colS, valS, rows, x_policy, lane);
+            return true;
+        }
+        // entries b + h + 2i of row r, in order
+        const int trips = (int)__reduce_max_sync(FULL, (unsigned)((e - b + 1 - h) >> 1));
+#pragma unroll 1
+        for (int i = 0; i < trips; i += 2) {
+            const int k0 = b + h + 2 * i;
+            const double p0 = lds_f64_lt(k0, e, valS + 8 * k0), p1 = lds_f64_lt(k0 + 2, e, valS + 8 * k0 + 16);
+            acc += p0;
+            acc += p1;
+        }
+        return true;
     }
-    // entries b + h + 2i and b + h + 2i + 2 of row r per step; a masked
-    // entry multiplies 0.0 by x at the item's first remainder column
+    if (maxlen > 32) {
+        acc += flat_rows<false>(p, rpS, colS, valS, rows, x_policy, lane);
+        return false;
+    }
+    // entries b + h + 2i and b + h + 2i + 2 of row r per step (stencils, <= 4
+    // entries per row: one round of gathers); a masked entry multiplies 0.0 by
+    // x at the item's first remainder column
     const int cdef = lds_s32(colS);
     const int trips = maxlen <= 4 ? 1 : (int)__reduce_max_sync(FULL, (unsigned)((e - b + 1 - h) >> 1));
 #pragma unroll 1
@@ -183,6 +245,7 @@ __device__ __forceinline__ void remainder(const Params &p, uint32_t rpS, uint32_
         acc = fma(v0, x0, acc);
         acc = fma(v1, x1, acc);
     }
+    return false;
 }
 
 // Row-group item (internal.cuh): ntr consecutive tile rows without stored
@@ -192,14 +255,16 @@ __device__ __forceinline__ void remainder(const Params &p, uint32_t rpS, uint32_
 // are summed by the whole warp with an xor tree.  y is written once per row.
 // A tile row's sums depend only on its own entries, so grouping never
 // changes a bit of y.
-__device__ __forceinline__ void group_item(const Params &p, const WItem &it, uint32_t slot, uint64_t x_policy,
-                                           int lane) {
+template <bool PRE>
+__device__ __forceinline__ bool group_item(const Params &p, const WItem &it, uint32_t slot, uint64_t x_policy,
+                                           uint32_t xcS, int lane) {
     const int ntr = (int)(it.jt_rows_pay & 0xFFu);
     const int rows_last = (int)((it.jt_rows_pay >> 8) & 31u);
     const uint32_t total = it.val_tot >> 16, rp = it.rp_col & 0xFFFFu;
     const bool has_rem = total > rp;
     const uint32_t rpS = slot + rp, colS = slot + (it.rp_col >> 16), valS = slot + (it.val_tot & 0xFFFFu);
     const int h = lane >> 4, r = lane & 15;
+    if (PRE && has_rem) rem_products(p, colS, valS, lds_s32(rpS + 4 * (16 * (ntr - 1) + rows_last)), x_policy, xcS, lane);
 #pragma unroll 1
     for (int g = 0; g < ntr; g += 2) {
         const int gg = g + h;
@@ -215,10 +280,10 @@ __device__ __forceinline__ void group_item(const Params &p, const WItem &it, uin
 #pragma unroll 1
             for (int t = 0; t < trips; ++t) {
                 const int k = b + 4 * t;
-                s0 += rem_product(p, k, ee, colS, valS, x_policy);
-                s1 += rem_product(p, k + 1, ee, colS, valS, x_policy);
-                s2 += rem_product(p, k + 2, ee, colS, valS, x_policy);
-                s3 += rem_product(p, k + 3, ee, colS, valS, x_policy);
+                s0 += rem_product<PRE>(p, k, ee, colS, valS, x_policy);
+                s1 += rem_product<PRE>(p, k + 1, ee, colS, valS, x_policy);
+                s2 += rem_product<PRE>(p, k + 2, ee, colS, valS, x_policy);
+                s3 += rem_product<PRE>(p, k + 3, ee, colS, valS, x_policy);
             }
             acc = (s0 + s1) + (s2 + s3);
             uint32_t lm = __ballot_sync(FULL, lng);
@@ -232,10 +297,10 @@ __device__ __forceinline__ void group_item(const Params &p, const WItem &it, uin
 #pragma unroll 1
                 for (int t = 0; t < t2; ++t) {
                     const int k = bb + lane + 128 * t;
-                    q0 += rem_product(p, k, e2, colS, valS, x_policy);
-                    q1 += rem_product(p, k + 32, e2, colS, valS, x_policy);
-                    q2 += rem_product(p, k + 64, e2, colS, valS, x_policy);
-                    q3 += rem_product(p, k + 96, e2, colS, valS, x_policy);
+                    q0 += rem_product<PRE>(p, k, e2, colS, valS, x_policy);
+                    q1 += rem_product<PRE>(p, k + 32, e2, colS, valS, x_policy);
+                    q2 += rem_product<PRE>(p, k + 64, e2, colS, valS, x_policy);
+                    q3 += rem_product<PRE>(p, k + 96, e2, colS, valS, x_policy);
                 }
                 double sq = (q0 + q1) + (q2 + q3);
                 sq += __shfl_xor_sync(FULL, sq, 16);
@@ -249,6 +314,7 @@ __device__ __forceinline__ void group_item(const Params &p, const WItem &it, uin
         const int64_t row = 16 * ((int64_t)it.I + gg) + r;
         if (gg < ntr && row < p.m) p.y[row] = acc;
     }
+    return PRE && has_rem;
 }
 
 // ADPT's COO run (blob_parts): the item's COO tiles and HYB COO parts as one
@@ -361,22 +427,24 @@ __device__ __forceinline__ void issue_x(const Params &p, int J, int nt, uint32_t
 }
 
 // steps 2-4 of an item whose blob is in `slot` and whose x segments are in
-// flight into `xs`: remainder, tiles, y (or the split-row carry)
-__device__ __forceinline__ void compute_item(const Params &p, const WItem &it, uint32_t slot, uint32_t xs,
-                                             uint32_t racc, uint64_t x_policy, int lane, double &carry) {
-    if (it.jt_rows_pay & 0xFFu) {  // row-group item (no tiles, no x segments)
-        group_item(p, it, slot, x_policy, lane);
-        return;
-    }
+// flight into `xs`: remainder, tiles, y (or the split-row carry).  Returns
+// true if the slot was written (products), so the caller fences the generic
+// proxy writes before the next TMA copy into the slot.
+template <bool PRE>
+__device__ __forceinline__ bool compute_item(const Params &p, const WItem &it, uint32_t slot, uint32_t xs,
+                                             uint32_t racc, uint64_t x_policy, uint32_t xcS, int lane, double &carry) {
+    if (it.jt_rows_pay & 0xFFu)  // row-group item (no tiles, no x segments)
+        return group_item<PRE>(p, it, slot, x_policy, xcS, lane);
     const int h = lane >> 4, r = lane & 15;
     const uint32_t total = it.val_tot >> 16;
     // 2. fused CSR remainder, while the x segments land
     double acc = 0.0;
     const uint32_t rp = it.rp_col & 0xFFFFu;
     const bool run = it.groups >> 31;  // the rp/col/val parts hold a COO run (ADPT), not a remainder
+    bool wrote = false;
     if (total > rp && !run)
-        remainder(p, slot + rp, slot + (it.rp_col >> 16), slot + (it.val_tot & 0xFFFFu),
-                  (int)((it.jt_rows_pay >> 8) & 31u), x_policy, lane, acc);
+        wrote = remainder<PRE>(p, slot + rp, slot + (it.rp_col >> 16), slot + (it.val_tot & 0xFFFFu),
+                  (int)((it.jt_rows_pay >> 8) & 31u), x_policy, xcS, lane, acc);
     if (p.x_vec) cp_async_wait_all();
     __syncwarp();
     if (run)
@@ -443,6 +511,7 @@ __device__ __forceinline__ void compute_item(const Params &p, const WItem &it, u
             }
         }
     }
+    return wrote;
 }
 
 // Dense-row kernel: WARPS warps per CTA, several CTAs per SM, one blob in
@@ -493,7 +562,8 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, MINB) tilespmv
         }
         TSP_STAMP(gw, k - kbeg, 1);
         TSP_INFO(gw, k - kbeg, k, it);
-        compute_item(p, it, slot, xs, racc, x_policy, lane, carry);
+        if (compute_item<false>(p, it, slot, xs, racc, x_policy, 0u, lane, carry))
+            fence_proxy_async();  // products written to the slot before the next TMA copy into it
         __syncwarp();  // slot and x scratch free for the next item
         TSP_STAMP(gw, k - kbeg, 3);
     }
@@ -509,9 +579,13 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, MINB) tilespmv
 // Each warp claims its next unit when it starts one, so the claim and the
 // unit's bounds are in flight while the current unit runs.
 // XT tiles per item (an x stage of XT segments per warp)
-template <int WARPS, int SLOT, int XT>
-__global__ void __launch_bounds__(WarpCfg<WARPS, SLOT, XT>::kThreads, 1) tilespmv_fp64_sm(const Params p) {
-    using Cfg = WarpCfg<WARPS, SLOT, XT>;
+// XC > 0 (GATHER): an x cache of the XC most-gathered remainder columns in
+// shared memory, filled at launch (schedule.cu: blob columns ~slot), and
+// every remainder through the product pre-pass
+template <int WARPS, int SLOT, int XT, int XC>
+__global__ void __launch_bounds__(WarpCfg<WARPS, SLOT, XT, XC>::kThreads, 1) tilespmv_fp64_sm(const Params p) {
+    using Cfg = WarpCfg<WARPS, SLOT, XT, XC>;
+    constexpr bool PRE = XC > 0;
     extern __shared__ __align__(128) uint8_t smem[];
     __shared__ int s_next;
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -534,8 +608,9 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT, XT>::kThreads, 1) tilespm
     const uint64_t stream_policy = policy_evict_first(), x_policy = policy_evict_last();
     int k = -1, ke = 0, nb = -1, ne = 0;
     if (ub + warp < ue) {
-        k = __ldg(p.units + ub + warp);
-        ke = __ldg(p.units + ub + warp + 1);
+        const int2 u = __ldg(p.units + ub + warp);
+        k = u.x;
+        ke = u.y;
     }
     int kb = k;
     WItem nxt{};
@@ -544,13 +619,23 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT, XT>::kThreads, 1) tilespm
         nxt = load_witem(p.witems, k);
         Jn = lane < 16 ? __ldg(p.jcols + (int64_t)k * 16 + lane) : 0;
     }
-    bool waited = false;
+    bool waited = false, issued = false;
+    const uint32_t xcS = smem_u32(smem) + Cfg::kXc;
+    if (XC > 0 && p.xc_n > 0) {  // the first blob in flight, then the x cache (x is the previous kernel's)
+        if (k >= 0) issue_blob(p, nxt, slot, bar, stream_policy, lane);
+        issued = true;
+        griddep_wait();
+        waited = true;
+        for (int i = threadIdx.x; i < p.xc_n; i += Cfg::kThreads) sts_f64(xcS + 8u * i, __ldg(p.x + __ldg(p.xc_cols + i)));
+        __syncthreads();
+    }
     int j = 0;
     while (k >= 0) {
         const WItem it = nxt;
         const int J = Jn;
         TSP_STAMP(gw, j, 0);
-        issue_blob(p, it, slot, bar, stream_policy, lane);
+        if (!issued) issue_blob(p, it, slot, bar, stream_policy, lane);
+        issued = false;
         // the matrix is immutable; x and y may belong to the previous kernel
         if (!waited) {
             griddep_wait();
@@ -562,8 +647,9 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT, XT>::kThreads, 1) tilespm
             c = __shfl_sync(FULL, c, 0);
             nb = -1;
             if (c < ue) {
-                nb = __ldg(p.units + c);
-                ne = __ldg(p.units + c + 1);
+                const int2 u = __ldg(p.units + c);
+                nb = u.x;
+                ne = u.y;
             }
         }
         // 1. x segments, issued before the blob lands (J came with the record)
@@ -579,7 +665,8 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT, XT>::kThreads, 1) tilespm
         }
         TSP_STAMP(gw, j, 1);
         TSP_INFO(gw, j, k, it);
-        compute_item(p, it, slot, xs, racc, x_policy, lane, carry);
+        if (compute_item<PRE>(p, it, slot, xs, racc, x_policy, xcS, lane, carry))
+            fence_proxy_async();  // products written to the slot before the next TMA copy into it
         __syncwarp();  // slot and x scratch free for the next item
         TSP_STAMP(gw, j, 3);
         ++j;
@@ -597,16 +684,16 @@ KernelChoice kernel_choice(int kernel) {
     if (kernel == TILESPMV_KERNEL_DENSE_ROWS) {
         using Cfg = WarpCfg<4, 10752>;
         return {"tilespmv_fp64_warp<4,10752>", tilespmv_fp64_warp<4, 10752, 4>, Cfg::kThreads, (int)Cfg::kSmem,
-                10752, kItemTiles, false};
+                10752, kItemTiles, false, 0};
     }
     if (kernel == TILESPMV_KERNEL_GATHER) {
-        using Cfg = WarpCfg<32, 3328, 4>;
-        return {"tilespmv_fp64_sm<32,3328,4>", tilespmv_fp64_sm<32, 3328, 4>, Cfg::kThreads, (int)Cfg::kSmem, 3328, 4,
-                true};
+        using Cfg = WarpCfg<32, kGatherSlot, 4, kXCache>;
+        return {"tilespmv_fp64_sm<32,3136,4,1024>", tilespmv_fp64_sm<32, kGatherSlot, 4, kXCache>, Cfg::kThreads,
+                (int)Cfg::kSmem, kGatherSlot, 4, true, kXCache};
     }
     using Cfg = WarpCfg<32, 4608>;
-    return {"tilespmv_fp64_sm<32,4608>", tilespmv_fp64_sm<32, 4608, kItemTiles>, Cfg::kThreads, (int)Cfg::kSmem, 4608,
-            kItemTiles, true};
+    return {"tilespmv_fp64_sm<32,4608>", tilespmv_fp64_sm<32, 4608, kItemTiles, 0>, Cfg::kThreads, (int)Cfg::kSmem,
+            4608, kItemTiles, true, 0};
 }
 
 }  // namespace tsp

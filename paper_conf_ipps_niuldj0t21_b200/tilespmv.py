@@ -47,7 +47,7 @@ class Info(ctypes.Structure):
                 ("meta_bytes", ctypes.c_int64), ("alg_bytes", ctypes.c_int64),
                 ("flops", ctypes.c_int64), ("num_items", ctypes.c_int64),
                 ("num_split_rows", ctypes.c_int64), ("device_bytes", ctypes.c_int64),
-                ("create_ms", ctypes.c_double), ("kernel", ctypes.c_int32), ("reserved", ctypes.c_int32)]
+                ("create_ms", ctypes.c_double), ("kernel", ctypes.c_int32), ("xcache_cols", ctypes.c_int32)]
 
     def as_dict(self) -> dict:
         d = {}

@@ -9,6 +9,9 @@ Times one launch between two events in several settings (median of 40):
            (the SM shared-memory carve-out is already the kernel's)
   idle     stream idle, events recorded around a launch from Python
   graph    as held, the launch replayed from a one-node CUDA graph
+and, for scale, the same settings for a 1-element torch kernel (the launch
+floor) and a torch copy moving the SpMV's algorithmic bytes (half read, half
+written; replicas rotated so L2 holds none of it).
 """
 import os
 import sys
@@ -35,10 +38,31 @@ with torch.cuda.graph(g):
 torch.cuda.synchronize()
 
 
-def t(kind, n=40):
+tiny = torch.zeros(1, device=dev)
+alg0 = Ms[0].info()["alg_bytes"]
+half = alg0 // 16  # doubles per copy side
+srcs = [torch.rand(half, dtype=torch.float64, device=dev) for _ in range(R)]
+dsts = [torch.empty_like(srcs[0]) for _ in range(R)]
+
+
+def t(kind, n=40, what="spmv"):
     out = []
     for i in range(n + 3):
         j = i % R
+        if what != "spmv":
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            torch.cuda.synchronize()
+            torch.cuda._sleep(400_000)
+            e0.record(s)
+            if what == "tiny":
+                tiny.add_(1.0)
+            else:
+                dsts[j].copy_(srcs[j])
+            e1.record(s)
+            torch.cuda.synchronize()
+            if i >= 3:
+                out.append(e0.elapsed_time(e1) * 1e3)
+            continue
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         torch.cuda.synchronize()
         if kind != "idle":
@@ -61,3 +85,6 @@ alg = Ms[0].info()["alg_bytes"]
 for kind in ("held", "warm", "idle", "graph", "held", "warm"):
     us = t(kind)
     print(f"{wl}/{mode} {kind:6s} {us:8.2f} us  frac {alg / (us * 1e-6) / 1e9 / 6547.8:.3f}", flush=True)
+for what in ("tiny", "copy", "tiny", "copy"):
+    us = t("held", what=what)
+    print(f"{what:5s} (held) {us:8.2f} us" + (f"  copy of {alg0 / 1e6:.1f} MB traffic: frac {alg0 / (us * 1e-6) / 1e9 / 6547.8:.3f}" if what == "copy" else ""), flush=True)

@@ -99,7 +99,7 @@ def test_default_spmv_kernel_has_no_register_spills(tmp_path):
     checked = 0
     for b in blocks[1:]:
         name = b.split("'")[1]
-        names = ("tilespmv_fp64_smILi32ELi4608ELi16EE", "tilespmv_fp64_smILi32ELi3328ELi4EE",
+        names = ("tilespmv_fp64_smILi32ELi4608ELi16E", "tilespmv_fp64_smILi32ELi3136ELi4E",
                  "tilespmv_fp64_warpILi4ELi10752")
         assert "tilespmv_fp64" not in name or any(n in name for n in names), name
         if any(n in name for n in names):

@@ -372,3 +372,33 @@ def test_row_slices_bitwise_equal_full(cuda_device, name, mode, kernel):
         with TM.from_host_csr(S, mode=mode, device=cuda_device, kernel=kernel) as M:
             ys = M.run(xd).cpu().numpy()
         assert np.array_equal(ys.view(np.uint64), yfull[r0:r1].view(np.uint64)), (name, mode, r0, r1)
+
+
+@pytest.mark.parametrize("name", ["rmat12", "heavy_row"])
+def test_gather_xcache(cuda_device, name):
+    """GATHER's shared-memory x cache holds the most-gathered remainder
+    columns: as many as there are columns gathered at least twice, at most
+    1024 (xcache_cols); the other kernels have none.  x is NaN on every
+    16-column segment that no matrix entry references (tile kernels multiply
+    whole segments), so a cache slot filled from a column outside the
+    matrix's segments would poison y."""
+    import torch
+    TM = tm()
+    if name == "heavy_row":
+        A = [a for a in _special() if a.name == "heavy_row"][0]
+        x = gen.dense_x(A.n, 101)
+    else:
+        A, x = gen.make(name)
+    yref, absy = O.spmv(A, x)
+    seg = np.zeros((A.n + 15) // 16, bool)
+    seg[A.colidx >> 4] = True
+    xp = np.where(seg[np.arange(A.n) >> 4], x, np.nan)
+    with TM.from_host_csr(A, mode="DEFERRED", device=cuda_device, kernel="GATHER", keep_layout=True) as M:
+        rem = M.export("remCol")
+        cnt = np.bincount(rem, minlength=A.n)
+        assert M.info()["xcache_cols"] == min(1024, int((cnt >= 2).sum()))
+        assert name != "rmat12" or M.info()["xcache_cols"] == 1024
+        y = M.run(torch.from_numpy(xp).to(cuda_device)).cpu().numpy()
+        assert_spmv_close(y, yref, absy, f"{name}/GATHER x cache")
+    with TM.from_host_csr(A, mode="DEFERRED", device=cuda_device, kernel="SM_QUEUE") as M:
+        assert M.info()["xcache_cols"] == 0
