@@ -105,6 +105,11 @@ constexpr int64_t kItemFixedCost = 2048;
 // 320 per tile row of a group moves R-MAT from 108.8 to 102.9 us
 // (profiles/r02_ab/group_row_cost_rmat20.txt; 160: 104.1, 640: 104.0)
 constexpr int64_t kGroupRowCost = 320;
+// ... with the GATHER kernel's product pre-pass a row-group item costs close
+// to what its bytes say (R-MAT traces: 4.71 us for 2,224 B against 5.47 us
+// for a 2,911 B remainder-only item); 80 per tile row measured best (R-MAT
+// 0 / 80 / 160 / 320: 90.8 / 86.5 / 86.9 / 88.4 us, profiles/r02_ab2)
+constexpr int64_t kGroupRowCostPre = 80;
 __host__ __device__ __forceinline__ int item_nt(const Item &it) { return (it.part_nt >> 24) & 31; }
 __host__ __device__ __forceinline__ int item_part(const Item &it) { return it.part_nt & 0xFFFFFF; }
 __host__ __device__ __forceinline__ bool item_local(const Item &it) { return (it.part_nt >> 29) & 1; }

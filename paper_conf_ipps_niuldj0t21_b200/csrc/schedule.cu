@@ -545,11 +545,12 @@ __global__ void k_blob_fill(Item *items, int64_t nitems, int64_t m, int64_t n, c
 }
 
 // item cost for the CTA chunking: bytes staged + a fixed per-item overhead
-__global__ void k_item_cost(const Item *items, int64_t n, int64_t m, int64_t fixed, int64_t *cost) {
+__global__ void k_item_cost(const Item *items, int64_t n, int64_t m, int64_t fixed, int64_t group_row,
+                            int64_t *cost) {
     int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     if (k >= n) return;
     const Item it = items[k];
-    cost[k] = (int64_t)blob_parts(it, m).total + 40 * (item_nt(it)) + fixed + kGroupRowCost * it.ntr;
+    cost[k] = (int64_t)blob_parts(it, m).total + 40 * (item_nt(it)) + fixed + group_row * it.ntr;
 }
 
 __global__ void k_warp_first(const int64_t *begin, const WItem *witems, const int32_t *jcols, int W, WFirst *wf) {
@@ -895,7 +896,8 @@ static int configure_sm_queue(Matrix &M, int G, cudaStream_t st) {
     int64_t *cost = costb.as<int64_t>(), *incl = cost + n;
     int32_t *flag = flagb.as<int32_t>(), *pos = flag + (n + 1), *ustart = ub.as<int32_t>();
     const unsigned nb = (unsigned)((n + 1 + 255) / 256);
-    k_item_cost<<<nb, 256, 0, st>>>(M.items, n, M.m, kItemFixedCost, cost);
+    k_item_cost<<<nb, 256, 0, st>>>(M.items, n, M.m, kItemFixedCost,
+                                    M.kernel == TILESPMV_KERNEL_GATHER ? kGroupRowCostPre : kGroupRowCost, cost);
     if (int rc = scan([&](void *t, size_t &b) { return cub::DeviceScan::InclusiveSum(t, b, cost, incl, (int)n, st); }, st)) return rc;
     TSP_CK(cudaMemsetAsync(flag + n, 0, sizeof(int32_t), st));
     k_unit_flags<<<nb, 256, 0, st>>>(M.items, n, kLocalParts, flag);
@@ -956,7 +958,7 @@ int configure_launch(Matrix &M, cudaStream_t st) {
         if (int rc = costb.alloc(2 * M.num_items * sizeof(int64_t))) return rc;
         int64_t *cost = costb.as<int64_t>(), *incl = cost + M.num_items;
         k_item_cost<<<(unsigned)((M.num_items + 255) / 256), 256, 0, st>>>(M.items, M.num_items, M.m, kItemFixedCost,
-                                                                         cost);
+                                                                         kGroupRowCost, cost);
         if (int rc = scan([&](void *t, size_t &b) { return cub::DeviceScan::InclusiveSum(t, b, cost, incl, (int)M.num_items, st); }, st))
             return rc;
         k_cta_begin<<<(W + 1 + 255) / 256, 256, 0, st>>>(incl, M.items, M.num_items, W, kLocalParts, M.cta_begin);
