@@ -363,35 +363,45 @@ def time_single(launch, dev, reps, n=SINGLE_LAUNCHES):
     host's Python enqueue.  Two ways to launch: `eager` (tilespmv_run, a
     cudaLaunchKernelEx from the host) and `graph` (the same call captured as
     a one-node CUDA graph per replica, replayed).  Returns median / p10 /
-    p90 ms of each."""
+    p90 ms of each.  The same pair around a 1-element torch kernel gives the floor of this
+    measurement (`launch_floor_ms`: launch latency and event overhead with no
+    work)."""
     import torch
     stream = torch.cuda.current_stream(dev)
+    tiny = torch.zeros(1, device=dev)
     graphs = []
     for j in range(reps):
         g = torch.cuda.CUDAGraph()
         with torch.cuda.graph(g):
             launch(j)
         graphs.append(g)
+    tg = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(tg):
+        tiny.add_(1.0)
     torch.cuda.synchronize(dev)
     out = {}
     for kind in ("eager", "graph"):
-        ts = []
+        ts, fs = [], []
         for i in range(n + 3):
-            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-            torch.cuda.synchronize(dev)
-            torch.cuda._sleep(400_000)
-            e0.record(stream)
-            if kind == "graph":
-                graphs[i % reps].replay()
-            else:
-                launch(i)
-            e1.record(stream)
-            torch.cuda.synchronize(dev)
-            if i >= 3:
-                ts.append(e0.elapsed_time(e1))
+            for what, acc in (("spmv", ts), ("tiny", fs)):
+                e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                torch.cuda.synchronize(dev)
+                torch.cuda._sleep(400_000)
+                e0.record(stream)
+                if what == "tiny":
+                    tg.replay() if kind == "graph" else tiny.add_(1.0)
+                elif kind == "graph":
+                    graphs[i % reps].replay()
+                else:
+                    launch(i)
+                e1.record(stream)
+                torch.cuda.synchronize(dev)
+                if i >= 3:
+                    acc.append(e0.elapsed_time(e1))
         t = np.array(ts)
         out[kind] = {"median_ms": float(np.median(t)), "p10_ms": float(np.percentile(t, 10)),
-                     "p90_ms": float(np.percentile(t, 90)), "launches": n}
+                     "p90_ms": float(np.percentile(t, 90)), "launches": n,
+                     "launch_floor_ms": float(np.median(fs))}
     return out
 
 
@@ -439,7 +449,8 @@ def measure_workload(A, x_h, mode, steps, warmup, dev, use_graph=True, single=Tr
             v["frac"] = v["achieved_gbs"] / peak
             v["gflops"] = 2.0 * A.nnz / (v["median_ms"] * 1e-3) / 1e9
         s["note"] = ("one launch between events, no kernel of ours before it: includes the front-end launch "
-                     "latency and the cold prologue that PDL hides in back-to-back runs")
+                     "latency and the cold prologue that PDL hides in back-to-back runs; launch_floor_ms is the "
+                     "same measurement of a 1-element torch kernel")
         res["single_launch"] = s
     if check:
         torch.cuda.synchronize(dev)
