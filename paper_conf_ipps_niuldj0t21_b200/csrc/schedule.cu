@@ -1020,6 +1020,9 @@ int launch_spmv(const Matrix &M, const double *d_x, double *d_y, cudaStream_t st
     p.m = M.m;
     p.n = M.n;
     p.x_vec = (reinterpret_cast<uintptr_t>(d_x) & 15u) == 0;
+    p.blob_bytes = M.blob_bytes;
+    p.num_items = M.num_items;
+    p.slot_bytes = M.item_bytes;
     const KernelChoice kc = kernel_choice(M.kernel);
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3(M.grid);

@@ -4,6 +4,16 @@
 
 #include "internal.cuh"
 
+// TSP_CHECKED (scripts/checked_small.py only): device-side bounds checks of
+// every blob copy, x read, x segment and unit index against the handle's
+// sizes; a failed check is a device assert.  Off in the product build.
+#ifdef TSP_CHECKED
+#include <cassert>
+#define TSP_CHECK(c) assert(c)
+#else
+#define TSP_CHECK(c) ((void)0)
+#endif
+
 namespace tsp {
 
 constexpr unsigned FULL = 0xffffffffu;
@@ -25,6 +35,8 @@ struct Params {
     double *y;
     int64_t m, n;
     int x_vec;                 // x is 16-byte aligned: x segments load as double2
+    int64_t blob_bytes, num_items;  // sizes for the TSP_CHECKED build's bounds checks
+    int slot_bytes;
     const int32_t *xc_cols;    // GATHER: the columns of the shared-memory x cache
     int xc_n;                  // (their number, <= the kernel's cache slots)
 };

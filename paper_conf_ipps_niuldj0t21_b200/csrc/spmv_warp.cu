@@ -122,6 +122,7 @@ __device__ __forceinline__ void rem_products(const Params &p, uint32_t colS, uin
             xv[j] = 0.0;
             if (k < E) {
                 const int c = lds_s32(colS + 4 * k);  // < 0: slot ~c of the CTA's x cache (GATHER)
+                TSP_CHECK(c < 0 ? ~c < p.xc_n : c < p.n);
                 xv[j] = c < 0 ? lds_f64(xcS + 8u * (uint32_t)~c) : ldg_hint(p.x + (uint32_t)c, x_policy);
             }
         }
@@ -143,6 +144,7 @@ __device__ __forceinline__ double rem_product(const Params &p, int k, int e, uin
     int c;
     double v;
     lds_entry_lt(k, e, colS + 4 * k, valS + 8 * k, c, v);
+    TSP_CHECK(c >= 0 && c < p.n);
     const double pr = __dmul_rn(v, ldg_hint(p.x + (uint32_t)c, x_policy));
     return k < e ? pr : 0.0;
 }
@@ -241,6 +243,7 @@ __device__ __forceinline__ bool remainder(const Params &p, uint32_t rpS, uint32_
         double v0, v1;
         lds_entry_or(k0, e, colS + 4 * k0, valS + 8 * k0, cdef, c0, v0);
         lds_entry_or(k1, e, colS + 4 * k1, valS + 8 * k1, cdef, c1, v1);
+        TSP_CHECK(c0 >= 0 && c0 < p.n && c1 >= 0 && c1 < p.n);
         const double x0 = ldg_hint(p.x + (uint32_t)c0, x_policy), x1 = ldg_hint(p.x + (uint32_t)c1, x_policy);
         acc = fma(v0, x0, acc);
         acc = fma(v1, x1, acc);
@@ -376,6 +379,7 @@ __device__ __forceinline__ void run_group(int np, uint32_t &d, uint32_t xs, int 
 __device__ __forceinline__ void issue_blob(const Params &p, const WItem &it, uint32_t slot, uint32_t bar,
                                            uint64_t policy, int lane) {
     const uint32_t total = it.val_tot >> 16;
+    TSP_CHECK(total <= (uint32_t)p.slot_bytes && (int64_t)it.blob16 * 16 + total <= p.blob_bytes);
     if (lane == 0 && total) {
         mbar_expect_tx(bar, total);
         bulk_g2s_hint(slot, p.blob + (size_t)it.blob16 * 16, total, bar, policy);
@@ -396,6 +400,7 @@ __device__ __forceinline__ void issue_x(const Params &p, int J, int nt, uint32_t
         for (int kk = 0; kk < XT / 4; ++kk) {
             const int t = 4 * kk + (lane >> 3);
             const uint32_t Jt = (uint32_t)__shfl_sync(FULL, J, t);
+            TSP_CHECK(t >= nt || (int64_t)Jt * 16 + 16 <= p.n);
             if (t < nt) cp_async16(xs_l + 128 * t, xq + 16u * Jt, 16u, x_policy);
         }
         cp_async_commit();
@@ -626,6 +631,7 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT, XT, XC>::kThreads, 1) til
         issued = true;
         griddep_wait();
         waited = true;
+        for (int i = threadIdx.x; i < p.xc_n; i += Cfg::kThreads) TSP_CHECK(p.xc_cols[i] >= 0 && p.xc_cols[i] < p.n);
         for (int i = threadIdx.x; i < p.xc_n; i += Cfg::kThreads) sts_f64(xcS + 8u * i, __ldg(p.x + __ldg(p.xc_cols + i)));
         __syncthreads();
     }
@@ -647,7 +653,9 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT, XT, XC>::kThreads, 1) til
             c = __shfl_sync(FULL, c, 0);
             nb = -1;
             if (c < ue) {
+                TSP_CHECK(c >= ub);
                 const int2 u = __ldg(p.units + c);
+                TSP_CHECK(u.x >= 0 && u.x < u.y && u.y <= p.num_items);
                 nb = u.x;
                 ne = u.y;
             }
@@ -655,6 +663,7 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT, XT, XC>::kThreads, 1) til
         // 1. x segments, issued before the blob lands (J came with the record)
         issue_x<XT>(p, J, (it.part_nt >> 24) & 31, xs, x_policy, lane, (it.groups >> 30) & 1u);
         const int kn = k + 1 < ke ? k + 1 : nb;
+        TSP_CHECK(kn < p.num_items);
         if (kn >= 0) {  // the next record and its columns, in flight during this item
             nxt = load_witem(p.witems, kn);
             Jn = lane < 16 ? __ldg(p.jcols + (int64_t)kn * 16 + lane) : 0;
