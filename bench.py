@@ -48,6 +48,7 @@ SECONDARY = [("fem", "DEFERRED"), ("rmat20", "DEFERRED"), ("mixed", "ADPT"), ("m
              # the optional byte-cost selection mode (not the paper's rule)
              ("fem", "BYTES")]
 SINGLE_LAUNCHES = 60  # single-launch timing: median of this many isolated launches
+CHUNKS = 4            # N > 1, --exchange chunked: chunks per rank
 
 
 def log(*a):
@@ -496,7 +497,10 @@ def measure_sharded(workload, mode, steps, warmup, dev, rank, P, group, exchange
                    (SURVEY 8(e), the north star's exchange);
       halo      -- neighbour-only NCCL send/recv of the x rows each peer's
                    columns touch, overlapped with the interior SpMV; the
-                   boundary SpMVs run after it lands.
+                   boundary SpMVs run after it lands (SURVEY 8(f) f1);
+      chunked   -- the all-gather in CHUNKS pieces, each rank's chunk i sent
+                   to every peer (NCCL send/recv) while chunk i + 1 computes
+                   (SURVEY 8(e), B200-native improvement 1).
     x stays fixed across steps (the exchanged rows equal what is there), so
     the timed work is exactly one iteration's and values stay finite.  Times
     are device events on the compute stream, max over ranks: the step, the
@@ -504,7 +508,8 @@ def measure_sharded(workload, mode, steps, warmup, dev, rank, P, group, exchange
     import torch
     import torch.distributed as dist
     from paper_conf_ipps_niuldj0t21_b200 import TiledMatrix
-    from paper_conf_ipps_niuldj0t21_b200.sharded import HaloSpMV, ShardedSpMV, build_shard_handles, plan_halo
+    from paper_conf_ipps_niuldj0t21_b200.sharded import (ChunkedAllGatherSpMV, HaloSpMV, ShardedSpMV,
+                                                         build_shard_handles, chunk_bounds, plan_halo)
     from synthetic import gen
 
     t0 = time.perf_counter()
@@ -525,6 +530,9 @@ def measure_sharded(workload, mode, steps, warmup, dev, rank, P, group, exchange
     if exchange == "halo":
         plan = plan_halo(A.rowptr, A.colidx, bounds, rank, P, group)
         parts = plan.parts
+    elif exchange == "chunked":
+        cb = chunk_bounds(bounds, CHUNKS)[rank]
+        plan, parts = None, [(cb[i], cb[i + 1], True) for i in range(CHUNKS)]
     else:
         plan, parts = None, [(a, b, True)]
     mats, _, _ = build_shard_handles(create, [(r0, r1) for r0, r1, _ in parts], A.nnz, mode=mode,
@@ -548,9 +556,13 @@ def measure_sharded(workload, mode, steps, warmup, dev, rank, P, group, exchange
                 e[2 + 2 * i].record(stream)
         return f
 
-    if exchange == "halo":
+    if exchange in ("halo", "chunked"):
         y = torch.empty(n, dtype=torch.float64, device=dev)
-        H = HaloSpMV(plan, [timed_run(i, M) for i, M in enumerate(mats)], group=group, host_staging=one_gpu)
+        if exchange == "halo":
+            H = HaloSpMV(plan, [timed_run(i, M) for i, M in enumerate(mats)], group=group, host_staging=one_gpu)
+        else:
+            H = ChunkedAllGatherSpMV([timed_run(i, M) for i, M in enumerate(mats)], bounds, rank, P, group=group,
+                                     host_staging=one_gpu)
 
         def step(ev=None):
             cur[0] = ev
@@ -612,7 +624,10 @@ def measure_sharded(workload, mode, steps, warmup, dev, rank, P, group, exchange
                         "frac": achieved / peak, "traffic": None, "peak_source": peak_src,
                         "alg_bytes_per_launch": infos[dom]["alg_bytes"],
                         "kernel": mats[dom].kernel_name() + (" (interior part)" if exchange == "halo" else "")}}
-    if exchange == "halo":
+    if exchange == "chunked":
+        res["exchange"] = {"kind": f"all-gather in {CHUNKS} chunks (NCCL send/recv of chunk i while chunk i+1 "
+                                   "computes)", "bytes_per_rank": 8 * (n - (b - a))}
+    elif exchange == "halo":
         res["exchange"] = {"kind": "halo (NCCL send/recv, overlapped with the interior SpMV)",
                            "recv_bytes_rank": 8 * plan.recv_elems, "send_bytes_rank": 8 * plan.send_elems,
                            "parts_rank": [[r0, r1, bool(it)] for r0, r1, it in parts]}
@@ -627,7 +642,7 @@ def measure_sharded(workload, mode, steps, warmup, dev, rank, P, group, exchange
         def e2e_step():
             x[a:b].copy_(hx, non_blocking=True)
             step()
-            hy.copy_(y[a:b] if exchange == "halo" else sh.local_out(), non_blocking=True)
+            hy.copy_(y[a:b] if exchange in ("halo", "chunked") else sh.local_out(), non_blocking=True)
             stream.synchronize()
 
         for _ in range(2):
@@ -676,13 +691,14 @@ def run_ours(args):
         res = measure_sharded(args.workload, args.mode, args.steps, args.warmup, dev, rank, P, group,
                               args.exchange, args.e2e_steps, one_gpu)
         if not args.no_secondary:  # the other exchange, same shards
-            other = "halo" if args.exchange == "allgather" else "allgather"
-            r2 = measure_sharded(args.workload, args.mode, args.steps, args.warmup, dev, rank, P, group,
-                                 other, 0, one_gpu)
-            secondary[f"exchange_{other}"] = {
-                "value": r2["value"], "unit": UNIT, "ms_per_step": r2["ms_per_step"],
-                "breakdown_ms_max_over_ranks": r2["breakdown_ms_max_over_ranks"],
-                "exchange": r2["exchange"], "roofline": r2["roofline"], "clocks": r2["clocks"]}
+            others = [e for e in ("allgather", "halo", "chunked") if e != args.exchange]
+            for other in others:
+                r2 = measure_sharded(args.workload, args.mode, args.steps, args.warmup, dev, rank, P, group,
+                                     other, 0, one_gpu)
+                secondary[f"exchange_{other}"] = {
+                    "value": r2["value"], "unit": UNIT, "ms_per_step": r2["ms_per_step"],
+                    "breakdown_ms_max_over_ranks": r2["breakdown_ms_max_over_ranks"],
+                    "exchange": r2["exchange"], "roofline": r2["roofline"], "clocks": r2["clocks"]}
         m, n, nnz = res["m"], res["n"], res["nnz"]
     else:
         t0 = time.perf_counter()
@@ -728,8 +744,10 @@ def run_ours(args):
                "e2e": res.get("e2e"),
                "gpu_launches": args.steps * res.get("launches_per_step", 1),
                "clocks": res["clocks"],
-               "step": (("SpMV + NCCL all-gather of y" if args.exchange == "allgather" else
-                         "halo exchange overlapped with the interior SpMV + boundary SpMVs")
+               "step": ({"allgather": "SpMV + NCCL all-gather of y",
+                         "halo": "halo exchange overlapped with the interior SpMV + boundary SpMVs",
+                         "chunked": f"{CHUNKS} chunk SpMVs, each chunk sent to every peer while the next "
+                                    "computes"}[args.exchange]
                         if P > 1 else "one SpMV launch"),
                "timing": {"launch_mode": res["launch_mode"], "replicas_rotated": res["reps"],
                           "host_enqueue_us_per_step": res.get("host_enqueue_us_per_step")},
@@ -759,9 +777,10 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--workload", default=DEFAULT_WORKLOAD)
     ap.add_argument("--mode", default="DEFERRED", choices=["ADPT", "DEFERRED", "AUTO", "FORCE_CSR", "BYTES"])
-    ap.add_argument("--exchange", default="allgather", choices=["allgather", "halo"],
-                    help="N>1: all-gather of y (north star, default) or the neighbour-only x exchange; "
-                         "the other one is timed as a secondary entry")
+    ap.add_argument("--exchange", default="allgather", choices=["allgather", "halo", "chunked"],
+                    help="N>1: all-gather of y (north star, default), the neighbour-only x exchange, or the all-gather in "
+                         "chunks overlapped with the SpMV; "
+                         "the others are timed as secondary entries")
     ap.add_argument("--e2e-steps", type=int, default=20)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-secondary", action="store_true")

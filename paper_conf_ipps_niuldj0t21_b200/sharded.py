@@ -292,3 +292,82 @@ class HaloSpMV:
                 continue
             f(x_cur, x_next[r0:r1])
         return x_next
+
+
+# ----------------------------------------------------------------------------
+# All-gather overlapped with the SpMV (SURVEY §8(e), B200-native improvement
+# 1): every rank's rows are cut into C chunks on tile-row boundaries; chunk i
+# is computed, then sent to every peer while chunk i + 1 computes, and every
+# peer's chunk i is received in place into x_{k+1}.  With NCCL the sends of
+# chunk i wait (on NCCL's stream) only for chunk i's kernel.  Each chunk is its
+# own handle built from its row slice, so every row is summed exactly as on
+# one GPU and x_{k+1} equals the 1-GPU iterate bitwise.
+# ----------------------------------------------------------------------------
+
+def chunk_bounds(bounds, chunks: int) -> list[list[int]]:
+    """For every rank r, chunks + 1 row boundaries of [bounds[r], bounds[r+1])
+    on tile-row (16-row) boundaries, the tile rows split as evenly as
+    possible by count.  Pure host logic: every rank computes every rank's."""
+    out = []
+    for r in range(len(bounds) - 1):
+        a, b = int(bounds[r]), int(bounds[r + 1])
+        T = (b - a + 15) // 16
+        out.append([min(a + 16 * ((T * i) // chunks), b) for i in range(chunks)] + [b])
+    return out
+
+
+class ChunkedAllGatherSpMV:
+    """One rank's side of the chunked, overlapped all-gather iterated SpMV.
+
+    spmvs[i] is a callable (x_full, y_out) for this rank's chunk i (normally
+    the TiledMatrix.run of that row slice); x buffers are full length."""
+
+    def __init__(self, spmvs, bounds, rank: int, world: int, group=None, host_staging: bool = False):
+        """host_staging: move the chunks through host buffers (a backend such as
+        gloo that cannot send device tensors; development runs only)."""
+        self.spmvs, self.rank, self.world, self.group = list(spmvs), rank, world, group
+        self.cb = chunk_bounds(bounds, len(self.spmvs))
+        self.host_staging = host_staging
+
+    @property
+    def parts(self):
+        c = self.cb[self.rank]
+        return [(c[i], c[i + 1]) for i in range(len(self.spmvs))]
+
+    def _ops(self, x, i, staged):
+        import torch.distributed as dist
+        a, b = self.cb[self.rank][i], self.cb[self.rank][i + 1]
+        ops = []
+        for q in range(self.world):
+            if q == self.rank:
+                continue
+            lo, hi = self.cb[q][i], self.cb[q][i + 1]
+            if b > a:
+                t = x[a:b].cpu() if self.host_staging else x[a:b]
+                ops.append(dist.P2POp(dist.isend, t, q, group=self.group))
+            if hi > lo:
+                if self.host_staging:
+                    h = x.new_empty(hi - lo, device="cpu")
+                    staged.append((x[lo:hi], h))
+                    ops.append(dist.P2POp(dist.irecv, h, q, group=self.group))
+                else:
+                    ops.append(dist.P2POp(dist.irecv, x[lo:hi], q, group=self.group))
+        return ops
+
+    def step(self, x_cur, x_next):
+        """x_next = A x_cur on every rank (own rows computed, peers' received)."""
+        import torch.distributed as dist
+        works, staged = [], []
+        for i, f in enumerate(self.spmvs):
+            a, b = self.cb[self.rank][i], self.cb[self.rank][i + 1]
+            if b > a:
+                f(x_cur, x_next[a:b])
+            if self.world > 1 and dist.is_available() and dist.is_initialized():
+                ops = self._ops(x_next, i, staged)
+                if ops:
+                    works += dist.batch_isend_irecv(ops)
+        for w in works:
+            w.wait()
+        for dst, h in staged:
+            dst.copy_(h)
+        return x_next

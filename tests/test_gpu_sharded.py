@@ -40,7 +40,8 @@ def _rank_worker(rank, world, port, name, exchange, q):
         import torch
         import torch.distributed as dist
         from paper_conf_ipps_niuldj0t21_b200 import TiledMatrix
-        from paper_conf_ipps_niuldj0t21_b200.sharded import (HaloSpMV, ShardedSpMV, build_shard_handles,
+        from paper_conf_ipps_niuldj0t21_b200.sharded import (ChunkedAllGatherSpMV, HaloSpMV, ShardedSpMV,
+                                                             build_shard_handles, chunk_bounds,
                                                              partition_tile_rows, plan_halo)
         os.environ["MASTER_ADDR"] = "127.0.0.1"
         os.environ["MASTER_PORT"] = str(port)
@@ -69,6 +70,21 @@ def _rank_worker(rank, world, port, name, exchange, q):
                 torch.cuda.synchronize()
                 outs.append(xk.cpu().numpy())
             M.close()
+        elif exchange == "chunked":  # all-gather overlapped with the SpMV, 3 chunks per rank
+            cb = chunk_bounds(b, 3)[rank]
+            hs, md, kn = build_shard_handles(create, [(cb[i], cb[i + 1]) for i in range(3)], S.nnz)
+            C = ChunkedAllGatherSpMV([lambda xf, yo, M=M: M.run(xf, yo) for M in hs], b, rank, world,
+                                     host_staging=True)
+            xa = torch.from_numpy(x.copy()).to(dev)
+            xb = torch.full((A.n,), float("nan"), dtype=torch.float64, device=dev)
+            for _ in range(ITERS):
+                C.step(xa, xb)
+                torch.cuda.synchronize()
+                outs.append(xb.cpu().numpy())
+                xa, xb = xb, xa
+                xb.fill_(float("nan"))  # every row must be computed or received
+            for M in hs:
+                M.close()
         else:
             plan = plan_halo(S.rowptr, S.colidx, b, rank, world)
             hs, md, kn = build_shard_handles(create, [(r0, r1) for r0, r1, _ in plan.parts], S.nnz)
@@ -90,7 +106,7 @@ def _rank_worker(rank, world, port, name, exchange, q):
         q.put((rank, None, traceback.format_exc(), None))
 
 
-@pytest.mark.parametrize("exchange", ["allgather", "halo"])
+@pytest.mark.parametrize("exchange", ["allgather", "halo", "chunked"])
 @pytest.mark.parametrize("name", ["stencil27_40", "rmat12", "lap2d_37x29", "mixed_small"])
 def test_sharded_cuda_iterates_bitwise_equal_one_gpu(cuda_device, name, exchange):
     import torch
@@ -126,7 +142,7 @@ def test_sharded_cuda_iterates_bitwise_equal_one_gpu(cuda_device, name, exchange
         for k in range(ITERS):
             got = outs[k] if exchange == "halo" else outs[k][b[r]:b[r + 1]]
             assert np.array_equal(got.view(np.uint64), ref[k][b[r]:b[r + 1]].view(np.uint64)), (name, exchange, r, k)
-            if exchange == "allgather":  # every rank holds the whole iterate
+            if exchange in ("allgather", "chunked"):  # every rank holds the whole iterate
                 assert np.array_equal(outs[k].view(np.uint64), ref[k].view(np.uint64))
 
 

@@ -271,3 +271,85 @@ def test_build_shard_handles_resolves_auto_globally():
         assert kn == KERNELS["GATHER"], (rank, kn)
         assert hs == [(MODES["DEFERRED"], KERNELS["GATHER"])] * 2
         assert closed == 2  # the two provisional SM_QUEUE handles
+
+
+# ---------------------------------------------------------------------------
+# chunked all-gather overlapped with the SpMV (SURVEY §8(e) improvement 1)
+# ---------------------------------------------------------------------------
+
+def _chunked_worker(rank, world, port, name, chunks, iters, q):
+    try:
+        from oracle import oracle as O
+        from paper_conf_ipps_niuldj0t21_b200.sharded import ChunkedAllGatherSpMV, chunk_bounds
+        from synthetic import gen
+        os.environ["MASTER_ADDR"] = "127.0.0.1"
+        os.environ["MASTER_PORT"] = str(port)
+        dist.init_process_group("gloo", rank=rank, world_size=world)
+        A, x = gen.make(name)
+        b = partition_tile_rows(A.m, world)
+        cb = chunk_bounds(b, chunks)[rank]
+
+        def part_spmv(r0, r1):
+            P = A.row_slice(r0, r1)
+
+            def f(xf, yout):
+                y, _ = O.spmv(P, xf.numpy())
+                yout.copy_(torch.from_numpy(y))
+            return f
+
+        C = ChunkedAllGatherSpMV([part_spmv(cb[i], cb[i + 1]) for i in range(chunks)], b, rank, world)
+        xa = torch.from_numpy(x.copy())
+        xb = torch.full((A.n,), float("nan"), dtype=torch.float64)  # every row must be written or received
+        outs = []
+        for k in range(iters):
+            C.step(xa, xb)
+            outs.append(xb.numpy().copy())
+            xa, xb = xb, xa
+            xb.fill_(float("nan"))
+        q.put((rank, b, outs))
+        dist.destroy_process_group()
+    except Exception:  # pragma: no cover
+        import traceback
+        q.put((rank, None, traceback.format_exc()))
+
+
+@pytest.mark.parametrize("name,world,chunks", [("stencil27_21", 2, 3), ("rmat12", 3, 4), ("lap2d_37x29", 2, 5)])
+def test_chunked_allgather_equals_unsharded(name, world, chunks):
+    """Every rank holds the full x_{k+1}, bitwise equal to the unsharded
+    oracle iterate (x_{k+1} starts as NaN: a row neither computed nor received
+    would show)."""
+    from oracle import oracle as O
+    from synthetic import gen
+    iters = 3
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _port()
+    procs = [ctx.Process(target=_chunked_worker, args=(r, world, port, name, chunks, iters, q))
+             for r in range(world)]
+    for p in procs:
+        p.start()
+    res = [q.get(timeout=300) for _ in range(world)]
+    for p in procs:
+        p.join(timeout=60)
+    for r, b, outs in res:
+        assert b is not None, outs
+    A, x = gen.make(name)
+    ref, xk = [], x.copy()
+    for _ in range(iters):
+        xk, _ = O.spmv(A, xk)
+        ref.append(xk.copy())
+    for r, b, outs in res:
+        for k in range(iters):
+            assert np.array_equal(outs[k].view(np.uint64), ref[k].view(np.uint64)), (name, r, k)
+
+
+def test_chunk_bounds():
+    from paper_conf_ipps_niuldj0t21_b200.sharded import chunk_bounds
+    b = partition_tile_rows(8_000_000, 8)
+    cb = chunk_bounds(b, 4)
+    assert cb[0] == [0, 250_000, 500_000, 750_000, 1_000_000]   # C5 at N = 8: 15,625 tile rows per chunk
+    for bounds, C in [([0, 37, 100], 3), ([0, 16, 17], 4), ([0, 0, 48], 2), (partition_tile_rows(1000, 3), 7)]:
+        for r, c in enumerate(chunk_bounds(bounds, C)):
+            assert len(c) == C + 1 and c[0] == bounds[r] and c[-1] == bounds[r + 1]
+            assert all(c[i] <= c[i + 1] for i in range(C))
+            assert all((v - bounds[r]) % 16 == 0 for v in c[:-1])
