@@ -27,4 +27,5 @@ TILESPMV_BENCH_ONE_GPU=1 timeout 900 python -m torch.distributed.run --nnodes=1 
    --master-addr 127.0.0.1 --master-port 29533 bench.py --gpus 2 --steps 5 --warmup 3 --workload stencil27_40 \
    --e2e-steps 2 > $OUT/n2_devcheck.json 2> $OUT/n2_devcheck.err; echo "rc=$?" >> $OUT/n2_devcheck.err
 timeout 300 python bench.py --impl reference --steps 20 --warmup 5 > $OUT/reference.json 2> $OUT/reference.err
+timeout 800 python scripts/checked_small.py > $OUT/checked_small.log 2>&1; echo "rc=$?" >> $OUT/checked_small.log
 echo done > $OUT/DONE
