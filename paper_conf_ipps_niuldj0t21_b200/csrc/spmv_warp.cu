@@ -593,13 +593,16 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT, XT, XC>::kThreads, 1) til
     constexpr bool PRE = XC > 0;
     extern __shared__ __align__(128) uint8_t smem[];
     __shared__ int s_next;
+    __shared__ __align__(8) uint64_t s_xc_bar;  // GATHER: the x cache is filled (every warp arrives once)
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const uint32_t xs = smem_u32(smem) + (uint32_t)warp * Cfg::kX;
     const uint32_t slot = smem_u32(smem) + WARPS * Cfg::kX + (uint32_t)warp * Cfg::kPer;
     const uint32_t racc = slot + SLOT, bar = racc + Cfg::kRacc;
+    const uint32_t xc_bar = smem_u32(&s_xc_bar);
     const int ub = (int)__ldg(p.cta_begin + blockIdx.x), ue = (int)__ldg(p.cta_begin + blockIdx.x + 1);
     if (lane == 0) {
         mbar_init(bar, 1);
+        if (XC > 0 && warp == 0) mbar_init(xc_bar, WARPS);
         fence_mbar_init();
     }
     if (threadIdx.x == 0) s_next = ub + WARPS;  // units ub .. ub+WARPS-1 are the warps' first
@@ -624,16 +627,18 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT, XT, XC>::kThreads, 1) til
         nxt = load_witem(p.witems, k);
         Jn = lane < 16 ? __ldg(p.jcols + (int64_t)k * 16 + lane) : 0;
     }
-    bool waited = false, issued = false;
+    bool waited = false, issued = false, xc_wait = false;
     const uint32_t xcS = smem_u32(smem) + Cfg::kXc;
-    if (XC > 0 && p.xc_n > 0) {  // the first blob in flight, then the x cache (x is the previous kernel's)
+    if (XC > 0 && p.xc_n > 0) {  // the first blob in flight, then the warp's share of the x cache
         if (k >= 0) issue_blob(p, nxt, slot, bar, stream_policy, lane);
         issued = true;
-        griddep_wait();
+        griddep_wait();  // x is the previous kernel's
         waited = true;
         for (int i = threadIdx.x; i < p.xc_n; i += Cfg::kThreads) TSP_CHECK(p.xc_cols[i] >= 0 && p.xc_cols[i] < p.n);
         for (int i = threadIdx.x; i < p.xc_n; i += Cfg::kThreads) sts_f64(xcS + 8u * i, __ldg(p.x + __ldg(p.xc_cols + i)));
-        __syncthreads();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(xc_bar);  // release: the warp's cache entries
+        xc_wait = true;  // the whole cache is needed only once the first blob has landed
     }
     int j = 0;
     while (k >= 0) {
@@ -671,6 +676,10 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT, XT, XC>::kThreads, 1) til
         if (it.val_tot >> 16) {
             mbar_wait(bar, phase);
             phase ^= 1u;
+        }
+        if (XC > 0 && xc_wait) {  // acquire: every warp's cache entries
+            mbar_wait(xc_bar, 0);
+            xc_wait = false;
         }
         TSP_STAMP(gw, j, 1);
         TSP_INFO(gw, j, k, it);
