@@ -328,6 +328,87 @@ __device__ __forceinline__ void half_coo_scan(uint32_t V, uint32_t rc, int n, ui
     if ((rows >> (16 * h + r)) & 1u) acc += lds_f64(Sh + 8 * r);
 }
 
+// ------------------------------------------ split routines (odd groups) ----
+// A format group with an odd number of tiles ends in a pair whose second
+// tile is a masked copy of the first.  That last tile then runs on BOTH
+// halves: half h takes the tile's entries / slots / columns / full rows of
+// parity h, and the halves' partial row sums meet in the final
+// acc(r) + acc(r + 16) like every other pair's.  Which tiles split depends
+// only on the item's content (the group's tile count), so every row's
+// summation order stays content-defined.
+
+// Dns: half h multiplies columns 8h .. 8h + 7
+__device__ __forceinline__ void split_dns(uint32_t P, uint32_t X, int r, int h, double &acc) {
+    const uint32_t V = P + 8 * r + 1024 * h, Xh = X + 64 * h;
+    double a0 = 0.0, a1 = 0.0;
+#pragma unroll
+    for (int c = 0; c < 8; c += 2) {
+        const double2 xc = lds_v2f64(Xh + 8 * c);
+        a0 = fma(lds_f64(V + 128 * c), xc.x, a0);
+        a1 = fma(lds_f64(V + 128 * c + 128), xc.y, a1);
+    }
+    acc += a0 + a1;
+}
+
+// CSR: half h takes entries h, h + 2, ... of row r (tm: the tile's longest row)
+__device__ __forceinline__ void split_csr(uint32_t RP, int nz, int tm, uint32_t X, int r, int h, double &acc) {
+    const int beg = (int)lds_u8(RP + r);
+    const int end = r < 15 ? (int)lds_u8(RP + r + 1) : nz;
+    const int len = end - beg;
+    const uint32_t V = RP + 8 * (beg - nz);
+#pragma unroll 1
+    for (int j0 = h; j0 < tm; j0 += 4) {
+        double v[2], xv[2];
+#pragma unroll
+        for (int q = 0; q < 2; ++q) {
+            const int j = j0 + 2 * q, e = beg + j;
+            const uint32_t b = lds_u8(RP + 16 + (min(e, 255) >> 1));
+            xv[q] = lds_f64(X + 8 * ((b >> (4 * (e & 1))) & 15u));
+            v[q] = lds_f64_lt(j, len, V + 8 * j);
+        }
+        acc = fma(v[0], xv[0], acc);
+        acc = fma(v[1], xv[1], acc);
+    }
+}
+
+// ELL: half h takes slots h, h + 2, ... (w: the width)
+__device__ __forceinline__ void split_ell(uint32_t P, int w, uint32_t X, int r, int h, double &acc) {
+    const uint32_t ci = P + 128 * w + (r >> 1), V = P + 8 * r;
+    const uint32_t rot = (r & 1) ? 31u : 3u;
+#pragma unroll 1
+    for (int k = h; k < w; k += 2) {
+        const uint32_t b = lds_u8(ci + 8 * k);
+        acc = fma(lds_f64(V + 128 * k), lds_f64(xaddr(__funnelshift_l(b, b, rot), X)), acc);
+    }
+}
+
+// DnsCol: half h takes full columns q = h, h + 2, ...
+__device__ __forceinline__ void split_dnscol(uint32_t P, int nc, uint32_t X, int r, int h, double &acc) {
+    const uint32_t cid = P + 128 * nc;
+#pragma unroll 1
+    for (int q = h; q < nc; q += 2)
+        acc = fma(lds_f64(P + 8 * (16 * q + r)), lds_f64(X + 8 * (lds_u8(cid + q) & 15u)), acc);
+}
+
+// DnsRow (P:173's mapping): half h takes full rows q = h, h + 2, ..., lane c
+// of the half multiplies value q*16 + c by x[c], a 16-lane tree sums the row
+// and the lane of rowid[q] adds it
+__device__ __forceinline__ void split_dnsrow(uint32_t P, int nr, uint32_t X, int r, int h, double &acc) {
+    const uint32_t rid = P + 128 * nr;
+    const double xc = lds_f64(X + 8 * r);
+    const int trips = (nr + 1) >> 1;  // warp-uniform: both halves hold the same tile
+#pragma unroll 1
+    for (int t = 0; t < trips; ++t) {
+        const int q = 2 * t + h;
+        double s = lds_f64_lt(q, nr, P + 8 * (16 * q + r)) * xc;
+        s += __shfl_xor_sync(FULL, s, 8);
+        s += __shfl_xor_sync(FULL, s, 4);
+        s += __shfl_xor_sync(FULL, s, 2);
+        s += __shfl_xor_sync(FULL, s, 1);
+        if (q < nr && (int)lds_u8(rid + q) == r) acc += s;
+    }
+}
+
 // HYB in the TM kernels: the ELL part as ELL, the COO part with the
 // lane-per-entry scan in passes of 16 entries
 __device__ __forceinline__ void half_hyb_scan(uint32_t P, int w, int nz, uint32_t X, int r, int h, uint32_t S, bool ok,
