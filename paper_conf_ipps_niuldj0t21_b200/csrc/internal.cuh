@@ -15,6 +15,9 @@ constexpr int kTile = 16;  // P:20 "the size is always 16 by 16"
 
 // Format codes (same numbering as the ABI, P:96 order).
 enum : uint8_t { F_CSR = 0, F_COO = 1, F_ELL = 2, F_HYB = 3, F_DNS = 4, F_DNSROW = 5, F_DNSCOL = 6 };
+// execution-descriptor code of a merged CSR pair (schedule.cu, CSR2): COO
+// tiles never get descriptors, so their code is free on the execution side
+constexpr uint8_t F_CSR2 = F_COO;
 
 // ---------------------------------------------------------------------------
 // SpMV schedule.  A work item is a byte-bounded piece of one tile row: a run

@@ -34,6 +34,7 @@ struct TileView {
     const int32_t *tileColIdx;
     int run;        // ADPT / BYTES: COO data as a COO run
     int local_rem;  // DEFERRED: remainders that fit the x stage as a local run (rem_local)
+    const uint8_t *payload;  // canonical level-2 payload (CSR2 merge test and re-encoding)
 };
 
 // Bytes tile g occupies in its item's blob payload, and the entries it adds
@@ -233,14 +234,56 @@ __device__ __forceinline__ int dsc_format(const TileView &T, int g) {
     return f;
 }
 
+// CSR2 (execution copy only; the canonical tiling is untouched): two CSR
+// tiles of an item at adjacent tile columns J, J + 1 whose merged rows hold
+// at most 3 entries each -- the dy = +-1 half-bands of a 27-point stencil,
+// where tile J holds rows 0..8 and tile J + 1 rows 7..15 -- run as ONE tile
+// whose 5-bit columns index both x segments (staged side by side), so a lane
+// does its row's 3 entries once instead of two half-empty tiles.  Encoding:
+// val[nz] row-major (row r: tile J's entries, then tile J + 1's), rowptr[16]
+// u8, one column byte per entry (0..31); never larger than the two tiles'
+// canonical payloads (checked), written over them in the blob.  Only without
+// a COO run; descriptor format code F_CSR2 = 1 (COO tiles never get
+// descriptors: DEFERRED extracts them, ADPT/BYTES move them into the run).
+__device__ __forceinline__ bool csr2_mergeable(const TileView &T, int g) {
+    if (T.run || T.tileFmt[g] != F_CSR || T.tileFmt[g + 1] != F_CSR) return false;
+    if (T.tileColIdx[g + 1] != T.tileColIdx[g] + 1) return false;
+    const int na = T.tileNnz[g + 1] - T.tileNnz[g], nb = T.tileNnz[g + 2] - T.tileNnz[g + 1];
+    if (up16(9u * (uint32_t)(na + nb) + 16u) > (T.tileOff[g + 2] - T.tileOff[g]) * 16u) return false;
+    const uint8_t *ra = T.payload + (size_t)T.tileOff[g] * 16 + 8 * na;
+    const uint8_t *rb = T.payload + (size_t)T.tileOff[g + 1] * 16 + 8 * nb;
+    for (int r = 0; r < 16; ++r) {
+        const int la = (r < 15 ? ra[r + 1] : na) - ra[r], lb = (r < 15 ? rb[r + 1] : nb) - rb[r];
+        if (la + lb > 3) return false;
+    }
+    return true;
+}
+
+// execution format of every tile of the item (pairs merged greedily left to
+// right): dsc_format, F_CSR2 for a merged pair's first tile, -1 for no descriptor
+__device__ __forceinline__ void exec_formats(const Item &it, const TileView &T, int8_t *ef) {
+    const int nt = item_nt(it);
+    for (int t = 0; t < nt; ++t) {
+        if (t + 1 < nt && csr2_mergeable(T, it.tb + t)) {
+            ef[t] = F_CSR2;
+            ef[t + 1] = -1;
+            ++t;
+        } else {
+            ef[t] = (int8_t)dsc_format(T, it.tb + t);
+        }
+    }
+}
+
 __global__ void k_dsc_count(Item *items, int64_t n, TileView T, int32_t *ndsc) {
     int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     if (k >= n) return;
     const Item it = items[k];
     const int nt = item_nt(it);
     int cnt[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+    int8_t ef[kItemTiles];
+    exec_formats(it, T, ef);
     for (int t = 0; t < nt; ++t) {
-        const int f = dsc_format(T, it.tb + t);
+        const int f = ef[t];
         if (f >= 0) cnt[f]++;
     }
     int total = 0;
@@ -267,17 +310,20 @@ __global__ void k_dsc_write(Item *items, int64_t n, const int32_t *dbeg, const i
             o += pt;
         }
     }
+    int8_t ef[kItemTiles];
+    exec_formats(it, T, ef);
     for (int f = 0; f < 7; ++f) {
         uint2 last = make_uint2(0u, 0u);
         int c = 0;
         for (int t = 0; t < nt; ++t) {
             const int g = it.tb + t;
-            if (dsc_format(T, g) != f) continue;
+            if (ef[t] != f) continue;
             const bool hyb_ell = T.tileFmt[g] == F_HYB;  // (run) the ELL(w) part of a HYB tile
             uint2 d;
             d.x = off[t] | ((uint32_t)t << 21) | ((uint32_t)f << 29);
-            d.y = (uint32_t)T.tileAux[g] |
-                  ((hyb_ell ? 16u * T.tileAux[g] : (uint32_t)(T.tileNnz[g + 1] - T.tileNnz[g])) << 8);
+            d.y = f == F_CSR2 ? (uint32_t)(T.tileNnz[g + 2] - T.tileNnz[g]) << 8
+                              : (uint32_t)T.tileAux[g] |
+                                    ((hyb_ell ? 16u * T.tileAux[g] : (uint32_t)(T.tileNnz[g + 1] - T.tileNnz[g])) << 8);
             dlist[pos++] = d;
             last = d;
             c++;
@@ -371,8 +417,10 @@ __global__ void k_blob_fill(Item *items, int64_t nitems, int64_t m, int64_t n, c
         w.rp_col = b.rp | (b.col << 16);
         w.val_tot = b.val | (b.total << 16);
         int cnt[7] = {0, 0, 0, 0, 0, 0, 0};
+        int8_t ef[kItemTiles];
+        exec_formats(it, T, ef);
         for (int t = 0; t < nt; ++t) {
-            const int f = dsc_format(T, it.tb + t);
+            const int f = ef[t];
             if (f >= 0) cnt[f]++;
         }
         uint32_t g = 0;
@@ -398,7 +446,7 @@ __global__ void k_blob_fill(Item *items, int64_t nitems, int64_t m, int64_t n, c
             const uint2 d = dlist[it.dbeg + i];
             const uint32_t off = d.x & 0x1FFFFFu, t = (d.x >> 21) & 0xFFu, f = d.x >> 29;
             const uint32_t nz = (d.y >> 8) & 0x1FFu;
-            e.x = b.pay + off + (f == F_CSR ? 8u * nz : 0u) - 8u * (uint32_t)i;
+            e.x = b.pay + off + (f == F_CSR || f == F_CSR2 ? 8u * nz : 0u) - 8u * (uint32_t)i;
             e.y = (d.y & 0x1Fu) | (t << 7) | (nz << 11) | (d.y & 0x80000000u);
             if (f == F_CSR) {
                 const uint8_t *rp = payload + (size_t)T.tileOff[it.tb + t] * 16 + 8u * nz;
@@ -408,8 +456,8 @@ __global__ void k_blob_fill(Item *items, int64_t nitems, int64_t m, int64_t n, c
                 }
             } else if (f == F_ELL) {
                 tm = d.y & 0x1Fu;
-            } else if (f == F_COO) {
-                tm = nz;  // <= 11
+            } else if (f == F_CSR2) {
+                tm = 3;  // merged rows hold <= 3 entries (csr2_mergeable)
             }
         }
         const uint32_t tmo = __shfl_xor_sync(0xFFFFFFFFu, tm, 1);
@@ -438,6 +486,39 @@ __global__ void k_blob_fill(Item *items, int64_t nitems, int64_t m, int64_t n, c
         const uint4 *ps = reinterpret_cast<const uint4 *>(payload + (size_t)it.offb * 16);
         uint4 *pd = reinterpret_cast<uint4 *>(dst + b.pay);
         for (uint32_t i = lane; i < it.offe - it.offb; i += 32) pd[i] = ps[i];
+        __syncwarp();
+        // CSR2 pairs re-encoded over their two tiles' bytes (lane r: row r)
+        int8_t ef[kItemTiles];
+        exec_formats(it, T, ef);
+        for (int t = 0; t < nt; ++t) {
+            if (ef[t] != F_CSR2) continue;
+            const int g = it.tb + t;
+            const int na = T.tileNnz[g + 1] - T.tileNnz[g], nb = T.tileNnz[g + 2] - T.tileNnz[g + 1], nz = na + nb;
+            const uint8_t *sa = payload + (size_t)T.tileOff[g] * 16, *sb = payload + (size_t)T.tileOff[g + 1] * 16;
+            const uint8_t *ra = sa + 8 * na, *rb = sb + 8 * nb;
+            uint8_t *o = dst + b.pay + (T.tileOff[g] - it.offb) * 16u;
+            const uint32_t span = (T.tileOff[g + 2] - T.tileOff[g]) * 16u;
+            __syncwarp();
+            for (uint32_t i = lane; i < span; i += 32) o[i] = 0;
+            __syncwarp();
+            if (lane < 16) {
+                const int r = lane;
+                const int ba = ra[r], ea = r < 15 ? ra[r + 1] : na, bb = rb[r], eb = r < 15 ? rb[r + 1] : nb;
+                const int mp = ba + bb;  // merged row start
+                o[8 * nz + r] = (uint8_t)mp;
+                double *ov = reinterpret_cast<double *>(o);
+                uint8_t *oc = o + 8 * nz + 16;
+                int q = mp;
+                for (int k = ba; k < ea; ++k, ++q) {
+                    ov[q] = reinterpret_cast<const double *>(sa)[k];
+                    oc[q] = (uint8_t)((sa[8 * na + 16 + (k >> 1)] >> (4 * (k & 1))) & 15);
+                }
+                for (int k = bb; k < eb; ++k, ++q) {
+                    ov[q] = reinterpret_cast<const double *>(sb)[k];
+                    oc[q] = (uint8_t)(16 + ((sb[8 * nb + 16 + (k >> 1)] >> (4 * (k & 1))) & 15));
+                }
+            }
+        }
     } else {  // tile by tile: COO tiles left out, HYB(w) tiles as their ELL(w) part
         uint32_t o = b.pay;
         for (int t = 0; t < nt; ++t) {
@@ -658,7 +739,7 @@ __global__ void k_unit_bounds(const int32_t *ustart, const int32_t *uidx, int64_
 TileView tile_view(const Matrix &M) {
     return {M.tilePtr, M.tileOff, M.tileFmt, M.tileAux, M.tileNnz, M.tileColIdx,
             M.mode == TILESPMV_MODE_ADPT || M.mode == TILESPMV_MODE_BYTES ? 1 : 0,
-            M.mode == TILESPMV_MODE_DEFERRED ? 1 : 0};
+            M.mode == TILESPMV_MODE_DEFERRED ? 1 : 0, M.payload};
 }
 
 // stream-ordered temporary device buffer

@@ -328,6 +328,25 @@ __device__ __forceinline__ void half_coo_scan(uint32_t V, uint32_t rc, int n, ui
     if ((rows >> (16 * h + r)) & 1u) acc += lds_f64(Sh + 8 * r);
 }
 
+// CSR2 (schedule.cu: two CSR tiles at adjacent tile columns merged, every
+// merged row <= 3 entries): like CSR, but one column byte per entry (0..31)
+// indexing the two x segments staged side by side from X
+__device__ __forceinline__ void half_csr2_n3(uint32_t RP, int nz, uint32_t X, int r, bool ok, double &acc) {
+    const int beg = (int)lds_u8(RP + r);
+    const int end = r < 15 ? (int)lds_u8(RP + r + 1) : nz;
+    const int len = ok ? end - beg : 0;
+    const uint32_t ca = RP + 16 + beg, wa = ca & ~3u;
+    const uint32_t u = funnel_r(lds_u32(wa), lds_u32(wa + 4), 8u * (ca & 3u));
+    const uint32_t V = RP + 8 * (beg - nz);
+    // byte j of u times 8: the entry's x offset from X (<= 248)
+    const double x0 = lds_f64(X + ((u << 3) & 0xF8u)), x1 = lds_f64(X + ((u >> 5) & 0xF8u)),
+                 x2 = lds_f64(X + ((u >> 13) & 0xF8u));
+    const double v0 = lds_f64_lt(0, len, V), v1 = lds_f64_lt(1, len, V + 8), v2 = lds_f64_lt(2, len, V + 16);
+    acc = fma(v0, x0, acc);
+    acc = fma(v1, x1, acc);
+    acc = fma(v2, x2, acc);
+}
+
 // ------------------------------------------ split routines (odd groups) ----
 // A format group with an odd number of tiles ends in a pair whose second
 // tile is a masked copy of the first.  That last tile then runs on BOTH

@@ -379,10 +379,7 @@ __device__ __forceinline__ void run_group(int np, uint32_t &d, uint32_t xs, int 
         if (F == F_DNS) half_dns(P, X, r, ok, acc);
         if (F == F_DNSCOL) half_dnscol(P, aux, X, r, ok, acc);
         if (F == F_DNSROW) half_dnsrow_tree(P, aux, X, r, ok, acc);
-        if (F == F_COO) {  // tiny tiles (power-law, stencil corners): walk; else scan
-            if (tm <= 2) half_coo_n<2>(P, P + 8 * nz, nz, X, r, ok, acc);
-            else half_coo_scan(P, P + 8 * nz, nz, X, r, lane_h, racc, ok, acc);
-        }
+        if (F == F_CSR2) half_csr2_n3(P, nz, X, r, ok, acc);  // merged CSR pairs (schedule.cu)
         if (F == F_HYB) half_hyb_scan(P, aux, nz, X, r, lane_h, racc, ok, acc);
     }
 }
@@ -477,7 +474,7 @@ __device__ __forceinline__ bool compute_item(const Params &p, const WItem &it, u
         // those groups without per-pair dispatch
         if ((g >> 28) & 1u) run_group<F_CSR, 3>((int)(g & 15u), d, xs, r, acc);
         else run_group<F_CSR>((int)(g & 15u), d, xs, r, acc);
-        if (g & 0xF0u) run_group<F_COO>((int)((g >> 4) & 15u), d, xs, r, acc, racc);
+        if (g & 0xF0u) run_group<F_CSR2>((int)((g >> 4) & 15u), d, xs, r, acc);
         if ((g >> 29) & 1u) run_group<F_ELL, 3>((int)((g >> 8) & 15u), d, xs, r, acc);
         else run_group<F_ELL>((int)((g >> 8) & 15u), d, xs, r, acc);
         if (g & 0x0FFFF000u) {  // one test skips the four rarer formats
