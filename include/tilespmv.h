@@ -115,7 +115,7 @@ typedef struct {
     double create_ms;                   /* wall time of tilespmv_create_from_csr */
     int32_t kernel;                     /* resolved TILESPMV_KERNEL_* (never AUTO) */
     int32_t xcache_cols;                /* GATHER kernel: remainder columns held in its shared-memory
-                                           x cache (the most-gathered ones, <= 1024); 0 otherwise */
+                                           x cache (the most-gathered ones, <= 2048); 0 otherwise */
 } tilespmv_info_t;
 
 /* Build a tiled matrix from a canonical device CSR ("converting a basic

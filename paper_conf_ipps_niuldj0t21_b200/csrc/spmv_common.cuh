@@ -202,9 +202,10 @@ struct KernelChoice {
     int xcache;       // slots of the shared-memory x cache (0: none)
 };
 // GATHER kernel: x cache slots (8 B each) and slot bytes, sized so the
-// kernel's 130 KB of shared memory stays in the 132 KB carve-out step
-// (R-MAT: 1,024 / 3,136 B 88.4 us; 4,096 / 3,328 B, 164 KB step, 93.0 us)
-constexpr int kXCache = 1024;
+// kernel's 131 KB of shared memory stays in the 132 KB carve-out step
+// (R-MAT: 1,024 / 3,136 B 88.4 us; 4,096 / 3,328 B, 164 KB step, 93.0 us;
+// 2,048 / 3,136 B once the COO-scan scratch went: 83.5 us)
+constexpr int kXCache = 2048;
 constexpr int kGatherSlot = 3136;
 // TILESPMV_KERNEL_SM_QUEUE, _DENSE_ROWS or _GATHER
 KernelChoice kernel_choice(int kernel);

@@ -169,19 +169,6 @@ __device__ __forceinline__ void half_dnsrow_tree(uint32_t P, int nr, uint32_t X,
     }
 }
 
-// COO with at most N entries per tile of the pair (tm <= N): every lane of
-// the half walks the entries, the lane of the entry's row adds it
-template <int N>
-__device__ __forceinline__ void half_coo_n(uint32_t V, uint32_t rc, int n, uint32_t X, int r, bool ok, double &acc) {
-    const int nq = ok ? n : 0;
-#pragma unroll
-    for (int j = 0; j < N; ++j) {
-        const uint32_t b = lds_u8(rc + j);
-        const double v = lds_f64_lt(j, (int)(b >> 4) == r ? nq : 0, V + 8 * j);
-        acc = fma(v, lds_f64(X + 8 * (b & 15u)), acc);
-    }
-}
-
 // ------------------------------- routines with the pair's extent known -----
 // The schedule stores in every descriptor the longest row (CSR) or width
 // (ELL) of the two tiles of its half-warp pair (bits 20-24), so the trip count
@@ -283,51 +270,6 @@ __device__ __forceinline__ void half_ell_n(uint32_t P, int w, uint32_t X, int r,
     ell_steps<N>(P + 8 * r, P + 128 * w + (r >> 1), (r & 1) ? 31u : 3u, X, 0, ok ? w : 0, acc);
 }
 
-// COO (n <= 11 by the selection rule; Alg. 3) with one lane
-// per entry: lane j of the half multiplies entry j; an inclusive segmented
-// scan over the half (entries are row-major, so a row's entries are adjacent
-// lanes) leaves each row's sum on the row's last entry, which stores it in
-// the warp's row scratch S (16 doubles per half) for the row's lane.
-// base: first entry of this pass (HYB's COO part may hold more than 16
-// entries and runs in passes of 16; a row that straddles two passes gets two
-// partial sums, added in pass order)
-__device__ __forceinline__ void half_coo_scan(uint32_t V, uint32_t rc, int n, uint32_t X, int r, int h, uint32_t S,
-                                              bool ok, double &acc, int base = 0) {
-    const int nq = ok ? n : 0;
-    const bool have = base + r < nq;
-    uint32_t b = 0;
-    double p = 0.0;
-    if (have) {
-        b = lds_u8(rc + base + r);
-        p = lds_f64(V + 8 * (base + r)) * lds_f64(X + 8 * (b & 15u));
-    }
-    const int row = have ? (int)(b >> 4) : 16 + r;  // idle lanes: a row of their own
-    {  // (every lane executes every shuffle: no shuffle inside a short-circuit)
-        const double pp = __shfl_up_sync(FULL, p, 1, 16);
-        const int r1 = __shfl_up_sync(FULL, row, 1, 16);
-        if (r >= 1 && r1 == row) p += pp;
-    }
-    // rows of three or more entries are rare in a COO tile (n <= 11): the
-    // longer steps run only when some row needs them
-    const int r2 = __shfl_up_sync(FULL, row, 2, 16);
-    if (__any_sync(FULL, r >= 2 && r2 == row)) {
-#pragma unroll
-        for (int off = 2; off < 16; off <<= 1) {
-            const double pp = __shfl_up_sync(FULL, p, off, 16);
-            const int rr = __shfl_up_sync(FULL, row, off, 16);
-            if (r >= off && rr == row) p += pp;
-        }
-    }
-    const int rnext = __shfl_down_sync(FULL, row, 1, 16);
-    const bool tail = have && (base + r == nq - 1 || r == 15 || rnext != row);
-    const uint32_t rows = __reduce_or_sync(FULL, tail ? 1u << (16 * h + row) : 0u);
-    const uint32_t Sh = S + 128 * h;
-    __syncwarp();  // the previous pair's reads of S are done
-    if (tail) sts_f64(Sh + 8 * row, p);
-    __syncwarp();
-    if ((rows >> (16 * h + r)) & 1u) acc += lds_f64(Sh + 8 * r);
-}
-
 // CSR2 (schedule.cu: two CSR tiles at adjacent tile columns merged, every
 // merged row <= 3 entries): like CSR, but one column byte per entry (0..31)
 // indexing the two x segments staged side by side from X
@@ -426,25 +368,6 @@ __device__ __forceinline__ void split_dnsrow(uint32_t P, int nr, uint32_t X, int
         s += __shfl_xor_sync(FULL, s, 1);
         if (q < nr && (int)lds_u8(rid + q) == r) acc += s;
     }
-}
-
-// HYB in the TM kernels: the ELL part as ELL, the COO part with the
-// lane-per-entry scan in passes of 16 entries
-__device__ __forceinline__ void half_hyb_scan(uint32_t P, int w, int nz, uint32_t X, int r, int h, uint32_t S, bool ok,
-                                              double &acc) {
-    const int kc = nz - 16 * w;
-    const uint32_t ei = P + 128 * w + 8 * kc;
-    const int wq = ok ? w : 0;
-    const int trips = (int)__reduce_max_sync(FULL, (unsigned)wq);
-    const uint32_t sh = 4 * (r & 1);
-    for (int k = 0; k < trips; ++k) {
-        const double v = lds_f64_lt(k, wq, P + 8 * (16 * k + r));
-        const double xv = lds_f64(X + 8 * ((lds_u8(ei + 8 * k + (r >> 1)) >> sh) & 15u));
-        acc = fma(v, xv, acc);
-    }
-    const int passes = (int)__reduce_max_sync(FULL, (unsigned)(ok ? (kc + 15) >> 4 : 0));
-#pragma unroll 1
-    for (int c = 0; c < passes; ++c) half_coo_scan(P + 128 * w, ei + 8 * w, kc, X, r, h, S, ok, acc, 16 * c);
 }
 
 }  // namespace tsp

@@ -69,10 +69,9 @@ template <int WARPS, int SLOT, int XT = kItemTiles, int XC = 0>
 struct WarpCfg {
     static_assert(SLOT % 16 == 0 && SLOT <= kItemBytesMax && XT % 4 == 0 && XT <= kItemTiles, "slot size");
     // [x stage of every warp, XT x 128 B, 128-byte aligned] [per warp: slot |
-    // row-sum scratch of the COO scan (256 B) | mbarrier] [x cache: XC x 8 B]
+    // mbarrier] [x cache: XC x 8 B]
     static constexpr uint32_t kX = XT * 16 * 8;
-    static constexpr uint32_t kRacc = 256;
-    static constexpr uint32_t kPer = SLOT + kRacc + 16;
+    static constexpr uint32_t kPer = SLOT + 16;
     static constexpr uint32_t kXc = WARPS * (kX + kPer);  // x cache offset
     static constexpr uint32_t kSmem = kXc + XC * 8 + 256;  // +256: loads may overrun a slot
     static constexpr int kThreads = 32 * WARPS;
@@ -348,7 +347,7 @@ __device__ __forceinline__ void coo_run(uint32_t rpS, uint32_t xslS, uint32_t va
 // invalid << 31 (tm: the pair's longest CSR row / larger ELL width / larger
 // COO entry count).  N = 3: every CSR row / ELL width of the item is <= 3.
 template <int F, int N = 0>
-__device__ __forceinline__ void run_group(int np, uint32_t &d, uint32_t xs, int r, double &acc, uint32_t racc = 0) {
+__device__ __forceinline__ void run_group(int np, uint32_t &d, uint32_t xs, int r, double &acc) {
     const int lane_h = (int)(threadIdx.x >> 4) & 1;
     // (not the N = 3 CSR / ELL paths: a masked pair's straight-line steps
     // beat the split loop there, C5 +3.5%)
@@ -380,7 +379,6 @@ __device__ __forceinline__ void run_group(int np, uint32_t &d, uint32_t xs, int 
         if (F == F_DNSCOL) half_dnscol(P, aux, X, r, ok, acc);
         if (F == F_DNSROW) half_dnsrow_tree(P, aux, X, r, ok, acc);
         if (F == F_CSR2) half_csr2_n3(P, nz, X, r, ok, acc);  // merged CSR pairs (schedule.cu)
-        if (F == F_HYB) half_hyb_scan(P, aux, nz, X, r, lane_h, racc, ok, acc);
     }
 }
 
@@ -448,7 +446,7 @@ __device__ __forceinline__ void issue_x(const Params &p, int J, int nt, uint32_t
 // proxy writes before the next TMA copy into the slot.
 template <bool PRE>
 __device__ __forceinline__ bool compute_item(const Params &p, const WItem &it, uint32_t slot, uint32_t xs,
-                                             uint32_t racc, uint64_t x_policy, uint32_t xcS, int lane, double &carry) {
+                                             uint64_t x_policy, uint32_t xcS, int lane, double &carry) {
     if (it.jt_rows_pay & 0xFFu)  // row-group item (no tiles, no x segments)
         return group_item<PRE>(p, it, slot, x_policy, xcS, lane);
     const int h = lane >> 4, r = lane & 15;
@@ -477,8 +475,10 @@ __device__ __forceinline__ bool compute_item(const Params &p, const WItem &it, u
         if (g & 0xF0u) run_group<F_CSR2>((int)((g >> 4) & 15u), d, xs, r, acc);
         if ((g >> 29) & 1u) run_group<F_ELL, 3>((int)((g >> 8) & 15u), d, xs, r, acc);
         else run_group<F_ELL>((int)((g >> 8) & 15u), d, xs, r, acc);
-        if (g & 0x0FFFF000u) {  // one test skips the four rarer formats
-            run_group<F_HYB>((int)((g >> 12) & 15u), d, xs, r, acc, racc);
+        // HYB descriptors never occur: a HYB tile is ELL(w) + COO run (ADPT,
+        // BYTES) or ELL(w) + remainder (DEFERRED, reading R17)
+        TSP_CHECK(((g >> 12) & 15u) == 0);
+        if (g & 0x0FFF0000u) {  // one test skips the three rarer formats
             run_group<F_DNS>((int)((g >> 16) & 15u), d, xs, r, acc);
             run_group<F_DNSROW>((int)((g >> 20) & 15u), d, xs, r, acc);
             run_group<F_DNSCOL>((int)((g >> 24) & 15u), d, xs, r, acc);
@@ -540,7 +540,7 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, MINB) tilespmv
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const uint32_t xs = smem_u32(smem) + (uint32_t)warp * Cfg::kX;
     const uint32_t slot = smem_u32(smem) + WARPS * Cfg::kX + (uint32_t)warp * Cfg::kPer;
-    const uint32_t racc = slot + SLOT, bar = racc + Cfg::kRacc;
+    const uint32_t bar = slot + SLOT;
     if (lane == 0) {
         mbar_init(bar, 1);
         fence_mbar_init();
@@ -578,7 +578,7 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, MINB) tilespmv
         }
         TSP_STAMP(gw, k - kbeg, 1);
         TSP_INFO(gw, k - kbeg, k, it);
-        if (compute_item<false>(p, it, slot, xs, racc, x_policy, 0u, lane, carry))
+        if (compute_item<false>(p, it, slot, xs, x_policy, 0u, lane, carry))
             fence_proxy_async();  // products written to the slot before the next TMA copy into it
         __syncwarp();  // slot and x scratch free for the next item
         TSP_STAMP(gw, k - kbeg, 3);
@@ -608,7 +608,7 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT, XT, XC>::kThreads, 1) til
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const uint32_t xs = smem_u32(smem) + (uint32_t)warp * Cfg::kX;
     const uint32_t slot = smem_u32(smem) + WARPS * Cfg::kX + (uint32_t)warp * Cfg::kPer;
-    const uint32_t racc = slot + SLOT, bar = racc + Cfg::kRacc;
+    const uint32_t bar = slot + SLOT;
     const uint32_t xc_bar = smem_u32(&s_xc_bar);
     const int ub = (int)__ldg(p.cta_begin + blockIdx.x), ue = (int)__ldg(p.cta_begin + blockIdx.x + 1);
     if (lane == 0) {
@@ -694,7 +694,7 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT, XT, XC>::kThreads, 1) til
         }
         TSP_STAMP(gw, j, 1);
         TSP_INFO(gw, j, k, it);
-        if (compute_item<PRE>(p, it, slot, xs, racc, x_policy, xcS, lane, carry))
+        if (compute_item<PRE>(p, it, slot, xs, x_policy, xcS, lane, carry))
             fence_proxy_async();  // products written to the slot before the next TMA copy into it
         __syncwarp();  // slot and x scratch free for the next item
         TSP_STAMP(gw, j, 3);
@@ -717,7 +717,7 @@ KernelChoice kernel_choice(int kernel) {
     }
     if (kernel == TILESPMV_KERNEL_GATHER) {
         using Cfg = WarpCfg<32, kGatherSlot, 4, kXCache>;
-        return {"tilespmv_fp64_sm<32,3136,4,1024>", tilespmv_fp64_sm<32, kGatherSlot, 4, kXCache>, Cfg::kThreads,
+        return {"tilespmv_fp64_sm<32,3136,4,2048>", tilespmv_fp64_sm<32, kGatherSlot, 4, kXCache>, Cfg::kThreads,
                 (int)Cfg::kSmem, kGatherSlot, 4, true, kXCache};
     }
     using Cfg = WarpCfg<32, 4608>;

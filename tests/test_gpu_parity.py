@@ -378,7 +378,7 @@ def test_row_slices_bitwise_equal_full(cuda_device, name, mode, kernel):
 def test_gather_xcache(cuda_device, name):
     """GATHER's shared-memory x cache holds the most-gathered remainder
     columns: as many as there are columns gathered at least twice, at most
-    1024 (xcache_cols); the other kernels have none.  x is NaN on every
+    2048 (xcache_cols); the other kernels have none.  x is NaN on every
     16-column segment that no matrix entry references (tile kernels multiply
     whole segments), so a cache slot filled from a column outside the
     matrix's segments would poison y."""
@@ -396,8 +396,8 @@ def test_gather_xcache(cuda_device, name):
     with TM.from_host_csr(A, mode="DEFERRED", device=cuda_device, kernel="GATHER", keep_layout=True) as M:
         rem = M.export("remCol")
         cnt = np.bincount(rem, minlength=A.n)
-        assert M.info()["xcache_cols"] == min(1024, int((cnt >= 2).sum()))
-        assert name != "rmat12" or M.info()["xcache_cols"] == 1024
+        assert M.info()["xcache_cols"] == min(2048, int((cnt >= 2).sum()))
+        assert name != "rmat12" or M.info()["xcache_cols"] >= 1024
         y = M.run(torch.from_numpy(xp).to(cuda_device)).cpu().numpy()
         assert_spmv_close(y, yref, absy, f"{name}/GATHER x cache")
     with TM.from_host_csr(A, mode="DEFERRED", device=cuda_device, kernel="SM_QUEUE") as M:
