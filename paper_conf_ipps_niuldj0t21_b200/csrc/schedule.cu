@@ -242,11 +242,11 @@ __device__ __forceinline__ int dsc_format(const TileView &T, int g) {
 // does its row's 3 entries once instead of two half-empty tiles.  Encoding:
 // val[nz] row-major (row r: tile J's entries, then tile J + 1's), rowptr[16]
 // u8, one column byte per entry (0..31); never larger than the two tiles'
-// canonical payloads (checked), written over them in the blob.  Only without
-// a COO run; descriptor format code F_CSR2 = 1 (COO tiles never get
-// descriptors: DEFERRED extracts them, ADPT/BYTES move them into the run).
+// canonical payloads (checked), written where they would be in the blob.
+// Descriptor format code F_CSR2 = 1 (COO tiles never get descriptors:
+// DEFERRED extracts them, ADPT/BYTES move them into the run).
 __device__ __forceinline__ bool csr2_mergeable(const TileView &T, int g) {
-    if (T.run || T.tileFmt[g] != F_CSR || T.tileFmt[g + 1] != F_CSR) return false;
+    if (T.tileFmt[g] != F_CSR || T.tileFmt[g + 1] != F_CSR) return false;
     if (T.tileColIdx[g + 1] != T.tileColIdx[g] + 1) return false;
     const int na = T.tileNnz[g + 1] - T.tileNnz[g], nb = T.tileNnz[g + 2] - T.tileNnz[g + 1];
     if (up16(9u * (uint32_t)(na + nb) + 16u) > (T.tileOff[g + 2] - T.tileOff[g]) * 16u) return false;
@@ -257,6 +257,36 @@ __device__ __forceinline__ bool csr2_mergeable(const TileView &T, int g) {
         if (la + lb > 3) return false;
     }
     return true;
+}
+
+// the CSR2 encoding of tiles g, g + 1 at o (span: their canonical bytes,
+// zeroed first); lane r < 16 writes row r
+__device__ __forceinline__ void write_csr2(const TileView &T, int g, uint8_t *o, int lane) {
+    const int na = T.tileNnz[g + 1] - T.tileNnz[g], nb = T.tileNnz[g + 2] - T.tileNnz[g + 1], nz = na + nb;
+    const uint8_t *sa = T.payload + (size_t)T.tileOff[g] * 16, *sb = T.payload + (size_t)T.tileOff[g + 1] * 16;
+    const uint8_t *ra = sa + 8 * na, *rb = sb + 8 * nb;
+    const uint32_t span = (T.tileOff[g + 2] - T.tileOff[g]) * 16u;
+    __syncwarp();
+    for (uint32_t i = lane; i < span; i += 32) o[i] = 0;
+    __syncwarp();
+    if (lane < 16) {
+        const int r = lane;
+        const int ba = ra[r], ea = r < 15 ? ra[r + 1] : na, bb = rb[r], eb = r < 15 ? rb[r + 1] : nb;
+        const int mp = ba + bb;  // merged row start
+        o[8 * nz + r] = (uint8_t)mp;
+        double *ov = reinterpret_cast<double *>(o);
+        uint8_t *oc = o + 8 * nz + 16;
+        int q = mp;
+        for (int k = ba; k < ea; ++k, ++q) {
+            ov[q] = reinterpret_cast<const double *>(sa)[k];
+            oc[q] = (uint8_t)((sa[8 * na + 16 + (k >> 1)] >> (4 * (k & 1))) & 15);
+        }
+        for (int k = bb; k < eb; ++k, ++q) {
+            ov[q] = reinterpret_cast<const double *>(sb)[k];
+            oc[q] = (uint8_t)(16 + ((sb[8 * nb + 16 + (k >> 1)] >> (4 * (k & 1))) & 15));
+        }
+    }
+    __syncwarp();
 }
 
 // execution format of every tile of the item (pairs merged greedily left to
@@ -490,42 +520,25 @@ __global__ void k_blob_fill(Item *items, int64_t nitems, int64_t m, int64_t n, c
         // CSR2 pairs re-encoded over their two tiles' bytes (lane r: row r)
         int8_t ef[kItemTiles];
         exec_formats(it, T, ef);
-        for (int t = 0; t < nt; ++t) {
-            if (ef[t] != F_CSR2) continue;
-            const int g = it.tb + t;
-            const int na = T.tileNnz[g + 1] - T.tileNnz[g], nb = T.tileNnz[g + 2] - T.tileNnz[g + 1], nz = na + nb;
-            const uint8_t *sa = payload + (size_t)T.tileOff[g] * 16, *sb = payload + (size_t)T.tileOff[g + 1] * 16;
-            const uint8_t *ra = sa + 8 * na, *rb = sb + 8 * nb;
-            uint8_t *o = dst + b.pay + (T.tileOff[g] - it.offb) * 16u;
-            const uint32_t span = (T.tileOff[g + 2] - T.tileOff[g]) * 16u;
-            __syncwarp();
-            for (uint32_t i = lane; i < span; i += 32) o[i] = 0;
-            __syncwarp();
-            if (lane < 16) {
-                const int r = lane;
-                const int ba = ra[r], ea = r < 15 ? ra[r + 1] : na, bb = rb[r], eb = r < 15 ? rb[r + 1] : nb;
-                const int mp = ba + bb;  // merged row start
-                o[8 * nz + r] = (uint8_t)mp;
-                double *ov = reinterpret_cast<double *>(o);
-                uint8_t *oc = o + 8 * nz + 16;
-                int q = mp;
-                for (int k = ba; k < ea; ++k, ++q) {
-                    ov[q] = reinterpret_cast<const double *>(sa)[k];
-                    oc[q] = (uint8_t)((sa[8 * na + 16 + (k >> 1)] >> (4 * (k & 1))) & 15);
-                }
-                for (int k = bb; k < eb; ++k, ++q) {
-                    ov[q] = reinterpret_cast<const double *>(sb)[k];
-                    oc[q] = (uint8_t)(16 + ((sb[8 * nb + 16 + (k >> 1)] >> (4 * (k & 1))) & 15));
-                }
-            }
-        }
-    } else {  // tile by tile: COO tiles left out, HYB(w) tiles as their ELL(w) part
+        for (int t = 0; t < nt; ++t)
+            if (ef[t] == F_CSR2) write_csr2(T, it.tb + t, dst + b.pay + (T.tileOff[it.tb + t] - it.offb) * 16u, lane);
+    } else {  // tile by tile: COO tiles left out, HYB(w) tiles as their ELL(w) part, CSR2 pairs merged
         uint32_t o = b.pay;
+        int8_t ef[kItemTiles];
+        exec_formats(it, T, ef);
         for (int t = 0; t < nt; ++t) {
             const int g = it.tb + t;
             uint32_t pt, rt;
             tile_cost(T, g, pt, rt);
             const uint8_t *src = payload + (size_t)T.tileOff[g] * 16;
+            if (ef[t] == F_CSR2) {
+                uint32_t pt1, rt1;
+                tile_cost(T, g + 1, pt1, rt1);
+                write_csr2(T, g, dst + o, lane);
+                o += pt + pt1;
+                ++t;
+                continue;
+            }
             if (T.tileFmt[g] == F_HYB) {
                 const uint32_t w = T.tileAux[g], kc = rt;
                 const uint2 *vs = reinterpret_cast<const uint2 *>(src);  // ELL values, 16 w
