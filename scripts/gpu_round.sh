@@ -28,4 +28,6 @@ TILESPMV_BENCH_ONE_GPU=1 timeout 900 python -m torch.distributed.run --nnodes=1 
    --e2e-steps 2 > $OUT/n2_devcheck.json 2> $OUT/n2_devcheck.err; echo "rc=$?" >> $OUT/n2_devcheck.err
 timeout 300 python bench.py --impl reference --steps 20 --warmup 5 > $OUT/reference.json 2> $OUT/reference.err
 timeout 800 python scripts/checked_small.py > $OUT/checked_small.log 2>&1; echo "rc=$?" >> $OUT/checked_small.log
+timeout 1200 python scripts/paper_ablation.py > $OUT/ablation.jsonl 2> $OUT/ablation.err
+timeout 600 python scripts/cg_bench.py > $OUT/cg_stencil27_200.json 2> $OUT/cg.err
 echo done > $OUT/DONE
