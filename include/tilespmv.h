@@ -59,8 +59,9 @@ extern "C" {
                                         6 KiB (dense, FEM-like tile rows), else SM_QUEUE          */
 #define TILESPMV_KERNEL_SM_QUEUE 1   /* one 32-warp CTA per SM, 4.5 KiB items, shared-memory queue */
 #define TILESPMV_KERNEL_DENSE_ROWS 2 /* 16 warps per SM, 10.5 KiB items, static per-warp chunks    */
-#define TILESPMV_KERNEL_GATHER 3     /* SM_QUEUE with 3.25 KiB items of at most 4 tiles: 132 KiB of
-                                        shared memory per SM instead of 222 KiB leaves ~125 KiB of
+#define TILESPMV_KERNEL_GATHER 3     /* SM_QUEUE with ~3 KiB items of at most 4 tiles and a 16 KiB
+                                        x cache of the most-gathered remainder columns: 131 KiB of
+                                        shared memory per SM instead of 209 KiB leaves ~124 KiB of
                                         L1 to the remainder's x gathers                            */
 
 /* tile format codes, in the order of P:20 / P:96 */
