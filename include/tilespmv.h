@@ -146,6 +146,27 @@ int tilespmv_create_from_csr(tilespmv_handle_t *out, int64_t m, int64_t n, int64
  * must be serialised (the handle owns one split-row workspace).             */
 int tilespmv_run(tilespmv_handle_t h, const double *d_x, double *d_y, void *stream);
 
+/* tilespmv_run with a fused scatter epilogue (SURVEY §8(e), B200-native
+ * improvement 2): every row of y is stored to d_y AND to each of the n_peer
+ * device pointers d_peer_ys[t] (double[m] each; typically the peers' copies of
+ * the next iterate at this rank's row offset, mapped with tilespmv_ipc_open
+ * so the stores travel over NVLink), so tile-row sharded iterated SpMV needs
+ * no separate all-gather.  n_peer in 0..7 (0 = tilespmv_run).  Completion is
+ * the kernel's: the caller synchronises with the peers (e.g. a barrier after
+ * the stream) before they read.  Errors as tilespmv_run, plus INVALID_ARG for
+ * n_peer out of range or a NULL peer pointer.                                */
+int tilespmv_run_scatter(tilespmv_handle_t h, const double *d_x, double *d_y, double *const *d_peer_ys,
+                         int32_t n_peer, void *stream);
+
+/* CUDA IPC plumbing for tilespmv_run_scatter's peers (handles are 64 bytes).
+ * ipc_alloc: cudaMalloc(bytes) into *d_ptr and its IPC handle into handle[64];
+ * ipc_open: map a peer's handle (cudaIpcOpenMemHandle, lazy peer access);
+ * ipc_close / ipc_free undo them.  Errors: INVALID_ARG, CUDA.                 */
+int tilespmv_ipc_alloc(int64_t bytes, void **d_ptr, void *handle);
+int tilespmv_ipc_free(void *d_ptr);
+int tilespmv_ipc_open(const void *handle, void **d_ptr);
+int tilespmv_ipc_close(void *d_ptr);
+
 /* Host-buffer variant: copies h_x (double[n]) to a handle-owned device
  * buffer, runs, copies y back to h_y (double[m]) and synchronises `stream`.
  * h_x / h_y should be page-locked for asynchronous copies.                  */

@@ -159,6 +159,62 @@ int tilespmv_run(tilespmv_handle_t h, const double *d_x, double *d_y, void *stre
     return launch_spmv(*h, d_x, d_y, static_cast<cudaStream_t>(stream));
 }
 
+int tilespmv_run_scatter(tilespmv_handle_t h, const double *d_x, double *d_y, double *const *d_peer_ys,
+                         int32_t n_peer, void *stream) {
+    if (n_peer < 0 || n_peer > kMaxScatter) return set_error(TILESPMV_INVALID_ARG, "n_peer must be 0..7");
+    if (n_peer > 0 && !d_peer_ys) return set_error(TILESPMV_INVALID_ARG, "d_peer_ys is NULL");
+    double *ys[kMaxScatter] = {nullptr};
+    for (int t = 0; t < n_peer; ++t) {
+        if (h && h->m > 0 && !d_peer_ys[t]) return set_error(TILESPMV_INVALID_ARG, "a peer y is NULL");
+        ys[t] = d_peer_ys[t];
+    }
+    if (int rc = check_handle(h)) return rc;
+    if (h->m > 0 && !d_y) return set_error(TILESPMV_INVALID_ARG, "y is NULL");
+    if (h->n > 0 && !d_x) return set_error(TILESPMV_INVALID_ARG, "x is NULL");
+    if (h->m > 0 && h->n > 0) {
+        const char *xa = reinterpret_cast<const char *>(d_x), *ya = reinterpret_cast<const char *>(d_y);
+        if (xa < ya + 8 * h->m && ya < xa + 8 * h->n) return set_error(TILESPMV_INVALID_ARG, "x and y overlap");
+    }
+    return launch_spmv(*h, d_x, d_y, static_cast<cudaStream_t>(stream), ys, n_peer);
+}
+
+int tilespmv_ipc_alloc(int64_t bytes, void **d_ptr, void *handle) {
+    if (!d_ptr || !handle || bytes <= 0) return set_error(TILESPMV_INVALID_ARG, "bad ipc_alloc arguments");
+    *d_ptr = nullptr;
+    void *p = nullptr;
+    if (cudaMalloc(&p, (size_t)bytes) != cudaSuccess) return cuda_status(cudaGetLastError(), "cudaMalloc(ipc buffer)");
+    cudaIpcMemHandle_t hd;
+    cudaError_t e = cudaIpcGetMemHandle(&hd, p);
+    if (e != cudaSuccess) {
+        cudaFree(p);
+        return cuda_status(e, "cudaIpcGetMemHandle");
+    }
+    std::memcpy(handle, &hd, sizeof(hd));
+    *d_ptr = p;
+    return TILESPMV_OK;
+}
+
+int tilespmv_ipc_free(void *d_ptr) {
+    if (d_ptr && cudaFree(d_ptr) != cudaSuccess) return cuda_status(cudaGetLastError(), "cudaFree(ipc buffer)");
+    return TILESPMV_OK;
+}
+
+int tilespmv_ipc_open(const void *handle, void **d_ptr) {
+    if (!handle || !d_ptr) return set_error(TILESPMV_INVALID_ARG, "bad ipc_open arguments");
+    *d_ptr = nullptr;
+    cudaIpcMemHandle_t hd;
+    std::memcpy(&hd, handle, sizeof(hd));
+    cudaError_t e = cudaIpcOpenMemHandle(d_ptr, hd, cudaIpcMemLazyEnablePeerAccess);
+    if (e != cudaSuccess) return cuda_status(e, "cudaIpcOpenMemHandle");
+    return TILESPMV_OK;
+}
+
+int tilespmv_ipc_close(void *d_ptr) {
+    if (d_ptr && cudaIpcCloseMemHandle(d_ptr) != cudaSuccess)
+        return cuda_status(cudaGetLastError(), "cudaIpcCloseMemHandle");
+    return TILESPMV_OK;
+}
+
 int tilespmv_run_host(tilespmv_handle_t h, const double *h_x, double *h_y, void *stream) {
     if (int rc = check_handle(h)) return rc;
     if ((h->m > 0 && !h_y) || (h->n > 0 && !h_x)) return set_error(TILESPMV_INVALID_ARG, "NULL host buffer");

@@ -12,6 +12,7 @@
 namespace tsp {
 
 constexpr int kTile = 16;  // P:20 "the size is always 16 by 16"
+constexpr int kMaxScatter = 7;  // tilespmv_run_scatter: peers (the other 7 GPUs of one node)
 
 // Format codes (same numbering as the ABI, P:96 order).
 enum : uint8_t { F_CSR = 0, F_COO = 1, F_ELL = 2, F_HYB = 3, F_DNS = 4, F_DNSROW = 5, F_DNSCOL = 6 };
@@ -186,7 +187,8 @@ int build_schedule(Matrix &M, cudaStream_t stream);
 int build_tdesc(Matrix &M, cudaStream_t stream);
 int configure_launch(Matrix &M, cudaStream_t stream);
 void release_create_time(Matrix &M, cudaStream_t stream);
-int launch_spmv(const Matrix &M, const double *d_x, double *d_y, cudaStream_t stream);
+int launch_spmv(const Matrix &M, const double *d_x, double *d_y, cudaStream_t stream, double *const *yx = nullptr,
+                int nyx = 0);
 // cg.cu
 int cg_solve(const Matrix &M, const double *d_b, double *d_x, double tol, int maxit, int *iters, double *relres,
              cudaStream_t stream);

@@ -1031,6 +1031,7 @@ static int configure_sm_queue(Matrix &M, int G, cudaStream_t st) {
 int configure_launch(Matrix &M, cudaStream_t st) {
     const KernelChoice kc = kernel_choice(M.kernel);
     TSP_CK(cudaFuncSetAttribute(kc.fn, cudaFuncAttributeMaxDynamicSharedMemorySize, kc.smem));
+    TSP_CK(cudaFuncSetAttribute(kc.fn_scatter, cudaFuncAttributeMaxDynamicSharedMemorySize, kc.smem));
     int sms = 0, per_sm = 0;
     TSP_CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, M.device));
     TSP_CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kc.fn, kc.threads, kc.smem));
@@ -1095,9 +1096,11 @@ void release_create_time(Matrix &M, cudaStream_t st) {
     drop(M.remVal);
 }
 
-int launch_spmv(const Matrix &M, const double *d_x, double *d_y, cudaStream_t st) {
+int launch_spmv(const Matrix &M, const double *d_x, double *d_y, cudaStream_t st, double *const *yx, int nyx) {
     if (M.m == 0) return 0;
     Params p;
+    p.nyx = nyx;
+    for (int t = 0; t < kMaxScatter; ++t) p.yx[t] = t < nyx ? yx[t] : nullptr;
     p.blob = M.blob;
     p.witems = M.witems;
     p.jcols = M.jcols;
@@ -1130,7 +1133,7 @@ int launch_spmv(const Matrix &M, const double *d_x, double *d_y, cudaStream_t st
     attr[0].val.programmaticStreamSerializationAllowed = 1;
     cfg.attrs = attr;
     cfg.numAttrs = 1;
-    TSP_CK(cudaLaunchKernelEx(&cfg, kc.fn, p));
+    TSP_CK(cudaLaunchKernelEx(&cfg, nyx > 0 ? kc.fn_scatter : kc.fn, p));
     return 0;
 }
 

@@ -35,6 +35,8 @@ struct Params {
     double *y;
     int64_t m, n;
     int x_vec;                 // x is 16-byte aligned: x segments load as double2
+    int nyx;                   // tilespmv_run_scatter: peers' y copies (0: plain run)
+    double *yx[kMaxScatter];   // each row of y is also stored to yx[t][row], t < nyx
     int64_t blob_bytes, num_items;  // sizes for the TSP_CHECKED build's bounds checks
     int slot_bytes;
     const int32_t *xc_cols;    // GATHER: the columns of the shared-memory x cache
@@ -195,6 +197,7 @@ __device__ __forceinline__ void fma_if(bool pred, double a, double b, double &ac
 struct KernelChoice {
     const char *name;
     void (*fn)(Params);
+    void (*fn_scatter)(Params);  // the same kernel storing y to the peer copies too (tilespmv_run_scatter)
     int threads, smem;
     int slot_bytes;   // item budget the schedule must respect
     int item_tiles;   // tiles per item (x stage segments)

@@ -148,6 +148,19 @@ __device__ __forceinline__ double rem_product(const Params &p, int k, int e, uin
     return k < e ? pr : 0.0;
 }
 
+// y[row] = v, and the same value into every peer copy of y (the fused
+// scatter epilogue of tilespmv_run_scatter: the next iterate's rows stored
+// straight into the peers' x over NVLink; nyx = 0 for a plain run)
+// (SC: the scatter instantiation of each kernel; the plain one stores y only)
+template <bool SC>
+__device__ __forceinline__ void store_y(const Params &p, int64_t row, double v) {
+    p.y[row] = v;
+    if (SC) {
+#pragma unroll 1
+        for (int t = 0; t < p.nyx; ++t) p.yx[t][row] = v;
+    }
+}
+
 // Flat remainder pass for one tile row (rows <= 16, row pointers at
 // rq): rows of <= kShortRow products two lanes per row, longer rows a
 // half-warp per row (two rows at a time, the whole warp for the last one)
@@ -257,7 +270,7 @@ __device__ __forceinline__ bool remainder(const Params &p, uint32_t rpS, uint32_
 // are summed by the whole warp with an xor tree.  y is written once per row.
 // A tile row's sums depend only on its own entries, so grouping never
 // changes a bit of y.
-template <bool PRE>
+template <bool PRE, bool SC>
 __device__ __forceinline__ bool group_item(const Params &p, const WItem &it, uint32_t slot, uint64_t x_policy,
                                            uint32_t xcS, int lane) {
     const int ntr = (int)(it.jt_rows_pay & 0xFFu);
@@ -314,7 +327,7 @@ __device__ __forceinline__ bool group_item(const Params &p, const WItem &it, uin
             }
         }
         const int64_t row = 16 * ((int64_t)it.I + gg) + r;
-        if (gg < ntr && row < p.m) p.y[row] = acc;
+        if (gg < ntr && row < p.m) store_y<SC>(p, row, acc);
     }
     return PRE && has_rem;
 }
@@ -444,11 +457,11 @@ __device__ __forceinline__ void issue_x(const Params &p, int J, int nt, uint32_t
 // flight into `xs`: remainder, tiles, y (or the split-row carry).  Returns
 // true if the slot was written (products), so the caller fences the generic
 // proxy writes before the next TMA copy into the slot.
-template <bool PRE>
+template <bool PRE, bool SC>
 __device__ __forceinline__ bool compute_item(const Params &p, const WItem &it, uint32_t slot, uint32_t xs,
                                              uint64_t x_policy, uint32_t xcS, int lane, double &carry) {
     if (it.jt_rows_pay & 0xFFu)  // row-group item (no tiles, no x segments)
-        return group_item<PRE>(p, it, slot, x_policy, xcS, lane);
+        return group_item<PRE, SC>(p, it, slot, x_policy, xcS, lane);
     const int h = lane >> 4, r = lane & 15;
     const uint32_t total = it.val_tot >> 16;
     // 2. fused CSR remainder, while the x segments land
@@ -488,14 +501,14 @@ __device__ __forceinline__ bool compute_item(const Params &p, const WItem &it, u
     // 4. y, once per row
     const int64_t row = 16 * (int64_t)it.I + lane;
     if (it.split < 0) {
-        if (lane < 16 && row < p.m) p.y[row] = acc;
+        if (lane < 16 && row < p.m) store_y<SC>(p, row, acc);
     } else if (!((it.part_nt >> 30) & 1)) {  // a group of parts runs here, in part order
         carry += acc;
     } else {
         const double sum = carry + acc;
         carry = 0.0;
         if ((it.part_nt >> 29) & 1) {  // the row's only group
-            if (lane < 16 && row < p.m) p.y[row] = sum;
+            if (lane < 16 && row < p.m) store_y<SC>(p, row, sum);
         } else {  // hub row: one partial per group, the last group sums them in order
             const int2 si = p.split_info[it.split];
             const int ngroups = (si.y + kLocalParts - 1) / kLocalParts;
@@ -522,7 +535,7 @@ __device__ __forceinline__ bool compute_item(const Params &p, const WItem &it, u
                     for (int i = 0; i < 4; ++i) s += v[i];
                 }
                 s += __shfl_xor_sync(FULL, s, 16);
-                if (lane < 16 && row < p.m) p.y[row] = s;
+                if (lane < 16 && row < p.m) store_y<SC>(p, row, s);
                 if (lane == 0) p.counters[it.split] = 0;  // ready for the next run
             }
         }
@@ -533,7 +546,7 @@ __device__ __forceinline__ bool compute_item(const Params &p, const WItem &it, u
 // Dense-row kernel: WARPS warps per CTA, several CTAs per SM, one blob in
 // flight per warp; each warp owns a contiguous, cost-balanced, row-aligned
 // item chunk (schedule.cu) and its start record (chunk + first item).
-template <int WARPS, int SLOT, int MINB>
+template <int WARPS, int SLOT, int MINB, bool SC>
 __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, MINB) tilespmv_fp64_warp(const Params p) {
     using Cfg = WarpCfg<WARPS, SLOT>;
     extern __shared__ __align__(128) uint8_t smem[];
@@ -578,7 +591,7 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, MINB) tilespmv
         }
         TSP_STAMP(gw, k - kbeg, 1);
         TSP_INFO(gw, k - kbeg, k, it);
-        if (compute_item<false>(p, it, slot, xs, x_policy, 0u, lane, carry))
+        if (compute_item<false, SC>(p, it, slot, xs, x_policy, 0u, lane, carry))
             fence_proxy_async();  // products written to the slot before the next TMA copy into it
         __syncwarp();  // slot and x scratch free for the next item
         TSP_STAMP(gw, k - kbeg, 3);
@@ -598,7 +611,7 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT>::kThreads, MINB) tilespmv
 // XC > 0 (GATHER): an x cache of the XC most-gathered remainder columns in
 // shared memory, filled at launch (schedule.cu: blob columns ~slot), and
 // every remainder through the product pre-pass
-template <int WARPS, int SLOT, int XT, int XC>
+template <int WARPS, int SLOT, int XT, int XC, bool SC>
 __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT, XT, XC>::kThreads, 1) tilespmv_fp64_sm(const Params p) {
     using Cfg = WarpCfg<WARPS, SLOT, XT, XC>;
     constexpr bool PRE = XC > 0;
@@ -694,7 +707,7 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT, XT, XC>::kThreads, 1) til
         }
         TSP_STAMP(gw, j, 1);
         TSP_INFO(gw, j, k, it);
-        if (compute_item<PRE>(p, it, slot, xs, x_policy, xcS, lane, carry))
+        if (compute_item<PRE, SC>(p, it, slot, xs, x_policy, xcS, lane, carry))
             fence_proxy_async();  // products written to the slot before the next TMA copy into it
         __syncwarp();  // slot and x scratch free for the next item
         TSP_STAMP(gw, j, 3);
@@ -712,16 +725,19 @@ __global__ void __launch_bounds__(WarpCfg<WARPS, SLOT, XT, XC>::kThreads, 1) til
 KernelChoice kernel_choice(int kernel) {
     if (kernel == TILESPMV_KERNEL_DENSE_ROWS) {
         using Cfg = WarpCfg<4, 10752>;
-        return {"tilespmv_fp64_warp<4,10752>", tilespmv_fp64_warp<4, 10752, 4>, Cfg::kThreads, (int)Cfg::kSmem,
+        return {"tilespmv_fp64_warp<4,10752>", tilespmv_fp64_warp<4, 10752, 4, false>,
+                tilespmv_fp64_warp<4, 10752, 4, true>, Cfg::kThreads, (int)Cfg::kSmem,
                 10752, kItemTiles, false, 0};
     }
     if (kernel == TILESPMV_KERNEL_GATHER) {
         using Cfg = WarpCfg<32, kGatherSlot, 4, kXCache>;
-        return {"tilespmv_fp64_sm<32,3136,4,2048>", tilespmv_fp64_sm<32, kGatherSlot, 4, kXCache>, Cfg::kThreads,
+        return {"tilespmv_fp64_sm<32,3136,4,2048>", tilespmv_fp64_sm<32, kGatherSlot, 4, kXCache, false>,
+                tilespmv_fp64_sm<32, kGatherSlot, 4, kXCache, true>, Cfg::kThreads,
                 (int)Cfg::kSmem, kGatherSlot, 4, true, kXCache};
     }
     using Cfg = WarpCfg<32, 4608>;
-    return {"tilespmv_fp64_sm<32,4608>", tilespmv_fp64_sm<32, 4608, kItemTiles, 0>, Cfg::kThreads, (int)Cfg::kSmem,
+    return {"tilespmv_fp64_sm<32,4608>", tilespmv_fp64_sm<32, 4608, kItemTiles, 0, false>,
+            tilespmv_fp64_sm<32, 4608, kItemTiles, 0, true>, Cfg::kThreads, (int)Cfg::kSmem,
             4608, kItemTiles, true, 0};
 }
 

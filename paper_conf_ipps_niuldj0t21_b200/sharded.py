@@ -371,3 +371,70 @@ class ChunkedAllGatherSpMV:
         for dst, h in staged:
             dst.copy_(h)
         return x_next
+
+
+# ----------------------------------------------------------------------------
+# Scatter fused into the SpMV epilogue (SURVEY §8(e), B200-native
+# improvement 2): the kernel stores every y row both into the rank's own
+# x_{k+1} and, through CUDA IPC mappings (NVLink peer memory on a multi-GPU
+# node), straight into every peer's x_{k+1} at this rank's row offset
+# (tilespmv_run_scatter), so no collective moves y at all; one barrier per
+# step orders the iterations.  Two IPC buffers per rank ping-pong between
+# x_k and x_{k+1}.  Every row is still summed exactly as on one GPU.
+# ----------------------------------------------------------------------------
+
+class FusedScatterSpMV:
+    """One rank's side of the fused-scatter iterated SpMV.
+
+    M: this rank's TiledMatrix (its row slice, global columns); x0: the
+    replicated start vector (length n, CUDA)."""
+
+    def __init__(self, M, bounds, rank: int, world: int, x0, group=None):
+        import torch.distributed as dist
+        from .tilespmv import IpcBuffer
+        self.M, self.rank, self.world, self.group = M, rank, world, group
+        self.a, self.b = int(bounds[rank]), int(bounds[rank + 1])
+        n = int(x0.numel())
+        self.bufs = [IpcBuffer(n), IpcBuffer(n)]
+        self.bufs[0].tensor.copy_(x0)
+        mine = [buf.handle for buf in self.bufs]
+        allh = [None] * world
+        if world > 1:
+            dist.all_gather_object(allh, mine, group=group)
+        else:
+            allh = [mine]
+        self.opened = [IpcBuffer.open(allh[q][i]) for q in range(world) if q != rank for i in range(2)]
+        # peers' buffer i at this rank's row offset (opened: peer-major, buffer-minor)
+        self.peers = [[self.opened[2 * j + i] + 8 * self.a for j in range(world - 1)] for i in range(2)]
+        self.k = 0
+        self._barrier()
+
+    def _barrier(self):
+        import torch
+        import torch.distributed as dist
+        torch.cuda.current_stream().synchronize()
+        if self.world > 1 and dist.is_available() and dist.is_initialized():
+            dist.barrier(group=self.group)
+
+    @property
+    def x(self):
+        """The current iterate (every rank holds all of it)."""
+        return self.bufs[self.k % 2].tensor
+
+    def step(self):
+        """x_{k+1} = A x_k on every rank; returns x_{k+1}."""
+        cur, nxt = self.bufs[self.k % 2], self.bufs[(self.k + 1) % 2]
+        self.M.run_scatter(cur.tensor, nxt.tensor[self.a:self.b], self.peers[(self.k + 1) % 2])
+        self._barrier()  # every rank's stores into every x_{k+1} are complete
+        self.k += 1
+        return nxt.tensor
+
+    def close(self):
+        from .tilespmv import IpcBuffer
+        self._barrier()
+        for q in self.opened:
+            IpcBuffer.close(q)
+        self.opened = []
+        self._barrier()
+        for buf in self.bufs:
+            buf.free()

@@ -25,7 +25,8 @@ EXPORTED_SYMBOLS = ["tilespmv_create_from_csr", "tilespmv_run", "tilespmv_run_ho
                     "tilespmv_destroy", "tilespmv_get_info", "tilespmv_export_size",
                     "tilespmv_export", "tilespmv_status_string", "tilespmv_last_error",
                     "tilespmv_launch_shape", "tilespmv_kernel_name", "tilespmv_cg",
-                    "tilespmv_auto_kernel"]
+                    "tilespmv_auto_kernel", "tilespmv_run_scatter", "tilespmv_ipc_alloc",
+                    "tilespmv_ipc_free", "tilespmv_ipc_open", "tilespmv_ipc_close"]
 
 
 class TileSpMVError(RuntimeError):
@@ -93,6 +94,15 @@ def load(build_if_missing: bool = True):
     if hasattr(L, "tilespmv_auto_kernel"):  # (absent from round-1 builds used in A/B runs)
         L.tilespmv_auto_kernel.argtypes = [i64, i64, i64, i64]
         L.tilespmv_auto_kernel.restype = i32
+    if hasattr(L, "tilespmv_run_scatter"):  # (absent from older builds used in A/B runs)
+        L.tilespmv_run_scatter.argtypes = [p, p, p, ctypes.POINTER(p), i32, p]
+        L.tilespmv_ipc_alloc.argtypes = [i64, ctypes.POINTER(p), p]
+        L.tilespmv_ipc_free.argtypes = [p]
+        L.tilespmv_ipc_open.argtypes = [p, ctypes.POINTER(p)]
+        L.tilespmv_ipc_close.argtypes = [p]
+        for name in ("tilespmv_run_scatter", "tilespmv_ipc_alloc", "tilespmv_ipc_free", "tilespmv_ipc_open",
+                     "tilespmv_ipc_close"):
+            getattr(L, name).restype = ctypes.c_int
     L.tilespmv_kernel_name.argtypes = [p]
     L.tilespmv_kernel_name.restype = ctypes.c_char_p
     for name in ("tilespmv_create_from_csr", "tilespmv_run", "tilespmv_run_host",
@@ -189,6 +199,23 @@ class TiledMatrix:
         _check(rc, "tilespmv_run")
         return y
 
+    def run_scatter(self, x, y, peer_ptrs, stream=None):
+        """y = A @ x, every row also stored to each peer pointer (device
+        addresses of m doubles each, e.g. IpcBuffer.open peers at this rank's
+        row offset): tilespmv_run_scatter.  Asynchronous."""
+        import torch
+        if not (x.is_cuda and y.is_cuda and x.dtype == torch.float64 and y.dtype == torch.float64
+                and x.is_contiguous() and y.is_contiguous()):
+            raise TileSpMVError("x and y must be contiguous float64 CUDA tensors")
+        if x.numel() != self.n or y.numel() != self.m:
+            raise TileSpMVError(f"shape mismatch: A is {self.m}x{self.n}, x {x.numel()}, y {y.numel()}")
+        arr = (ctypes.c_void_p * max(len(peer_ptrs), 1))(*[int(q) for q in peer_ptrs])
+        rc = load().tilespmv_run_scatter(self._h, x.data_ptr() if self.n else None,
+                                         y.data_ptr() if self.m else None, arr, len(peer_ptrs),
+                                         _stream_ptr(stream))
+        _check(rc, "tilespmv_run_scatter")
+        return y
+
     def run_host(self, hx, hy, stream=None):
         """Host buffers (pinned torch CPU tensors or numpy arrays): H2D, run, D2H, sync."""
         def ptr(a):
@@ -260,3 +287,44 @@ class TiledMatrix:
 
     def __exit__(self, *a):
         self.close()
+
+
+class IpcBuffer:
+    """A cudaMalloc'd float64 buffer shareable with other processes (CUDA IPC
+    through the ABI's tilespmv_ipc_*): .tensor is a zero-copy torch view,
+    .handle the 64-byte IPC handle; IpcBuffer.open(handle) maps a peer's."""
+
+    def __init__(self, n: int):
+        _require_cuda()
+        L = load()
+        p, h = ctypes.c_void_p(), ctypes.create_string_buffer(64)
+        _check(L.tilespmv_ipc_alloc(8 * max(n, 1), ctypes.byref(p), h), "tilespmv_ipc_alloc")
+        self.ptr, self.n, self.handle = p.value, n, h.raw
+        self.tensor = _device_tensor(self.ptr, n)
+
+    @staticmethod
+    def open(handle: bytes) -> int:
+        """Maps a peer's buffer; returns its device address (close with close())."""
+        p = ctypes.c_void_p()
+        _check(load().tilespmv_ipc_open(ctypes.create_string_buffer(handle, 64), ctypes.byref(p)), "tilespmv_ipc_open")
+        return p.value
+
+    @staticmethod
+    def close(ptr: int):
+        _check(load().tilespmv_ipc_close(ctypes.c_void_p(ptr)), "tilespmv_ipc_close")
+
+    def free(self):
+        if self.ptr:
+            self.tensor = None
+            _check(load().tilespmv_ipc_free(ctypes.c_void_p(self.ptr)), "tilespmv_ipc_free")
+            self.ptr = None
+
+
+def _device_tensor(ptr: int, n: int):
+    """A float64 CUDA tensor viewing n doubles at device address ptr (no copy)."""
+    import torch
+
+    class _View:
+        __cuda_array_interface__ = {"shape": (n,), "typestr": "<f8", "data": (ptr, False), "version": 3,
+                                    "strides": None}
+    return torch.as_tensor(_View(), device=torch.device("cuda", torch.cuda.current_device()))

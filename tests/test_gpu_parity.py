@@ -402,3 +402,34 @@ def test_gather_xcache(cuda_device, name):
         assert_spmv_close(y, yref, absy, f"{name}/GATHER x cache")
     with TM.from_host_csr(A, mode="DEFERRED", device=cuda_device, kernel="SM_QUEUE") as M:
         assert M.info()["xcache_cols"] == 0
+
+
+def test_run_scatter_writes_every_copy(cuda_device):
+    """tilespmv_run_scatter (the fused scatter epilogue): y and every peer
+    copy hold the plain run's y bit for bit, for 0, 1 and 7 peers; a peer
+    pointer at an offset inside a longer buffer touches only its m rows."""
+    import torch
+    TM = tm()
+    for name in ("stencil27_21", "rmat12", "mixed_small"):
+        A, x = gen.make(name)
+        xd = torch.from_numpy(x).to(cuda_device)
+        with TM.from_host_csr(A, device=cuda_device) as M:
+            y0 = M.run(xd).cpu().numpy()
+            for npeer in (0, 1, 7):
+                bufs = [torch.full((A.m + 40,), float("nan"), dtype=torch.float64, device=cuda_device)
+                        for _ in range(npeer)]
+                y = torch.empty(A.m, dtype=torch.float64, device=cuda_device)
+                M.run_scatter(xd, y, [t.data_ptr() + 8 * 24 for t in bufs])
+                torch.cuda.synchronize()
+                assert np.array_equal(y.cpu().numpy().view(np.uint64), y0.view(np.uint64))
+                for t in bufs:
+                    h = t.cpu().numpy()
+                    assert np.array_equal(h[24:24 + A.m].view(np.uint64), y0.view(np.uint64))
+                    assert np.isnan(h[:24]).all() and np.isnan(h[24 + A.m:]).all()
+    from paper_conf_ipps_niuldj0t21_b200 import TileSpMVError
+    A, x = gen.make("lap2d_37x29")
+    with TM.from_host_csr(A, device=cuda_device) as M:
+        xd = torch.from_numpy(x).to(cuda_device)
+        y = torch.empty(A.m, dtype=torch.float64, device=cuda_device)
+        with pytest.raises(TileSpMVError):
+            M.run_scatter(xd, y, [y.data_ptr()] * 8)

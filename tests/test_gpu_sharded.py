@@ -40,8 +40,8 @@ def _rank_worker(rank, world, port, name, exchange, q):
         import torch
         import torch.distributed as dist
         from paper_conf_ipps_niuldj0t21_b200 import TiledMatrix
-        from paper_conf_ipps_niuldj0t21_b200.sharded import (ChunkedAllGatherSpMV, HaloSpMV, ShardedSpMV,
-                                                             build_shard_handles, chunk_bounds,
+        from paper_conf_ipps_niuldj0t21_b200.sharded import (ChunkedAllGatherSpMV, FusedScatterSpMV, HaloSpMV,
+                                                             ShardedSpMV, build_shard_handles, chunk_bounds,
                                                              partition_tile_rows, plan_halo)
         os.environ["MASTER_ADDR"] = "127.0.0.1"
         os.environ["MASTER_PORT"] = str(port)
@@ -69,6 +69,13 @@ def _rank_worker(rank, world, port, name, exchange, q):
                 xk = sh.step(xk).clone()
                 torch.cuda.synchronize()
                 outs.append(xk.cpu().numpy())
+            M.close()
+        elif exchange == "fused":  # the kernel stores y into every rank's x_{k+1} over CUDA IPC
+            (M,), md, kn = build_shard_handles(create, [(a0, a1)], S.nnz)
+            F = FusedScatterSpMV(M, b, rank, world, torch.from_numpy(x).to(dev))
+            for _ in range(ITERS):
+                outs.append(F.step().cpu().numpy())
+            F.close()
             M.close()
         elif exchange == "chunked":  # all-gather overlapped with the SpMV, 3 chunks per rank
             cb = chunk_bounds(b, 3)[rank]
@@ -106,7 +113,7 @@ def _rank_worker(rank, world, port, name, exchange, q):
         q.put((rank, None, traceback.format_exc(), None))
 
 
-@pytest.mark.parametrize("exchange", ["allgather", "halo", "chunked"])
+@pytest.mark.parametrize("exchange", ["allgather", "halo", "chunked", "fused"])
 @pytest.mark.parametrize("name", ["stencil27_40", "rmat12", "lap2d_37x29", "mixed_small"])
 def test_sharded_cuda_iterates_bitwise_equal_one_gpu(cuda_device, name, exchange):
     import torch
@@ -142,7 +149,7 @@ def test_sharded_cuda_iterates_bitwise_equal_one_gpu(cuda_device, name, exchange
         for k in range(ITERS):
             got = outs[k] if exchange == "halo" else outs[k][b[r]:b[r + 1]]
             assert np.array_equal(got.view(np.uint64), ref[k][b[r]:b[r + 1]].view(np.uint64)), (name, exchange, r, k)
-            if exchange in ("allgather", "chunked"):  # every rank holds the whole iterate
+            if exchange in ("allgather", "chunked", "fused"):  # every rank holds the whole iterate
                 assert np.array_equal(outs[k].view(np.uint64), ref[k].view(np.uint64))
 
 
