@@ -500,7 +500,11 @@ def measure_sharded(workload, mode, steps, warmup, dev, rank, P, group, exchange
                    boundary SpMVs run after it lands (SURVEY 8(f) f1);
       chunked   -- the all-gather in CHUNKS pieces, each rank's chunk i sent
                    to every peer (NCCL send/recv) while chunk i + 1 computes
-                   (SURVEY 8(e), B200-native improvement 1).
+                   (SURVEY 8(e), B200-native improvement 1);
+      fused     -- no collective: the SpMV kernel stores its y rows into every
+                   rank's x_{k+1} through CUDA IPC / NVLink mappings
+                   (tilespmv_run_scatter), one barrier per step (SURVEY 8(e),
+                   B200-native improvement 2).
     x stays fixed across steps (the exchanged rows equal what is there), so
     the timed work is exactly one iteration's and values stay finite.  Times
     are device events on the compute stream, max over ranks: the step, the
@@ -508,8 +512,8 @@ def measure_sharded(workload, mode, steps, warmup, dev, rank, P, group, exchange
     import torch
     import torch.distributed as dist
     from paper_conf_ipps_niuldj0t21_b200 import TiledMatrix
-    from paper_conf_ipps_niuldj0t21_b200.sharded import (ChunkedAllGatherSpMV, HaloSpMV, ShardedSpMV,
-                                                         build_shard_handles, chunk_bounds, plan_halo)
+    from paper_conf_ipps_niuldj0t21_b200.sharded import (ChunkedAllGatherSpMV, FusedScatterSpMV, HaloSpMV,
+                                                         ShardedSpMV, build_shard_handles, chunk_bounds, plan_halo)
     from synthetic import gen
 
     t0 = time.perf_counter()
@@ -556,7 +560,24 @@ def measure_sharded(workload, mode, steps, warmup, dev, rank, P, group, exchange
                 e[2 + 2 * i].record(stream)
         return f
 
-    if exchange in ("halo", "chunked"):
+    if exchange == "fused":
+        F = FusedScatterSpMV(mats[0], bounds, rank, P, x, group=group)
+        Mf = mats[0]
+
+        def step(ev=None):
+            cur[0] = ev
+            if ev is not None:
+                ev[0].record(stream)
+                ev[1].record(stream)
+            # x stays fixed: every step reads buffer 0 and scatters into buffer 1
+            Mf.run_scatter(F.bufs[0].tensor, F.bufs[1].tensor[a:b], F.peers[1])
+            if ev is not None:
+                ev[2].record(stream)
+            F._barrier()
+            if ev is not None:
+                ev[-1].record(stream)
+        y = F.bufs[1].tensor
+    elif exchange in ("halo", "chunked"):
         y = torch.empty(n, dtype=torch.float64, device=dev)
         if exchange == "halo":
             H = HaloSpMV(plan, [timed_run(i, M) for i, M in enumerate(mats)], group=group, host_staging=one_gpu)
@@ -624,7 +645,11 @@ def measure_sharded(workload, mode, steps, warmup, dev, rank, P, group, exchange
                         "frac": achieved / peak, "traffic": None, "peak_source": peak_src,
                         "alg_bytes_per_launch": infos[dom]["alg_bytes"],
                         "kernel": mats[dom].kernel_name() + (" (interior part)" if exchange == "halo" else "")}}
-    if exchange == "chunked":
+    if exchange == "fused":
+        res["exchange"] = {"kind": "fused scatter epilogue (y rows stored into every rank's x_{k+1} over CUDA IPC / "
+                                   "NVLink; one barrier per step, no collective)",
+                           "bytes_per_rank": 8 * (b - a) * (P - 1)}
+    elif exchange == "chunked":
         res["exchange"] = {"kind": f"all-gather in {CHUNKS} chunks (NCCL send/recv of chunk i while chunk i+1 "
                                    "computes)", "bytes_per_rank": 8 * (n - (b - a))}
     elif exchange == "halo":
@@ -642,7 +667,7 @@ def measure_sharded(workload, mode, steps, warmup, dev, rank, P, group, exchange
         def e2e_step():
             x[a:b].copy_(hx, non_blocking=True)
             step()
-            hy.copy_(y[a:b] if exchange in ("halo", "chunked") else sh.local_out(), non_blocking=True)
+            hy.copy_(y[a:b] if exchange in ("halo", "chunked", "fused") else sh.local_out(), non_blocking=True)
             stream.synchronize()
 
         for _ in range(2):
@@ -659,6 +684,8 @@ def measure_sharded(workload, mode, steps, warmup, dev, rank, P, group, exchange
                       "ms_per_step": e2e_s * 1e3, "steps": e2e_steps,
                       "call": "per rank: H2D own x rows -> step (exchange + SpMV) -> D2H own y rows; "
                               "bytes summed over ranks, time max over ranks"}
+    if exchange == "fused":
+        F.close()
     for M in mats:
         M.close()
     return res
@@ -691,7 +718,7 @@ def run_ours(args):
         res = measure_sharded(args.workload, args.mode, args.steps, args.warmup, dev, rank, P, group,
                               args.exchange, args.e2e_steps, one_gpu)
         if not args.no_secondary:  # the other exchange, same shards
-            others = [e for e in ("allgather", "halo", "chunked") if e != args.exchange]
+            others = [e for e in ("allgather", "halo", "chunked", "fused") if e != args.exchange]
             for other in others:
                 r2 = measure_sharded(args.workload, args.mode, args.steps, args.warmup, dev, rank, P, group,
                                      other, 0, one_gpu)
@@ -747,7 +774,8 @@ def run_ours(args):
                "step": ({"allgather": "SpMV + NCCL all-gather of y",
                          "halo": "halo exchange overlapped with the interior SpMV + boundary SpMVs",
                          "chunked": f"{CHUNKS} chunk SpMVs, each chunk sent to every peer while the next "
-                                    "computes"}[args.exchange]
+                                    "computes",
+                         "fused": "SpMV storing y into every rank's x_{k+1} (scatter epilogue) + barrier"}[args.exchange]
                         if P > 1 else "one SpMV launch"),
                "timing": {"launch_mode": res["launch_mode"], "replicas_rotated": res["reps"],
                           "host_enqueue_us_per_step": res.get("host_enqueue_us_per_step")},
@@ -777,9 +805,9 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--workload", default=DEFAULT_WORKLOAD)
     ap.add_argument("--mode", default="DEFERRED", choices=["ADPT", "DEFERRED", "AUTO", "FORCE_CSR", "BYTES"])
-    ap.add_argument("--exchange", default="allgather", choices=["allgather", "halo", "chunked"],
-                    help="N>1: all-gather of y (north star, default), the neighbour-only x exchange, or the all-gather in "
-                         "chunks overlapped with the SpMV; "
+    ap.add_argument("--exchange", default="allgather", choices=["allgather", "halo", "chunked", "fused"],
+                    help="N>1: all-gather of y (north star, default), the neighbour-only x exchange, the all-gather in "
+                         "chunks overlapped with the SpMV, or the fused scatter epilogue (no collective); "
                          "the others are timed as secondary entries")
     ap.add_argument("--e2e-steps", type=int, default=20)
     ap.add_argument("--no-cpu-baseline", action="store_true")
