@@ -54,6 +54,16 @@ def test_null_arguments_rejected_without_gpu():
     assert L.tilespmv_create_from_csr(ctypes.byref(h), -1, 1, 0, None, None, None, None, None) == -1
     assert L.tilespmv_create_from_csr(ctypes.byref(h), 1 << 31, 1, 0, None, None, None, None, None) == -3
     assert L.tilespmv_run(None, None, None, None) == -1
+    # the scatter epilogue and its IPC plumbing validate their arguments first
+    peers = (ctypes.c_void_p * 8)()
+    assert L.tilespmv_run_scatter(None, None, None, peers, 8, None) == -1   # more than 7 peers
+    assert L.tilespmv_run_scatter(None, None, None, None, 1, None) == -1    # NULL peer list
+    assert L.tilespmv_run_scatter(None, None, None, None, 0, None) == -1    # NULL handle
+    p = ctypes.c_void_p()
+    assert L.tilespmv_ipc_alloc(0, ctypes.byref(p), ctypes.create_string_buffer(64)) == -1
+    assert L.tilespmv_ipc_alloc(8, None, None) == -1
+    assert L.tilespmv_ipc_open(None, ctypes.byref(p)) == -1
+    assert L.tilespmv_ipc_close(None) == 0 and L.tilespmv_ipc_free(None) == 0  # NULL is a no-op
 
 
 def test_product_package_does_not_import_oracle():
